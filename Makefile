@@ -1,0 +1,36 @@
+# Native build: libdasp.so (product, sm_100a) + the test-side helper libraries.
+NVCC      ?= /usr/local/cuda/bin/nvcc
+ARCH      := -gencode arch=compute_100a,code=sm_100a
+NVFLAGS   := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-fopenmp -Xptxas -v
+CXXFLAGS  := -O3 -std=c++17 -fPIC -fopenmp -Wall -Wextra
+PKG       := paper_conf_sc_lu023_b200
+SRC       := $(PKG)/csrc
+OBJ       := build
+
+all: $(PKG)/libdasp.so oracle/liboracle.so synth/libsynth.so
+
+$(OBJ):
+	mkdir -p $(OBJ)
+
+$(OBJ)/builder.o: $(SRC)/builder.cpp $(SRC)/format.hpp include/dasp.h | $(OBJ)
+	g++ $(CXXFLAGS) -c $< -o $@
+
+$(OBJ)/kernels.o: $(SRC)/kernels.cu $(SRC)/kernels.cuh | $(OBJ)
+	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $(OBJ)/kernels.ptxas.txt || (cat $(OBJ)/kernels.ptxas.txt; false)
+
+$(OBJ)/api.o: $(SRC)/api.cu $(SRC)/kernels.cuh $(SRC)/format.hpp include/dasp.h | $(OBJ)
+	$(NVCC) $(NVFLAGS) -c $< -o $@
+
+$(PKG)/libdasp.so: $(OBJ)/builder.o $(OBJ)/kernels.o $(OBJ)/api.o
+	$(NVCC) $(ARCH) -shared -o $@ $^ -Xcompiler -fopenmp -lgomp
+
+oracle/liboracle.so: oracle/oracle.c
+	gcc -O2 -ffp-contract=off -fno-fast-math -fPIC -shared -o $@ $< -lm
+
+synth/libsynth.so: synth/synth.c
+	gcc -O2 -fopenmp -fPIC -shared -o $@ $< -lm
+
+clean:
+	rm -rf $(OBJ) $(PKG)/libdasp.so oracle/liboracle.so synth/libsynth.so
+
+.PHONY: all clean

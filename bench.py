@@ -1,0 +1,407 @@
+#!/usr/bin/env python3
+"""Benchmark of the DASP SpMV hot path on B200 (BASELINE.json metric:
+"FP64/FP16 SpMV GFLOPS & effective HBM GB/s (fraction of B200 peak), 1-8 GPUs").
+
+One step = one whole pass of the hot path: y_slab = alpha * A_slab * x (dasp_spmv: the fused
+long/medium/short kernel + the long-row finish kernel) over the configured synthetic matrix,
+and for N > 1 the in-place NCCL all-gather of the next x (iterated SpMV).
+Default workload (N = 1): configs[2], the power-law matrix with ~2e8 nnz in FP64.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--dtype f64|f16]
+                    [--variant mma|cudacore] [--impl dasp|reference]
+
+--impl reference times the CPU oracle (oracle/, test infrastructure) on a bounded sample of
+the same workload: this tier has no runnable reference implementation.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIG_DOC = {
+    "c1a": "random CSR n=4096, Poisson(16) row lengths (configs[0])",
+    "c1b": "class-coverage mix n=4096 (configs[0] variant)",
+    "c2": "3D 27-point stencil 128^3, 55,742,968 nnz (configs[1])",
+    "c2big": "3D 27-point stencil 162^3, 113,379,904 nnz (C2+)",
+    "c3": "power-law row lengths gamma=1.86 on [1,1e5] + 8 rows of 1e5, 12.5M rows, ~2.04e8 nnz (configs[2])",
+    "c5": "mixed-class mean row length ~64, row-partitioned (configs[4])",
+    "c6": "short rows only, len U{1..4} (mc2depi-like)",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--config", default="c3")
+    ap.add_argument("--scale", type=float, default=1.0)
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f16"])
+    ap.add_argument("--variant", default="mma", choices=["mma", "cudacore"])
+    ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget-s", type=float, default=12.0)
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+# ----------------------------------------------------------------------------------------------
+# clocks sampled DURING the timed region (B200_PROFILING.md clocks line)
+# ----------------------------------------------------------------------------------------------
+class ClockSampler:
+    REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown", 0x4: "sw_power_cap",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock", 0x2: "applications_clocks_setting",
+               0x1: "gpu_idle"}
+
+    def __init__(self, index):
+        self.index = index
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self.ok = True
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nvml = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.ok = False
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nvml.nvmlDeviceGetClockInfo(self.h, self.nvml.NVML_CLOCK_SM))
+                r = self.nvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def result(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------------------------------------
+# bytes per launch: CSR-equivalent and algorithmic (what the DASP format moves)
+# ----------------------------------------------------------------------------------------------
+def byte_model(info, dtype, beta_nonzero=False):
+    sv, sx, sy = (8, 8, 8) if dtype == "f64" else (2, 2, 4)
+    sa = sy
+    b1 = 2 if beta_nonzero else 1
+    m, n, nnz = info["m"], info["n"], info["nnz"]
+    G = 64 if dtype == "f64" else 256
+    ngp = info["n_groups_padded"]
+    nrb = info["rowblocks"]
+    nout = 64 * info["tiles_13"] + 32 * info["tiles_4"] + 64 * info["tiles_22"] + 128 * info["tiles_single"]
+    n_short_rows = info["n_len1"] + info["n_len2"] + info["n_len3"] + info["n_len4"]
+    main = (ngp * G * (sv + 4) + ngp * sa
+            + (info["nnz_reg_new"] + info["nnz_irreg"]) * (sv + 4) + 8 * (nrb + 1) + 8 * (8 * nrb + 1) + 4 * 8 * nrb
+            + info["row_medium"] * sy * b1
+            + info["nnz_short_new"] * (sv + 4) + 4 * nout + n_short_rows * sy * b1
+            + n * sx)
+    finish = (ngp * sa + 8 * (info["row_long"] + 1) + 4 * info["row_long"] + info["row_long"] * sy * b1
+              + info["n_empty"] * (4 + sy * b1))
+    csr_equiv = nnz * (sv + 4) + (m + 1) * 8 + n * sx + m * sy * b1
+    return {"main": main, "finish": finish, "total": main + finish, "csr_equiv": csr_equiv}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy burst)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_traffic(config, dtype, variant):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(f"{config}/{dtype}/{variant}")
+    except Exception:
+        return None
+
+
+# ----------------------------------------------------------------------------------------------
+# CPU oracle timing (cpu_baseline and --impl reference): bounded, strided row sample
+# ----------------------------------------------------------------------------------------------
+def row_sample(A, target_nnz):
+    import synth
+    if A.nnz <= target_nnz:
+        return A, 1
+    stride = int(np.ceil(A.nnz / target_nnz))
+    rows = np.arange(0, A.m, stride)
+    starts, ends = A.row_ptr[rows], A.row_ptr[rows + 1]
+    lens = ends - starts
+    rp = np.zeros(len(rows) + 1, dtype=np.int64)
+    np.cumsum(lens, out=rp[1:])
+    idx = np.repeat(starts - rp[:-1], lens) + np.arange(rp[-1])
+    return synth.CSR(len(rows), A.n, rp, A.col[idx], A.val[idx]), stride
+
+
+def time_oracle(A, x, dtype, budget_s):
+    import oracle
+    val = A.val if dtype == "f64" else A.val.astype(np.float16).astype(np.float64)
+    xv = x if dtype == "f64" else x.astype(np.float16).astype(np.float64)
+    oracle.spmv(A.row_ptr[:2], A.col[:1], val[:1], xv)  # load the library
+    reps, t_total = 0, 0.0
+    while t_total < budget_s and reps < 50:
+        t0 = time.perf_counter()
+        oracle.spmv(A.row_ptr, A.col, val, xv)
+        t_total += time.perf_counter() - t0
+        reps += 1
+    return t_total / reps, reps
+
+
+# ----------------------------------------------------------------------------------------------
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.gpus != world and world > 1:
+        print(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}", file=sys.stderr)
+    import synth
+
+    spec = synth.config(args.config, scale=args.scale)
+    workload = args.config if args.scale == 1.0 else f"{args.config}@{args.scale}"
+    metric = "FP64/FP16 SpMV GFLOPS & effective HBM GB/s (fraction of B200 peak), 1-8 GPUs"
+
+    if args.impl == "reference":
+        return run_reference(args, spec, workload, metric, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_lu023_b200 import dasp
+    from paper_conf_sc_lu023_b200.multigpu import SlabSpMV, build_slab
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    variant = dasp.DASP_VARIANT_MMA if args.variant == "mma" else dasp.DASP_VARIANT_CUDACORE
+
+    # ---- inputs: this rank's slab (whole matrix at N = 1), generated per row ----
+    t0 = time.perf_counter()
+    lens = synth.row_lengths(spec)
+
+    def gen_rows(r0, nr):
+        return synth.generate(spec, r0, nr)
+
+    def reduce_max(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    slab = build_slab(gen_rows, lens, rank, world, reduce_max)
+    gen_s = time.perf_counter() - t0
+    if args.dtype == "f16":
+        if world > 1:
+            raise SystemExit("FP16 multi-GPU is not part of the north star (x f16 vs y f32)")
+        slab.val = slab.val.astype(np.float16)
+    x_global = synth.vector(101, spec.n)
+
+    t1 = time.perf_counter()
+    if world == 1:
+        # single GPU: plain SpMV over resident inputs, y overwritten every step
+        plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
+                                     device=local, variant=variant)
+        xdt = torch.float64 if args.dtype == "f64" else torch.float16
+        ydt = torch.float64 if args.dtype == "f64" else torch.float32
+        xd = torch.from_numpy(x_global).to(xdt).to(dev)
+        yd = torch.zeros(slab.rows, dtype=ydt, device=dev)
+        stream = torch.cuda.current_stream(dev)
+        alpha = 1.0
+
+        def step():
+            dasp.dasp_spmv(plan, xd, yd, alpha, 0.0, stream, variant=variant, check=False)
+    else:
+        it = SlabSpMV(slab, world, rank, dev, args.dtype, variant=variant)
+        plan = it.plan
+        it.set_x(x_global)
+        alpha = 1.0 / max(slab.inf_norm, 1e-300)   # iterated SpMV stays bounded
+        stream = torch.cuda.current_stream(dev)
+
+        def step():
+            it.step(alpha)
+    plan_s = time.perf_counter() - t1
+    info = plan.info
+
+    # ---- warm-up, then K timed steps (barrier + synchronize on both sides, CUDA events) ----
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    dasp.dasp_plan_set_timing(plan, args.steps)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize(dev)
+    ms_total = ev0.elapsed_time(ev1)
+    if world > 1:
+        t = torch.tensor([ms_total], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+        dist.barrier()
+    kern = dasp.dasp_plan_read_timing(plan)
+    ms_step = ms_total / args.steps
+
+    nnz_total = int(lens.sum())
+    flops_step = 2.0 * nnz_total
+    gflops = flops_step / (ms_step * 1e-3) / 1e9
+    bm = byte_model(info, args.dtype)
+    # whole-job CSR-equivalent bytes: sum over ranks (slab models), else the local one
+    csr_bytes = bm["csr_equiv"]
+    if world > 1:
+        t = torch.tensor([float(csr_bytes)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t)
+        csr_bytes = float(t.item())
+    eff_gbs = csr_bytes / (ms_step * 1e-3) / 1e9
+
+    # ---- roofline of the dominant kernel (the fused main kernel), per launch ----
+    peak, peak_src = load_peaks()
+    main_ms, main_n = kern["dasp_main_kernel"]
+    fin_ms, fin_n = kern["dasp_finish_kernel"]
+    main_avg = main_ms / max(main_n, 1)
+    achieved = bm["main"] / (main_avg * 1e-3) / 1e9 if main_n else None
+    traffic = load_traffic(workload, args.dtype, args.variant)
+    roofline = {"kernel": "dasp_main_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak if achieved else None, "traffic": traffic,
+                "alg_bytes_per_launch": bm["main"], "avg_launch_ms": main_avg,
+                "share_of_step": (main_ms / max(main_n, 1)) / ms_step if main_n else None,
+                "finish_avg_ms": fin_ms / fin_n if fin_n else 0.0, "peak_source": peak_src}
+
+    # ---- e2e: the same metric through the C-ABI with HOST buffers (copies inside the timed region) ----
+    e2e = None
+    if world == 1 and args.e2e_steps > 0:
+        xdt_np = np.float64 if args.dtype == "f64" else np.float16
+        xh = torch.from_numpy(x_global.astype(xdt_np)).pin_memory()
+        yh = torch.empty(slab.rows, dtype=torch.float64 if args.dtype == "f64" else torch.float32).pin_memory()
+        dasp.dasp_spmv_host(plan, xh.data_ptr(), yh.data_ptr(), 1.0, 0.0, stream)
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            dasp.dasp_spmv_host(plan, xh.data_ptr(), yh.data_ptr(), 1.0, 0.0, stream)
+        dt = (time.perf_counter() - t0) / args.e2e_steps
+        e2e = {"value": flops_step / dt / 1e9, "unit": "GFLOPS", "ms_per_step": dt * 1e3,
+               "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
+               "d2h_bytes_per_step": int(yh.numel() * yh.element_size()), "api": "dasp_spmv_host"}
+
+    # ---- CPU oracle on the host cores (rank 0, N = 1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        A = synth.CSR(slab.rows, spec.n, slab.row_ptr, slab.col,
+                      slab.val.astype(np.float64) if args.dtype == "f16" else slab.val)
+        target = max(1, int(min(A.nnz, 1.5e8)))
+        S, stride = row_sample(A, target)
+        per, reps = time_oracle(S, x_global, args.dtype, args.cpu_budget_s)
+        cpu = {"value": 2.0 * S.nnz / per / 1e9, "unit": "GFLOPS", "cores": 1, "kind": "oracle",
+               "sample": f"every {stride}th row of {workload} ({S.m} rows, {S.nnz} nnz), {reps} reps, "
+                         f"single-thread double-double CSR loop"}
+
+    if rank == 0:
+        clocks = clk.result()
+        line = {
+            "metric": metric, "value": gflops, "unit": "GFLOPS", "n_gpus": world, "steps": args.steps,
+            "warmup": max(args.warmup, 3), "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+            "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config),
+                       "m": int(spec.m), "n": int(spec.n), "nnz": nnz_total, "variant": args.variant,
+                       "parallelism": f"row-slab x{world}" + (" + NCCL all-gather of x" if world > 1 else ""),
+                       "l2": "inputs larger than L2 (packed A streamed every step); x stays L2-resident "
+                             "across steps as in the paper's averaged back-to-back runs"},
+            "effective_gbs": eff_gbs, "effective_frac_of_peak": eff_gbs / peak,
+            "alg_gbs_step": bm["total"] * world / (ms_step * 1e-3) / 1e9 if world == 1 else None,
+            "gpu_launches": int(info["launches_per_spmv"]) * args.steps,
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,
+                     "rows": {"empty": info["n_empty"], "short": info["n_len1"] + info["n_len2"] + info["n_len3"]
+                              + info["n_len4"], "medium": info["row_medium"], "long": info["row_long"]},
+                     "nnz": {"short": info["nnz_short"], "medium": info["nnz_medium"], "long": info["nnz_long"]},
+                     "fill_rate": (info["nnz_long_new"] + info["nnz_reg_new"] + info["nnz_irreg"]
+                                   + info["nnz_short_new"]) / max(info["nnz"], 1) - 1.0,
+                     "medium_rb_per_warp": info["medium_rb_per_warp"]},
+        }
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_reference(args, spec, workload, metric, rank, world):
+    """--impl reference: the CPU oracle, bounded per-step sample of the same workload."""
+    if rank != 0:
+        return
+    import synth
+    lens = synth.row_lengths(spec)
+    nnz = int(lens.sum())
+    A = synth.generate(spec)
+    if args.dtype == "f16":
+        A.val = A.val.astype(np.float16).astype(np.float64)
+    x = synth.vector(101, spec.n)
+    total = args.steps + max(args.warmup, 3)
+    per_step_nnz = int(np.clip(90.0 * 2.5e8 / total, 2e5, nnz))   # ~90 s of oracle work in all
+    S, stride = row_sample(A, per_step_nnz)
+    import oracle
+    xv = x.astype(np.float16).astype(np.float64) if args.dtype == "f16" else x
+    for _ in range(max(args.warmup, 3)):
+        oracle.spmv(S.row_ptr, S.col, S.val, xv)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.spmv(S.row_ptr, S.col, S.val, xv)
+    dt = (time.perf_counter() - t0) / args.steps
+    v = 2.0 * S.nnz / dt / 1e9
+    line = {"impl": "reference", "metric": metric, "value": v, "unit": "GFLOPS", "n_gpus": world,
+            "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+            "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config), "nnz": nnz},
+            "cpu_baseline": {"value": v, "unit": "GFLOPS", "cores": 1, "kind": "oracle",
+                             "sample": f"every {stride}th row ({S.m} rows, {S.nnz} nnz) per step"},
+            "e2e": {"value": v, "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,208 @@
+/*
+ * dasp.h — C-ABI of the B200-native DASP SpMV hot path (libdasp.so).
+ *
+ * Operation (the hot path): general sparse matrix-vector multiply
+ *
+ *        y = alpha * A * x + beta * y
+ *
+ * with A in CSR (Val, ColIdx, RowPtr; §2.1 of /root/reference/PAPER.md, cited P:Lnnn)
+ * and x, y dense.  Alg. 1 defines the result; DASP (§3) computes it
+ * by binning rows into long / medium / short classes, packing each class into
+ * small padded MMA-shaped blocks, computing block inner products on the MMA
+ * units and writing y.  alpha/beta are the BLAS generalisation of Alg. 1 l.7
+ * asked for by BASELINE.json north_star (reading R16).
+ *
+ * Precisions (north_star):
+ *   DASP_R_64F : val f64, x f64, y f64; products and sums in f64 (DMMA m8n8k4).
+ *   DASP_R_16F : val f16 (IEEE binary16 bits), x f16, y f32; products exact in f32 and sums
+ *                in f32 (HMMA m16n8k16 f16->f32, R14/R15).  alpha/beta are applied
+ *                in f32.
+ *
+ * No torch or CUDA types cross this boundary: device pointers are plain pointers, the CUDA
+ * stream is passed as `void*` (a cudaStream_t, NULL = legacy default stream).
+ *
+ * Error behaviour: every entry point returns a dasp_status_t; nothing aborts or throws
+ * across the ABI.  Asynchronous device faults surface at the caller's next synchronisation.
+ */
+#ifndef DASP_H
+#define DASP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dasp_plan_s* dasp_plan_t;
+
+typedef enum { DASP_R_64F = 0, DASP_R_16F = 1 } dasp_dtype_t;
+
+typedef enum {
+    DASP_OK = 0,
+    DASP_ERR_INVALID_ARG = 1,   /* null/negative/aliasing argument (see each call)            */
+    DASP_ERR_INVALID_CSR = 2,   /* row_ptr[0]!=0, decreasing row_ptr, row_ptr[m]!=nnz, col out of range */
+    DASP_ERR_OUT_OF_MEMORY = 3, /* host or device allocation failed                           */
+    DASP_ERR_CUDA = 4,          /* a CUDA runtime call or kernel launch failed                */
+    DASP_ERR_UNSUPPORTED = 5,   /* e.g. dasp_spmv on a host-only plan                         */
+    DASP_ERR_INTERNAL = 6
+} dasp_status_t;
+
+/* Compute variant of the block inner products (north_star (3)): the same packed arrays are
+ * read either way; only the arithmetic differs.                                            */
+typedef enum {
+    DASP_VARIANT_DEFAULT = 0,   /* the plan's default (options.variant)                       */
+    DASP_VARIANT_MMA = 1,       /* DMMA m8n8k4 (FP64) / HMMA m16n8k16 (FP16) + diagonal
+                                   extraction by shuffles (Alg. 2-4)              */
+    DASP_VARIANT_CUDACORE = 2   /* per-lane FMA + warp-shuffle segmented reduction            */
+} dasp_variant_t;
+
+typedef struct {
+    int32_t device;             /* CUDA device ordinal; -1 = host-only plan (builder only)   */
+    int32_t variant;            /* default variant of dasp_spmv (DASP_VARIANT_MMA if 0)       */
+    int32_t validate;           /* 1: O(nnz) CSR validation (default); 0: skip               */
+    int32_t keep_host;          /* 1: keep the host staging copy of the packed arrays        */
+    int32_t medium_rb_per_warp; /* row-blocks per warp in the medium kernel (P:L271-273
+                                   LOOP_NUM); 0 = automatic                                   */
+    int32_t num_threads;        /* host builder threads; 0 = all available                   */
+} dasp_options_t;
+
+/* Fills `opts` with the defaults: device 0, MMA variant, validate, no keep_host, auto LOOP_NUM. */
+void dasp_options_default(dasp_options_t* opts);
+
+/* Plan statistics (Fig. 12's class shares; build cost). */
+typedef struct {
+    int64_t m, n, nnz;
+    int32_t dtype, device;
+    int64_t n_empty, n_len1, n_len2, n_len3, n_len4;   /* short classes + empty rows (R1)   */
+    int64_t row_medium, row_long;
+    int64_t rowblocks;                                 /* ceil(row_medium/8) (R7)   */
+    int64_t n_groups, n_groups_padded;                 /* long groups of 2*MMA_M*MMA_K      */
+    int64_t tiles_13, tiles_4, tiles_22, tiles_single; /* short tiles of 32 4-slot rows /128 singles */
+    int64_t nnz_long_new, nnz_reg_new, nnz_irreg, nnz_short_new; /* P:L156-164 array sizes  */
+    int64_t nnz_long, nnz_medium, nnz_short;           /* real nonzeros per class           */
+    int64_t device_bytes;                              /* device memory held by the plan    */
+    int64_t alg_bytes_beta0;                           /* bytes one dasp_spmv must move with
+                                                          beta == 0 (DESIGN.md §6 B_alg)     */
+    int64_t alg_bytes_beta1;                           /* ... with beta != 0                */
+    int32_t medium_rb_per_warp;
+    int32_t launches_per_spmv;                         /* kernels one dasp_spmv enqueues    */
+    double build_ms, upload_ms;                        /* host build; host->device upload   */
+} dasp_plan_info_t;
+
+/*
+ * dasp_plan_create — preprocessing (§3.2; Fig. 13 cost).
+ *
+ *   m, n, nnz : rows, columns, nonzeros (m, n, nnz >= 0; n <= INT32_MAX).  Rectangular ok.
+ *   row_ptr   : HOST int64[m+1], row_ptr[0] = 0, non-decreasing, row_ptr[m] = nnz.
+ *   col_idx   : HOST int32[nnz], 0 <= col < n.  Unsorted columns and duplicates are allowed
+ *               (duplicates are summed like any other entry).
+ *   val       : HOST double[nnz] (DASP_R_64F) or uint16_t[nnz] binary16 bits (DASP_R_16F).
+ *   opts      : NULL for defaults.
+ *
+ * Copies everything it needs (the caller may free the CSR on return), builds the DASP
+ * arrays on the host (multithreaded) and uploads them to `opts->device` (skipped for a
+ * host-only plan).  Returns INVALID_ARG (plan_out NULL, negative sizes, n > INT32_MAX,
+ * null arrays with nnz/m > 0), INVALID_CSR (validation failure), OUT_OF_MEMORY or CUDA.
+ * On error *plan_out is set to NULL.
+ */
+dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz,
+                               const int64_t* row_ptr, const int32_t* col_idx, const void* val,
+                               dasp_dtype_t dtype, const dasp_options_t* opts);
+
+/*
+ * dasp_spmv — the hot path (§3.3, Alg. 2-5):  y = alpha*A*x + beta*y.
+ *
+ *   x : DEVICE pointer on the plan's device, n elements (f64, or f16 bits for DASP_R_16F).
+ *   y : DEVICE pointer, m elements (f64, or f32 for DASP_R_16F).  Read only if beta != 0
+ *       (BLAS convention: beta == 0 overwrites y, NaNs in y do not propagate).
+ *   stream : cudaStream_t as void* (NULL = default stream).  Enqueue only; no host sync.
+ *
+ * alpha == 0 is a quick path (y = beta*y; A and x are not read).  m == 0 is a no-op.
+ * Calls on one plan must be stream-ordered (the long-row partial-sum workspace is shared).
+ * Returns INVALID_ARG (null plan; x == y; x NULL with n > 0 and alpha != 0; y NULL with
+ * m > 0), UNSUPPORTED (host-only plan) or CUDA (launch error).
+ */
+dasp_status_t dasp_spmv(dasp_plan_t plan, const void* x, void* y, double alpha, double beta,
+                        void* stream);
+
+/* As dasp_spmv with an explicit compute variant (dasp_variant_t). */
+dasp_status_t dasp_spmv_ex(dasp_plan_t plan, const void* x, void* y, double alpha, double beta,
+                           void* stream, int32_t variant);
+
+/*
+ * dasp_spmv_host — end-to-end call with HOST buffers: copies x (and y if beta != 0) to
+ * plan-owned device buffers, runs dasp_spmv on `stream`, copies y back and synchronises
+ * `stream`.  x_host: n elements, y_host: m elements, same element types as dasp_spmv.
+ * Pinned (page-locked) host buffers give full PCIe/C2C bandwidth; pageable ones work.
+ */
+dasp_status_t dasp_spmv_host(dasp_plan_t plan, const void* x_host, void* y_host, double alpha,
+                             double beta, void* stream);
+
+/* Frees every host and device buffer of the plan.  No call on the plan may be in flight
+ * (the call synchronises the plan's device).  NULL is accepted. */
+dasp_status_t dasp_plan_destroy(dasp_plan_t plan);
+
+/* Static string for a status code. */
+const char* dasp_status_string(dasp_status_t s);
+
+/* Fills *out with the plan's statistics. */
+dasp_status_t dasp_plan_get_info(dasp_plan_t plan, dasp_plan_info_t* out);
+
+/* Packed arrays of the plan (DESIGN.md §4 FORMAT), for the builder's byte-for-byte test. */
+typedef enum {
+    DASP_ARR_LONG_VAL = 0, DASP_ARR_LONG_COL, DASP_ARR_GROUP_PTR, DASP_ARR_LONG_OUT,
+    DASP_ARR_RB_PTR, DASP_ARR_REG_VAL, DASP_ARR_REG_COL, DASP_ARR_IRR_PTR, DASP_ARR_IRR_VAL,
+    DASP_ARR_IRR_COL, DASP_ARR_MED_OUT, DASP_ARR_SHORT_VAL, DASP_ARR_SHORT_COL,
+    DASP_ARR_SHORT_OUT, DASP_ARR_EMPTY_ROWS, DASP_ARR_COUNT
+} dasp_array_t;
+
+/*
+ * dasp_plan_copy_array — copies packed array `id` into HOST memory `dst` (device plans copy
+ * from device memory and synchronise; host-only or keep_host plans copy from the staging
+ * copy).  *bytes: in = capacity of dst, out = size of the array.  dst == NULL only queries
+ * the size.  Returns INVALID_ARG for an unknown id or too small a capacity.
+ */
+dasp_status_t dasp_plan_copy_array(dasp_plan_t plan, int32_t id, void* dst, int64_t* bytes);
+
+/*
+ * dasp_partition_rows — nnz-balanced contiguous row slabs for the multi-GPU mode (§8(e)):
+ * starts[0] = 0, starts[nparts] = m, starts[p] = the first row r with row_ptr[r] >=
+ * p*nnz/nparts (binary search on HOST row_ptr[m+1]).  nparts >= 1.
+ */
+dasp_status_t dasp_partition_rows(const int64_t* row_ptr, int64_t m, int32_t nparts, int64_t* starts);
+
+/*
+ * dasp_remap_columns — column remap of a slab into the padded, all-gathered x layout:
+ * global column c owned by part p (starts[p] <= c < starts[p+1]) becomes
+ * p*S + (c - starts[p]) with S = max_p (starts[p+1]-starts[p]).  In place on HOST col[nnz]
+ * (valid for square matrices partitioned like their rows).  Returns S through *stride.
+ */
+dasp_status_t dasp_remap_columns(int32_t* col, int64_t nnz, const int64_t* starts, int32_t nparts,
+                                 int64_t* stride);
+
+/* Kernel ids of the per-kernel timing below. */
+typedef enum {
+    DASP_K_MAIN = 0,      /* fused long-phase-1 + medium + short/single kernel (Alg. 2 l.1-16, Alg. 3-5) */
+    DASP_K_FINISH = 1,    /* long phase 2 (Alg. 2 l.17-25) + empty rows */
+    DASP_K_SCALE = 2,     /* alpha == 0 quick path */
+    DASP_K_COUNT = 3
+} dasp_kernel_t;
+
+/*
+ * Per-kernel device timing with CUDA events recorded on the launch stream (for bench.py's
+ * roofline line).  dasp_plan_set_timing(plan, capacity): record events for up to `capacity`
+ * subsequent dasp_spmv calls (0 disables).  dasp_plan_read_timing synchronises, returns for
+ * each kernel id the summed milliseconds and the number of timed launches, and resets.
+ */
+dasp_status_t dasp_plan_set_timing(dasp_plan_t plan, int32_t capacity);
+dasp_status_t dasp_plan_read_timing(dasp_plan_t plan, double* ms_per_kernel /* [DASP_K_COUNT] */,
+                                    int64_t* launches_per_kernel /* [DASP_K_COUNT] */);
+
+/* Library version string. */
+const char* dasp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DASP_H */

@@ -1,0 +1,408 @@
+// api.cu — the C-ABI of libdasp.so (include/dasp.h): plan creation (host build + upload),
+// the SpMV launch sequence, host-buffer end-to-end call, introspection, multi-GPU helpers
+// and per-kernel event timing.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "format.hpp"
+#include "kernels.cuh"
+
+using dasp::HostFormat;
+
+struct TimingRec {
+    int kernel;
+    cudaEvent_t a, b;
+};
+
+struct dasp_plan_s {
+    int dtype = 0, device = -1, variant = DASP_VARIANT_MMA, rbw = 1;
+    bool keep_host = false;
+    HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
+    void* d[DASP_ARR_COUNT] = {};
+    int64_t bytes[DASP_ARR_COUNT] = {};
+    void* d_partial = nullptr;
+    void* d_xh = nullptr;                 // dasp_spmv_host staging
+    void* d_yh = nullptr;
+    int64_t device_bytes = 0;
+    double build_ms = 0, upload_ms = 0;
+    int64_t w_long = 0, w_med = 0, w_short = 0;
+    // timing
+    int32_t timing_cap = 0, timing_calls = 0;
+    std::vector<TimingRec> recs;
+    std::vector<cudaEvent_t> pool;
+    size_t pool_used = 0;
+};
+
+namespace {
+
+int sx(int dtype) { return dtype == DASP_R_64F ? 8 : 2; }
+int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
+
+// LOOP_NUM of P:L271-273 (R11): row-blocks per warp from the number of medium rows
+int auto_rbw(int64_t row_medium) {
+    if (row_medium < 59990) return 1;
+    if (row_medium < 400000) return 2;
+    return 4;
+}
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+void free_device(dasp_plan_s* p) {
+    for (auto& ptr : p->d) {
+        if (ptr) cudaFree(ptr);
+        ptr = nullptr;
+    }
+    if (p->d_partial) cudaFree(p->d_partial);
+    if (p->d_xh) cudaFree(p->d_xh);
+    if (p->d_yh) cudaFree(p->d_yh);
+    p->d_partial = p->d_xh = p->d_yh = nullptr;
+    for (auto& r : p->recs) { (void)r; }
+    for (auto e : p->pool) cudaEventDestroy(e);
+    p->pool.clear();
+    p->recs.clear();
+}
+
+cudaEvent_t take_event(dasp_plan_s* p) {
+    if (p->pool_used == p->pool.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        p->pool.push_back(e);
+    }
+    return p->pool[p->pool_used++];
+}
+
+// launch wrapper recording events when timing is on
+template <typename F>
+cudaError_t timed(dasp_plan_s* p, int kernel, cudaStream_t s, bool on, F&& launch) {
+    if (!on) return launch();
+    cudaEvent_t a = take_event(p), b = take_event(p);
+    if (a) cudaEventRecord(a, s);
+    cudaError_t e = launch();
+    if (b) cudaEventRecord(b, s);
+    if (a && b) p->recs.push_back({kernel, a, b});
+    return e;
+}
+
+int64_t alg_bytes(const dasp_plan_s* p, bool beta) {
+    const HostFormat& f = p->host;
+    const int64_t s_v = f.geo.sv, s_x = sx(p->dtype), s_y = sy(p->dtype), s_a = s_y;
+    const int64_t nmp = f.nrb * 8;
+    const int64_t nout = 64 * f.t13 + 32 * f.t4 + 64 * f.t22 + 128 * f.ts;
+    int64_t b = 0;
+    b += f.n_groups_padded * f.geo.G * (s_v + 4) + 2 * f.n_groups_padded * s_a + 8 * (f.row_long + 1) + 4 * f.row_long;
+    b += (f.nnz_reg_new + f.nnz_irreg) * (s_v + 4) + 8 * (f.nrb + 1) + 8 * (nmp + 1) + 4 * nmp;
+    b += f.nnz_short_new * (s_v + 4) + 4 * nout;
+    b += 4 * f.n0;
+    b += f.n * s_x + f.m * s_y * (beta ? 2 : 1);
+    return b;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* dasp_version(void) { return "dasp-b200 0.1 (sm_100a)"; }
+
+void dasp_options_default(dasp_options_t* o) {
+    if (!o) return;
+    o->device = 0;
+    o->variant = DASP_VARIANT_MMA;
+    o->validate = 1;
+    o->keep_host = 0;
+    o->medium_rb_per_warp = 0;
+    o->num_threads = 0;
+}
+
+const char* dasp_status_string(dasp_status_t s) {
+    switch (s) {
+    case DASP_OK: return "DASP_OK";
+    case DASP_ERR_INVALID_ARG: return "DASP_ERR_INVALID_ARG";
+    case DASP_ERR_INVALID_CSR: return "DASP_ERR_INVALID_CSR";
+    case DASP_ERR_OUT_OF_MEMORY: return "DASP_ERR_OUT_OF_MEMORY";
+    case DASP_ERR_CUDA: return "DASP_ERR_CUDA";
+    case DASP_ERR_UNSUPPORTED: return "DASP_ERR_UNSUPPORTED";
+    case DASP_ERR_INTERNAL: return "DASP_ERR_INTERNAL";
+    }
+    return "DASP_ERR_UNKNOWN";
+}
+
+dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr,
+                               const int32_t* col_idx, const void* val, dasp_dtype_t dtype, const dasp_options_t* opts) {
+    if (!plan_out) return DASP_ERR_INVALID_ARG;
+    *plan_out = nullptr;
+    if (m < 0 || n < 0 || nnz < 0 || n > 0x7fffffffLL || m > 0x7fffffffLL) return DASP_ERR_INVALID_ARG;
+    if (dtype != DASP_R_64F && dtype != DASP_R_16F) return DASP_ERR_INVALID_ARG;
+    if (!row_ptr || (nnz > 0 && (!col_idx || !val))) return DASP_ERR_INVALID_ARG;
+    dasp_options_t o;
+    dasp_options_default(&o);
+    if (opts) o = *opts;
+    if (o.variant != DASP_VARIANT_MMA && o.variant != DASP_VARIANT_CUDACORE) o.variant = DASP_VARIANT_MMA;
+    if (o.validate && row_ptr[m] != nnz) return DASP_ERR_INVALID_CSR;
+
+    dasp_plan_s* p = new (std::nothrow) dasp_plan_s;
+    if (!p) return DASP_ERR_OUT_OF_MEMORY;
+    p->dtype = dtype;
+    p->device = o.device;
+    p->variant = o.variant;
+    p->keep_host = o.keep_host != 0 || o.device < 0;
+
+    auto t0 = std::chrono::steady_clock::now();
+    int st = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0);
+    auto t1 = std::chrono::steady_clock::now();
+    p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    if (st != DASP_OK) {
+        delete p;
+        return static_cast<dasp_status_t>(st);
+    }
+    HostFormat& f = p->host;
+    p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium);
+    p->w_long = f.n_groups_padded / f.geo.UG;
+    p->w_med = (f.nrb + p->rbw - 1) / p->rbw;
+    p->w_short = f.t13 + f.t4 + f.t22 + f.ts;
+    for (int a = 0; a < DASP_ARR_COUNT; ++a) p->bytes[a] = f.arr[a].bytes;
+
+    if (p->device >= 0) {
+        DeviceGuard guard(p->device);
+        for (int a = 0; a < DASP_ARR_COUNT; ++a) {
+            if (p->bytes[a] == 0) continue;
+            // 256 B alignment from cudaMalloc keeps every lane's 16/32 B vector load aligned
+            if (cudaMalloc(&p->d[a], static_cast<size_t>(p->bytes[a])) != cudaSuccess) {
+                free_device(p); f.release(); delete p;
+                return DASP_ERR_OUT_OF_MEMORY;
+            }
+            p->device_bytes += p->bytes[a];
+        }
+        const int64_t pb = std::max<int64_t>(f.n_groups_padded, 1) * sy(dtype);
+        if (cudaMalloc(&p->d_partial, static_cast<size_t>(pb)) != cudaSuccess) {
+            free_device(p); f.release(); delete p;
+            return DASP_ERR_OUT_OF_MEMORY;
+        }
+        p->device_bytes += pb;
+        auto u0 = std::chrono::steady_clock::now();
+        for (int a = 0; a < DASP_ARR_COUNT; ++a) {
+            if (p->bytes[a] == 0) continue;
+            if (cudaMemcpy(p->d[a], f.arr[a].ptr, static_cast<size_t>(p->bytes[a]), cudaMemcpyHostToDevice) != cudaSuccess) {
+                free_device(p); f.release(); delete p;
+                return DASP_ERR_CUDA;
+            }
+        }
+        auto u1 = std::chrono::steady_clock::now();
+        p->upload_ms = std::chrono::duration<double, std::milli>(u1 - u0).count();
+        if (!p->keep_host) f.release();
+    }
+    *plan_out = p;
+    return DASP_OK;
+}
+
+dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, double beta, void* stream, int32_t variant) {
+    if (!p) return DASP_ERR_INVALID_ARG;
+    if (p->device < 0) return DASP_ERR_UNSUPPORTED;
+    const HostFormat& f = p->host;
+    if (f.m == 0) return DASP_OK;
+    if (!y) return DASP_ERR_INVALID_ARG;
+    if (x == y) return DASP_ERR_INVALID_ARG;
+    if (variant == DASP_VARIANT_DEFAULT) variant = p->variant;
+    if (variant != DASP_VARIANT_MMA && variant != DASP_VARIANT_CUDACORE) return DASP_ERR_INVALID_ARG;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    DeviceGuard guard(p->device);
+    const bool on = p->timing_calls < p->timing_cap;
+    if (on) ++p->timing_calls;
+    cudaError_t e;
+    if (alpha == 0.0) {  // quick path: y = beta*y
+        if (beta == 1.0) return DASP_OK;
+        e = timed(p, DASP_K_SCALE, s, on, [&] { return dasp::launch_scale(y, f.m, beta, p->dtype, s); });
+        return e == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
+    }
+    if (!x && f.n > 0) return DASP_ERR_INVALID_ARG;
+    dasp::MainParams mp;
+    mp.long_val = p->d[DASP_ARR_LONG_VAL];
+    mp.long_col = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_COL]);
+    mp.partial = p->d_partial;
+    mp.rb_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_RB_PTR]);
+    mp.reg_val = p->d[DASP_ARR_REG_VAL];
+    mp.reg_col = static_cast<const int32_t*>(p->d[DASP_ARR_REG_COL]);
+    mp.irr_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_IRR_PTR]);
+    mp.irr_val = p->d[DASP_ARR_IRR_VAL];
+    mp.irr_col = static_cast<const int32_t*>(p->d[DASP_ARR_IRR_COL]);
+    mp.med_out = static_cast<const int32_t*>(p->d[DASP_ARR_MED_OUT]);
+    mp.short_val = p->d[DASP_ARR_SHORT_VAL];
+    mp.short_col = static_cast<const int32_t*>(p->d[DASP_ARR_SHORT_COL]);
+    mp.short_out = static_cast<const int32_t*>(p->d[DASP_ARR_SHORT_OUT]);
+    mp.x = x;
+    mp.y = y;
+    mp.alpha = alpha;
+    mp.beta = beta;
+    mp.nrb = f.nrb;
+    mp.t13 = f.t13; mp.t4 = f.t4; mp.t22 = f.t22; mp.ts = f.ts;
+    mp.w_long = p->w_long;
+    mp.w_med = p->w_med;
+    mp.w_total = p->w_long + p->w_med + p->w_short;
+    mp.rbw = p->rbw;
+    e = timed(p, DASP_K_MAIN, s, on, [&] { return dasp::launch_main(mp, p->dtype, variant, 0, mp.w_total, s); });
+    if (e != cudaSuccess) return DASP_ERR_CUDA;
+    const int64_t n0 = beta == 1.0 ? 0 : f.n0;
+    if (f.row_long + n0 > 0) {
+        dasp::FinishParams fp;
+        fp.partial = p->d_partial;
+        fp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
+        fp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
+        fp.empty_rows = static_cast<const int32_t*>(p->d[DASP_ARR_EMPTY_ROWS]);
+        fp.y = y;
+        fp.alpha = alpha;
+        fp.beta = beta;
+        fp.row_long = f.row_long;
+        fp.n0 = n0;
+        e = timed(p, DASP_K_FINISH, s, on, [&] { return dasp::launch_finish(fp, p->dtype, s); });
+        if (e != cudaSuccess) return DASP_ERR_CUDA;
+    }
+    return DASP_OK;
+}
+
+dasp_status_t dasp_spmv(dasp_plan_t p, const void* x, void* y, double alpha, double beta, void* stream) {
+    return dasp_spmv_ex(p, x, y, alpha, beta, stream, DASP_VARIANT_DEFAULT);
+}
+
+dasp_status_t dasp_spmv_host(dasp_plan_t p, const void* x_host, void* y_host, double alpha, double beta, void* stream) {
+    if (!p) return DASP_ERR_INVALID_ARG;
+    if (p->device < 0) return DASP_ERR_UNSUPPORTED;
+    const HostFormat& f = p->host;
+    if (f.m == 0) return DASP_OK;
+    if (!y_host || (!x_host && f.n > 0 && alpha != 0.0)) return DASP_ERR_INVALID_ARG;
+    DeviceGuard guard(p->device);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const size_t xb = static_cast<size_t>(f.n) * sx(p->dtype), yb = static_cast<size_t>(f.m) * sy(p->dtype);
+    if (!p->d_xh && xb && cudaMalloc(&p->d_xh, xb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
+    if (!p->d_yh && cudaMalloc(&p->d_yh, yb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
+    if (xb && alpha != 0.0 && cudaMemcpyAsync(p->d_xh, x_host, xb, cudaMemcpyHostToDevice, s) != cudaSuccess) return DASP_ERR_CUDA;
+    if (beta != 0.0 && cudaMemcpyAsync(p->d_yh, y_host, yb, cudaMemcpyHostToDevice, s) != cudaSuccess) return DASP_ERR_CUDA;
+    dasp_status_t st = dasp_spmv(p, p->d_xh, p->d_yh, alpha, beta, stream);
+    if (st != DASP_OK) return st;
+    if (cudaMemcpyAsync(y_host, p->d_yh, yb, cudaMemcpyDeviceToHost, s) != cudaSuccess) return DASP_ERR_CUDA;
+    return cudaStreamSynchronize(s) == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
+}
+
+dasp_status_t dasp_plan_destroy(dasp_plan_t p) {
+    if (!p) return DASP_OK;
+    if (p->device >= 0) {
+        DeviceGuard guard(p->device);
+        cudaDeviceSynchronize();
+        free_device(p);
+    }
+    p->host.release();
+    delete p;
+    return DASP_OK;
+}
+
+dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
+    if (!p || !o) return DASP_ERR_INVALID_ARG;
+    const HostFormat& f = p->host;
+    std::memset(o, 0, sizeof(*o));
+    o->m = f.m; o->n = f.n; o->nnz = f.nnz;
+    o->dtype = p->dtype; o->device = p->device;
+    o->n_empty = f.n0; o->n_len1 = f.n1; o->n_len2 = f.n2; o->n_len3 = f.n3; o->n_len4 = f.n4;
+    o->row_medium = f.row_medium; o->row_long = f.row_long; o->rowblocks = f.nrb;
+    o->n_groups = f.n_groups; o->n_groups_padded = f.n_groups_padded;
+    o->tiles_13 = f.t13; o->tiles_4 = f.t4; o->tiles_22 = f.t22; o->tiles_single = f.ts;
+    o->nnz_long_new = f.nnz_long_new; o->nnz_reg_new = f.nnz_reg_new; o->nnz_irreg = f.nnz_irreg;
+    o->nnz_short_new = f.nnz_short_new;
+    o->nnz_long = f.nnz_long; o->nnz_medium = f.nnz_medium; o->nnz_short = f.nnz_short;
+    o->device_bytes = p->device_bytes;
+    o->alg_bytes_beta0 = alg_bytes(p, false);
+    o->alg_bytes_beta1 = alg_bytes(p, true);
+    o->medium_rb_per_warp = p->rbw;
+    o->launches_per_spmv = (p->w_long + p->w_med + p->w_short > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
+    o->build_ms = p->build_ms;
+    o->upload_ms = p->upload_ms;
+    return DASP_OK;
+}
+
+dasp_status_t dasp_plan_copy_array(dasp_plan_t p, int32_t id, void* dst, int64_t* bytes) {
+    if (!p || !bytes || id < 0 || id >= DASP_ARR_COUNT) return DASP_ERR_INVALID_ARG;
+    const int64_t nb = p->bytes[id];
+    if (!dst) { *bytes = nb; return DASP_OK; }
+    if (*bytes < nb) { *bytes = nb; return DASP_ERR_INVALID_ARG; }
+    *bytes = nb;
+    if (nb == 0) return DASP_OK;
+    if (p->host.arr[id].ptr) {
+        std::memcpy(dst, p->host.arr[id].ptr, static_cast<size_t>(nb));
+        return DASP_OK;
+    }
+    if (p->device < 0 || !p->d[id]) return DASP_ERR_INTERNAL;
+    DeviceGuard guard(p->device);
+    return cudaMemcpy(dst, p->d[id], static_cast<size_t>(nb), cudaMemcpyDeviceToHost) == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
+}
+
+dasp_status_t dasp_partition_rows(const int64_t* row_ptr, int64_t m, int32_t nparts, int64_t* starts) {
+    if (!row_ptr || !starts || nparts < 1 || m < 0) return DASP_ERR_INVALID_ARG;
+    const int64_t nnz = row_ptr[m];
+    starts[0] = 0;
+    for (int32_t q = 1; q < nparts; ++q) {
+        // first row r with row_ptr[r] >= q*nnz/nparts (balanced by nonzeros)
+        const int64_t target = static_cast<int64_t>((static_cast<__int128>(nnz) * q) / nparts);
+        const int64_t* it = std::lower_bound(row_ptr, row_ptr + m + 1, target);
+        int64_t r = it - row_ptr;
+        starts[q] = std::max(starts[q - 1], std::min(r, m));
+    }
+    starts[nparts] = m;
+    return DASP_OK;
+}
+
+dasp_status_t dasp_remap_columns(int32_t* col, int64_t nnz, const int64_t* starts, int32_t nparts, int64_t* stride) {
+    if ((!col && nnz > 0) || !starts || nparts < 1 || !stride) return DASP_ERR_INVALID_ARG;
+    int64_t S = 0;
+    for (int32_t q = 0; q < nparts; ++q) S = std::max(S, starts[q + 1] - starts[q]);
+    if (S * nparts > 0x7fffffffLL) return DASP_ERR_INVALID_ARG;
+    *stride = S;
+    const int64_t n = starts[nparts];
+    int bad = 0;
+#pragma omp parallel for schedule(static) reduction(| : bad)
+    for (int64_t k = 0; k < nnz; ++k) {
+        const int64_t c = col[k];
+        if (c < 0 || c >= n) { bad |= 1; continue; }
+        const int64_t q = std::upper_bound(starts, starts + nparts + 1, c) - starts - 1;
+        col[k] = static_cast<int32_t>(q * S + (c - starts[q]));
+    }
+    return bad ? DASP_ERR_INVALID_ARG : DASP_OK;
+}
+
+dasp_status_t dasp_plan_set_timing(dasp_plan_t p, int32_t capacity) {
+    if (!p || capacity < 0) return DASP_ERR_INVALID_ARG;
+    p->timing_cap = capacity;
+    p->timing_calls = 0;
+    return DASP_OK;
+}
+
+dasp_status_t dasp_plan_read_timing(dasp_plan_t p, double* ms, int64_t* launches) {
+    if (!p || !ms || !launches) return DASP_ERR_INVALID_ARG;
+    for (int k = 0; k < DASP_K_COUNT; ++k) { ms[k] = 0; launches[k] = 0; }
+    if (p->device < 0) return DASP_OK;
+    DeviceGuard guard(p->device);
+    for (auto& r : p->recs) {
+        if (cudaEventSynchronize(r.b) != cudaSuccess) return DASP_ERR_CUDA;
+        float t = 0;
+        if (cudaEventElapsedTime(&t, r.a, r.b) != cudaSuccess) return DASP_ERR_CUDA;
+        ms[r.kernel] += t;
+        launches[r.kernel] += 1;
+    }
+    p->recs.clear();
+    p->pool_used = 0;
+    p->timing_calls = 0;
+    return DASP_OK;
+}
+
+}  // extern "C"

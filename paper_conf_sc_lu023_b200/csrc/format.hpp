@@ -1,0 +1,54 @@
+// format.hpp — host-side DASP format (DESIGN.md §4 FORMAT) shared by the production builder,
+// the plan/ABI code and (as launch metadata) the CUDA kernels.  Not shared with oracle/.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+
+#include "../../include/dasp.h"
+
+namespace dasp {
+
+// Per-dtype block geometry.  FP64: mma.sync m8n8k4 (MMA_M=8, MMA_N=8, MMA_K=4).
+// FP16: mma.sync m16n8k16 with A rows 0-7 live (R14), so the block is 8 x 16.
+struct Geometry {
+    int sv;   // bytes per value
+    int K;    // MMA_K (slots per row per block)
+    int BE;   // elements per 8 x K block
+    int EPL;  // elements per lane per block (BE / 32)
+    int G;    // long-row group = 2 * MMA_M * MMA_K
+    int UG;   // groups per long warp unit (R18): one unit = 32 lanes x (UG*G/32) elements
+    int CW;   // medium chunk width in blocks (R18)
+};
+
+inline Geometry geometry(int dtype) {
+    if (dtype == DASP_R_64F) return Geometry{8, 4, 32, 1, 64, 4, 4};
+    return Geometry{2, 16, 128, 4, 256, 2, 2};
+}
+
+constexpr int MAX_LEN = 256;
+constexpr int MMA_M = 8;
+constexpr int32_t PAD_COL = -1;  // R12: sentinel column of pads (x read as 0)
+constexpr int SHORT_TILE = 128;  // elements per short tile (32 four-slot rows)
+
+struct HostBuf {
+    void* ptr = nullptr;
+    int64_t bytes = 0;
+};
+
+struct HostFormat {
+    Geometry geo{};
+    int dtype = 0;
+    int64_t m = 0, n = 0, nnz = 0;
+    int64_t n0 = 0, n1 = 0, n2 = 0, n3 = 0, n4 = 0, row_medium = 0, row_long = 0;
+    int64_t nrb = 0, n_groups = 0, n_groups_padded = 0, t13 = 0, t4 = 0, t22 = 0, ts = 0;
+    int64_t nnz_long_new = 0, nnz_reg_new = 0, nnz_irreg = 0, nnz_short_new = 0;
+    int64_t nnz_long = 0, nnz_medium = 0, nnz_short = 0;
+    HostBuf arr[DASP_ARR_COUNT];
+    void release();
+};
+
+// Builds the format on the host.  Returns a dasp_status_t.
+int build_format(HostFormat& f, int dtype, int64_t m, int64_t n, const int64_t* row_ptr,
+                 const int32_t* col, const void* val, int nthreads, bool validate);
+
+}  // namespace dasp

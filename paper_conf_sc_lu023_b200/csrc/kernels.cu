@@ -1,0 +1,525 @@
+// kernels.cu — sm_100a kernels of the DASP SpMV hot path (§3.3, Alg. 2-5).
+//
+// One fused launch covers the three row classes (warp-uniform dispatch on the global warp
+// index), plus a small "finish" launch for long-row phase 2 (Alg. 2 l.17-25)
+// and empty rows.  Every block inner product is computed by one of two variants that read
+// the SAME packed arrays (north_star (3)):
+//   VAR_MMA      legacy warp MMA: DMMA m8n8k4 f64 (Listing 1) / HMMA m16n8k16
+//                f16->f32; the block dot products sit on the diagonal of C (Fig. 4)
+//                and are extracted with shuffles (Alg. 2 l.10-13, Alg. 3 l.13-17).
+//   VAR_CUDACORE per-lane FMA and a warp-shuffle segmented reduction.
+// The packed val/col streams are read with 128/256-bit L1::no_allocate loads carrying an
+// L2 evict_first policy (the paper's "cache bypass", R17) so that x stays in L2;
+// x is gathered through the read-only path.  Pads carry column -1 and read x = 0 (R12).
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.cuh"
+
+namespace dasp {
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+enum { VAR_MMA = 1, VAR_CUDACORE = 2 };
+
+// ------------------------------------------------------------------------------------------
+// memory helpers
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t stream_policy() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ void ld4_f64(const double* a, uint64_t pol, double (&v)[4]) {
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f64 {%0,%1,%2,%3}, [%4], %5;"
+        : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(a), "l"(pol));
+}
+__device__ __forceinline__ void ld2_f64(const double* a, uint64_t pol, double& v0, double& v1) {
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;"
+        : "=d"(v0), "=d"(v1) : "l"(a), "l"(pol));
+}
+__device__ __forceinline__ double ld1_f64(const double* a, uint64_t pol) {
+    double v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(a), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void ld8_b32(const void* a, uint64_t pol, uint32_t (&v)[8]) {
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+        : "l"(a), "l"(pol));
+}
+__device__ __forceinline__ void ld4_b32(const void* a, uint64_t pol, uint32_t (&v)[4]) {
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.b32 {%0,%1,%2,%3}, [%4], %5;"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "l"(a), "l"(pol));
+}
+__device__ __forceinline__ void ld2_b32(const void* a, uint64_t pol, uint32_t& v0, uint32_t& v1) {
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.b32 {%0,%1}, [%2], %3;"
+        : "=r"(v0), "=r"(v1) : "l"(a), "l"(pol));
+}
+__device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
+    uint32_t v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+    return v;
+}
+// x gather: column -1 (pad, R12) reads 0 without touching memory
+__device__ __forceinline__ double gx(const double* x, uint32_t c) {
+    return static_cast<int32_t>(c) >= 0 ? __ldg(x + static_cast<int32_t>(c)) : 0.0;
+}
+__device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
+    return static_cast<int32_t>(c) >= 0 ? __ldg(reinterpret_cast<const unsigned short*>(x) + static_cast<int32_t>(c))
+                                        : static_cast<uint16_t>(0);
+}
+__device__ __forceinline__ float h2f(uint16_t h) { return __half2float(__ushort_as_half(h)); }
+__device__ __forceinline__ float2 u2f2(uint32_t u) {  // two packed binary16 -> two f32 (exact)
+    return make_float2(h2f(static_cast<uint16_t>(u & 0xffffu)), h2f(static_cast<uint16_t>(u >> 16)));
+}
+__device__ __forceinline__ uint32_t pack2(uint16_t lo, uint16_t hi) { return static_cast<uint32_t>(lo) | (static_cast<uint32_t>(hi) << 16); }
+
+// ------------------------------------------------------------------------------------------
+// MMA wrappers (Listing 1) and diagonal extraction (Fig. 4)
+// ------------------------------------------------------------------------------------------
+// C(8x8) += A(8x4) * B(4x8); lane (g = lane>>2, t = lane&3) holds A[g][t], B[t][g],
+// C[g][2t], C[g][2t+1].
+__device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                 : "+d"(c0), "+d"(c1) : "d"(a), "d"(b));
+}
+// C(16x8) += A(16x16) * B(16x8), f16 inputs, f32 accumulate.  Rows 8-15 of A are zero
+// (R14): a0 = A[g][2t..2t+1], a2 = A[g][2t+8..2t+9]; b0 = B[2t..2t+1][g], b1 = B[2t+8..2t+9][g];
+// c0,c1 = C[g][2t..2t+1].
+__device__ __forceinline__ void hmma(float& c0, float& c1, uint32_t a0, uint32_t a2, uint32_t b0, uint32_t b1) {
+    float c2 = 0.f, c3 = 0.f;
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+        : "+f"(c0), "+f"(c1), "+f"(c2), "+f"(c3)
+        : "r"(a0), "r"(0u), "r"(a2), "r"(0u), "r"(b0), "r"(b1));
+}
+// C[g][g] lives in lane 4g + (g>>1), register g&1.  Returns it to every lane of quad g.
+template <typename A>
+__device__ __forceinline__ A diag_to_quad(A c0, A c1, int lane) {
+    const int g = lane >> 2;
+    A d = (g & 1) ? c1 : c0;
+    return __shfl_sync(FULL, d, 4 * g + (g >> 1));
+}
+__device__ __forceinline__ bool is_diag_holder(int lane) {
+    const int g = lane >> 2;
+    return (lane & 3) == (g >> 1);
+}
+
+template <int DT> struct Tr;
+template <> struct Tr<0> {  // FP64
+    using V = double; using Y = double; using A = double; using X = double;
+    static constexpr int K = 4, BE = 32, EPL = 1, G = 64, UG = 4, CW = 4;
+};
+template <> struct Tr<1> {  // FP16 storage, FP32 accumulate
+    using V = uint16_t; using Y = float; using A = float; using X = uint16_t;
+    static constexpr int K = 16, BE = 128, EPL = 4, G = 256, UG = 2, CW = 2;
+};
+
+// y[row] = alpha*acc + beta*y[row] (beta == 0: y not read, R16)
+template <int DT>
+__device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typename Tr<DT>::A acc) {
+    using Y = typename Tr<DT>::Y;
+    if (row < 0) return;
+    Y* y = static_cast<Y*>(P.y);
+    Y r = static_cast<Y>(P.alpha) * acc;
+    if (P.beta != 0.0) r += static_cast<Y>(P.beta) * y[row];
+    y[row] = r;
+}
+
+// ------------------------------------------------------------------------------------------
+// long rows, phase 1 (Alg. 2 l.1-16): one warp = one unit of UG consecutive groups
+// ------------------------------------------------------------------------------------------
+template <int VAR>
+__device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol) {
+    const int64_t base = u * 256 + lane * 8;            // lane holds 8 consecutive elements
+    const double* lv = static_cast<const double*>(P.long_val) + base;
+    double v[8];
+    uint32_t c[8];
+    ld4_f64(lv, pol, *reinterpret_cast<double(*)[4]>(&v[0]));
+    ld4_f64(lv + 4, pol, *reinterpret_cast<double(*)[4]>(&v[4]));
+    ld8_b32(P.long_col + base, pol, c);
+    const double* x = static_cast<const double*>(P.x);
+    double xv[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) xv[j] = gx(x, c[j]);
+    double part;
+    if constexpr (VAR == VAR_MMA) {
+        double c0 = 0.0, c1 = 0.0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) dmma(c0, c1, v[j], xv[j]);   // 8 m8n8k4 = 4 groups of 64
+        double d = diag_to_quad(c0, c1, lane);                  // rows 2q, 2q+1 = group q
+        part = (lane & 3) == 0 ? d : 0.0;
+        part += __shfl_xor_sync(FULL, part, 4);
+    } else {
+        part = 0.0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) part = fma(v[j], xv[j], part);
+        part += __shfl_xor_sync(FULL, part, 1);
+        part += __shfl_xor_sync(FULL, part, 2);
+        part += __shfl_xor_sync(FULL, part, 4);
+    }
+    if ((lane & 7) == 0) static_cast<double*>(P.partial)[u * 4 + (lane >> 3)] = part;
+}
+
+template <int VAR>
+__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol) {
+    const int64_t base = u * 512 + lane * 16;           // lane holds 16 consecutive elements
+    uint32_t vv[8], c[16];
+    ld8_b32(static_cast<const uint16_t*>(P.long_val) + base, pol, vv);
+    ld8_b32(P.long_col + base, pol, *reinterpret_cast<uint32_t(*)[8]>(&c[0]));
+    ld8_b32(P.long_col + base + 8, pol, *reinterpret_cast<uint32_t(*)[8]>(&c[8]));
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    uint16_t xh[16];
+#pragma unroll
+    for (int j = 0; j < 16; ++j) xh[j] = gxh(x, c[j]);
+    float part;
+    if constexpr (VAR == VAR_MMA) {
+        float c0 = 0.f, c1 = 0.f;
+#pragma unroll
+        for (int h = 0; h < 4; ++h)   // elements 4h..4h+3 -> A[g][2t,2t+1,2t+8,2t+9]
+            hmma(c0, c1, vv[2 * h], vv[2 * h + 1], pack2(xh[4 * h], xh[4 * h + 1]), pack2(xh[4 * h + 2], xh[4 * h + 3]));
+        float d = diag_to_quad(c0, c1, lane);                   // rows 4q..4q+3 = group q
+        part = (lane & 3) == 0 ? d : 0.f;
+        part += __shfl_xor_sync(FULL, part, 4);
+        part += __shfl_xor_sync(FULL, part, 8);
+    } else {
+        part = 0.f;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            float2 af = u2f2(vv[j]);
+            part = fmaf(af.x, h2f(xh[2 * j]), part);
+            part = fmaf(af.y, h2f(xh[2 * j + 1]), part);
+        }
+#pragma unroll
+        for (int o = 1; o < 16; o <<= 1) part += __shfl_xor_sync(FULL, part, o);
+    }
+    if ((lane & 15) == 0) static_cast<float*>(P.partial)[u * 2 + (lane >> 4)] = part;
+}
+
+// ------------------------------------------------------------------------------------------
+// medium rows (Alg. 3): row-block = 8 rows; regular 8 x K blocks in lane-interleaved chunks
+// of CW blocks (R18), then the irregular tails with 4 lanes per row, then y.
+// ------------------------------------------------------------------------------------------
+template <int VAR>
+__device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
+    const int g = lane >> 2, t = lane & 3;
+    const int64_t base = P.rb_ptr[rb];
+    const int64_t nreg = (P.rb_ptr[rb + 1] - base) >> 5;
+    const double* rv = static_cast<const double*>(P.reg_val) + base;
+    const int32_t* rc = P.reg_col + base;
+    const double* x = static_cast<const double*>(P.x);
+    double c0 = 0.0, c1 = 0.0, part = 0.0;
+    const int64_t nfull = nreg >> 2;
+    for (int64_t ch = 0; ch < nfull; ++ch) {           // full chunks: 4 blocks, 32 B + 16 B per lane
+        double v[4];
+        uint32_t c[4];
+        ld4_f64(rv + ch * 128 + lane * 4, pol, v);
+        ld4_b32(rc + ch * 128 + lane * 4, pol, c);
+        double xv[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) xv[j] = gx(x, c[j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, v[j], xv[j]);
+            else part = fma(v[j], xv[j], part);
+        }
+    }
+    const int rem = static_cast<int>(nreg - (nfull << 2));
+    if (rem) {                                          // last chunk, width rem
+        const int64_t cb = nfull * 128 + lane * rem;
+        for (int j = 0; j < rem; ++j) {
+            double v = ld1_f64(rv + cb + j, pol);
+            double xv = gx(x, ld1_b32(rc + cb + j, pol));
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, v, xv);
+            else part = fma(v, xv, part);
+        }
+    }
+    if constexpr (VAR == VAR_MMA) {                     // Alg. 3 l.13-17: diagonal -> lane 4g
+        double d = diag_to_quad(c0, c1, lane);
+        part = t == 0 ? d : 0.0;
+    }
+    const int64_t i = rb * 8 + g;                      // Alg. 3 l.20-24: irregular part
+    const int64_t ib = P.irr_ptr[i], ie = P.irr_ptr[i + 1];
+    const double* iv = static_cast<const double*>(P.irr_val);
+    for (int64_t k = ib + t; k < ie; k += 4) part = fma(ld1_f64(iv + k, pol), gx(x, ld1_b32(P.irr_col + k, pol)), part);
+    part += __shfl_xor_sync(FULL, part, 1);
+    part += __shfl_xor_sync(FULL, part, 2);
+    if (t == 0) store_y<0>(P, P.med_out[i], part);     // Alg. 3 l.25 through the output map (R9)
+}
+
+template <int VAR>
+__device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
+    const int g = lane >> 2, t = lane & 3;
+    const int64_t base = P.rb_ptr[rb];
+    const int64_t nreg = (P.rb_ptr[rb + 1] - base) >> 7;
+    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + base;
+    const int32_t* rc = P.reg_col + base;
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    float c0 = 0.f, c1 = 0.f, part = 0.f;
+    auto block = [&](uint32_t a0, uint32_t a2, const uint32_t* c) {
+        uint16_t xh[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) xh[e] = gxh(x, c[e]);
+        if constexpr (VAR == VAR_MMA) {
+            hmma(c0, c1, a0, a2, pack2(xh[0], xh[1]), pack2(xh[2], xh[3]));
+        } else {
+            float2 lo = u2f2(a0);
+            float2 hi = u2f2(a2);
+            part = fmaf(lo.x, h2f(xh[0]), part);
+            part = fmaf(lo.y, h2f(xh[1]), part);
+            part = fmaf(hi.x, h2f(xh[2]), part);
+            part = fmaf(hi.y, h2f(xh[3]), part);
+        }
+    };
+    const int64_t nfull = nreg >> 1;
+    for (int64_t ch = 0; ch < nfull; ++ch) {           // 2 blocks: 16 B + 32 B per lane
+        uint32_t v[4], c[8];
+        ld4_b32(rv + ch * 256 + lane * 8, pol, v);
+        ld8_b32(rc + ch * 256 + lane * 8, pol, c);
+        block(v[0], v[1], &c[0]);
+        block(v[2], v[3], &c[4]);
+    }
+    if (nreg & 1) {
+        uint32_t v0, v1, c[4];
+        ld2_b32(rv + nfull * 256 + lane * 4, pol, v0, v1);
+        ld4_b32(rc + nfull * 256 + lane * 4, pol, c);
+        block(v0, v1, c);
+    }
+    if constexpr (VAR == VAR_MMA) {
+        float d = diag_to_quad(c0, c1, lane);
+        part = t == 0 ? d : 0.f;
+    }
+    const int64_t i = rb * 8 + g;
+    const int64_t ib = P.irr_ptr[i], ie = P.irr_ptr[i + 1];
+    const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
+    for (int64_t k = ib + t; k < ie; k += 4)
+        part = fmaf(h2f(__ldg(iv + k)), h2f(gxh(x, __ldg(reinterpret_cast<const uint32_t*>(P.irr_col) + k))), part);
+    part += __shfl_xor_sync(FULL, part, 1);
+    part += __shfl_xor_sync(FULL, part, 2);
+    if (t == 0) store_y<1>(P, P.med_out[i], part);
+}
+
+// ------------------------------------------------------------------------------------------
+// short rows (Alg. 4) and singles (Alg. 5): one tile of 32 four-slot rows
+// ------------------------------------------------------------------------------------------
+// cat 0 = 1&3 (seg0 = slot 0, seg1 = slots 1-3), 1 = len-4, 2 = 2&2 (slots 0-1 | 2-3)
+__device__ __forceinline__ int seg_of(int cat, int slot) { return cat == 0 ? (slot > 0) : (cat == 2 ? (slot >> 1) : 0); }
+
+template <int VAR>
+__device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
+                                               uint64_t pol) {
+    const int g = lane >> 2, t = lane & 3;
+    double v[4];
+    uint32_t c[4];
+    ld4_f64(static_cast<const double*>(P.short_val) + tile * 128 + lane * 4, pol, v);
+    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
+    const double* x = static_cast<const double*>(P.x);
+    double xv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) xv[j] = gx(x, c[j]);
+    const int nseg = cat == 1 ? 1 : 2;
+    const int myseg = seg_of(cat, t);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {                       // 4-slot row r = 8j + g, slot t
+        for (int s = 0; s < nseg; ++s) {
+            const int o = nseg == 2 ? 16 * j + 8 * s + g : 8 * j + g;
+            if constexpr (VAR == VAR_MMA) {             // x masked to the segment (Alg. 4 l.7-11)
+                double c0 = 0.0, c1 = 0.0;
+                dmma(c0, c1, v[j], myseg == s ? xv[j] : 0.0);
+                if (is_diag_holder(lane)) store_y<0>(P, P.short_out[obase + o], (g & 1) ? c1 : c0);
+            } else {
+                double p = myseg == s ? v[j] * xv[j] : 0.0;
+                p += __shfl_xor_sync(FULL, p, 1);
+                p += __shfl_xor_sync(FULL, p, 2);
+                if (t == 0) store_y<0>(P, P.short_out[obase + o], p);
+            }
+        }
+    }
+}
+
+template <int VAR>
+__device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
+                                               uint64_t pol) {
+    const int g = lane >> 2, t = lane & 3;
+    uint32_t a0, a2, c[4];
+    ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
+    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    uint16_t xh[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) xh[e] = gxh(x, c[e]);
+    // element e: four-slot row group q = (e<2 ? 0 : 2) + (t>>1), slot 2(t&1) + (e&1)
+    const int nseg = cat == 1 ? 1 : 2;
+    const int seg0 = seg_of(cat, 2 * (t & 1)), seg1 = seg_of(cat, 2 * (t & 1) + 1);
+    if constexpr (VAR == VAR_MMA) {
+        for (int q = 0; q < 4; ++q) {
+            const bool lo = q == (t >> 1), hi = q == 2 + (t >> 1);
+            for (int s = 0; s < nseg; ++s) {
+                const bool m0 = seg0 == s, m1 = seg1 == s;
+                uint32_t b0 = lo ? pack2(m0 ? xh[0] : 0, m1 ? xh[1] : 0) : 0u;
+                uint32_t b1 = hi ? pack2(m0 ? xh[2] : 0, m1 ? xh[3] : 0) : 0u;
+                float c0 = 0.f, c1 = 0.f;
+                hmma(c0, c1, a0, a2, b0, b1);
+                const int o = nseg == 2 ? 16 * q + 8 * s + g : 8 * q + g;
+                if (is_diag_holder(lane)) store_y<1>(P, P.short_out[obase + o], (g & 1) ? c1 : c0);
+            }
+        }
+    } else {
+        float2 vl = u2f2(a0);
+        float2 vh = u2f2(a2);
+        const float p0 = vl.x * h2f(xh[0]), p1 = vl.y * h2f(xh[1]), p2 = vh.x * h2f(xh[2]), p3 = vh.y * h2f(xh[3]);
+        for (int s = 0; s < nseg; ++s) {
+            float slo = (seg0 == s ? p0 : 0.f) + (seg1 == s ? p1 : 0.f);   // group t>>1
+            float shi = (seg0 == s ? p2 : 0.f) + (seg1 == s ? p3 : 0.f);   // group 2 + (t>>1)
+            slo += __shfl_xor_sync(FULL, slo, 1);
+            shi += __shfl_xor_sync(FULL, shi, 1);
+            if ((t & 1) == 0) {
+                const int qlo = t >> 1, qhi = 2 + (t >> 1);
+                store_y<1>(P, P.short_out[obase + (nseg == 2 ? 16 * qlo + 8 * s + g : 8 * qlo + g)], slo);
+                store_y<1>(P, P.short_out[obase + (nseg == 2 ? 16 * qhi + 8 * s + g : 8 * qhi + g)], shi);
+            }
+        }
+    }
+}
+
+// singles (Alg. 5): lane handles 4 consecutive len-1 rows on CUDA cores
+template <int DT>
+__device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, int64_t obase, int lane, uint64_t pol) {
+    uint32_t c[4], o[4];
+    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
+    ld4_b32(P.short_out + obase + lane * 4, pol, o);
+    if constexpr (DT == 0) {
+        double v[4];
+        ld4_f64(static_cast<const double*>(P.short_val) + tile * 128 + lane * 4, pol, v);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) store_y<0>(P, static_cast<int32_t>(o[j]), v[j] * gx(static_cast<const double*>(P.x), c[j]));
+    } else {
+        uint32_t a0, a2;
+        ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
+        float2 lo = u2f2(a0);
+        float2 hi = u2f2(a2);
+        const float v[4] = {lo.x, lo.y, hi.x, hi.y};
+        const uint16_t* x = static_cast<const uint16_t*>(P.x);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) store_y<1>(P, static_cast<int32_t>(o[j]), v[j] * h2f(gxh(x, c[j])));
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// the fused main kernel
+// ------------------------------------------------------------------------------------------
+template <int DT, int VAR>
+__global__ void __launch_bounds__(MAIN_THREADS) dasp_main_kernel(const MainParams P, int64_t w_begin, int64_t w_end) {
+    const int lane = threadIdx.x & 31;
+    int64_t w = w_begin + (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) / 32;
+    if (w >= w_end) return;
+    const uint64_t pol = stream_policy();
+    if (w < P.w_long) {
+        if constexpr (DT == 0) long_unit_f64<VAR>(P, w, lane, pol);
+        else long_unit_f16<VAR>(P, w, lane, pol);
+        return;
+    }
+    w -= P.w_long;
+    if (w < P.w_med) {
+        const int64_t rb0 = w * P.rbw;
+        const int64_t rb1 = rb0 + P.rbw < P.nrb ? rb0 + P.rbw : P.nrb;
+        for (int64_t rb = rb0; rb < rb1; ++rb) {
+            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb, lane, pol);
+            else medium_rb_f16<VAR>(P, rb, lane, pol);
+        }
+        return;
+    }
+    int64_t tile = w - P.w_med;                         // short tiles: [1&3][len4][2&2][singles]
+    int cat;
+    int64_t obase;
+    if (tile < P.t13) { cat = 0; obase = tile * 64; }
+    else if (tile < P.t13 + P.t4) { cat = 1; obase = 64 * P.t13 + (tile - P.t13) * 32; }
+    else if (tile < P.t13 + P.t4 + P.t22) { cat = 2; obase = 64 * P.t13 + 32 * P.t4 + (tile - P.t13 - P.t4) * 64; }
+    else {
+        obase = 64 * P.t13 + 32 * P.t4 + 64 * P.t22 + (tile - P.t13 - P.t4 - P.t22) * 128;
+        singles_tile<DT>(P, tile, obase, lane, pol);
+        return;
+    }
+    if constexpr (DT == 0) short_tile_f64<VAR>(P, cat, tile, obase, lane, pol);
+    else short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
+}
+
+// long phase 2 (Alg. 2 l.17-25): one warp per long row, lane-strided sum of the group partials
+// in a fixed order, butterfly reduction (deterministic, R19); then the empty rows (R1).
+template <int DT>
+__global__ void __launch_bounds__(256) dasp_finish_kernel(const FinishParams P) {
+    using A = typename Tr<DT>::A;
+    using Y = typename Tr<DT>::Y;
+    const int lane = threadIdx.x & 31;
+    const int64_t w = (static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x) / 32;
+    Y* y = static_cast<Y*>(P.y);
+    if (w < P.row_long) {
+        const A* part = static_cast<const A*>(P.partial);
+        A s = 0;
+        for (int64_t k = P.group_ptr[w] + lane; k < P.group_ptr[w + 1]; k += 32) s += part[k];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+        if (lane == 0) {
+            const int32_t row = P.long_out[w];
+            Y r = static_cast<Y>(P.alpha) * s;
+            if (P.beta != 0.0) r += static_cast<Y>(P.beta) * y[row];
+            y[row] = r;
+        }
+        return;
+    }
+    const int64_t e = (w - P.row_long) * 32 + lane;
+    if (e < P.n0) {
+        const int32_t row = P.empty_rows[e];
+        y[row] = P.beta != 0.0 ? static_cast<Y>(P.beta) * y[row] : Y(0);
+    }
+}
+
+template <int DT>
+__global__ void dasp_scale_kernel(void* yv, int64_t m, double beta) {
+    using Y = typename Tr<DT>::Y;
+    Y* y = static_cast<Y*>(yv);
+    for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < m;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x)
+        y[i] = beta != 0.0 ? static_cast<Y>(beta) * y[i] : Y(0);
+}
+
+}  // namespace
+
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t w_begin, int64_t w_end, cudaStream_t s) {
+    if (w_end <= w_begin) return cudaSuccess;
+    const int64_t warps = w_end - w_begin;
+    const int64_t blocks = (warps * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
+    if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
+    if (dtype == 0) {
+        if (variant == VAR_MMA) dasp_main_kernel<0, VAR_MMA><<<grid, block, 0, s>>>(p, w_begin, w_end);
+        else dasp_main_kernel<0, VAR_CUDACORE><<<grid, block, 0, s>>>(p, w_begin, w_end);
+    } else {
+        if (variant == VAR_MMA) dasp_main_kernel<1, VAR_MMA><<<grid, block, 0, s>>>(p, w_begin, w_end);
+        else dasp_main_kernel<1, VAR_CUDACORE><<<grid, block, 0, s>>>(p, w_begin, w_end);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s) {
+    const int64_t warps = p.row_long + (p.n0 + 31) / 32;
+    if (warps == 0) return cudaSuccess;
+    dim3 grid(static_cast<unsigned>((warps * 32 + 255) / 256)), block(256);
+    if (dtype == 0) dasp_finish_kernel<0><<<grid, block, 0, s>>>(p);
+    else dasp_finish_kernel<1><<<grid, block, 0, s>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s) {
+    if (m == 0) return cudaSuccess;
+    int64_t blocks = (m + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (dtype == 0) dasp_scale_kernel<0><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta);
+    else dasp_scale_kernel<1><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta);
+    return cudaGetLastError();
+}
+
+}  // namespace dasp

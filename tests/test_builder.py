@@ -1,0 +1,141 @@
+"""Production builder (libdasp.so, host-only plans) vs the oracle's literal builder: byte for byte
+(north_star: "bit-exact for the format builder's indexing and permutation"),
+plus the C-ABI surface that needs no GPU.  CPU only."""
+import ctypes
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from paper_conf_sc_lu023_b200 import dasp
+from tests.format_decode import check_roundtrip
+
+COUNT_MAP = {"n0": "n_empty", "n1": "n_len1", "n2": "n_len2", "n3": "n_len3", "n4": "n_len4",
+             "row_medium": "row_medium", "row_long": "row_long", "nrb": "rowblocks", "n_groups": "n_groups",
+             "n_groups_padded": "n_groups_padded", "t13": "tiles_13", "t4": "tiles_4", "t22": "tiles_22",
+             "ts": "tiles_single", "nnz_long_new": "nnz_long_new", "nnz_reg_new": "nnz_reg_new",
+             "nnz_irreg": "nnz_irreg", "nnz_short_new": "nnz_short_new", "m": "m", "n": "n", "nnz": "nnz"}
+
+
+def host_plan(A, dt, **kw):
+    val = A.val if dt == "f64" else A.val.astype(np.float16)
+    return dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dt, device=-1, **kw)
+
+
+def matrices():
+    yield "c1a", synth.generate(synth.config("c1a"))
+    yield "c1b", synth.generate(synth.config("c1b"))
+    yield "c2s", synth.generate(synth.config("c2", scale=16 / 128))
+    yield "c3s", synth.generate(synth.config("c3", scale=0.002))
+    yield "c5s", synth.generate(synth.config("c5", scale=2e-5))
+    yield "c6s", synth.generate(synth.config("c6", scale=0.01))
+    lens = [0, 1, 2, 3, 4, 5, 9, 17, 31, 33, 64, 255, 256, 257, 300, 1000, 2049, 4, 4, 3, 2, 1, 1, 1, 7, 6]
+    yield "lens", synth.from_lengths(lens * 5, n=3000)
+
+
+CASES = list(matrices())
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("name,A", CASES, ids=[c[0] for c in CASES])
+def test_builder_bit_exact_vs_oracle(name, A, dt):
+    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt)
+    plan = host_plan(A, dt)
+    info = plan.info
+    for k, v in ref.counts.items():
+        assert info[COUNT_MAP[k]] == v, k
+    for arr in dasp.ARRAYS:
+        got = dasp.dasp_plan_copy_array(plan, arr)
+        want = ref.arrays[arr]
+        assert got.shape == want.shape, arr
+        assert np.array_equal(got, want), arr
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_builder_roundtrip_via_abi(dt):
+    A = synth.generate(synth.config("c1b"))
+    plan = host_plan(A, dt)
+    info = plan.info
+    counts = {k: info[v] for k, v in COUNT_MAP.items()}
+
+    def get(name):
+        b = dasp.dasp_plan_copy_array(plan, name)
+        if name.endswith("_val"):
+            return b.view(np.float64 if dt == "f64" else np.float16)
+        if name in ("group_ptr", "rb_ptr", "irr_ptr"):
+            return b.view(np.int64)
+        return b.view(np.int32)
+    check_roundtrip(A, counts, get, dt)
+    assert info["nnz_long"] + info["nnz_medium"] + info["nnz_short"] == A.nnz
+
+
+def test_builder_threads_deterministic():
+    A = synth.generate(synth.config("c3", scale=0.004))
+    p1, p8 = host_plan(A, "f64", num_threads=1), host_plan(A, "f64", num_threads=8)
+    for arr in dasp.ARRAYS:
+        assert np.array_equal(dasp.dasp_plan_copy_array(p1, arr), dasp.dasp_plan_copy_array(p8, arr)), arr
+
+
+def test_exports_every_header_symbol():
+    import re
+    hdr = open(__file__.replace("tests/test_builder.py", "include/dasp.h")).read()
+    declared = set(re.findall(r"\b(dasp_[a-z_]+)\s*\(", hdr))
+    assert declared == set(dasp.EXPORTS)
+    lib = ctypes.CDLL(dasp.LIB_PATH)
+    for s in declared:
+        assert getattr(lib, s) is not None
+
+
+def test_status_strings_and_errors():
+    L = dasp.lib()
+    assert L.dasp_status_string(2) == b"DASP_ERR_INVALID_CSR"
+    A = synth.generate(synth.config("c1a"))
+    bad = A.row_ptr.copy()
+    bad[5], bad[6] = bad[6], bad[5] - 1            # decreasing row_ptr
+    with pytest.raises(dasp.DaspError) as e:
+        dasp.dasp_plan_create(bad, A.col, A.val, A.m, A.n, "f64", device=-1)
+    assert e.value.status == 2
+    col = A.col.copy()
+    col[7] = A.n                                    # column out of range
+    with pytest.raises(dasp.DaspError) as e:
+        dasp.dasp_plan_create(A.row_ptr, col, A.val, A.m, A.n, "f64", device=-1)
+    assert e.value.status == 2
+    with pytest.raises(dasp.DaspError) as e:
+        dasp.dasp_plan_create(A.row_ptr, A.col, A.val, A.m, -1, "f64", device=-1)
+    assert e.value.status == 1
+    h = ctypes.c_void_p()
+    assert L.dasp_plan_create(None, 1, 1, 0, None, None, None, 0, None) == 1
+    assert L.dasp_plan_create(ctypes.byref(h), 1, 1, 0, None, None, None, 0, None) == 1
+    # spmv on a host-only plan is unsupported, not a crash
+    p = dasp.dasp_plan_create(A.row_ptr, A.col, A.val, A.m, A.n, "f64", device=-1)
+    assert L.dasp_spmv(p.handle, 16, 32, 1.0, 0.0, None) == 5
+    assert L.dasp_spmv(None, 16, 32, 1.0, 0.0, None) == 1
+
+
+def test_degenerate_plans():
+    for m, n in [(0, 0), (5, 3), (3, 0)]:
+        rp = np.zeros(m + 1, dtype=np.int64)
+        p = dasp.dasp_plan_create(rp, np.zeros(0, np.int32), np.zeros(0), m, n, "f64", device=-1)
+        info = p.info
+        assert info["n_empty"] == m and info["nnz"] == 0 and info["launches_per_spmv"] == (1 if m else 0)
+
+
+def test_partition_rows_balanced():
+    A = synth.generate(synth.config("c3", scale=0.004))
+    for P in [1, 2, 3, 4, 8]:
+        s = dasp.dasp_partition_rows(A.row_ptr, P)
+        assert s[0] == 0 and s[-1] == A.m and (np.diff(s) >= 0).all()
+        for q in range(1, P):   # first row whose start offset reaches q*nnz/P
+            target = (A.nnz * q) // P
+            assert A.row_ptr[s[q]] >= target and (s[q] == 0 or A.row_ptr[s[q] - 1] < target)
+
+
+def test_remap_columns_padded_layout():
+    A = synth.generate(synth.config("c1b"))
+    s = dasp.dasp_partition_rows(A.row_ptr, 3)
+    col = A.col.copy()
+    S = dasp.dasp_remap_columns(col, s)
+    assert S == np.diff(s).max()
+    owner = np.searchsorted(s, A.col, side="right") - 1
+    assert np.array_equal(col, owner * S + (A.col - s[owner]))

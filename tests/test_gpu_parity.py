@@ -1,0 +1,238 @@
+"""GPU parity: libdasp.so kernels (through the C-ABI) vs the CPU oracle on the same seeded inputs.
+
+Bar (BASELINE.json north_star): FP64 |y - y_ref| <= 1e-12 * sum|a_ij x_j| per row; FP16
+<= 2e-3 * sum|a_ij x_j| against the FP64 oracle fed the same fp16 values; bit-exact on
+small-integer inputs (P5), identity / diagonal / permutation matrices (P2), and for the
+device copy of the packed format vs the oracle builder.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_sc_lu023_b200 import dasp  # noqa: E402
+
+VARIANTS = [dasp.DASP_VARIANT_MMA, dasp.DASP_VARIANT_CUDACORE]
+VNAME = {dasp.DASP_VARIANT_MMA: "mma", dasp.DASP_VARIANT_CUDACORE: "cudacore"}
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    torch.cuda.init()
+
+
+def make(A, dt, **kw):
+    val = A.val if dt == "f64" else A.val.astype(np.float16)
+    return dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dt, device=0, **kw)
+
+
+def run(plan, x_np, dt, alpha=1.0, beta=0.0, y0=None, variant=0):
+    xd = torch.from_numpy(np.ascontiguousarray(x_np.astype(np.float64 if dt == "f64" else np.float16))).cuda()
+    ydt = torch.float64 if dt == "f64" else torch.float32
+    if y0 is None:
+        y = torch.full((plan.m,), float("nan"), dtype=ydt, device="cuda")
+    else:
+        y = torch.from_numpy(np.ascontiguousarray(y0)).to(ydt).cuda()
+    dasp.dasp_spmv(plan, xd, y, alpha, beta, variant=variant)
+    torch.cuda.synchronize()
+    return y.cpu().numpy().astype(np.float64)
+
+
+def oracle_ref(A, x, dt, alpha=1.0, beta=0.0, y0=None):
+    if dt == "f16":
+        val = A.val.astype(np.float16).astype(np.float64)
+        x = x.astype(np.float16).astype(np.float64)
+        if y0 is not None:
+            y0 = y0.astype(np.float32).astype(np.float64)
+    else:
+        val = A.val
+    return oracle.spmv(A.row_ptr, A.col, val, x, alpha, beta, y0)
+
+
+def cases():
+    yield "c1a", lambda vm: synth.generate(synth.config("c1a", val_mode=vm))
+    yield "c1b", lambda vm: synth.generate(synth.config("c1b", val_mode=vm))
+    yield "c2s", lambda vm: synth.generate(synth.config("c2", scale=24 / 128, val_mode=vm))
+    yield "c3s", lambda vm: synth.generate(synth.config("c3", scale=0.01, val_mode=vm))
+    yield "c5s", lambda vm: synth.generate(synth.config("c5", scale=4e-4, val_mode=vm))
+    yield "c6s", lambda vm: synth.generate(synth.config("c6", scale=0.05, val_mode=vm))
+    lens = [0, 1, 2, 3, 4, 5, 9, 17, 31, 33, 64, 255, 256, 257, 300, 1000, 2049, 4, 4, 3, 2, 1, 1, 1, 7, 6]
+    yield "lens", lambda vm: synth.from_lengths(lens * 7, n=5000, val_mode=vm)
+
+
+CASES = list(cases())
+
+
+@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("name,gen", CASES, ids=[c[0] for c in CASES])
+def test_parity_random_values(name, gen, dt, variant):
+    A = gen(synth.VAL_UNIFORM)
+    x = synth.vector(11, A.n)
+    plan = make(A, dt)
+    y = run(plan, x, dt, variant=variant)
+    y_ref, s = oracle_ref(A, x, dt)
+    ok = oracle.tolerance_ok(y, y_ref, s, dt)
+    bad = np.flatnonzero(~ok)
+    assert ok.all(), f"{len(bad)} rows off, first {bad[:5]}: {y[bad[:5]]} vs {y_ref[bad[:5]]}"
+
+
+# P5: small-integer values make every summation order exact -> bit-exact in both dtypes,
+# which also pins the MMA fragment layout and the diagonal lanes (Fig. 4).
+@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("name,gen", CASES, ids=[c[0] for c in CASES])
+def test_parity_integer_bit_exact(name, gen, dt, variant):
+    A = gen(synth.VAL_INT)
+    x = synth.vector(12, A.n, synth.VAL_INT)
+    plan = make(A, dt)
+    y = run(plan, x, dt, variant=variant)
+    y_ref, _ = oracle_ref(A, x, dt)
+    assert np.array_equal(y, y_ref)
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_identity_diagonal_permutation_exact(dt):
+    n = 5003
+    rng = np.random.default_rng(3)
+    x = rng.uniform(-1, 1, n)
+    ar = np.arange(n + 1, dtype=np.int64)
+    for val, col in [(np.ones(n), np.arange(n)), (rng.uniform(-4, 4, n), np.arange(n)),
+                     (np.ones(n), rng.permutation(n))]:
+        A = synth.CSR(n, n, ar, col.astype(np.int32), val)
+        for v in VARIANTS:
+            y = run(make(A, dt), x, dt, variant=v)
+            y_ref, _ = oracle_ref(A, x, dt)
+            if dt == "f16":   # one fp16 x fp16 product is exact in fp32, then rounded to y's fp32
+                y_ref = y_ref.astype(np.float32).astype(np.float64)
+            assert np.array_equal(y, y_ref)
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_alpha_beta(dt):
+    A = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
+    x = synth.vector(1, A.n, synth.VAL_INT)
+    y0 = synth.vector(2, A.m, synth.VAL_INT)
+    plan = make(A, dt)
+    for alpha, beta in [(2.0, -1.0), (-0.5, 3.0), (1.0, 1.0), (0.0, 2.0), (0.0, 0.0), (3.0, 0.0)]:
+        for v in VARIANTS:
+            y = run(plan, x, dt, alpha, beta, y0, variant=v)
+            y_ref, _ = oracle_ref(A, x, dt, alpha, beta, y0)
+            assert np.array_equal(y, y_ref), (alpha, beta, v)
+    # beta == 0: y is not read (NaN in y must not propagate)
+    y = run(plan, x, dt, 1.0, 0.0, np.full(A.m, np.nan))
+    assert np.isfinite(y).all()
+
+
+# P11: pads carry a sentinel column, so an Inf in x only reaches rows that store that column
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_inf_in_x_only_reaches_referencing_rows(dt):
+    A = synth.generate(synth.config("c1b"))
+    x = synth.vector(4, A.n)
+    plan = make(A, dt)
+    base = run(plan, x, dt)
+    x2 = x.copy()
+    x2[0] = np.inf
+    for v in VARIANTS:
+        y = run(plan, x2, dt, variant=v)
+        touches = np.zeros(A.m, bool)
+        rows = np.repeat(np.arange(A.m), np.diff(A.row_ptr))
+        touches[rows[A.col == 0]] = True
+        assert np.array_equal(y[~touches], run(plan, x, dt, variant=v)[~touches])
+        assert not np.isfinite(y[touches]).any() or touches.sum() == 0
+    assert np.isfinite(base).all()
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_device_arrays_match_oracle_builder(dt):
+    A = synth.generate(synth.config("c1b"))
+    plan = make(A, dt)   # keep_host off: copy_array reads back the uploaded device buffers
+    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt)
+    for arr in dasp.ARRAYS:
+        assert np.array_equal(dasp.dasp_plan_copy_array(plan, arr), ref.arrays[arr]), arr
+
+
+def test_deterministic_and_variants_agree():
+    A = synth.generate(synth.config("c3", scale=0.01))
+    x = synth.vector(5, A.n)
+    plan = make(A, "f64")
+    a = run(plan, x, "f64")
+    b = run(plan, x, "f64")
+    assert np.array_equal(a, b)
+    c = run(plan, x, "f64", variant=dasp.DASP_VARIANT_CUDACORE)
+    y_ref, s = oracle_ref(A, x, "f64")
+    assert oracle.tolerance_ok(c, y_ref, s).all()
+
+
+def test_empty_and_degenerate():
+    for m, n in [(0, 0), (7, 3), (1, 1)]:
+        A = synth.CSR(m, n, np.zeros(m + 1, dtype=np.int64), np.zeros(0, np.int32), np.zeros(0))
+        for dt in ["f64", "f16"]:
+            plan = make(A, dt)
+            if m:
+                y = run(plan, np.ones(n), dt, 1.0, 0.0, np.full(m, np.nan))
+                assert np.array_equal(y, np.zeros(m))
+                y = run(plan, np.ones(n), dt, 1.0, 2.0, np.arange(m, dtype=np.float64))
+                assert np.array_equal(y, 2.0 * np.arange(m))
+
+
+def test_spmv_host_end_to_end():
+    A = synth.generate(synth.config("c1b"))
+    x = synth.vector(6, A.n)
+    plan = make(A, "f64")
+    y = np.full(A.m, np.nan)
+    dasp.dasp_spmv_host(plan, x, y)
+    y_ref, s = oracle.spmv_csr(A, x)
+    assert oracle.tolerance_ok(y, y_ref, s).all()
+    y0 = synth.vector(7, A.m)
+    y = y0.copy()
+    dasp.dasp_spmv_host(plan, x, y, 2.0, -1.0)
+    y_ref, s = oracle.spmv_csr(A, x, 2.0, -1.0, y0)
+    assert oracle.tolerance_ok(y, y_ref, s).all()
+
+
+def test_bad_device_args():
+    A = synth.generate(synth.config("c1a"))
+    plan = make(A, "f64")
+    x = torch.zeros(A.n, dtype=torch.float64, device="cuda")
+    with pytest.raises(ValueError):
+        dasp.dasp_spmv(plan, x, torch.zeros(A.m, dtype=torch.float32, device="cuda"))
+    with pytest.raises(dasp.DaspError):
+        dasp.dasp_spmv(plan, x, x, check=False)   # aliasing x == y
+
+
+# full-size configs, in the launch configuration bench.py times: sampled rows vs the oracle
+def _sampled_parity(A, dt, nsample=20000, seed=0):
+    x = synth.vector(13, A.n)
+    plan = make(A, dt)
+    y = run(plan, x, dt)
+    rng = np.random.default_rng(seed)
+    lens = np.diff(A.row_ptr)
+    rows = np.unique(np.concatenate([rng.integers(0, A.m, nsample), np.flatnonzero(lens > 256)[:2000],
+                                     [0, A.m - 1]]))
+    starts, ends = A.row_ptr[rows], A.row_ptr[rows + 1]
+    sub_rp = np.concatenate([[0], np.cumsum(ends - starts)]).astype(np.int64)
+    idx = np.concatenate([np.arange(s, e) for s, e in zip(starts, ends)]) if len(rows) else np.zeros(0, np.int64)
+    sub = synth.CSR(len(rows), A.n, sub_rp, A.col[idx], A.val[idx])
+    y_ref, s = oracle_ref(sub, x, dt)
+    ok = oracle.tolerance_ok(y[rows], y_ref, s, dt)
+    assert ok.all(), f"{(~ok).sum()} sampled rows off"
+    return plan
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_full_size_stencil_sampled(dt):
+    A = synth.generate(synth.config("c2"))
+    _sampled_parity(A, dt)
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+def test_full_size_powerlaw_sampled(dt):
+    A = synth.generate(synth.config("c3"))
+    _sampled_parity(A, dt)
