@@ -48,6 +48,7 @@ def parse():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f16"])
     ap.add_argument("--variant", default="mma", choices=["mma", "cudacore"])
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
+    ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=12.0)
@@ -241,7 +242,7 @@ def main():
     if world == 1:
         # single GPU: plain SpMV over resident inputs, y overwritten every step
         plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
-                                     device=local, variant=variant)
+                                     device=local, variant=variant, medium_rb_per_warp=args.rbw)
         xdt = torch.float64 if args.dtype == "f64" else torch.float16
         ydt = torch.float64 if args.dtype == "f64" else torch.float32
         xd = torch.from_numpy(x_global).to(xdt).to(dev)

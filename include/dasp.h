@@ -65,9 +65,14 @@ typedef struct {
     int32_t medium_rb_per_warp; /* row-blocks per warp in the medium kernel (P:L271-273
                                    LOOP_NUM); 0 = automatic                                   */
     int32_t num_threads;        /* host builder threads; 0 = all available                   */
+    int64_t panel_rows;         /* rows per panel (R28): each panel of consecutive
+                                   rows is classified, sorted and pieced on its own so x and y
+                                   windows stay L2-resident; 0 = automatic, -1 = one panel
+                                   (the paper's global format)                        */
 } dasp_options_t;
 
-/* Fills `opts` with the defaults: device 0, MMA variant, validate, no keep_host, auto LOOP_NUM. */
+/* Fills `opts` with the defaults: device 0, MMA variant, validate, no keep_host, auto LOOP_NUM,
+ * automatic panel size. */
 void dasp_options_default(dasp_options_t* opts);
 
 /* Plan statistics (Fig. 12's class shares; build cost). */
@@ -87,6 +92,7 @@ typedef struct {
     int64_t alg_bytes_beta1;                           /* ... with beta != 0                */
     int32_t medium_rb_per_warp;
     int32_t launches_per_spmv;                         /* kernels one dasp_spmv enqueues    */
+    int64_t panel_rows, n_panels;                      /* resolved panel size and count     */
     double build_ms, upload_ms;                        /* host build; host->device upload   */
 } dasp_plan_info_t;
 
@@ -154,7 +160,10 @@ typedef enum {
     DASP_ARR_LONG_VAL = 0, DASP_ARR_LONG_COL, DASP_ARR_GROUP_PTR, DASP_ARR_LONG_OUT,
     DASP_ARR_RB_PTR, DASP_ARR_REG_VAL, DASP_ARR_REG_COL, DASP_ARR_IRR_PTR, DASP_ARR_IRR_VAL,
     DASP_ARR_IRR_COL, DASP_ARR_MED_OUT, DASP_ARR_SHORT_VAL, DASP_ARR_SHORT_COL,
-    DASP_ARR_SHORT_OUT, DASP_ARR_EMPTY_ROWS, DASP_ARR_COUNT
+    DASP_ARR_SHORT_OUT, DASP_ARR_EMPTY_ROWS,
+    DASP_ARR_PANELS,        /* int64 [n_panels][12]: row0, rows, unit0, nunits, rb0, nrb, tile0,
+                               t13, t4, t22, ts, out0                           */
+    DASP_ARR_COUNT
 } dasp_array_t;
 
 /*

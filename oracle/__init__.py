@@ -27,9 +27,10 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 
 ARRAYS = ["long_val", "long_col", "group_ptr", "long_out", "rb_ptr", "reg_val", "reg_col", "irr_ptr",
-          "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows"]
+          "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows", "panels"]
 COUNTS = ["m", "n", "nnz", "n0", "n1", "n2", "n3", "n4", "row_medium", "row_long", "nrb", "n_groups",
-          "n_groups_padded", "t13", "t4", "t22", "ts", "nnz_long_new", "nnz_reg_new", "nnz_irreg", "nnz_short_new"]
+          "n_groups_padded", "t13", "t4", "t22", "ts", "nnz_long_new", "nnz_reg_new", "nnz_irreg", "nnz_short_new",
+          "panel_rows", "n_panels"]
 
 
 def build_lib() -> str:
@@ -49,7 +50,7 @@ def _L():
         lib = ctypes.CDLL(_SO)
         vp, i64, d = ctypes.c_void_p, ctypes.c_int64, ctypes.c_double
         lib.oracle_spmv.argtypes = [i64, vp, vp, vp, vp, d, d, vp, vp, vp]
-        lib.oracle_build.argtypes = [ctypes.c_int, i64, i64, vp, vp, vp]
+        lib.oracle_build.argtypes = [ctypes.c_int, i64, i64, vp, vp, vp, i64]
         lib.oracle_build.restype = vp
         lib.oracle_free.argtypes = [vp]
         lib.oracle_fmt_count.argtypes = [vp, ctypes.c_char_p]
@@ -104,13 +105,13 @@ def tolerance_ok(y, y_ref, s, dtype="f64"):
 class Format:
     """The oracle builder's arrays (numpy copies) and counts."""
 
-    def __init__(self, A, dtype="f64"):
+    def __init__(self, A, dtype="f64", panel_rows=0):
         lib = _L()
         dt = 0 if dtype == "f64" else 1
         val = np.ascontiguousarray(A.val.astype(np.float64 if dt == 0 else np.float16))
         rp = np.ascontiguousarray(A.row_ptr, dtype=np.int64)
         col = np.ascontiguousarray(A.col, dtype=np.int32)
-        h = lib.oracle_build(dt, A.m, A.n, _p(rp), _p(col), _p(val))
+        h = lib.oracle_build(dt, A.m, A.n, _p(rp), _p(col), _p(val), int(panel_rows))
         try:
             self.counts = {c: int(lib.oracle_fmt_count(h, c.encode())) for c in COUNTS}
             self.arrays = {}
@@ -127,10 +128,11 @@ class Format:
         b = self.arrays[name]
         if name.endswith("_val"):
             return b.view(np.float64 if self.dtype == "f64" else np.float16)
-        if name in ("group_ptr", "rb_ptr", "irr_ptr"):
+        if name in ("group_ptr", "rb_ptr", "irr_ptr", "panels"):
             return b.view(np.int64)
         return b.view(np.int32)
 
 
-def build(A, dtype="f64") -> Format:
-    return Format(A, dtype)
+def build(A, dtype="f64", panel_rows=0) -> Format:
+    """panel_rows <= 0: one panel (the paper's global format); else panels of that many rows."""
+    return Format(A, dtype, panel_rows)

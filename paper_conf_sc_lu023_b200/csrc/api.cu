@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -30,7 +31,12 @@ struct dasp_plan_s {
     void* d_yh = nullptr;
     int64_t device_bytes = 0;
     double build_ms = 0, upload_ms = 0;
-    int64_t w_long = 0, w_med = 0, w_short = 0;
+    int64_t blocks = 0;                   // grid of the fused main kernel
+    void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
+    void* d_blk_panel = nullptr;          // int32 panel of every block
+    int32_t xmode = 0;                    // x gather policy (kernels.cuh MainParams::xmode)
+    size_t apw_bytes = 0;                 // L2 persisting access-policy window over x (0 = off)
+    float apw_hit = 1.0f;
     // timing
     int32_t timing_cap = 0, timing_calls = 0;
     std::vector<TimingRec> recs;
@@ -44,6 +50,10 @@ int sx(int dtype) { return dtype == DASP_R_64F ? 8 : 2; }
 int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
 
 // LOOP_NUM of P:L271-273 (R11): row-blocks per warp from the number of medium rows
+// automatic panel: ~1M rows keeps a panel's x window and y (8 B each per row) well inside the
+// ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
+constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
+
 int auto_rbw(int64_t row_medium) {
     if (row_medium < 59990) return 1;
     if (row_medium < 400000) return 2;
@@ -68,6 +78,9 @@ void free_device(dasp_plan_s* p) {
         ptr = nullptr;
     }
     if (p->d_partial) cudaFree(p->d_partial);
+    if (p->d_panels) cudaFree(p->d_panels);
+    if (p->d_blk_panel) cudaFree(p->d_blk_panel);
+    p->d_panels = p->d_blk_panel = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -126,6 +139,7 @@ void dasp_options_default(dasp_options_t* o) {
     o->keep_host = 0;
     o->medium_rb_per_warp = 0;
     o->num_threads = 0;
+    o->panel_rows = 0;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -162,7 +176,10 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     p->keep_host = o.keep_host != 0 || o.device < 0;
 
     auto t0 = std::chrono::steady_clock::now();
-    int st = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0);
+    // panel size (R28): -1 one panel (the paper's global format); 0 automatic; env override
+    int64_t panel_rows = o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
+    if (const char* pr = std::getenv("DASP_PANEL_ROWS")) panel_rows = std::atoll(pr);
+    int st = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0, panel_rows);
     auto t1 = std::chrono::steady_clock::now();
     p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
     if (st != DASP_OK) {
@@ -171,9 +188,25 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     }
     HostFormat& f = p->host;
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium);
-    p->w_long = f.n_groups_padded / f.geo.UG;
-    p->w_med = (f.nrb + p->rbw - 1) / p->rbw;
-    p->w_short = f.t13 + f.t4 + f.t22 + f.ts;
+    // per-panel launch descriptors: warps = long units + medium warps + tiles
+    std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
+    std::vector<int32_t> blk_panel;
+    {
+        const int64_t* pt = static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr);
+        int64_t blk = 0;
+        for (int64_t q = 0; q < f.n_panels; ++q) {
+            const int64_t* e = pt + q * dasp::PANEL_FIELDS;
+            dasp::PanelDesc& d = desc[q];
+            d.blk0 = blk;
+            d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5]; d.nmw = (e[5] + p->rbw - 1) / p->rbw;
+            d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
+            const int64_t warps = d.nunits + d.nmw + d.t13 + d.t4 + d.t22 + d.ts;
+            const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
+            blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
+            blk += nb;
+        }
+        p->blocks = blk;
+    }
     for (int a = 0; a < DASP_ARR_COUNT; ++a) p->bytes[a] = f.arr[a].bytes;
 
     if (p->device >= 0) {
@@ -193,6 +226,34 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
             return DASP_ERR_OUT_OF_MEMORY;
         }
         p->device_bytes += pb;
+        const size_t db = desc.size() * sizeof(dasp::PanelDesc), bb = std::max<size_t>(blk_panel.size(), 1) * 4;
+        if (cudaMalloc(&p->d_panels, std::max<size_t>(db, 1)) != cudaSuccess || cudaMalloc(&p->d_blk_panel, bb) != cudaSuccess) {
+            free_device(p); f.release(); delete p;
+            return DASP_ERR_OUT_OF_MEMORY;
+        }
+        if ((db && cudaMemcpy(p->d_panels, desc.data(), db, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            (!blk_panel.empty() && cudaMemcpy(p->d_blk_panel, blk_panel.data(), blk_panel.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)) {
+            free_device(p); f.release(); delete p;
+            return DASP_ERR_CUDA;
+        }
+        p->device_bytes += db + bb;
+        // x residency in L2 (R17): evict_last gathers and/or a persisting access-policy window
+        const char* xm = std::getenv("DASP_XMODE");
+        p->xmode = xm ? std::atoi(xm) : 0;
+        const char* apw = std::getenv("DASP_X_APW");
+        if (apw && std::atoi(apw) > 0) {
+            cudaDeviceProp prop;
+            if (cudaGetDeviceProperties(&prop, p->device) == cudaSuccess && prop.persistingL2CacheMaxSize > 0) {
+                const size_t xb = static_cast<size_t>(f.n) * sx(dtype);
+                size_t lim = std::min<size_t>(static_cast<size_t>(prop.persistingL2CacheMaxSize), xb);
+                size_t win = std::min<size_t>(static_cast<size_t>(prop.accessPolicyMaxWindowSize), xb);
+                if (lim > 0 && win > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim) == cudaSuccess) {
+                    p->apw_bytes = win;
+                    p->apw_hit = std::min(1.0f, static_cast<float>(lim) / static_cast<float>(win));
+                }
+            }
+            cudaGetLastError();
+        }
         auto u0 = std::chrono::steady_clock::now();
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
             if (p->bytes[a] == 0) continue;
@@ -247,13 +308,20 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
     mp.y = y;
     mp.alpha = alpha;
     mp.beta = beta;
-    mp.nrb = f.nrb;
-    mp.t13 = f.t13; mp.t4 = f.t4; mp.t22 = f.t22; mp.ts = f.ts;
-    mp.w_long = p->w_long;
-    mp.w_med = p->w_med;
-    mp.w_total = p->w_long + p->w_med + p->w_short;
+    mp.panels = static_cast<const dasp::PanelDesc*>(p->d_panels);
+    mp.blk_panel = static_cast<const int32_t*>(p->d_blk_panel);
     mp.rbw = p->rbw;
-    e = timed(p, DASP_K_MAIN, s, on, [&] { return dasp::launch_main(mp, p->dtype, variant, 0, mp.w_total, s); });
+    mp.xmode = p->xmode;
+    mp.class_mask = 7;
+    // DASP_PROFILE_CLASS (profiling only; the other classes' rows are then NOT computed):
+    // 1 = long units, 2 = medium warps, 3 = short tiles
+    if (const char* pc = std::getenv("DASP_PROFILE_CLASS")) {
+        const int c = std::atoi(pc);
+        if (c >= 1 && c <= 3) mp.class_mask = 1 << (c - 1);
+    }
+    e = timed(p, DASP_K_MAIN, s, on, [&] {
+        return dasp::launch_main(mp, p->dtype, variant, p->blocks, s, x, p->apw_bytes, p->apw_hit);
+    });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
     const int64_t n0 = beta == 1.0 ? 0 : f.n0;
     if (f.row_long + n0 > 0) {
@@ -325,7 +393,9 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta0 = alg_bytes(p, false);
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
-    o->launches_per_spmv = (p->w_long + p->w_med + p->w_short > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
+    o->launches_per_spmv = (p->blocks > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
+    o->panel_rows = f.panel_rows;
+    o->n_panels = f.n_panels;
     o->build_ms = p->build_ms;
     o->upload_ms = p->upload_ms;
     return DASP_OK;

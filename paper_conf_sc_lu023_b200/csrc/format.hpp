@@ -29,6 +29,7 @@ constexpr int MAX_LEN = 256;
 constexpr int MMA_M = 8;
 constexpr int32_t PAD_COL = -1;  // R12: sentinel column of pads (x read as 0)
 constexpr int SHORT_TILE = 128;  // elements per short tile (32 four-slot rows)
+constexpr int PANEL_FIELDS = 12; // row0, rows, unit0, nunits, rb0, nrb, tile0, t13, t4, t22, ts, out0
 
 struct HostBuf {
     void* ptr = nullptr;
@@ -43,12 +44,14 @@ struct HostFormat {
     int64_t nrb = 0, n_groups = 0, n_groups_padded = 0, t13 = 0, t4 = 0, t22 = 0, ts = 0;
     int64_t nnz_long_new = 0, nnz_reg_new = 0, nnz_irreg = 0, nnz_short_new = 0;
     int64_t nnz_long = 0, nnz_medium = 0, nnz_short = 0;
+    int64_t panel_rows = 0;   // rows per panel (R28); >= m: one panel = the paper's global format
+    int64_t n_panels = 0;
     HostBuf arr[DASP_ARR_COUNT];
     void release();
 };
 
 // Builds the format on the host.  Returns a dasp_status_t.
 int build_format(HostFormat& f, int dtype, int64_t m, int64_t n, const int64_t* row_ptr,
-                 const int32_t* col, const void* val, int nthreads, bool validate);
+                 const int32_t* col, const void* val, int nthreads, bool validate, int64_t panel_rows);
 
 }  // namespace dasp

@@ -63,13 +63,40 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
     return v;
 }
-// x gather: column -1 (pad, R12) reads 0 without touching memory
-__device__ __forceinline__ double gx(const double* x, uint32_t c) {
-    return static_cast<int32_t>(c) >= 0 ? __ldg(x + static_cast<int32_t>(c)) : 0.0;
+// x gather: column -1 (pad, R12) reads 0 without touching memory.  x lines carry an L2
+// evict_last policy so the streamed A arrays (evict_first) do not push x out of L2.
+__device__ __forceinline__ uint64_t x_policy() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
 }
-__device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
-    return static_cast<int32_t>(c) >= 0 ? __ldg(reinterpret_cast<const unsigned short*>(x) + static_cast<int32_t>(c))
-                                        : static_cast<uint16_t>(0);
+struct XLoad {
+    uint64_t pol;
+    int mode;   // 0: plain read-only load, 1: L2 evict_last hint
+};
+__device__ __forceinline__ double ldx(const double* p, const XLoad& xl) {
+    if (xl.mode == 1) {
+        double v;
+        asm("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(xl.pol));
+        return v;
+    }
+    return __ldg(p);
+}
+__device__ __forceinline__ uint16_t ldxh(const uint16_t* p, const XLoad& xl) {
+    if (xl.mode == 1) {
+        uint16_t v;
+        asm("ld.global.nc.L2::cache_hint.b16 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(xl.pol));
+        return v;
+    }
+    return __ldg(reinterpret_cast<const unsigned short*>(p));
+}
+#define gx(x, c) gx_(x, c, XL)
+#define gxh(x, c) gxh_(x, c, XL)
+__device__ __forceinline__ double gx_(const double* x, uint32_t c, const XLoad& XL) {
+    return static_cast<int32_t>(c) >= 0 ? ldx(x + static_cast<int32_t>(c), XL) : 0.0;
+}
+__device__ __forceinline__ uint16_t gxh_(const uint16_t* x, uint32_t c, const XLoad& XL) {
+    return static_cast<int32_t>(c) >= 0 ? ldxh(x + static_cast<int32_t>(c), XL) : static_cast<uint16_t>(0);
 }
 __device__ __forceinline__ float h2f(uint16_t h) { return __half2float(__ushort_as_half(h)); }
 __device__ __forceinline__ float2 u2f2(uint32_t u) {  // two packed binary16 -> two f32 (exact)
@@ -133,7 +160,7 @@ __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typena
 // long rows, phase 1 (Alg. 2 l.1-16): one warp = one unit of UG consecutive groups
 // ------------------------------------------------------------------------------------------
 template <int VAR>
-__device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol) {
+__device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol, const XLoad& XL) {
     const int64_t base = u * 256 + lane * 8;            // lane holds 8 consecutive elements
     const double* lv = static_cast<const double*>(P.long_val) + base;
     double v[8];
@@ -165,7 +192,7 @@ __device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, in
 }
 
 template <int VAR>
-__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol) {
+__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol, const XLoad& XL) {
     const int64_t base = u * 512 + lane * 16;           // lane holds 16 consecutive elements
     uint32_t vv[8], c[16];
     ld8_b32(static_cast<const uint16_t*>(P.long_val) + base, pol, vv);
@@ -204,7 +231,7 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
 // of CW blocks (R18), then the irregular tails with 4 lanes per row, then y.
 // ------------------------------------------------------------------------------------------
 template <int VAR>
-__device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
+__device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, int lane, uint64_t pol, const XLoad& XL) {
     const int g = lane >> 2, t = lane & 3;
     const int64_t base = P.rb_ptr[rb];
     const int64_t nreg = (P.rb_ptr[rb + 1] - base) >> 5;
@@ -251,7 +278,7 @@ __device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, i
 }
 
 template <int VAR>
-__device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
+__device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, int lane, uint64_t pol, const XLoad& XL) {
     const int g = lane >> 2, t = lane & 3;
     const int64_t base = P.rb_ptr[rb];
     const int64_t nreg = (P.rb_ptr[rb + 1] - base) >> 7;
@@ -310,7 +337,7 @@ __device__ __forceinline__ int seg_of(int cat, int slot) { return cat == 0 ? (sl
 
 template <int VAR>
 __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol) {
+                                               uint64_t pol, const XLoad& XL) {
     const int g = lane >> 2, t = lane & 3;
     double v[4];
     uint32_t c[4];
@@ -342,7 +369,7 @@ __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int
 
 template <int VAR>
 __device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol) {
+                                               uint64_t pol, const XLoad& XL) {
     const int g = lane >> 2, t = lane & 3;
     uint32_t a0, a2, c[4];
     ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
@@ -387,7 +414,7 @@ __device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int
 
 // singles (Alg. 5): lane handles 4 consecutive len-1 rows on CUDA cores
 template <int DT>
-__device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, int64_t obase, int lane, uint64_t pol) {
+__device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, int64_t obase, int lane, uint64_t pol, const XLoad& XL) {
     uint32_t c[4], o[4];
     ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
     ld4_b32(P.short_out + obase + lane * 4, pol, o);
@@ -411,40 +438,48 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
 // ------------------------------------------------------------------------------------------
 // the fused main kernel
 // ------------------------------------------------------------------------------------------
+#ifndef DASP_MIN_BLOCKS
+#define DASP_MIN_BLOCKS 1
+#endif
 template <int DT, int VAR>
-__global__ void __launch_bounds__(MAIN_THREADS) dasp_main_kernel(const MainParams P, int64_t w_begin, int64_t w_end) {
+__global__ void __launch_bounds__(MAIN_THREADS, DASP_MIN_BLOCKS) dasp_main_kernel(const MainParams P) {
     const int lane = threadIdx.x & 31;
-    int64_t w = w_begin + (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) / 32;
-    if (w >= w_end) return;
+    const PanelDesc D = P.panels[P.blk_panel[blockIdx.x]];
+    int64_t w = (static_cast<int64_t>(blockIdx.x) - D.blk0) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
     const uint64_t pol = stream_policy();
-    if (w < P.w_long) {
-        if constexpr (DT == 0) long_unit_f64<VAR>(P, w, lane, pol);
-        else long_unit_f16<VAR>(P, w, lane, pol);
+    const XLoad XL{x_policy(), P.xmode};
+    if (w < D.nunits) {                                  // long rows, phase 1
+        if (!(P.class_mask & 1)) return;
+        if constexpr (DT == 0) long_unit_f64<VAR>(P, D.unit0 + w, lane, pol, XL);
+        else long_unit_f16<VAR>(P, D.unit0 + w, lane, pol, XL);
         return;
     }
-    w -= P.w_long;
-    if (w < P.w_med) {
-        const int64_t rb0 = w * P.rbw;
-        const int64_t rb1 = rb0 + P.rbw < P.nrb ? rb0 + P.rbw : P.nrb;
+    w -= D.nunits;
+    if (w < D.nmw) {                                     // medium rows
+        if (!(P.class_mask & 2)) return;
+        const int64_t rb0 = D.rb0 + w * P.rbw;
+        const int64_t rb1 = min(rb0 + P.rbw, D.rb0 + D.nrb);
         for (int64_t rb = rb0; rb < rb1; ++rb) {
-            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb, lane, pol);
-            else medium_rb_f16<VAR>(P, rb, lane, pol);
+            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb, lane, pol, XL);
+            else medium_rb_f16<VAR>(P, rb, lane, pol, XL);
         }
         return;
     }
-    int64_t tile = w - P.w_med;                         // short tiles: [1&3][len4][2&2][singles]
+    int64_t t = w - D.nmw;                               // short tiles: [1&3][len4][2&2][singles]
+    if (t >= D.t13 + D.t4 + D.t22 + D.ts || !(P.class_mask & 4)) return;
+    const int64_t tile = D.tile0 + t;
     int cat;
     int64_t obase;
-    if (tile < P.t13) { cat = 0; obase = tile * 64; }
-    else if (tile < P.t13 + P.t4) { cat = 1; obase = 64 * P.t13 + (tile - P.t13) * 32; }
-    else if (tile < P.t13 + P.t4 + P.t22) { cat = 2; obase = 64 * P.t13 + 32 * P.t4 + (tile - P.t13 - P.t4) * 64; }
+    if (t < D.t13) { cat = 0; obase = D.out0 + t * 64; }
+    else if (t < D.t13 + D.t4) { cat = 1; obase = D.out0 + 64 * D.t13 + (t - D.t13) * 32; }
+    else if (t < D.t13 + D.t4 + D.t22) { cat = 2; obase = D.out0 + 64 * D.t13 + 32 * D.t4 + (t - D.t13 - D.t4) * 64; }
     else {
-        obase = 64 * P.t13 + 32 * P.t4 + 64 * P.t22 + (tile - P.t13 - P.t4 - P.t22) * 128;
-        singles_tile<DT>(P, tile, obase, lane, pol);
+        obase = D.out0 + 64 * D.t13 + 32 * D.t4 + 64 * D.t22 + (t - D.t13 - D.t4 - D.t22) * 128;
+        singles_tile<DT>(P, tile, obase, lane, pol, XL);
         return;
     }
-    if constexpr (DT == 0) short_tile_f64<VAR>(P, cat, tile, obase, lane, pol);
-    else short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
+    if constexpr (DT == 0) short_tile_f64<VAR>(P, cat, tile, obase, lane, pol, XL);
+    else short_tile_f16<VAR>(P, cat, tile, obase, lane, pol, XL);
 }
 
 // long phase 2 (Alg. 2 l.17-25): one warp per long row, lane-strided sum of the group partials
@@ -488,19 +523,41 @@ __global__ void dasp_scale_kernel(void* yv, int64_t m, double beta) {
 
 }  // namespace
 
-cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t w_begin, int64_t w_end, cudaStream_t s) {
-    if (w_end <= w_begin) return cudaSuccess;
-    const int64_t warps = w_end - w_begin;
-    const int64_t blocks = (warps * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
-    if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-    dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
-    if (dtype == 0) {
-        if (variant == VAR_MMA) dasp_main_kernel<0, VAR_MMA><<<grid, block, 0, s>>>(p, w_begin, w_end);
-        else dasp_main_kernel<0, VAR_CUDACORE><<<grid, block, 0, s>>>(p, w_begin, w_end);
-    } else {
-        if (variant == VAR_MMA) dasp_main_kernel<1, VAR_MMA><<<grid, block, 0, s>>>(p, w_begin, w_end);
-        else dasp_main_kernel<1, VAR_CUDACORE><<<grid, block, 0, s>>>(p, w_begin, w_end);
+template <typename Kern>
+static cudaError_t launch_ex(Kern kernel, unsigned blocks, cudaStream_t s, const void* apw_base, size_t apw_bytes,
+                             float apw_hit, const MainParams& p) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(blocks);
+    cfg.blockDim = dim3(MAIN_THREADS);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    if (apw_bytes) {
+        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(apw_base);
+        attr[0].val.accessPolicyWindow.num_bytes = apw_bytes;
+        attr[0].val.accessPolicyWindow.hitRatio = apw_hit;
+        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
     }
+    return cudaLaunchKernelEx(&cfg, kernel, p);
+}
+
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
+                        const void* apw_base, size_t apw_bytes, float apw_hit) {
+    if (blocks <= 0) return cudaSuccess;
+    if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    const unsigned nb = static_cast<unsigned>(blocks);
+    cudaError_t e;
+    if (dtype == 0) {
+        if (variant == VAR_MMA) e = launch_ex(dasp_main_kernel<0, VAR_MMA>, nb, s, apw_base, apw_bytes, apw_hit, p);
+        else e = launch_ex(dasp_main_kernel<0, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
+    } else {
+        if (variant == VAR_MMA) e = launch_ex(dasp_main_kernel<1, VAR_MMA>, nb, s, apw_base, apw_bytes, apw_hit, p);
+        else e = launch_ex(dasp_main_kernel<1, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
+    }
+    if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 

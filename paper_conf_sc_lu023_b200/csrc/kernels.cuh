@@ -6,10 +6,21 @@
 
 namespace dasp {
 
-// Everything the fused main kernel reads.  Warp ranges (global warp index w):
-//   [0, w_long)                 long phase 1: one unit of UG groups per warp (Alg. 2 l.1-16)
-//   [w_long, w_long + w_med)    medium: `rbw` row-blocks per warp (Alg. 3, LOOP_NUM P:L271)
-//   [w_long + w_med, w_total)   short: one tile per warp (1&3 | len4 | 2&2 | singles; Alg. 4-5)
+constexpr int MAIN_THREADS = 256;
+constexpr int WARPS_PER_BLOCK = MAIN_THREADS / 32;
+
+// One row panel (R28) as the fused kernel sees it.  A panel owns the blocks
+// [blk0, blk0 + ceil(warps/8)); its warps are, in order:
+//   nunits long units (UG groups each; Alg. 2 l.1-16), nmw medium warps (rbw row-blocks each;
+//   Alg. 3, LOOP_NUM P:L271), then one warp per short tile (1&3 | len4 | 2&2 | singles).
+struct PanelDesc {
+    int64_t blk0;
+    int64_t unit0, nunits;
+    int64_t rb0, nrb, nmw;
+    int64_t tile0, t13, t4, t22, ts, out0;
+};
+
+// Everything the fused main kernel reads.
 struct MainParams {
     const void* long_val;
     const int32_t* long_col;
@@ -24,13 +35,14 @@ struct MainParams {
     const void* short_val;
     const int32_t* short_col;
     const int32_t* short_out;
+    const PanelDesc* panels;
+    const int32_t* blk_panel; // panel of every block
     const void* x;
     void* y;
     double alpha, beta;
-    int64_t nrb;
-    int64_t t13, t4, t22, ts;
-    int64_t w_long, w_med, w_total;
     int32_t rbw;
+    int32_t xmode;            // x gather cache policy: 0 plain, 1 L2 evict_last
+    int32_t class_mask;       // bit 0 long, bit 1 medium, bit 2 short (profiling; 7 = all)
 };
 
 struct FinishParams {
@@ -44,12 +56,10 @@ struct FinishParams {
 };
 
 // variant: 1 = MMA (DMMA/HMMA diagonal trick), 2 = CUDA-core.  dtype: 0 = FP64, 1 = FP16.
-// w_begin/w_end select a sub-range of the main kernel's warps (whole range for a normal call).
-cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t w_begin, int64_t w_end,
-                        cudaStream_t s);
+// apw_bytes > 0: launch with an L2 access-policy window (persisting) over [apw_base, +apw_bytes)
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
+                        const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s);
 cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s);
-
-constexpr int MAIN_THREADS = 256;
 
 }  // namespace dasp

@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdasp.so")
+LIB_PATH = os.environ.get("DASP_LIB", os.path.join(_HERE, "libdasp.so"))   # override: experiment builds
 
 DASP_R_64F, DASP_R_16F = 0, 1
 DASP_VARIANT_DEFAULT, DASP_VARIANT_MMA, DASP_VARIANT_CUDACORE = 0, 1, 2
@@ -21,7 +21,7 @@ DASP_K_MAIN, DASP_K_FINISH, DASP_K_SCALE, DASP_K_COUNT = 0, 1, 2, 3
 KERNEL_NAMES = ["dasp_main_kernel", "dasp_finish_kernel", "dasp_scale_kernel"]
 
 ARRAYS = ["long_val", "long_col", "group_ptr", "long_out", "rb_ptr", "reg_val", "reg_col", "irr_ptr",
-          "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows"]
+          "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows", "panels"]
 STATUS = ["DASP_OK", "DASP_ERR_INVALID_ARG", "DASP_ERR_INVALID_CSR", "DASP_ERR_OUT_OF_MEMORY",
           "DASP_ERR_CUDA", "DASP_ERR_UNSUPPORTED", "DASP_ERR_INTERNAL"]
 
@@ -42,7 +42,7 @@ class DaspError(RuntimeError):
 class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("variant", ctypes.c_int32), ("validate", ctypes.c_int32),
                 ("keep_host", ctypes.c_int32), ("medium_rb_per_warp", ctypes.c_int32),
-                ("num_threads", ctypes.c_int32)]
+                ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -54,6 +54,7 @@ class PlanInfo(ctypes.Structure):
                    "nnz_long_new", "nnz_reg_new", "nnz_irreg", "nnz_short_new", "nnz_long", "nnz_medium",
                    "nnz_short", "device_bytes", "alg_bytes_beta0", "alg_bytes_beta1")] + \
                [("medium_rb_per_warp", ctypes.c_int32), ("launches_per_spmv", ctypes.c_int32),
+                ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64),
                 ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double)]
 
     def as_dict(self):
@@ -150,11 +151,11 @@ class Plan:
 
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                      variant: int = DASP_VARIANT_MMA, validate: bool = True, keep_host: bool = False,
-                     medium_rb_per_warp: int = 0, num_threads: int = 0) -> Plan:
+                     medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
-    (dtype "f16"; passed as binary16 bits)."""
+    (dtype "f16"; passed as binary16 bits).  panel_rows: 0 automatic, -1 one global panel."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     if dtype == "f64":
@@ -172,6 +173,7 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     _lib.dasp_options_default(ctypes.byref(opts))
     opts.device, opts.variant, opts.validate = device, variant, int(validate)
     opts.keep_host, opts.medium_rb_per_warp, opts.num_threads = int(keep_host), medium_rb_per_warp, num_threads
+    opts.panel_rows = panel_rows
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))

@@ -48,8 +48,11 @@ def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, re
     starts = slab_bounds(row_lengths, world)
     r0, r1 = int(starts[rank]), int(starts[rank + 1])
     A = generate_rows(r0, r1 - r0)
-    col = np.ascontiguousarray(A.col, dtype=np.int32).copy()
-    S = dasp.dasp_remap_columns(col, starts)
+    if world == 1:                      # one slab: no remap (also valid for rectangular matrices)
+        col, S = np.ascontiguousarray(A.col, dtype=np.int32), A.n
+    else:
+        col = np.ascontiguousarray(A.col, dtype=np.int32).copy()
+        S = dasp.dasp_remap_columns(col, starts)
     absval = np.abs(A.val.astype(np.float64))
     lens = np.diff(A.row_ptr)
     rs = np.zeros(len(lens))

@@ -12,6 +12,7 @@ Configs (BASELINE.json ``configs``):
 * ``c3``   power-law lengths on [1,1e5], 12.5M rows, ~2e8 nnz             (configs[2])
 * ``c5``   mixed-class, mean length ~64, row 1-norm <= 1                  (configs[4])
 * ``c6``   short-only rows, len U{1..4}                                   (mc2depi-like)
+* ``c7``   long-only rows, len log-uniform [257, 2e4], 40K rows, ~1.8e8 nnz (per-class probe)
 """
 from __future__ import annotations
 
@@ -174,13 +175,23 @@ def config(name: str, seed: int | None = None, val_mode: int = VAL_UNIFORM, scal
         m = s(62_500_000)
         return Spec(SYN_MIXED64, m, m, 5 if seed is None else seed, val_mode, local_frac=0.5, local_w=4096,
                     zipf_s=1.1, name=name)
+    if name == "c7":  # long rows only: lengths log-uniform on [257, 2e4], columns as c3
+        m = s(40_000)
+        return Spec(SYN_LENLIST, m, 12_500_000, 7 if seed is None else seed, val_mode,
+                    lenlist=_long_lengths(m, 7 if seed is None else seed), local_frac=0.5, local_w=4096,
+                    zipf_s=1.1, name=name)
     if name == "c6":
         m = s(525_000)
         return Spec(SYN_SHORT, m, m, 6 if seed is None else seed, val_mode, name=name)
     raise KeyError(name)
 
 
+def _long_lengths(m, seed):
+    rng = np.random.default_rng(seed)
+    return np.exp(rng.uniform(np.log(257), np.log(20000), m)).astype(np.int64)
+
+
 def from_lengths(lens, n: int, seed: int = 7, val_mode: int = VAL_UNIFORM, name: str = "lenlist") -> CSR:
     lens = np.asarray(lens, dtype=np.int64)
-    spec = Spec(SYN_LENLIST, len(lens), n, seed, val_mode, lenlist=lens, name=name)
+    spec = Spec(SYN_LENLIST, len(lens), n, seed, val_mode, lenlist=lens, local_frac=0.0, name=name)
     return generate(spec)

@@ -208,6 +208,9 @@ static void row_cols(int kind, const synth_params* p, int64_t row, int64_t L, in
         }
         return; /* already ascending and distinct */
     }
+    case SYN_LENLIST:
+        if (p->local_frac <= 0.0) goto uniform;
+        /* fall through: local + Zipf columns */
     case SYN_POWERLAW:
     case SYN_MIXED64: {
         double one_minus_s = 1.0 - p->zipf_s;
@@ -228,7 +231,8 @@ static void row_cols(int kind, const synth_params* p, int64_t row, int64_t L, in
         }
         break;
     }
-    default: /* uniform columns */
+    default:
+    uniform: /* uniform columns */
         for (int64_t k = 0; k < L; ++k) c[k] = (int64_t)(u01(rng3(s, (uint64_t)row, K_COL(k))) * (double)n);
     }
     make_distinct(c, L, n);

@@ -32,21 +32,22 @@ def decode(F, get, dtype):
     def emit(row, c, v):
         rows.setdefault(int(row), []).append((int(c), int(v)))
 
-    # long
+    # long: each row's groups hold its elements then trailing pads; every other slot is a pad
     lv, lc, gp, lo = _bits(get("long_val")), get("long_col"), get("group_ptr"), get("long_out")
     assert len(lv) == F["n_groups_padded"] * G
+    covered = np.zeros(len(lc), dtype=bool)
     for r in range(F["row_long"]):
         seg_c = lc[gp[r] * G: gp[r + 1] * G]
         seg_v = lv[gp[r] * G: gp[r + 1] * G]
+        covered[gp[r] * G: gp[r + 1] * G] = True
         real = seg_c != PAD
         nreal = int(real.sum())
         assert real[:nreal].all(), "long pads must trail the row"
         for c, v in zip(seg_c[:nreal], seg_v[:nreal]):
             emit(lo[r], c, v)
         pads += list(zip(seg_c[nreal:], seg_v[nreal:]))
-    tail_c = lc[F["n_groups"] * G:]
-    pads += list(zip(tail_c, lv[F["n_groups"] * G:]))
-    assert (tail_c == PAD).all()
+    pads += list(zip(lc[~covered], lv[~covered]))
+    assert (lc[~covered] == PAD).all()
 
     # medium: regular chunks, then irregular tails
     rv, rc, rbp = _bits(get("reg_val")), get("reg_col"), get("rb_ptr")
@@ -82,52 +83,53 @@ def decode(F, get, dtype):
                 emit(row, c, v)
             rows.setdefault(int(row), [])
 
-    # short tiles
+    # short tiles, panel by panel: [1&3][len4][2&2][singles] per panel
     sv, sc, so = _bits(get("short_val")), get("short_col"), get("short_out")
-    tile0, out0 = 0, 0
-    for cat, ntl in enumerate([F["t13"], F["t4"], F["t22"]]):
-        two = cat != 1
-        for tl in range(ntl):
-            grid = {}
-            for lane in range(32):
-                g, t = lane >> 2, lane & 3
-                for j in range(4):
-                    if dtype == "f64":
-                        r, c = 8 * j + g, t
+    panels = get("panels").reshape(-1, 12)
+    for pn in panels:
+        tile0, t13, t4, t22, ts, out0 = (int(v) for v in pn[6:12])
+        for cat, ntl in enumerate([t13, t4, t22]):
+            two = cat != 1
+            for tl in range(ntl):
+                grid = {}
+                for lane in range(32):
+                    g, t = lane >> 2, lane & 3
+                    for j in range(4):
+                        if dtype == "f64":
+                            r, c = 8 * j + g, t
+                        else:
+                            r = 8 * ((t >> 1) + (0 if j < 2 else 2)) + g
+                            c = 2 * (t & 1) + (j & 1)
+                        at = (tile0 + tl) * 128 + lane * 4 + j
+                        grid[(r, c)] = (sc[at], sv[at])
+                for r in range(32):
+                    cells = [grid[(r, c)] for c in range(4)]
+                    if two:
+                        o = out0 + tl * 64 + 16 * (r // 8) + (r % 8)
+                        ra, rb_ = so[o], so[o + 8]
+                        split = 1 if cat == 0 else 2
+                        segs = [(ra, cells[:split]), (rb_, cells[split:])]
                     else:
-                        r = 8 * ((t >> 1) + (0 if j < 2 else 2)) + g
-                        c = 2 * (t & 1) + (j & 1)
-                    at = (tile0 + tl) * 128 + lane * 4 + j
-                    grid[(r, c)] = (sc[at], sv[at])
-            for r in range(32):
-                cells = [grid[(r, c)] for c in range(4)]
-                if two:
-                    o = out0 + tl * 64 + 16 * (r // 8) + (r % 8)
-                    ra, rb_ = so[o], so[o + 8]
-                    split = 1 if cat == 0 else 2
-                    segs = [(ra, cells[:split]), (rb_, cells[split:])]
-                else:
-                    segs = [(so[out0 + tl * 32 + r], cells)]
-                for row, seg in segs:
-                    real = [(c, v) for c, v in seg if c != PAD]
-                    assert all(c != PAD for c, _ in seg[:len(real)])
-                    pads += [(c, v) for c, v in seg if c == PAD]
-                    if row < 0:
-                        assert not real
-                        continue
-                    for c, v in real:
-                        emit(row, c, v)
-        tile0 += ntl
-        out0 += ntl * (64 if two else 32)
-    ns_region = F["ts"] * 128
-    for q in range(ns_region):
-        at = tile0 * 128 + q
-        row = so[out0 + q]
-        if row < 0:
-            assert sc[at] == PAD
-            pads.append((sc[at], sv[at]))
-        else:
-            emit(row, sc[at], sv[at])
+                        segs = [(so[out0 + tl * 32 + r], cells)]
+                    for row, seg in segs:
+                        real = [(c, v) for c, v in seg if c != PAD]
+                        assert all(c != PAD for c, _ in seg[:len(real)])
+                        pads += [(c, v) for c, v in seg if c == PAD]
+                        if row < 0:
+                            assert not real
+                            continue
+                        for c, v in real:
+                            emit(row, c, v)
+            tile0 += ntl
+            out0 += ntl * (64 if two else 32)
+        for q in range(ts * 128):
+            at = tile0 * 128 + q
+            row = so[out0 + q]
+            if row < 0:
+                assert sc[at] == PAD
+                pads.append((sc[at], sv[at]))
+            else:
+                emit(row, sc[at], sv[at])
 
     for e in get("empty_rows"):
         assert int(e) not in rows

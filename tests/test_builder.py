@@ -15,7 +15,8 @@ COUNT_MAP = {"n0": "n_empty", "n1": "n_len1", "n2": "n_len2", "n3": "n_len3", "n
              "row_medium": "row_medium", "row_long": "row_long", "nrb": "rowblocks", "n_groups": "n_groups",
              "n_groups_padded": "n_groups_padded", "t13": "tiles_13", "t4": "tiles_4", "t22": "tiles_22",
              "ts": "tiles_single", "nnz_long_new": "nnz_long_new", "nnz_reg_new": "nnz_reg_new",
-             "nnz_irreg": "nnz_irreg", "nnz_short_new": "nnz_short_new", "m": "m", "n": "n", "nnz": "nnz"}
+             "nnz_irreg": "nnz_irreg", "nnz_short_new": "nnz_short_new", "m": "m", "n": "n", "nnz": "nnz",
+             "panel_rows": "panel_rows", "n_panels": "n_panels"}
 
 
 def host_plan(A, dt, **kw):
@@ -37,11 +38,14 @@ def matrices():
 CASES = list(matrices())
 
 
+@pytest.mark.parametrize("panel", [0, -1, 1, 97, 1000])
 @pytest.mark.parametrize("dt", ["f64", "f16"])
 @pytest.mark.parametrize("name,A", CASES, ids=[c[0] for c in CASES])
-def test_builder_bit_exact_vs_oracle(name, A, dt):
-    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt)
-    plan = host_plan(A, dt)
+def test_builder_bit_exact_vs_oracle(name, A, dt, panel):
+    if panel in (1, 97) and A.m > 20000:
+        pytest.skip("tiny panels on the small matrices only")
+    plan = host_plan(A, dt, panel_rows=panel)
+    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt, panel_rows=plan.info["panel_rows"])
     info = plan.info
     for k, v in ref.counts.items():
         assert info[COUNT_MAP[k]] == v, k
@@ -53,9 +57,10 @@ def test_builder_bit_exact_vs_oracle(name, A, dt):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f16"])
-def test_builder_roundtrip_via_abi(dt):
+@pytest.mark.parametrize("panel", [-1, 333])
+def test_builder_roundtrip_via_abi(dt, panel):
     A = synth.generate(synth.config("c1b"))
-    plan = host_plan(A, dt)
+    plan = host_plan(A, dt, panel_rows=panel)
     info = plan.info
     counts = {k: info[v] for k, v in COUNT_MAP.items()}
 
@@ -63,7 +68,7 @@ def test_builder_roundtrip_via_abi(dt):
         b = dasp.dasp_plan_copy_array(plan, name)
         if name.endswith("_val"):
             return b.view(np.float64 if dt == "f64" else np.float16)
-        if name in ("group_ptr", "rb_ptr", "irr_ptr"):
+        if name in ("group_ptr", "rb_ptr", "irr_ptr", "panels"):
             return b.view(np.int64)
         return b.view(np.int32)
     check_roundtrip(A, counts, get, dt)
@@ -72,9 +77,10 @@ def test_builder_roundtrip_via_abi(dt):
 
 def test_builder_threads_deterministic():
     A = synth.generate(synth.config("c3", scale=0.004))
-    p1, p8 = host_plan(A, "f64", num_threads=1), host_plan(A, "f64", num_threads=8)
-    for arr in dasp.ARRAYS:
-        assert np.array_equal(dasp.dasp_plan_copy_array(p1, arr), dasp.dasp_plan_copy_array(p8, arr)), arr
+    for panel in [-1, 4096, 50]:    # inner-parallel and one-thread-per-panel paths
+        p1, p8 = host_plan(A, "f64", num_threads=1, panel_rows=panel), host_plan(A, "f64", num_threads=8, panel_rows=panel)
+        for arr in dasp.ARRAYS:
+            assert np.array_equal(dasp.dasp_plan_copy_array(p1, arr), dasp.dasp_plan_copy_array(p8, arr)), arr
 
 
 def test_exports_every_header_symbol():

@@ -97,6 +97,26 @@ def test_parity_integer_bit_exact(name, gen, dt, variant):
     assert np.array_equal(y, y_ref)
 
 
+# R28 panels: every panel size gives the same exact integer results (and parity on reals)
+@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("panel", [-1, 1, 97, 1000, 50000])
+def test_parity_panels(panel, dt, variant):
+    A = synth.generate(synth.config("c3", scale=0.01, val_mode=synth.VAL_INT))
+    x = synth.vector(21, A.n, synth.VAL_INT)
+    if panel == 1:
+        A = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
+        x = synth.vector(21, A.n, synth.VAL_INT)
+    plan = make(A, dt, panel_rows=panel)
+    y = run(plan, x, dt, variant=variant)
+    y_ref, _ = oracle_ref(A, x, dt)
+    assert np.array_equal(y, y_ref)
+    y0 = synth.vector(22, A.m, synth.VAL_INT)
+    y = run(plan, x, dt, 2.0, -3.0, y0, variant=variant)
+    y_ref, _ = oracle_ref(A, x, dt, 2.0, -3.0, y0)
+    assert np.array_equal(y, y_ref)
+
+
 @pytest.mark.parametrize("dt", ["f64", "f16"])
 def test_identity_diagonal_permutation_exact(dt):
     n = 5003
@@ -150,10 +170,11 @@ def test_inf_in_x_only_reaches_referencing_rows(dt):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f16"])
-def test_device_arrays_match_oracle_builder(dt):
+@pytest.mark.parametrize("panel", [-1, 500])
+def test_device_arrays_match_oracle_builder(dt, panel):
     A = synth.generate(synth.config("c1b"))
-    plan = make(A, dt)   # keep_host off: copy_array reads back the uploaded device buffers
-    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt)
+    plan = make(A, dt, panel_rows=panel)   # keep_host off: copy_array reads back the device buffers
+    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt, panel_rows=plan.info["panel_rows"])
     for arr in dasp.ARRAYS:
         assert np.array_equal(dasp.dasp_plan_copy_array(plan, arr), ref.arrays[arr]), arr
 

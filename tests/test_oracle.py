@@ -194,6 +194,33 @@ def test_p6_roundtrip(name, dt):
     assert c["nnz_long_new"] == sum(-(-L // G) * G for L in np.diff(A.row_ptr) if L > 256)
 
 
+# R28 panels: the panelized format is the paper's format of each panel, concatenated
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("R", [1, 97, 1000, 4096])
+def test_panels_roundtrip_and_concatenation(dt, R):
+    A = synth.generate(synth.config("c1b"))
+    Ad = A if dt == "f64" else A.to_fp16()
+    F = oracle.build(Ad, dt, panel_rows=R)
+    c = F.counts
+    assert c["n_panels"] == -(-A.m // R) and c["panel_rows"] == R
+    check_roundtrip(A, c, F.view, dt)
+    pn = F.view("panels").reshape(-1, 12)
+    # each panel's share equals the global format of that panel's rows alone
+    for q in [0, len(pn) // 2, len(pn) - 1]:
+        r0, rows = int(pn[q, 0]), int(pn[q, 1])
+        sub = synth.CSR(rows, A.n, A.row_ptr[r0:r0 + rows + 1] - A.row_ptr[r0],
+                        A.col[A.row_ptr[r0]:A.row_ptr[r0 + rows]], Ad.val[A.row_ptr[r0]:A.row_ptr[r0 + rows]])
+        G = oracle.build(sub, dt)
+        g = G.counts
+        assert int(pn[q, 5]) == g["nrb"]
+        assert tuple(int(v) for v in pn[q, 7:11]) == (g["t13"], g["t4"], g["t22"], g["ts"])
+        t0, nt = int(pn[q, 6]), g["t13"] + g["t4"] + g["t22"] + g["ts"]
+        sv = F.view("short_col")[t0 * 128:(t0 + nt) * 128]
+        assert np.array_equal(sv, G.view("short_col"))
+        so = F.view("short_out")[int(pn[q, 11]):int(pn[q, 11]) + len(G.view("short_out"))]
+        assert np.array_equal(so, np.where(G.view("short_out") >= 0, G.view("short_out") + r0, -1))
+
+
 def test_medium_sort_is_stable_descending():
     lens = [7, 9, 7, 12, 9, 7, 5, 12, 30, 7]
     A = synth.from_lengths(lens, n=64)
@@ -212,4 +239,4 @@ def test_empty_and_degenerate():
     assert F.counts["n0"] == 5 and F.counts["nrb"] == 0 and F.counts["n_groups"] == 0
     A0 = synth.CSR(0, 0, np.zeros(1, dtype=np.int64), np.zeros(0, np.int32), np.zeros(0))
     F0 = oracle.build(A0, "f64")
-    assert all(v == 0 for v in F0.counts.values())
+    assert all(v == 0 for k, v in F0.counts.items() if k not in ("panel_rows", "n_panels"))
