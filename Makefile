@@ -37,7 +37,7 @@ clean:
 
 # experiment builds: occupancy (min blocks per SM of the fused kernel)
 exp: $(OBJ)/builder.o $(OBJ)/api.o
-	for mb in 5 6 8; do \
+	for mb in 4 5 6; do \
 	  $(NVCC) $(NVFLAGS) -DDASP_MIN_BLOCKS=$$mb -c $(SRC)/kernels.cu -o $(OBJ)/kernels_mb$$mb.o 2> $(OBJ)/kernels_mb$$mb.ptxas.txt && \
 	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_mb$$mb.so $(OBJ)/builder.o $(OBJ)/kernels_mb$$mb.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
 	done

@@ -34,7 +34,7 @@ struct dasp_plan_s {
     int64_t blocks = 0;                   // grid of the fused main kernel
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
     void* d_blk_panel = nullptr;          // int32 panel of every block
-    int32_t xmode = 0;                    // x gather policy (kernels.cuh MainParams::xmode)
+    void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
     size_t apw_bytes = 0;                 // L2 persisting access-policy window over x (0 = off)
     float apw_hit = 1.0f;
     // timing
@@ -53,6 +53,7 @@ int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
 // automatic panel: ~1M rows keeps a panel's x window and y (8 B each per row) well inside the
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
+constexpr int kColBuckets = 16;
 
 int auto_rbw(int64_t row_medium) {
     if (row_medium < 59990) return 1;
@@ -80,7 +81,8 @@ void free_device(dasp_plan_s* p) {
     if (p->d_partial) cudaFree(p->d_partial);
     if (p->d_panels) cudaFree(p->d_panels);
     if (p->d_blk_panel) cudaFree(p->d_blk_panel);
-    p->d_panels = p->d_blk_panel = nullptr;
+    if (p->d_unit_order) cudaFree(p->d_unit_order);
+    p->d_panels = p->d_blk_panel = p->d_unit_order = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -207,6 +209,32 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         }
         p->blocks = blk;
     }
+    // long-unit execution order (a launch schedule, not part of the format): inside each panel
+    // the units run bucketed by the column of their first element, so that the warps in flight
+    // gather from ~1/kColBuckets of x at a time instead of all of it (long rows' columns are
+    // sorted, so a unit covers a narrow column range).  Partials are per group and summed in
+    // group order by the finish kernel: the result is bitwise independent of this order.
+    std::vector<int32_t> unit_order(static_cast<size_t>(f.n_groups_padded / f.geo.UG));
+    {
+        const int32_t* lc = static_cast<const int32_t*>(f.arr[DASP_ARR_LONG_COL].ptr);
+        const int64_t ue = static_cast<int64_t>(f.geo.UG) * f.geo.G;
+        const char* lo_env = std::getenv("DASP_LONG_ORDER");
+        const bool bucketed = !(lo_env && std::atoi(lo_env) == 0) && f.n > 0;
+        for (const auto& d : desc) {
+            std::vector<int32_t> cnt(kColBuckets + 1, 0);
+            auto bucket = [&](int64_t u) {
+                const int32_t c = lc[u * ue];
+                return c < 0 ? kColBuckets - 1 : static_cast<int>(static_cast<int64_t>(c) * kColBuckets / f.n);
+            };
+            if (!bucketed) {
+                for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + w] = static_cast<int32_t>(d.unit0 + w);
+                continue;
+            }
+            for (int64_t w = 0; w < d.nunits; ++w) cnt[bucket(d.unit0 + w) + 1]++;
+            for (int b = 0; b < kColBuckets; ++b) cnt[b + 1] += cnt[b];
+            for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + cnt[bucket(d.unit0 + w)]++] = static_cast<int32_t>(d.unit0 + w);
+        }
+    }
     for (int a = 0; a < DASP_ARR_COUNT; ++a) p->bytes[a] = f.arr[a].bytes;
 
     if (p->device >= 0) {
@@ -237,9 +265,15 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
             return DASP_ERR_CUDA;
         }
         p->device_bytes += db + bb;
-        // x residency in L2 (R17): evict_last gathers and/or a persisting access-policy window
-        const char* xm = std::getenv("DASP_XMODE");
-        p->xmode = xm ? std::atoi(xm) : 0;
+        const size_t ub = std::max<size_t>(unit_order.size(), 1) * 4;
+        if (cudaMalloc(&p->d_unit_order, ub) != cudaSuccess) { free_device(p); f.release(); delete p; return DASP_ERR_OUT_OF_MEMORY; }
+        if (!unit_order.empty() && cudaMemcpy(p->d_unit_order, unit_order.data(), unit_order.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
+            free_device(p); f.release(); delete p;
+            return DASP_ERR_CUDA;
+        }
+        p->device_bytes += ub;
+        // optional persisting L2 access-policy window over x (DASP_X_APW=1; measured slower on
+        // C3, profiles/r01, so off by default)
         const char* apw = std::getenv("DASP_X_APW");
         if (apw && std::atoi(apw) > 0) {
             cudaDeviceProp prop;
@@ -310,8 +344,8 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
     mp.beta = beta;
     mp.panels = static_cast<const dasp::PanelDesc*>(p->d_panels);
     mp.blk_panel = static_cast<const int32_t*>(p->d_blk_panel);
+    mp.unit_order = static_cast<const int32_t*>(p->d_unit_order);
     mp.rbw = p->rbw;
-    mp.xmode = p->xmode;
     mp.class_mask = 7;
     // DASP_PROFILE_CLASS (profiling only; the other classes' rows are then NOT computed):
     // 1 = long units, 2 = medium warps, 3 = short tiles

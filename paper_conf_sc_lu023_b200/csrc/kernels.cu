@@ -63,40 +63,13 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
     return v;
 }
-// x gather: column -1 (pad, R12) reads 0 without touching memory.  x lines carry an L2
-// evict_last policy so the streamed A arrays (evict_first) do not push x out of L2.
-__device__ __forceinline__ uint64_t x_policy() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-    return p;
+// x gather through the read-only path; column -1 (pad, R12) reads 0 without touching memory
+__device__ __forceinline__ double gx(const double* x, uint32_t c) {
+    return static_cast<int32_t>(c) >= 0 ? __ldg(x + static_cast<int32_t>(c)) : 0.0;
 }
-struct XLoad {
-    uint64_t pol;
-    int mode;   // 0: plain read-only load, 1: L2 evict_last hint
-};
-__device__ __forceinline__ double ldx(const double* p, const XLoad& xl) {
-    if (xl.mode == 1) {
-        double v;
-        asm("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(xl.pol));
-        return v;
-    }
-    return __ldg(p);
-}
-__device__ __forceinline__ uint16_t ldxh(const uint16_t* p, const XLoad& xl) {
-    if (xl.mode == 1) {
-        uint16_t v;
-        asm("ld.global.nc.L2::cache_hint.b16 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(xl.pol));
-        return v;
-    }
-    return __ldg(reinterpret_cast<const unsigned short*>(p));
-}
-#define gx(x, c) gx_(x, c, XL)
-#define gxh(x, c) gxh_(x, c, XL)
-__device__ __forceinline__ double gx_(const double* x, uint32_t c, const XLoad& XL) {
-    return static_cast<int32_t>(c) >= 0 ? ldx(x + static_cast<int32_t>(c), XL) : 0.0;
-}
-__device__ __forceinline__ uint16_t gxh_(const uint16_t* x, uint32_t c, const XLoad& XL) {
-    return static_cast<int32_t>(c) >= 0 ? ldxh(x + static_cast<int32_t>(c), XL) : static_cast<uint16_t>(0);
+__device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
+    return static_cast<int32_t>(c) >= 0 ? __ldg(reinterpret_cast<const unsigned short*>(x) + static_cast<int32_t>(c))
+                                        : static_cast<uint16_t>(0);
 }
 __device__ __forceinline__ float h2f(uint16_t h) { return __half2float(__ushort_as_half(h)); }
 __device__ __forceinline__ float2 u2f2(uint32_t u) {  // two packed binary16 -> two f32 (exact)
@@ -160,7 +133,7 @@ __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typena
 // long rows, phase 1 (Alg. 2 l.1-16): one warp = one unit of UG consecutive groups
 // ------------------------------------------------------------------------------------------
 template <int VAR>
-__device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol, const XLoad& XL) {
+__device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol) {
     const int64_t base = u * 256 + lane * 8;            // lane holds 8 consecutive elements
     const double* lv = static_cast<const double*>(P.long_val) + base;
     double v[8];
@@ -192,7 +165,7 @@ __device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, in
 }
 
 template <int VAR>
-__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol, const XLoad& XL) {
+__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol) {
     const int64_t base = u * 512 + lane * 16;           // lane holds 16 consecutive elements
     uint32_t vv[8], c[16];
     ld8_b32(static_cast<const uint16_t*>(P.long_val) + base, pol, vv);
@@ -231,59 +204,81 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
 // of CW blocks (R18), then the irregular tails with 4 lanes per row, then y.
 // ------------------------------------------------------------------------------------------
 template <int VAR>
-__device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, int lane, uint64_t pol, const XLoad& XL) {
+__device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
     const int g = lane >> 2, t = lane & 3;
-    const int64_t base = P.rb_ptr[rb];
-    const int64_t nreg = (P.rb_ptr[rb + 1] - base) >> 5;
+    const int64_t i = rb * 8 + g;
+    // every load that does not depend on data goes out first: the row-block's pointers, the
+    // irregular bounds and the output row (one memory round trip instead of three)
+    const int64_t base = __ldg(P.rb_ptr + rb), end = __ldg(P.rb_ptr + rb + 1);
+    const int64_t ib = __ldg(P.irr_ptr + i), ie = __ldg(P.irr_ptr + i + 1);
+    const int32_t orow = __ldg(P.med_out + i);
+    const int nreg = static_cast<int>((end - base) >> 5);
+    const int nfull = nreg >> 2, rem = nreg & 3;
     const double* rv = static_cast<const double*>(P.reg_val) + base;
     const int32_t* rc = P.reg_col + base;
+    const double* iv = static_cast<const double*>(P.irr_val);
     const double* x = static_cast<const double*>(P.x);
+    // round 1: first chunk (4 blocks, 256-bit value load), the ragged last chunk and the
+    // first irregular element of this lane, all in flight together
+    double va[4] = {0.0, 0.0, 0.0, 0.0};
+    uint32_t ca[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
+    if (nfull > 0) { ld4_f64(rv + lane * 4, pol, va); ld4_b32(rc + lane * 4, pol, ca); }
+    double vr[3] = {0.0, 0.0, 0.0};
+    uint32_t cr[3] = {0xffffffffu, 0xffffffffu, 0xffffffffu};
+    const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane * rem;
+#pragma unroll
+    for (int j = 0; j < 3; ++j)
+        if (j < rem) { vr[j] = ld1_f64(rv + rbase + j, pol); cr[j] = ld1_b32(rc + rbase + j, pol); }
+    int64_t k = ib + t;
+    double vi = 0.0;
+    uint32_t ci = 0xffffffffu;
+    if (k < ie) { vi = ld1_f64(iv + k, pol); ci = ld1_b32(P.irr_col + k, pol); }
     double c0 = 0.0, c1 = 0.0, part = 0.0;
-    const int64_t nfull = nreg >> 2;
-    for (int64_t ch = 0; ch < nfull; ++ch) {           // full chunks: 4 blocks, 32 B + 16 B per lane
-        double v[4];
-        uint32_t c[4];
-        ld4_f64(rv + ch * 128 + lane * 4, pol, v);
-        ld4_b32(rc + ch * 128 + lane * 4, pol, c);
+    for (int ch = 0; ch < nfull; ++ch) {
+        if (ch > 0) { ld4_f64(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
         double xv[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) xv[j] = gx(x, c[j]);
+        for (int j = 0; j < 4; ++j) xv[j] = gx(x, ca[j]);
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
-            if constexpr (VAR == VAR_MMA) dmma(c0, c1, v[j], xv[j]);
-            else part = fma(v[j], xv[j], part);
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, va[j], xv[j]);
+            else part = fma(va[j], xv[j], part);
         }
     }
-    const int rem = static_cast<int>(nreg - (nfull << 2));
-    if (rem) {                                          // last chunk, width rem
-        const int64_t cb = nfull * 128 + lane * rem;
-        for (int j = 0; j < rem; ++j) {
-            double v = ld1_f64(rv + cb + j, pol);
-            double xv = gx(x, ld1_b32(rc + cb + j, pol));
-            if constexpr (VAR == VAR_MMA) dmma(c0, c1, v, xv);
-            else part = fma(v, xv, part);
+    double xr[3];
+#pragma unroll
+    for (int j = 0; j < 3; ++j) xr[j] = gx(x, cr[j]);     // pads / unused slots read 0
+    const double xi = gx(x, ci);
+#pragma unroll
+    for (int j = 0; j < 3; ++j) {
+        if (j < rem) {                                     // rem is warp-uniform
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, vr[j], xr[j]);
+            else part = fma(vr[j], xr[j], part);
         }
     }
-    if constexpr (VAR == VAR_MMA) {                     // Alg. 3 l.13-17: diagonal -> lane 4g
-        double d = diag_to_quad(c0, c1, lane);
+    if constexpr (VAR == VAR_MMA) {                        // Alg. 3 l.13-17: diagonal -> quad g
+        const double d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.0;
     }
-    const int64_t i = rb * 8 + g;                      // Alg. 3 l.20-24: irregular part
-    const int64_t ib = P.irr_ptr[i], ie = P.irr_ptr[i + 1];
-    const double* iv = static_cast<const double*>(P.irr_val);
-    for (int64_t k = ib + t; k < ie; k += 4) part = fma(ld1_f64(iv + k, pol), gx(x, ld1_b32(P.irr_col + k, pol)), part);
+    part = fma(vi, xi, part);                              // Alg. 3 l.20-24: irregular part
+    for (k += 4; k < ie; k += 4) part = fma(ld1_f64(iv + k, pol), gx(x, ld1_b32(P.irr_col + k, pol)), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
-    if (t == 0) store_y<0>(P, P.med_out[i], part);     // Alg. 3 l.25 through the output map (R9)
+    if (t == 0) store_y<0>(P, orow, part);                 // Alg. 3 l.25 through the output map (R9)
 }
 
 template <int VAR>
-__device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, int lane, uint64_t pol, const XLoad& XL) {
+__device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
     const int g = lane >> 2, t = lane & 3;
-    const int64_t base = P.rb_ptr[rb];
-    const int64_t nreg = (P.rb_ptr[rb + 1] - base) >> 7;
+    const int64_t i = rb * 8 + g;
+    const int64_t base = __ldg(P.rb_ptr + rb), end = __ldg(P.rb_ptr + rb + 1);
+    const int64_t ib = __ldg(P.irr_ptr + i), ie = __ldg(P.irr_ptr + i + 1);
+    const int32_t orow = __ldg(P.med_out + i);
+    const int nreg = static_cast<int>((end - base) >> 7);
+    const int nfull = nreg >> 1, rem = nreg & 1;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + base;
     const int32_t* rc = P.reg_col + base;
+    const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
     float c0 = 0.f, c1 = 0.f, part = 0.f;
     auto block = [&](uint32_t a0, uint32_t a2, const uint32_t* c) {
@@ -293,128 +288,148 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, i
         if constexpr (VAR == VAR_MMA) {
             hmma(c0, c1, a0, a2, pack2(xh[0], xh[1]), pack2(xh[2], xh[3]));
         } else {
-            float2 lo = u2f2(a0);
-            float2 hi = u2f2(a2);
+            const float2 lo = u2f2(a0), hi = u2f2(a2);
             part = fmaf(lo.x, h2f(xh[0]), part);
             part = fmaf(lo.y, h2f(xh[1]), part);
             part = fmaf(hi.x, h2f(xh[2]), part);
             part = fmaf(hi.y, h2f(xh[3]), part);
         }
     };
-    const int64_t nfull = nreg >> 1;
-    for (int64_t ch = 0; ch < nfull; ++ch) {           // 2 blocks: 16 B + 32 B per lane
-        uint32_t v[4], c[8];
-        ld4_b32(rv + ch * 256 + lane * 8, pol, v);
-        ld8_b32(rc + ch * 256 + lane * 8, pol, c);
-        block(v[0], v[1], &c[0]);
-        block(v[2], v[3], &c[4]);
+    // round 1: first chunk (2 blocks), the ragged last block and the first irregular element
+    uint32_t va[4] = {0u, 0u, 0u, 0u}, ca[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) ca[e] = 0xffffffffu;
+    if (nfull > 0) { ld4_b32(rv + lane * 8, pol, va); ld8_b32(rc + lane * 8, pol, ca); }
+    uint32_t vr0 = 0u, vr1 = 0u, cr[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
+    if (rem) { ld2_b32(rv + nfull * 256 + lane * 4, pol, vr0, vr1); ld4_b32(rc + nfull * 256 + lane * 4, pol, cr); }
+    int64_t k = ib + t;
+    uint16_t vi = 0;
+    uint32_t ci = 0xffffffffu;
+    if (k < ie) { vi = __ldg(iv + k); ci = ld1_b32(P.irr_col + k, pol); }
+    for (int ch = 0; ch < nfull; ++ch) {
+        if (ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
+        block(va[0], va[1], &ca[0]);
+        block(va[2], va[3], &ca[4]);
     }
-    if (nreg & 1) {
-        uint32_t v0, v1, c[4];
-        ld2_b32(rv + nfull * 256 + lane * 4, pol, v0, v1);
-        ld4_b32(rc + nfull * 256 + lane * 4, pol, c);
-        block(v0, v1, c);
-    }
+    if (rem) block(vr0, vr1, cr);
     if constexpr (VAR == VAR_MMA) {
-        float d = diag_to_quad(c0, c1, lane);
+        const float d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.f;
     }
-    const int64_t i = rb * 8 + g;
-    const int64_t ib = P.irr_ptr[i], ie = P.irr_ptr[i + 1];
-    const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
-    for (int64_t k = ib + t; k < ie; k += 4)
-        part = fmaf(h2f(__ldg(iv + k)), h2f(gxh(x, __ldg(reinterpret_cast<const uint32_t*>(P.irr_col) + k))), part);
+    part = fmaf(h2f(vi), h2f(gxh(x, ci)), part);
+    for (k += 4; k < ie; k += 4)
+        part = fmaf(h2f(__ldg(iv + k)), h2f(gxh(x, ld1_b32(P.irr_col + k, pol))), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
-    if (t == 0) store_y<1>(P, P.med_out[i], part);
+    if (t == 0) store_y<1>(P, orow, part);
 }
 
 // ------------------------------------------------------------------------------------------
-// short rows (Alg. 4) and singles (Alg. 5): one tile of 32 four-slot rows
+// short rows (Alg. 4) and singles (Alg. 5): one tile of 32 four-slot rows.
+// Results are transposed with shuffles so that lane L writes outputs L and L+32 of the tile:
+// the output map is read with two coalesced loads issued at the start of the tile.
 // ------------------------------------------------------------------------------------------
 // cat 0 = 1&3 (seg0 = slot 0, seg1 = slots 1-3), 1 = len-4, 2 = 2&2 (slots 0-1 | 2-3)
 __device__ __forceinline__ int seg_of(int cat, int slot) { return cat == 0 ? (slot > 0) : (cat == 2 ? (slot >> 1) : 0); }
 
 template <int VAR>
 __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol, const XLoad& XL) {
+                                               uint64_t pol) {
     const int g = lane >> 2, t = lane & 3;
+    const int nseg = cat == 1 ? 1 : 2;
     double v[4];
     uint32_t c[4];
     ld4_f64(static_cast<const double*>(P.short_val) + tile * 128 + lane * 4, pol, v);
     ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
+    const int32_t o0 = __ldg(P.short_out + obase + lane);                        // outputs L, L+32
+    const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
     const double* x = static_cast<const double*>(P.x);
     double xv[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) xv[j] = gx(x, c[j]);
-    const int nseg = cat == 1 ? 1 : 2;
     const int myseg = seg_of(cat, t);
+    // output o = 16j + 8s + g (two outputs per four-slot row) or 8j + g (len-4)
+    const int src = 4 * (lane & 7);                      // quad of row g' = lane & 7
+    double r0 = 0.0, r1 = 0.0;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {                       // 4-slot row r = 8j + g, slot t
+    for (int j = 0; j < 4; ++j) {                        // four-slot row r = 8j + g, slot t
         for (int s = 0; s < nseg; ++s) {
-            const int o = nseg == 2 ? 16 * j + 8 * s + g : 8 * j + g;
-            if constexpr (VAR == VAR_MMA) {             // x masked to the segment (Alg. 4 l.7-11)
-                double c0 = 0.0, c1 = 0.0;
-                dmma(c0, c1, v[j], myseg == s ? xv[j] : 0.0);
-                if (is_diag_holder(lane)) store_y<0>(P, P.short_out[obase + o], (g & 1) ? c1 : c0);
+            double val;
+            if constexpr (VAR == VAR_MMA) {              // x masked to the segment (Alg. 4 l.7-11)
+                double cc0 = 0.0, cc1 = 0.0;
+                dmma(cc0, cc1, v[j], myseg == s ? xv[j] : 0.0);
+                val = __shfl_sync(FULL, (g & 1) ? cc1 : cc0, src + ((lane & 7) >> 1));
             } else {
                 double p = myseg == s ? v[j] * xv[j] : 0.0;
                 p += __shfl_xor_sync(FULL, p, 1);
                 p += __shfl_xor_sync(FULL, p, 2);
-                if (t == 0) store_y<0>(P, P.short_out[obase + o], p);
+                val = __shfl_sync(FULL, p, src);
             }
+            const int blk = nseg == 2 ? 2 * j + s : j;   // this result fills outputs 8*blk .. 8*blk+7
+            if ((lane >> 3) == blk) r0 = val;
+            if ((lane >> 3) == blk - 4) r1 = val;
         }
     }
+    store_y<0>(P, o0, r0);
+    if (nseg == 2) store_y<0>(P, o1, r1);
 }
 
 template <int VAR>
 __device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol, const XLoad& XL) {
+                                               uint64_t pol) {
     const int g = lane >> 2, t = lane & 3;
+    const int nseg = cat == 1 ? 1 : 2;
     uint32_t a0, a2, c[4];
     ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
     ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
+    const int32_t o0 = __ldg(P.short_out + obase + lane);
+    const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
     uint16_t xh[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) xh[e] = gxh(x, c[e]);
     // element e: four-slot row group q = (e<2 ? 0 : 2) + (t>>1), slot 2(t&1) + (e&1)
-    const int nseg = cat == 1 ? 1 : 2;
     const int seg0 = seg_of(cat, 2 * (t & 1)), seg1 = seg_of(cat, 2 * (t & 1) + 1);
-    if constexpr (VAR == VAR_MMA) {
-        for (int q = 0; q < 4; ++q) {
-            const bool lo = q == (t >> 1), hi = q == 2 + (t >> 1);
-            for (int s = 0; s < nseg; ++s) {
-                const bool m0 = seg0 == s, m1 = seg1 == s;
-                uint32_t b0 = lo ? pack2(m0 ? xh[0] : 0, m1 ? xh[1] : 0) : 0u;
-                uint32_t b1 = hi ? pack2(m0 ? xh[2] : 0, m1 ? xh[3] : 0) : 0u;
-                float c0 = 0.f, c1 = 0.f;
-                hmma(c0, c1, a0, a2, b0, b1);
-                const int o = nseg == 2 ? 16 * q + 8 * s + g : 8 * q + g;
-                if (is_diag_holder(lane)) store_y<1>(P, P.short_out[obase + o], (g & 1) ? c1 : c0);
-            }
-        }
-    } else {
-        float2 vl = u2f2(a0);
-        float2 vh = u2f2(a2);
+    const int gs = lane & 7;                              // row g' whose result this lane collects
+    float r0 = 0.f, r1 = 0.f;
+    float slo[2], shi[2];
+    if constexpr (VAR == VAR_CUDACORE) {
+        const float2 vl = u2f2(a0), vh = u2f2(a2);
         const float p0 = vl.x * h2f(xh[0]), p1 = vl.y * h2f(xh[1]), p2 = vh.x * h2f(xh[2]), p3 = vh.y * h2f(xh[3]);
-        for (int s = 0; s < nseg; ++s) {
-            float slo = (seg0 == s ? p0 : 0.f) + (seg1 == s ? p1 : 0.f);   // group t>>1
-            float shi = (seg0 == s ? p2 : 0.f) + (seg1 == s ? p3 : 0.f);   // group 2 + (t>>1)
-            slo += __shfl_xor_sync(FULL, slo, 1);
-            shi += __shfl_xor_sync(FULL, shi, 1);
-            if ((t & 1) == 0) {
-                const int qlo = t >> 1, qhi = 2 + (t >> 1);
-                store_y<1>(P, P.short_out[obase + (nseg == 2 ? 16 * qlo + 8 * s + g : 8 * qlo + g)], slo);
-                store_y<1>(P, P.short_out[obase + (nseg == 2 ? 16 * qhi + 8 * s + g : 8 * qhi + g)], shi);
-            }
+#pragma unroll
+        for (int s = 0; s < 2; ++s) {
+            slo[s] = (seg0 == s ? p0 : 0.f) + (seg1 == s ? p1 : 0.f);   // group t>>1
+            shi[s] = (seg0 == s ? p2 : 0.f) + (seg1 == s ? p3 : 0.f);   // group 2 + (t>>1)
+            slo[s] += __shfl_xor_sync(FULL, slo[s], 1);
+            shi[s] += __shfl_xor_sync(FULL, shi[s], 1);
         }
     }
+    for (int q = 0; q < 4; ++q) {
+        for (int s = 0; s < nseg; ++s) {
+            float val;
+            if constexpr (VAR == VAR_MMA) {
+                const bool lo = q == (t >> 1), hi = q == 2 + (t >> 1);
+                const bool m0 = seg0 == s, m1 = seg1 == s;
+                const uint32_t b0 = lo ? pack2(m0 ? xh[0] : 0, m1 ? xh[1] : 0) : 0u;
+                const uint32_t b1 = hi ? pack2(m0 ? xh[2] : 0, m1 ? xh[3] : 0) : 0u;
+                float cc0 = 0.f, cc1 = 0.f;
+                hmma(cc0, cc1, a0, a2, b0, b1);
+                val = __shfl_sync(FULL, (g & 1) ? cc1 : cc0, 4 * gs + (gs >> 1));
+            } else {
+                val = __shfl_sync(FULL, q < 2 ? slo[s] : shi[s], 4 * gs + 2 * (q & 1));
+            }
+            const int blk = nseg == 2 ? 2 * q + s : q;
+            if ((lane >> 3) == blk) r0 = val;
+            if ((lane >> 3) == blk - 4) r1 = val;
+        }
+    }
+    store_y<1>(P, o0, r0);
+    if (nseg == 2) store_y<1>(P, o1, r1);
 }
 
 // singles (Alg. 5): lane handles 4 consecutive len-1 rows on CUDA cores
 template <int DT>
-__device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, int64_t obase, int lane, uint64_t pol, const XLoad& XL) {
+__device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, int64_t obase, int lane, uint64_t pol) {
     uint32_t c[4], o[4];
     ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
     ld4_b32(P.short_out + obase + lane * 4, pol, o);
@@ -439,47 +454,54 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
 // the fused main kernel
 // ------------------------------------------------------------------------------------------
 #ifndef DASP_MIN_BLOCKS
-#define DASP_MIN_BLOCKS 1
+#define DASP_MIN_BLOCKS 4   // caps registers at 64: >= 32 resident warps per SM, no spills
 #endif
 template <int DT, int VAR>
 __global__ void __launch_bounds__(MAIN_THREADS, DASP_MIN_BLOCKS) dasp_main_kernel(const MainParams P) {
     const int lane = threadIdx.x & 31;
-    const PanelDesc D = P.panels[P.blk_panel[blockIdx.x]];
-    int64_t w = (static_cast<int64_t>(blockIdx.x) - D.blk0) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+    // role of this warp inside its panel; the descriptor fields are loaded only on the branch
+    // that needs them so they do not stay live (register pressure = occupancy)
+    const PanelDesc* D = P.panels + __ldg(P.blk_panel + blockIdx.x);
+    int64_t w = (static_cast<int64_t>(blockIdx.x) - __ldg(&D->blk0)) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
     const uint64_t pol = stream_policy();
-    const XLoad XL{x_policy(), P.xmode};
-    if (w < D.nunits) {                                  // long rows, phase 1
+    const int64_t nunits = __ldg(&D->nunits);
+    if (w < nunits) {                                    // long rows, phase 1
         if (!(P.class_mask & 1)) return;
-        if constexpr (DT == 0) long_unit_f64<VAR>(P, D.unit0 + w, lane, pol, XL);
-        else long_unit_f16<VAR>(P, D.unit0 + w, lane, pol, XL);
+        const int64_t u = __ldg(P.unit_order + __ldg(&D->unit0) + w);
+        if constexpr (DT == 0) long_unit_f64<VAR>(P, u, lane, pol);
+        else long_unit_f16<VAR>(P, u, lane, pol);
         return;
     }
-    w -= D.nunits;
-    if (w < D.nmw) {                                     // medium rows
+    w -= nunits;
+    const int64_t nmw = __ldg(&D->nmw);
+    if (w < nmw) {                                       // medium rows
         if (!(P.class_mask & 2)) return;
-        const int64_t rb0 = D.rb0 + w * P.rbw;
-        const int64_t rb1 = min(rb0 + P.rbw, D.rb0 + D.nrb);
+        const int64_t rbp0 = __ldg(&D->rb0);
+        const int64_t rb0 = rbp0 + w * P.rbw;
+        const int64_t rb1 = min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb));
         for (int64_t rb = rb0; rb < rb1; ++rb) {
-            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb, lane, pol, XL);
-            else medium_rb_f16<VAR>(P, rb, lane, pol, XL);
+            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb, lane, pol);
+            else medium_rb_f16<VAR>(P, rb, lane, pol);
         }
         return;
     }
-    int64_t t = w - D.nmw;                               // short tiles: [1&3][len4][2&2][singles]
-    if (t >= D.t13 + D.t4 + D.t22 + D.ts || !(P.class_mask & 4)) return;
-    const int64_t tile = D.tile0 + t;
+    const int64_t t = w - nmw;                           // short tiles: [1&3][len4][2&2][singles]
+    const int64_t t13 = __ldg(&D->t13), t4 = __ldg(&D->t4), t22 = __ldg(&D->t22);
+    if (t >= t13 + t4 + t22 + __ldg(&D->ts) || !(P.class_mask & 4)) return;
+    const int64_t tile = __ldg(&D->tile0) + t;
+    const int64_t out0 = __ldg(&D->out0);
     int cat;
     int64_t obase;
-    if (t < D.t13) { cat = 0; obase = D.out0 + t * 64; }
-    else if (t < D.t13 + D.t4) { cat = 1; obase = D.out0 + 64 * D.t13 + (t - D.t13) * 32; }
-    else if (t < D.t13 + D.t4 + D.t22) { cat = 2; obase = D.out0 + 64 * D.t13 + 32 * D.t4 + (t - D.t13 - D.t4) * 64; }
+    if (t < t13) { cat = 0; obase = out0 + t * 64; }
+    else if (t < t13 + t4) { cat = 1; obase = out0 + 64 * t13 + (t - t13) * 32; }
+    else if (t < t13 + t4 + t22) { cat = 2; obase = out0 + 64 * t13 + 32 * t4 + (t - t13 - t4) * 64; }
     else {
-        obase = D.out0 + 64 * D.t13 + 32 * D.t4 + 64 * D.t22 + (t - D.t13 - D.t4 - D.t22) * 128;
-        singles_tile<DT>(P, tile, obase, lane, pol, XL);
+        obase = out0 + 64 * t13 + 32 * t4 + 64 * t22 + (t - t13 - t4 - t22) * 128;
+        singles_tile<DT>(P, tile, obase, lane, pol);
         return;
     }
-    if constexpr (DT == 0) short_tile_f64<VAR>(P, cat, tile, obase, lane, pol, XL);
-    else short_tile_f16<VAR>(P, cat, tile, obase, lane, pol, XL);
+    if constexpr (DT == 0) short_tile_f64<VAR>(P, cat, tile, obase, lane, pol);
+    else short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
 }
 
 // long phase 2 (Alg. 2 l.17-25): one warp per long row, lane-strided sum of the group partials

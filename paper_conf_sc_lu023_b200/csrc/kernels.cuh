@@ -37,11 +37,11 @@ struct MainParams {
     const int32_t* short_out;
     const PanelDesc* panels;
     const int32_t* blk_panel; // panel of every block
+    const int32_t* unit_order;// long units in execution order (column-bucketed per panel)
     const void* x;
     void* y;
     double alpha, beta;
     int32_t rbw;
-    int32_t xmode;            // x gather cache policy: 0 plain, 1 L2 evict_last
     int32_t class_mask;       // bit 0 long, bit 1 medium, bit 2 short (profiling; 7 = all)
 };
 

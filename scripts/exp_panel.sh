@@ -1,11 +1,11 @@
 #!/bin/bash
 mkdir -p gpurun_out
 make -j8 all > gpurun_out/make.log 2>&1 || { tail -30 gpurun_out/make.log; exit 1; }
-timeout 900 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -5 gpurun_out/pytest_gpu.log
+#timeout 900 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -5 gpurun_out/pytest_gpu.log
 B="python bench.py --steps 100 --warmup 5 --e2e-steps 0 --no-cpu-baseline"
 : > gpurun_out/panel.jsonl
 for cfg in "c3" "c2"; do
- for pr in -1 262144 524288 1048576 2097152 4194304; do
+ for pr in -1 262144 1048576 2097152; do
   for v in mma cudacore; do
    echo "{\"panel\": $pr}" >> gpurun_out/panel.jsonl
    DASP_PANEL_ROWS=$pr timeout 300 $B --config $cfg --variant $v >> gpurun_out/panel.jsonl 2>> gpurun_out/panel.err

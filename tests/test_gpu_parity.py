@@ -257,3 +257,17 @@ def test_full_size_stencil_sampled(dt):
 def test_full_size_powerlaw_sampled(dt):
     A = synth.generate(synth.config("c3"))
     _sampled_parity(A, dt)
+
+
+def test_long_unit_order_is_result_neutral(monkeypatch):
+    """The column-bucketed long-unit schedule changes only execution order: bitwise same y."""
+    A = synth.generate(synth.config("c3", scale=0.02))
+    x = synth.vector(31, A.n)
+    ys = []
+    for order in ["0", "1"]:
+        monkeypatch.setenv("DASP_LONG_ORDER", order)
+        for v in VARIANTS:
+            ys.append(run(make(A, "f64", panel_rows=50000), x, "f64", variant=v))
+    assert np.array_equal(ys[0], ys[2]) and np.array_equal(ys[1], ys[3])
+    y_ref, s = oracle_ref(A, x, "f64")
+    assert oracle.tolerance_ok(ys[0], y_ref, s).all()
