@@ -47,9 +47,8 @@ inline int64_t reg_pos(const Geometry& geo, int64_t nreg, int g, int64_t s) {
     int64_t b = s / geo.K;
     int k = static_cast<int>(s % geo.K);
     int t, e;
-    if (geo.EPL == 1) { t = k; e = 0; }                       // m8n8k4: A[g][t]
-    else if (k < 8) { t = k >> 1; e = k & 1; }               // m16n8k16: a0,a1 = A[g][2t..2t+1]
-    else { t = (k - 8) >> 1; e = 2 + (k & 1); }               //           a4,a5 = A[g][2t+8..2t+9]
+    if (geo.EPL == 1) { t = k; e = 0; }                       // m8n8k4 f64: A[g][t]
+    else { t = k >> 1; e = k & 1; }                           // m16n8k8 f16: a0,a1 = A[g][2t..2t+1]
     int lane = 4 * g + t;
     int64_t c = b / geo.CW, jb = b % geo.CW;
     int64_t w = std::min<int64_t>(geo.CW, nreg - c * geo.CW);

@@ -9,7 +9,7 @@
 namespace dasp {
 
 // Per-dtype block geometry.  FP64: mma.sync m8n8k4 (MMA_M=8, MMA_N=8, MMA_K=4).
-// FP16: mma.sync m16n8k16 with A rows 0-7 live (R14), so the block is 8 x 16.
+// FP16: the minimum f16 shape mma.sync m16n8k8 with A rows 0-7 live (R14): 8 x 8 blocks.
 struct Geometry {
     int sv;   // bytes per value
     int K;    // MMA_K (slots per row per block)
@@ -22,7 +22,7 @@ struct Geometry {
 
 inline Geometry geometry(int dtype) {
     if (dtype == DASP_R_64F) return Geometry{8, 4, 32, 1, 64, 4, 4};
-    return Geometry{2, 16, 128, 4, 256, 2, 2};
+    return Geometry{2, 8, 64, 2, 128, 4, 4};
 }
 
 constexpr int MAX_LEN = 256;

@@ -86,15 +86,13 @@ __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b)
     asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
                  : "+d"(c0), "+d"(c1) : "d"(a), "d"(b));
 }
-// C(16x8) += A(16x16) * B(16x8), f16 inputs, f32 accumulate.  Rows 8-15 of A are zero
-// (R14): a0 = A[g][2t..2t+1], a2 = A[g][2t+8..2t+9]; b0 = B[2t..2t+1][g], b1 = B[2t+8..2t+9][g];
-// c0,c1 = C[g][2t..2t+1].
-__device__ __forceinline__ void hmma(float& c0, float& c1, uint32_t a0, uint32_t a2, uint32_t b0, uint32_t b1) {
+// C(16x8) += A(16x8) * B(8x8), f16 inputs, f32 accumulate (m16n8k8, the minimum f16 shape).
+// Rows 8-15 of A are zero (R14): a0 = A[g][2t..2t+1]; b0 = B[2t..2t+1][g]; c0,c1 = C[g][2t..2t+1].
+__device__ __forceinline__ void hmma(float& c0, float& c1, uint32_t a0, uint32_t b0) {
     float c2 = 0.f, c3 = 0.f;
-    asm volatile(
-        "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
-        : "+f"(c0), "+f"(c1), "+f"(c2), "+f"(c3)
-        : "r"(a0), "r"(0u), "r"(a2), "r"(0u), "r"(b0), "r"(b1));
+    asm volatile("mma.sync.aligned.m16n8k8.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5}, {%6}, {%0,%1,%2,%3};"
+                 : "+f"(c0), "+f"(c1), "+f"(c2), "+f"(c3)
+                 : "r"(a0), "r"(0u), "r"(b0));
 }
 // C[g][g] lives in lane 4g + (g>>1), register g&1.  Returns it to every lane of quad g.
 template <typename A>
@@ -115,7 +113,7 @@ template <> struct Tr<0> {  // FP64
 };
 template <> struct Tr<1> {  // FP16 storage, FP32 accumulate
     using V = uint16_t; using Y = float; using A = float; using X = uint16_t;
-    static constexpr int K = 16, BE = 128, EPL = 4, G = 256, UG = 2, CW = 2;
+    static constexpr int K = 8, BE = 64, EPL = 2, G = 128, UG = 4, CW = 4;
 };
 
 // y[row] = alpha*acc + beta*y[row] (beta == 0: y not read, R16)
@@ -179,24 +177,24 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
     if constexpr (VAR == VAR_MMA) {
         float c0 = 0.f, c1 = 0.f;
 #pragma unroll
-        for (int h = 0; h < 4; ++h)   // elements 4h..4h+3 -> A[g][2t,2t+1,2t+8,2t+9]
-            hmma(c0, c1, vv[2 * h], vv[2 * h + 1], pack2(xh[4 * h], xh[4 * h + 1]), pack2(xh[4 * h + 2], xh[4 * h + 3]));
-        float d = diag_to_quad(c0, c1, lane);                   // rows 4q..4q+3 = group q
+        for (int h = 0; h < 8; ++h)   // elements 2h, 2h+1 -> A[g][2t..2t+1] of one m16n8k8
+            hmma(c0, c1, vv[h], pack2(xh[2 * h], xh[2 * h + 1]));
+        const float d = diag_to_quad(c0, c1, lane);             // rows 2q, 2q+1 = group q
         part = (lane & 3) == 0 ? d : 0.f;
         part += __shfl_xor_sync(FULL, part, 4);
-        part += __shfl_xor_sync(FULL, part, 8);
     } else {
         part = 0.f;
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-            float2 af = u2f2(vv[j]);
+            const float2 af = u2f2(vv[j]);
             part = fmaf(af.x, h2f(xh[2 * j]), part);
             part = fmaf(af.y, h2f(xh[2 * j + 1]), part);
         }
-#pragma unroll
-        for (int o = 1; o < 16; o <<= 1) part += __shfl_xor_sync(FULL, part, o);
+        part += __shfl_xor_sync(FULL, part, 1);
+        part += __shfl_xor_sync(FULL, part, 2);
+        part += __shfl_xor_sync(FULL, part, 4);
     }
-    if ((lane & 15) == 0) static_cast<float*>(P.partial)[u * 2 + (lane >> 4)] = part;
+    if ((lane & 7) == 0) static_cast<float*>(P.partial)[u * 4 + (lane >> 3)] = part;
 }
 
 // ------------------------------------------------------------------------------------------
@@ -274,44 +272,49 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, i
     const int64_t base = __ldg(P.rb_ptr + rb), end = __ldg(P.rb_ptr + rb + 1);
     const int64_t ib = __ldg(P.irr_ptr + i), ie = __ldg(P.irr_ptr + i + 1);
     const int32_t orow = __ldg(P.med_out + i);
-    const int nreg = static_cast<int>((end - base) >> 7);
-    const int nfull = nreg >> 1, rem = nreg & 1;
+    const int nreg = static_cast<int>((end - base) >> 6);
+    const int nfull = nreg >> 2, rem = nreg & 3;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + base;
     const int32_t* rc = P.reg_col + base;
     const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
     float c0 = 0.f, c1 = 0.f, part = 0.f;
-    auto block = [&](uint32_t a0, uint32_t a2, const uint32_t* c) {
-        uint16_t xh[4];
-#pragma unroll
-        for (int e = 0; e < 4; ++e) xh[e] = gxh(x, c[e]);
+    // one 8x8 block: this lane's two slots 2t, 2t+1 of row g
+    auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) {
+        const uint16_t xa = gxh(x, ca), xb = gxh(x, cb);
         if constexpr (VAR == VAR_MMA) {
-            hmma(c0, c1, a0, a2, pack2(xh[0], xh[1]), pack2(xh[2], xh[3]));
+            hmma(c0, c1, a, pack2(xa, xb));
         } else {
-            const float2 lo = u2f2(a0), hi = u2f2(a2);
-            part = fmaf(lo.x, h2f(xh[0]), part);
-            part = fmaf(lo.y, h2f(xh[1]), part);
-            part = fmaf(hi.x, h2f(xh[2]), part);
-            part = fmaf(hi.y, h2f(xh[3]), part);
+            const float2 av = u2f2(a);
+            part = fmaf(av.x, h2f(xa), part);
+            part = fmaf(av.y, h2f(xb), part);
         }
     };
-    // round 1: first chunk (2 blocks), the ragged last block and the first irregular element
+    // round 1: first chunk (4 blocks: 16 B values, 32 B columns), the ragged last chunk and
+    // the first irregular element
     uint32_t va[4] = {0u, 0u, 0u, 0u}, ca[8];
 #pragma unroll
     for (int e = 0; e < 8; ++e) ca[e] = 0xffffffffu;
     if (nfull > 0) { ld4_b32(rv + lane * 8, pol, va); ld8_b32(rc + lane * 8, pol, ca); }
-    uint32_t vr0 = 0u, vr1 = 0u, cr[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
-    if (rem) { ld2_b32(rv + nfull * 256 + lane * 4, pol, vr0, vr1); ld4_b32(rc + nfull * 256 + lane * 4, pol, cr); }
+    uint32_t vr[3] = {0u, 0u, 0u}, cr[6];
+#pragma unroll
+    for (int e = 0; e < 6; ++e) cr[e] = 0xffffffffu;
+    const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2 * rem;
+#pragma unroll
+    for (int j = 0; j < 3; ++j)
+        if (j < rem) { vr[j] = ld1_b32(rv + rbase + 2 * j, pol); ld2_b32(rc + rbase + 2 * j, pol, cr[2 * j], cr[2 * j + 1]); }
     int64_t k = ib + t;
     uint16_t vi = 0;
     uint32_t ci = 0xffffffffu;
     if (k < ie) { vi = __ldg(iv + k); ci = ld1_b32(P.irr_col + k, pol); }
     for (int ch = 0; ch < nfull; ++ch) {
         if (ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
-        block(va[0], va[1], &ca[0]);
-        block(va[2], va[3], &ca[4]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) block(va[j], ca[2 * j], ca[2 * j + 1]);
     }
-    if (rem) block(vr0, vr1, cr);
+#pragma unroll
+    for (int j = 0; j < 3; ++j)
+        if (j < rem) block(vr[j], cr[2 * j], cr[2 * j + 1]);   // rem is warp-uniform
     if constexpr (VAR == VAR_MMA) {
         const float d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.f;
@@ -388,7 +391,8 @@ __device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int
     uint16_t xh[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) xh[e] = gxh(x, c[e]);
-    // element e: four-slot row group q = (e<2 ? 0 : 2) + (t>>1), slot 2(t&1) + (e&1)
+    // element e: four-slot row group q = (e<2 ? 0 : 2) + (t>>1), slot 2(t&1) + (e&1); elements
+    // 0,1 are this lane's slots of m16n8k8 block 0 (rows 0-15), elements 2,3 of block 1 (16-31)
     const int seg0 = seg_of(cat, 2 * (t & 1)), seg1 = seg_of(cat, 2 * (t & 1) + 1);
     const int gs = lane & 7;                              // row g' whose result this lane collects
     float r0 = 0.f, r1 = 0.f;
@@ -407,13 +411,13 @@ __device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int
     for (int q = 0; q < 4; ++q) {
         for (int s = 0; s < nseg; ++s) {
             float val;
-            if constexpr (VAR == VAR_MMA) {
-                const bool lo = q == (t >> 1), hi = q == 2 + (t >> 1);
+            if constexpr (VAR == VAR_MMA) {      // block q>>1, x masked to group q and segment s
+                const bool mine = (q & 1) == (t >> 1);
                 const bool m0 = seg0 == s, m1 = seg1 == s;
-                const uint32_t b0 = lo ? pack2(m0 ? xh[0] : 0, m1 ? xh[1] : 0) : 0u;
-                const uint32_t b1 = hi ? pack2(m0 ? xh[2] : 0, m1 ? xh[3] : 0) : 0u;
+                const int eb = (q >> 1) * 2;
+                const uint32_t b0 = mine ? pack2(m0 ? xh[eb] : 0, m1 ? xh[eb + 1] : 0) : 0u;
                 float cc0 = 0.f, cc1 = 0.f;
-                hmma(cc0, cc1, a0, a2, b0, b1);
+                hmma(cc0, cc1, (q >> 1) ? a2 : a0, b0);
                 val = __shfl_sync(FULL, (g & 1) ? cc1 : cc0, 4 * gs + (gs >> 1));
             } else {
                 val = __shfl_sync(FULL, q < 2 ? slo[s] : shi[s], 4 * gs + 2 * (q & 1));

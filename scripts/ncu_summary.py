@@ -1,0 +1,87 @@
+#!/usr/bin/env python3
+"""Summarise Nsight Compute reports of dasp_main_kernel into profiles/ (markdown + traffic JSON).
+
+    python scripts/ncu_summary.py OUT.md KEY=REPORT.ncu-rep [KEY=REPORT.ncu-rep ...]
+
+KEY is "<workload>/<dtype>/<variant>" (bench.py's lookup key for roofline.traffic).
+profiles/ncu_traffic.json receives dram__bytes_read.sum + dram__bytes_write.sum per launch.
+"""
+import csv
+import io
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+WANT = [
+    ("gpu__time_duration.sum", "duration"),
+    ("dram__bytes_read.sum", "DRAM read"),
+    ("dram__bytes_write.sum", "DRAM write"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "DRAM throughput % of peak"),
+    ("lts__t_sector_hit_rate.pct", "L2 hit %"),
+    ("l1tex__t_sector_hit_rate.pct", "L1 hit %"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved occupancy %"),
+    ("launch__registers_per_thread", "registers/thread"),
+    ("launch__grid_size", "grid"),
+    ("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active", "LSU pipe inst %"),
+    ("sm__inst_executed_pipe_tensor_subpipe_dmma.avg.pct_of_peak_sustained_active", "tensor DMMA inst %"),
+    ("sm__inst_executed_pipe_tensor_subpipe_hmma.avg.pct_of_peak_sustained_active", "tensor HMMA inst %"),
+    ("TPC.TriageCompute.sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed", "tensor pipe cycles active %"),
+    ("TPC.TriageCompute.sm__pipe_fp64_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed", "FP64 pipe cycles active %"),
+    ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", "FMA pipe inst %"),
+    ("sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active", "FP64 pipe inst %"),
+    ("smsp__inst_executed.sum", "warp instructions"),
+]
+
+
+def raw(rep):
+    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    h, u = rows[0], rows[1]
+    res = []
+    for r in rows[2:]:
+        res.append({h[i]: (u[i], r[i]) for i in range(len(h))})
+    return res
+
+
+def to_bytes(unit, v):
+    f = float(v.replace(",", ""))
+    return f * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(unit, 1)
+
+
+def main():
+    out_md = sys.argv[1]
+    traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
+    lines = ["# ncu summaries (dasp_main_kernel, `--set full --clock-control none`, one launch each)", ""]
+    for arg in sys.argv[2:]:
+        key, rep = arg.split("=", 1)
+        for k, d in enumerate(raw(rep)):
+            if "dasp_main_kernel" not in d.get("Kernel Name", ("", ""))[1]:
+                continue
+            lines.append(f"## {key}  ({os.path.basename(rep)})")
+            lines.append("")
+            lines.append("| metric | value |")
+            lines.append("|---|---|")
+            for m, name in WANT:
+                if m in d:
+                    lines.append(f"| {name} (`{m}`) | {d[m][1]} {d[m][0]} |")
+            stalls = sorted(((float(v[1].replace(",", "") or 0), m) for m, v in d.items()
+                             if m.startswith("smsp__pcsamp_warps_issue_stalled_") and not m.endswith("not_issued")),
+                            reverse=True)[:6]
+            lines.append("| top stall samples | " + ", ".join(f"{m.split('stalled_')[1]} {int(c)}" for c, m in stalls) + " |")
+            rd = to_bytes(*d["dram__bytes_read.sum"])
+            wr = to_bytes(*d["dram__bytes_write.sum"])
+            traffic[key] = rd + wr
+            lines.append("")
+            break
+    with open(out_md, "w") as f:
+        f.write("\n".join(lines) + "\n")
+    with open(traffic_path, "w") as f:
+        json.dump(traffic, f, indent=1, sort_keys=True)
+
+
+if __name__ == "__main__":
+    main()

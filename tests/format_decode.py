@@ -15,7 +15,7 @@ PAD = -1
 def params(dtype):
     if dtype == "f64":
         return dict(K=4, BE=32, EPL=1, G=64, UG=4, CW=4)
-    return dict(K=16, BE=128, EPL=4, G=256, UG=2, CW=2)
+    return dict(K=8, BE=64, EPL=2, G=128, UG=4, CW=4)
 
 
 def _bits(vals):
@@ -63,7 +63,7 @@ def decode(F, get, dtype):
             for lane in range(32):
                 g, t = lane >> 2, lane & 3
                 for e in range(EPL):
-                    slot = K * b + (t if EPL == 1 else (2 * t + e if e < 2 else 2 * t + 8 + e - 2))
+                    slot = K * b + (t if EPL == 1 else 2 * t + e)
                     at = base + lane * w * EPL + jb * EPL + e
                     slots[g][slot] = (rc[at], rv[at])
         for g in range(8):

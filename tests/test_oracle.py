@@ -147,12 +147,12 @@ def test_p9_stencil_closed_forms(g):
     if g == 128:
         assert (c["nnz_reg_new"], c["nnz_irreg"]) == (49_551_328, 6_191_640)
     if g == 16:
-        # FP16, K=16 (R14): len 27 -> 1 block + 11 irregular (block 1: 88/128 <= 96);
-        # len 18 -> 1 + 2; len 12 -> block 0 holds 96/128, not > 96 -> 0 + 12; len 8 -> 0 + 8
+        # FP16, K=8 (m16n8k8, R14): len 27 -> 3 blocks + 3 irregular (block 3: 24/64 <= 48);
+        # len 18 -> 2 + 2; len 12 -> block 1 holds 32/64 -> 1 + 4; len 8 -> 1 + 0
         F16 = oracle.build(A.to_fp16(), "f16")
         c16 = F16.counts
-        assert c16["nnz_reg_new"] == 16 * (h[27] + h[18])
-        assert c16["nnz_irreg"] == 11 * h[27] + 2 * h[18] + 12 * h[12] + 8 * h[8]
+        assert c16["nnz_reg_new"] == 24 * h[27] + 16 * h[18] + 8 * h[12] + 8 * h[8]
+        assert c16["nnz_irreg"] == 3 * h[27] + 2 * h[18] + 4 * h[12]
 
 
 # P8: closed-form short piecing counts (R13)
@@ -190,7 +190,7 @@ def test_p6_roundtrip(name, dt):
     check_roundtrip(A, F.counts, F.view, dt)
     c = F.counts
     assert c["n0"] + c["n1"] + c["n2"] + c["n3"] + c["n4"] + c["row_medium"] + c["row_long"] == A.m
-    G = 64 if dt == "f64" else 256
+    G = 64 if dt == "f64" else 128
     assert c["nnz_long_new"] == sum(-(-L // G) * G for L in np.diff(A.row_ptr) if L > 256)
 
 
