@@ -35,9 +35,10 @@ clean:
 
 .PHONY: all clean
 
-# experiment builds: occupancy (min blocks per SM of the fused kernel)
+# experiment builds: one libdasp_<VAR=value>.so per -D setting in EXPVARS
+EXPVARS ?= DASP_NSTAGE=3 DASP_NSTAGE=4
 exp: $(OBJ)/builder.o $(OBJ)/api.o
-	for mb in 4 5 6; do \
-	  $(NVCC) $(NVFLAGS) -DDASP_MIN_BLOCKS=$$mb -c $(SRC)/kernels.cu -o $(OBJ)/kernels_mb$$mb.o 2> $(OBJ)/kernels_mb$$mb.ptxas.txt && \
-	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_mb$$mb.so $(OBJ)/builder.o $(OBJ)/kernels_mb$$mb.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
+	for v in $(EXPVARS); do \
+	  $(NVCC) $(NVFLAGS) -D$$v -c $(SRC)/kernels.cu -o $(OBJ)/kernels_$$v.o 2> $(OBJ)/kernels_$$v.ptxas.txt && \
+	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$v.so $(OBJ)/builder.o $(OBJ)/kernels_$$v.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
 	done

@@ -50,6 +50,9 @@ def parse():
     ap.add_argument("--variant", default="mma", choices=["mma", "cudacore"])
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
+    ap.add_argument("--pipeline", action="store_true", help="use the TMA-staged persistent kernel")
+    ap.add_argument("--panel-rows", type=int, default=0, help="rows per panel (0 auto, -1 one global panel)")
+    ap.add_argument("--no-triad", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=12.0)
@@ -150,6 +153,28 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def stream_triad(dev, n=1 << 28, reps=20):
+    """STREAM triad a = b + s*c in FP64 on this GPU (3 x 2 GiB arrays, 24 B per element), best of
+    `reps`, CUDA events: the same-run HBM reference of SURVEY.md §8(d)."""
+    import torch
+    b = torch.rand(n, dtype=torch.float64, device=dev)
+    c = torch.rand(n, dtype=torch.float64, device=dev)
+    a = torch.empty_like(b)
+    best = float("inf")
+    for _ in range(3):
+        torch.add(b, c, alpha=3.0, out=a)
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        torch.add(b, c, alpha=3.0, out=a)
+        e1.record()
+        e1.synchronize()
+        best = min(best, e0.elapsed_time(e1))
+    del a, b, c
+    torch.cuda.empty_cache()
+    return 24.0 * n / (best * 1e-3) / 1e9
+
+
 def load_traffic(config, dtype, variant):
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
@@ -243,7 +268,8 @@ def main():
     if world == 1:
         # single GPU: plain SpMV over resident inputs, y overwritten every step
         plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
-                                     device=local, variant=variant, medium_rb_per_warp=args.rbw)
+                                     device=local, variant=variant, medium_rb_per_warp=args.rbw,
+                                     pipeline=args.pipeline, panel_rows=args.panel_rows)
         xdt = torch.float64 if args.dtype == "f64" else torch.float16
         ydt = torch.float64 if args.dtype == "f64" else torch.float32
         xd = torch.from_numpy(x_global).to(xdt).to(dev)
@@ -310,11 +336,13 @@ def main():
     main_avg = main_ms / max(main_n, 1)
     achieved = bm["main"] / (main_avg * 1e-3) / 1e9 if main_n else None
     traffic = load_traffic(workload, args.dtype, args.variant)
+    triad = None if args.no_triad else stream_triad(dev)
     roofline = {"kernel": "dasp_main_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak if achieved else None, "traffic": traffic,
                 "alg_bytes_per_launch": bm["main"], "avg_launch_ms": main_avg,
                 "share_of_step": (main_ms / max(main_n, 1)) / ms_step if main_n else None,
-                "finish_avg_ms": fin_ms / fin_n if fin_n else 0.0, "peak_source": peak_src}
+                "finish_avg_ms": fin_ms / fin_n if fin_n else 0.0, "peak_source": peak_src,
+                "stream_triad_gbs": triad, "frac_of_triad": achieved / triad if (achieved and triad) else None}
 
     # ---- e2e: the same metric through the C-ABI with HOST buffers (copies inside the timed region) ----
     e2e = None
@@ -352,6 +380,7 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config),
                        "m": int(spec.m), "n": int(spec.n), "nnz": nnz_total, "variant": args.variant,
+                       "kernel": "pipeline" if info.get("pipeline") else "direct", "panel_rows": info["panel_rows"],
                        "parallelism": f"row-slab x{world}" + (" + NCCL all-gather of x" if world > 1 else ""),
                        "l2": "inputs larger than L2 (packed A streamed every step); x stays L2-resident "
                              "across steps as in the paper's averaged back-to-back runs"},

@@ -69,6 +69,10 @@ typedef struct {
                                    rows is classified, sorted and pieced on its own so x and y
                                    windows stay L2-resident; 0 = automatic, -1 = one panel
                                    (the paper's global format)                        */
+    int32_t pipeline;           /* 1: persistent kernel whose producer lane stages every item's
+                                   packed arrays in shared memory with cp.async.bulk (TMA) and
+                                   mbarriers; 0 (default): one warp per item, loads straight to
+                                   registers (faster on B200 in our measurements) */
 } dasp_options_t;
 
 /* Fills `opts` with the defaults: device 0, MMA variant, validate, no keep_host, auto LOOP_NUM,
@@ -93,6 +97,7 @@ typedef struct {
     int32_t medium_rb_per_warp;
     int32_t launches_per_spmv;                         /* kernels one dasp_spmv enqueues    */
     int64_t panel_rows, n_panels;                      /* resolved panel size and count     */
+    int32_t pipeline;                                  /* 1 if the TMA-staged kernel is used */
     double build_ms, upload_ms;                        /* host build; host->device upload   */
 } dasp_plan_info_t;
 

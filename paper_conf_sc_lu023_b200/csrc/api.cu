@@ -35,6 +35,9 @@ struct dasp_plan_s {
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
     void* d_blk_panel = nullptr;          // int32 panel of every block
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
+    void* d_items = nullptr;              // uint64 item words of the pipelined kernel
+    int64_t n_items = 0, pipe_blocks = 0;
+    bool pipe = false;                    // persistent TMA-staged kernel (else the one-warp-per-item kernel)
     size_t apw_bytes = 0;                 // L2 persisting access-policy window over x (0 = off)
     float apw_hit = 1.0f;
     // timing
@@ -54,6 +57,7 @@ int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
+constexpr int64_t kAllocPad = 64;   // TMA windows may read up to 16 B past an array's end
 
 int auto_rbw(int64_t row_medium) {
     if (row_medium < 59990) return 1;
@@ -82,7 +86,8 @@ void free_device(dasp_plan_s* p) {
     if (p->d_panels) cudaFree(p->d_panels);
     if (p->d_blk_panel) cudaFree(p->d_blk_panel);
     if (p->d_unit_order) cudaFree(p->d_unit_order);
-    p->d_panels = p->d_blk_panel = p->d_unit_order = nullptr;
+    if (p->d_items) cudaFree(p->d_items);
+    p->d_panels = p->d_blk_panel = p->d_unit_order = p->d_items = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -142,6 +147,7 @@ void dasp_options_default(dasp_options_t* o) {
     o->medium_rb_per_warp = 0;
     o->num_threads = 0;
     o->panel_rows = 0;
+    o->pipeline = 0;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -235,6 +241,32 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
             for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + cnt[bucket(d.unit0 + w)]++] = static_cast<int32_t>(d.unit0 + w);
         }
     }
+    // item words of the pipelined kernel, panel by panel: long units (schedule order), medium
+    // row-blocks, short tiles (kind<<62 | payload; kernels.cu produce())
+    std::vector<uint64_t> items;
+    bool items_ok = true;
+    for (const auto& d : desc) {
+        for (int64_t w = 0; w < d.nunits; ++w) items.push_back((1ull << 62) | static_cast<uint64_t>(unit_order[d.unit0 + w]));
+        for (int64_t r = 0; r < d.nrb; ++r) items.push_back((2ull << 62) | static_cast<uint64_t>(d.rb0 + r));
+        const int64_t nt = d.t13 + d.t4 + d.t22 + d.ts;
+        for (int64_t t = 0; t < nt; ++t) {
+            int64_t cat, ob;
+            if (t < d.t13) { cat = 0; ob = d.out0 + t * 64; }
+            else if (t < d.t13 + d.t4) { cat = 1; ob = d.out0 + 64 * d.t13 + (t - d.t13) * 32; }
+            else if (t < d.t13 + d.t4 + d.t22) { cat = 2; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + (t - d.t13 - d.t4) * 64; }
+            else { cat = 3; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + 64 * d.t22 + (t - d.t13 - d.t4 - d.t22) * 128; }
+            const int64_t tile = d.tile0 + t;
+            if (tile >= (int64_t(1) << 27) || ob >= (int64_t(1) << 33)) items_ok = false;
+            items.push_back((3ull << 62) | (static_cast<uint64_t>(cat) << 60) | (static_cast<uint64_t>(tile) << 33) |
+                            static_cast<uint64_t>(ob));
+        }
+    }
+    p->n_items = static_cast<int64_t>(items.size());
+    {
+        // DASP_PIPE overrides the option (experiments)
+        const char* pe = std::getenv("DASP_PIPE");
+        p->pipe = items_ok && (pe ? std::atoi(pe) != 0 : o.pipeline != 0);
+    }
     for (int a = 0; a < DASP_ARR_COUNT; ++a) p->bytes[a] = f.arr[a].bytes;
 
     if (p->device >= 0) {
@@ -242,7 +274,7 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
             if (p->bytes[a] == 0) continue;
             // 256 B alignment from cudaMalloc keeps every lane's 16/32 B vector load aligned
-            if (cudaMalloc(&p->d[a], static_cast<size_t>(p->bytes[a])) != cudaSuccess) {
+            if (cudaMalloc(&p->d[a], static_cast<size_t>(p->bytes[a] + kAllocPad)) != cudaSuccess) {
                 free_device(p); f.release(); delete p;
                 return DASP_ERR_OUT_OF_MEMORY;
             }
@@ -272,6 +304,22 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
             return DASP_ERR_CUDA;
         }
         p->device_bytes += ub;
+        if (p->pipe) {
+            const size_t ib = std::max<size_t>(items.size(), 1) * 8;
+            int bps = 0, nsm = 0;
+            if (cudaMalloc(&p->d_items, ib) != cudaSuccess) { free_device(p); f.release(); delete p; return DASP_ERR_OUT_OF_MEMORY; }
+            if ((!items.empty() && cudaMemcpy(p->d_items, items.data(), items.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess) ||
+                dasp::pipe_occupancy(p->dtype, DASP_VARIANT_CUDACORE, &bps) != cudaSuccess ||   // sets both kernels'
+                dasp::pipe_occupancy(p->dtype, DASP_VARIANT_MMA, &bps) != cudaSuccess ||        // smem attribute
+                cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess) {
+                free_device(p); f.release(); delete p;
+                return DASP_ERR_CUDA;
+            }
+            // persistent grid: every SM full, never more warps than items
+            const int64_t wpb = dasp::pipe_warps_per_block();
+            p->pipe_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->n_items + wpb - 1) / wpb);
+            p->device_bytes += ib;
+        }
         // optional persisting L2 access-policy window over x (DASP_X_APW=1; measured slower on
         // C3, profiles/r01, so off by default)
         const char* apw = std::getenv("DASP_X_APW");
@@ -354,6 +402,9 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
         if (c >= 1 && c <= 3) mp.class_mask = 1 << (c - 1);
     }
     e = timed(p, DASP_K_MAIN, s, on, [&] {
+        if (p->pipe)
+            return dasp::launch_pipe(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_items), p->n_items,
+                                     p->pipe_blocks, s);
         return dasp::launch_main(mp, p->dtype, variant, p->blocks, s, x, p->apw_bytes, p->apw_hit);
     });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
@@ -430,6 +481,7 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->launches_per_spmv = (p->blocks > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
+    o->pipeline = p->pipe ? 1 : 0;
     o->build_ms = p->build_ms;
     o->upload_ms = p->upload_ms;
     return DASP_OK;

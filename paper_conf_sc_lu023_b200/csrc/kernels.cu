@@ -130,87 +130,125 @@ __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typena
 // ------------------------------------------------------------------------------------------
 // long rows, phase 1 (Alg. 2 l.1-16): one warp = one unit of UG consecutive groups
 // ------------------------------------------------------------------------------------------
+// Lane l reads the unit's 16-B value chunks l + 32j (j = 0..3): elements 2(l+32j), 2(l+32j)+1,
+// both in group j.  Every load instruction is one contiguous 512-B (values) / 256-B (columns)
+// span, and the 32 gathers of one instruction hit 64 consecutive, column-sorted elements of a
+// long row, so they share sectors in L1.  Group j is accumulated separately (4 accumulators)
+// and reduced over the warp.
 template <int VAR>
 __device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol) {
-    const int64_t base = u * 256 + lane * 8;            // lane holds 8 consecutive elements
-    const double* lv = static_cast<const double*>(P.long_val) + base;
+    const double* lv = static_cast<const double*>(P.long_val) + u * 256;
+    const int32_t* lc = P.long_col + u * 256;
+    const double* x = static_cast<const double*>(P.x);
     double v[8];
     uint32_t c[8];
-    ld4_f64(lv, pol, *reinterpret_cast<double(*)[4]>(&v[0]));
-    ld4_f64(lv + 4, pol, *reinterpret_cast<double(*)[4]>(&v[4]));
-    ld8_b32(P.long_col + base, pol, c);
-    const double* x = static_cast<const double*>(P.x);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        ld2_f64(lv + 2 * (lane + 32 * j), pol, v[2 * j], v[2 * j + 1]);
+        ld2_b32(lc + 2 * (lane + 32 * j), pol, c[2 * j], c[2 * j + 1]);
+    }
     double xv[8];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) xv[j] = gx(x, c[j]);
-    double part;
-    if constexpr (VAR == VAR_MMA) {
-        double c0 = 0.0, c1 = 0.0;
+    for (int e = 0; e < 8; ++e) xv[e] = gx(x, c[e]);
+    double gsum[4];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) dmma(c0, c1, v[j], xv[j]);   // 8 m8n8k4 = 4 groups of 64
-        double d = diag_to_quad(c0, c1, lane);                  // rows 2q, 2q+1 = group q
-        part = (lane & 3) == 0 ? d : 0.0;
-        part += __shfl_xor_sync(FULL, part, 4);
-    } else {
-        part = 0.0;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) part = fma(v[j], xv[j], part);
-        part += __shfl_xor_sync(FULL, part, 1);
-        part += __shfl_xor_sync(FULL, part, 2);
-        part += __shfl_xor_sync(FULL, part, 4);
+    for (int j = 0; j < 4; ++j) {
+        if constexpr (VAR == VAR_MMA) {                  // trace of C_j = sum of group j (Fig. 4 diagonal)
+            double c0 = 0.0, c1 = 0.0;
+            dmma(c0, c1, v[2 * j], xv[2 * j]);
+            dmma(c0, c1, v[2 * j + 1], xv[2 * j + 1]);
+            gsum[j] = is_diag_holder(lane) ? (((lane >> 2) & 1) ? c1 : c0) : 0.0;
+        } else {
+            gsum[j] = fma(v[2 * j], xv[2 * j], v[2 * j + 1] * xv[2 * j + 1]);
+        }
     }
-    if ((lane & 7) == 0) static_cast<double*>(P.partial)[u * 4 + (lane >> 3)] = part;
+    // 4-way transpose-reduce: after it lane l holds the full sum of group (l >> 3) & 3
+    {
+        const bool hi16 = lane & 16, hi8 = lane & 8;
+        double a0 = hi16 ? gsum[0] : gsum[2], a1 = hi16 ? gsum[1] : gsum[3];
+        double k0 = hi16 ? gsum[2] : gsum[0], k1 = hi16 ? gsum[3] : gsum[1];
+        k0 += __shfl_xor_sync(FULL, a0, 16);          // groups {0,1} on lanes 0-15, {2,3} on 16-31
+        k1 += __shfl_xor_sync(FULL, a1, 16);
+        double b = hi8 ? k0 : k1, kk = hi8 ? k1 : k0;
+        kk += __shfl_xor_sync(FULL, b, 8);             // lane l: group 2*(l>>4) + ((l>>3)&1)
+        kk += __shfl_xor_sync(FULL, kk, 4);
+        kk += __shfl_xor_sync(FULL, kk, 2);
+        kk += __shfl_xor_sync(FULL, kk, 1);
+        if ((lane & 7) == 0) static_cast<double*>(P.partial)[u * 4 + 2 * (lane >> 4) + ((lane >> 3) & 1)] = kk;
+    }
 }
 
+// FP16: lane l reads 8-B value chunks l + 32j (j = 0..3): halves 4(l+32j)..+3, all in group j
 template <int VAR>
 __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol) {
-    const int64_t base = u * 512 + lane * 16;           // lane holds 16 consecutive elements
-    uint32_t vv[8], c[16];
-    ld8_b32(static_cast<const uint16_t*>(P.long_val) + base, pol, vv);
-    ld8_b32(P.long_col + base, pol, *reinterpret_cast<uint32_t(*)[8]>(&c[0]));
-    ld8_b32(P.long_col + base + 8, pol, *reinterpret_cast<uint32_t(*)[8]>(&c[8]));
+    const uint16_t* lv = static_cast<const uint16_t*>(P.long_val) + u * 512;
+    const int32_t* lc = P.long_col + u * 512;
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    uint32_t vv[8], c[16];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        ld2_b32(lv + 4 * (lane + 32 * j), pol, vv[2 * j], vv[2 * j + 1]);
+        ld4_b32(lc + 4 * (lane + 32 * j), pol, *reinterpret_cast<uint32_t(*)[4]>(&c[4 * j]));
+    }
     uint16_t xh[16];
 #pragma unroll
-    for (int j = 0; j < 16; ++j) xh[j] = gxh(x, c[j]);
-    float part;
-    if constexpr (VAR == VAR_MMA) {
-        float c0 = 0.f, c1 = 0.f;
+    for (int e = 0; e < 16; ++e) xh[e] = gxh(x, c[e]);
+    float gsum[4];
 #pragma unroll
-        for (int h = 0; h < 8; ++h)   // elements 2h, 2h+1 -> A[g][2t..2t+1] of one m16n8k8
-            hmma(c0, c1, vv[h], pack2(xh[2 * h], xh[2 * h + 1]));
-        const float d = diag_to_quad(c0, c1, lane);             // rows 2q, 2q+1 = group q
-        part = (lane & 3) == 0 ? d : 0.f;
-        part += __shfl_xor_sync(FULL, part, 4);
-    } else {
-        part = 0.f;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const float2 af = u2f2(vv[j]);
-            part = fmaf(af.x, h2f(xh[2 * j]), part);
-            part = fmaf(af.y, h2f(xh[2 * j + 1]), part);
+    for (int j = 0; j < 4; ++j) {
+        if constexpr (VAR == VAR_MMA) {
+            float c0 = 0.f, c1 = 0.f;
+            hmma(c0, c1, vv[2 * j], pack2(xh[4 * j], xh[4 * j + 1]));
+            hmma(c0, c1, vv[2 * j + 1], pack2(xh[4 * j + 2], xh[4 * j + 3]));
+            gsum[j] = is_diag_holder(lane) ? (((lane >> 2) & 1) ? c1 : c0) : 0.f;
+        } else {
+            const float2 a = u2f2(vv[2 * j]), b = u2f2(vv[2 * j + 1]);
+            float sacc = a.x * h2f(xh[4 * j]);
+            sacc = fmaf(a.y, h2f(xh[4 * j + 1]), sacc);
+            sacc = fmaf(b.x, h2f(xh[4 * j + 2]), sacc);
+            gsum[j] = fmaf(b.y, h2f(xh[4 * j + 3]), sacc);
         }
-        part += __shfl_xor_sync(FULL, part, 1);
-        part += __shfl_xor_sync(FULL, part, 2);
-        part += __shfl_xor_sync(FULL, part, 4);
     }
-    if ((lane & 7) == 0) static_cast<float*>(P.partial)[u * 4 + (lane >> 3)] = part;
+    {
+        const bool hi16 = lane & 16, hi8 = lane & 8;
+        float a0 = hi16 ? gsum[0] : gsum[2], a1 = hi16 ? gsum[1] : gsum[3];
+        float k0 = hi16 ? gsum[2] : gsum[0], k1 = hi16 ? gsum[3] : gsum[1];
+        k0 += __shfl_xor_sync(FULL, a0, 16);
+        k1 += __shfl_xor_sync(FULL, a1, 16);
+        float b = hi8 ? k0 : k1, kk = hi8 ? k1 : k0;
+        kk += __shfl_xor_sync(FULL, b, 8);
+        kk += __shfl_xor_sync(FULL, kk, 4);
+        kk += __shfl_xor_sync(FULL, kk, 2);
+        kk += __shfl_xor_sync(FULL, kk, 1);
+        if ((lane & 7) == 0) static_cast<float*>(P.partial)[u * 4 + 2 * (lane >> 4) + ((lane >> 3) & 1)] = kk;
+    }
 }
 
 // ------------------------------------------------------------------------------------------
 // medium rows (Alg. 3): row-block = 8 rows; regular 8 x K blocks in lane-interleaved chunks
 // of CW blocks (R18), then the irregular tails with 4 lanes per row, then y.
 // ------------------------------------------------------------------------------------------
+// A row-block's metadata: its regular range, this lane's row's irregular range and output row.
+// The warp loads the NEXT row-block's metadata before working on the current one, so every
+// row-block after the first costs one memory round trip (stream loads) plus the gathers.
+struct RbMeta {
+    int64_t base, ib;         // regular region start; this lane's row's irregular start
+    int32_t nelem, ilen;      // regular elements (<= 64 blocks); irregular length (<= 256)
+    int32_t orow;
+};
+__device__ __forceinline__ RbMeta rb_meta(const MainParams& P, int64_t rb, int lane) {
+    const int64_t i = rb * 8 + (lane >> 2);
+    const int64_t base = __ldg(P.rb_ptr + rb), ib = __ldg(P.irr_ptr + i);
+    return RbMeta{base, ib, static_cast<int32_t>(__ldg(P.rb_ptr + rb + 1) - base),
+                  static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i)};
+}
+
 template <int VAR>
-__device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
-    const int g = lane >> 2, t = lane & 3;
-    const int64_t i = rb * 8 + g;
-    // every load that does not depend on data goes out first: the row-block's pointers, the
-    // irregular bounds and the output row (one memory round trip instead of three)
-    const int64_t base = __ldg(P.rb_ptr + rb), end = __ldg(P.rb_ptr + rb + 1);
-    const int64_t ib = __ldg(P.irr_ptr + i), ie = __ldg(P.irr_ptr + i + 1);
-    const int32_t orow = __ldg(P.med_out + i);
-    const int nreg = static_cast<int>((end - base) >> 5);
+__device__ __forceinline__ void medium_rb_f64(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
+    const int t = lane & 3;
+    const int64_t base = M.base, ib = M.ib, ie = M.ib + M.ilen;
+    const int32_t orow = M.orow;
+    const int nreg = M.nelem >> 5;
     const int nfull = nreg >> 2, rem = nreg & 3;
     const double* rv = static_cast<const double*>(P.reg_val) + base;
     const int32_t* rc = P.reg_col + base;
@@ -266,13 +304,11 @@ __device__ __forceinline__ void medium_rb_f64(const MainParams& P, int64_t rb, i
 }
 
 template <int VAR>
-__device__ __forceinline__ void medium_rb_f16(const MainParams& P, int64_t rb, int lane, uint64_t pol) {
-    const int g = lane >> 2, t = lane & 3;
-    const int64_t i = rb * 8 + g;
-    const int64_t base = __ldg(P.rb_ptr + rb), end = __ldg(P.rb_ptr + rb + 1);
-    const int64_t ib = __ldg(P.irr_ptr + i), ie = __ldg(P.irr_ptr + i + 1);
-    const int32_t orow = __ldg(P.med_out + i);
-    const int nreg = static_cast<int>((end - base) >> 6);
+__device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
+    const int t = lane & 3;
+    const int64_t base = M.base, ib = M.ib, ie = M.ib + M.ilen;
+    const int32_t orow = M.orow;
+    const int nreg = M.nelem >> 6;
     const int nfull = nreg >> 2, rem = nreg & 3;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + base;
     const int32_t* rc = P.reg_col + base;
@@ -378,15 +414,10 @@ __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int
 }
 
 template <int VAR>
-__device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol) {
+__device__ __forceinline__ void short_compute_f16(const MainParams& P, int cat, uint32_t a0, uint32_t a2, const uint32_t (&c)[4],
+                                                  int32_t o0, int32_t o1, int lane) {
     const int g = lane >> 2, t = lane & 3;
     const int nseg = cat == 1 ? 1 : 2;
-    uint32_t a0, a2, c[4];
-    ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
-    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
-    const int32_t o0 = __ldg(P.short_out + obase + lane);
-    const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
     uint16_t xh[4];
 #pragma unroll
@@ -429,6 +460,18 @@ __device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int
     }
     store_y<1>(P, o0, r0);
     if (nseg == 2) store_y<1>(P, o1, r1);
+}
+
+template <int VAR>
+__device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
+                                               uint64_t pol) {
+    const int nseg = cat == 1 ? 1 : 2;
+    uint32_t a0, a2, c[4];
+    ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
+    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
+    const int32_t o0 = __ldg(P.short_out + obase + lane);
+    const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
+    short_compute_f16<VAR>(P, cat, a0, a2, c, o0, o1, lane);
 }
 
 // singles (Alg. 5): lane handles 4 consecutive len-1 rows on CUDA cores
@@ -483,9 +526,12 @@ __global__ void __launch_bounds__(MAIN_THREADS, DASP_MIN_BLOCKS) dasp_main_kerne
         const int64_t rbp0 = __ldg(&D->rb0);
         const int64_t rb0 = rbp0 + w * P.rbw;
         const int64_t rb1 = min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb));
+        RbMeta cur = rb_meta(P, rb0, lane);
         for (int64_t rb = rb0; rb < rb1; ++rb) {
-            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb, lane, pol);
-            else medium_rb_f16<VAR>(P, rb, lane, pol);
+            const RbMeta nxt = rb + 1 < rb1 ? rb_meta(P, rb + 1, lane) : cur;   // prefetch
+            if constexpr (DT == 0) medium_rb_f64<VAR>(P, cur, lane, pol);
+            else medium_rb_f16<VAR>(P, cur, lane, pol);
+            cur = nxt;
         }
         return;
     }
@@ -547,6 +593,466 @@ __global__ void dasp_scale_kernel(void* yv, int64_t m, double beta) {
         y[i] = beta != 0.0 ? static_cast<Y>(beta) * y[i] : Y(0);
 }
 
+// ==========================================================================================
+// Persistent, TMA-staged pipeline.  Each warp walks the item list
+// (long unit | medium row-block | short tile, panel by panel) with stride = all warps of the
+// grid.  Lane 0 is the producer: NSTAGE items ahead it writes a small header into a
+// shared-memory stage and issues cp.async.bulk copies of the item's packed arrays (val, col,
+// output map, irregular windows) that complete on the stage's mbarrier; all 32 lanes then
+// consume the stage (x gathers from global, MMA / FMA, y stores).  In-flight stream bytes
+// live in shared memory instead of registers, so the SM keeps ~NSTAGE items per warp in
+// flight while the gathers of the current item are outstanding.
+// ==========================================================================================
+#ifndef DASP_NSTAGE
+#define DASP_NSTAGE 2
+#endif
+constexpr int NSTAGE = DASP_NSTAGE;
+constexpr int STAGE = 3328;                 // bytes per stage (64 B header + up to 3264 B data)
+constexpr int HDR = 64;
+enum { IT_LONG = 1, IT_MED = 2, IT_SHORT = 3, IT_MED_DIRECT = 4 };
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+
+// item word (host-built, api.cu): kind in bits 62-63;
+//   long: unit id | medium: row-block id | short: cat (60-61), tile (33-59), output base (0-32)
+__device__ __forceinline__ int item_kind(uint64_t w) { return static_cast<int>(w >> 62); }
+
+// medium pointers the producer needs one iteration before it issues the copies
+struct MedPtr {
+    int64_t base, end, irr0, irr1;
+};
+
+template <int DT>
+__device__ __forceinline__ void produce(const MainParams& P, uint64_t w, const MedPtr& mp, uint8_t* st, uint64_t* bar,
+                                        uint64_t pol) {
+    constexpr int sv = DT == 0 ? 8 : 2;
+    int64_t* h = reinterpret_cast<int64_t*>(st);
+    const int kind = item_kind(w);
+    const int64_t pay = static_cast<int64_t>(w & ((1ull << 62) - 1));
+    if (kind == IT_LONG) {
+        h[0] = IT_LONG;
+        h[1] = pay;
+        const uint32_t vb = 256 * 8, cb = 256 * 4;   // FP64: 256 elements; FP16: 512 elements
+        const uint32_t vbytes = DT == 0 ? vb : 512 * 2, cbytes = DT == 0 ? cb : 512 * 4;
+        const int64_t ne = DT == 0 ? 256 : 512;
+        mbar_expect_tx(bar, vbytes + cbytes);
+        bulk_g2s(st + HDR, static_cast<const uint8_t*>(P.long_val) + pay * ne * sv, vbytes, bar, pol);
+        bulk_g2s(st + HDR + vbytes, P.long_col + pay * ne, cbytes, bar, pol);
+    } else if (kind == IT_SHORT) {
+        const int cat = static_cast<int>((pay >> 60) & 3);
+        const int64_t tile = (pay >> 33) & ((1ll << 27) - 1);
+        const int64_t obase = pay & ((1ll << 33) - 1);
+        h[0] = IT_SHORT;
+        h[1] = tile;
+        h[2] = obase;
+        h[3] = cat;
+        const uint32_t vbytes = 128 * sv, cbytes = 128 * 4;
+        const uint32_t obytes = cat == 3 ? 128 * 4 : (cat == 1 ? 32 * 4 : 64 * 4);
+        mbar_expect_tx(bar, vbytes + cbytes + obytes);
+        bulk_g2s(st + HDR, static_cast<const uint8_t*>(P.short_val) + tile * 128 * sv, vbytes, bar, pol);
+        bulk_g2s(st + HDR + vbytes, P.short_col + tile * 128, cbytes, bar, pol);
+        bulk_g2s(st + HDR + vbytes + cbytes, P.short_out + obase, obytes, bar, pol);
+    } else {   // medium row-block
+        constexpr int BE = DT == 0 ? 32 : 64;
+        constexpr int VA = 16 / sv;                       // value elements per 16 B
+        const int64_t rb = pay;
+        const int64_t nreg = (mp.end - mp.base) / BE;
+        const int64_t ivb = mp.irr0 & ~static_cast<int64_t>(VA - 1), ive = (mp.irr1 + VA - 1) & ~static_cast<int64_t>(VA - 1);
+        const int64_t icb = mp.irr0 & ~int64_t(3), ice = (mp.irr1 + 3) & ~int64_t(3);
+        const uint32_t rv = static_cast<uint32_t>(nreg * BE * sv), rc = static_cast<uint32_t>(nreg * BE * 4);
+        const uint32_t iv = mp.irr1 > mp.irr0 ? static_cast<uint32_t>((ive - ivb) * sv) : 0u;
+        const uint32_t ic = mp.irr1 > mp.irr0 ? static_cast<uint32_t>((ice - icb) * 4) : 0u;
+        const uint32_t off_rv = HDR + 80 + 32, off_rc = off_rv + rv, off_iv = off_rc + rc, off_ic = off_iv + iv;
+        h[1] = rb;
+        h[2] = nreg;
+        h[3] = ivb;
+        h[4] = icb;
+        h[5] = off_iv;
+        h[6] = off_ic;
+        if (off_ic + ic > STAGE) {                       // does not fit: consumer reads global
+            h[0] = IT_MED_DIRECT;
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+            return;
+        }
+        h[0] = IT_MED;
+        mbar_expect_tx(bar, 80 + 32 + rv + rc + iv + ic);
+        bulk_g2s(st + HDR, P.irr_ptr + rb * 8, 80, bar, pol);            // irr_ptr[8rb .. 8rb+9]
+        bulk_g2s(st + HDR + 80, P.med_out + rb * 8, 32, bar, pol);
+        if (rv) {
+            bulk_g2s(st + off_rv, static_cast<const uint8_t*>(P.reg_val) + mp.base * sv, rv, bar, pol);
+            bulk_g2s(st + off_rc, P.reg_col + mp.base, rc, bar, pol);
+        }
+        if (iv) {
+            bulk_g2s(st + off_iv, static_cast<const uint8_t*>(P.irr_val) + ivb * sv, iv, bar, pol);
+            bulk_g2s(st + off_ic, P.irr_col + icb, ic, bar, pol);
+        }
+    }
+}
+
+// ---- consumers (all 32 lanes), FP64 ----
+template <int VAR>
+__device__ __forceinline__ void long_stage_f64(const MainParams& P, const uint8_t* st, int64_t u, int lane) {
+    // conflict-free reads: lane l takes 16-B chunks l + 32j, i.e. elements 2(l+32j), 2(l+32j)+1,
+    // both in group j of the unit
+    const double2* sv = reinterpret_cast<const double2*>(st + HDR);
+    const int2* sc = reinterpret_cast<const int2*>(st + HDR + 2048);
+    const double* x = static_cast<const double*>(P.x);
+    double v[8], xv[8];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const double2 a = sv[j * 32 + lane];
+        const int2 c = sc[j * 32 + lane];
+        v[2 * j] = a.x; v[2 * j + 1] = a.y;
+        xv[2 * j] = gx(x, static_cast<uint32_t>(c.x));
+        xv[2 * j + 1] = gx(x, static_cast<uint32_t>(c.y));
+    }
+    double gsum[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        if constexpr (VAR == VAR_MMA) {
+            double c0 = 0.0, c1 = 0.0;
+            dmma(c0, c1, v[2 * j], xv[2 * j]);
+            dmma(c0, c1, v[2 * j + 1], xv[2 * j + 1]);
+            gsum[j] = is_diag_holder(lane) ? (((lane >> 2) & 1) ? c1 : c0) : 0.0;   // trace terms
+        } else {
+            gsum[j] = fma(v[2 * j], xv[2 * j], v[2 * j + 1] * xv[2 * j + 1]);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) gsum[j] += __shfl_xor_sync(FULL, gsum[j], o);
+    if (lane < 4) static_cast<double*>(P.partial)[u * 4 + lane] = lane == 0 ? gsum[0] : lane == 1 ? gsum[1] : lane == 2 ? gsum[2] : gsum[3];
+}
+
+template <int VAR>
+__device__ __forceinline__ void short_compute_f64(const MainParams& P, int cat, const double (&v)[4], const uint32_t (&c)[4],
+                                                  int32_t o0, int32_t o1, int lane) {
+    const int g = lane >> 2, t = lane & 3;
+    const int nseg = cat == 1 ? 1 : 2;
+    const double* x = static_cast<const double*>(P.x);
+    double xv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) xv[j] = gx(x, c[j]);
+    const int myseg = seg_of(cat, t);
+    const int src = 4 * (lane & 7);
+    double r0 = 0.0, r1 = 0.0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        for (int s = 0; s < nseg; ++s) {
+            double val;
+            if constexpr (VAR == VAR_MMA) {
+                double cc0 = 0.0, cc1 = 0.0;
+                dmma(cc0, cc1, v[j], myseg == s ? xv[j] : 0.0);
+                val = __shfl_sync(FULL, (g & 1) ? cc1 : cc0, src + ((lane & 7) >> 1));
+            } else {
+                double p = myseg == s ? v[j] * xv[j] : 0.0;
+                p += __shfl_xor_sync(FULL, p, 1);
+                p += __shfl_xor_sync(FULL, p, 2);
+                val = __shfl_sync(FULL, p, src);
+            }
+            const int blk = nseg == 2 ? 2 * j + s : j;
+            if ((lane >> 3) == blk) r0 = val;
+            if ((lane >> 3) == blk - 4) r1 = val;
+        }
+    }
+    store_y<0>(P, o0, r0);
+    if (nseg == 2) store_y<0>(P, o1, r1);
+}
+
+template <int VAR>
+__device__ __forceinline__ void short_stage_f64(const MainParams& P, const uint8_t* st, int cat, int lane) {
+    const double2* sv = reinterpret_cast<const double2*>(st + HDR);
+    const uint4* sc = reinterpret_cast<const uint4*>(st + HDR + 1024);
+    const int32_t* so = reinterpret_cast<const int32_t*>(st + HDR + 1024 + 512);
+    const double2 a = sv[2 * lane], b = sv[2 * lane + 1];
+    const uint4 cc = sc[lane];
+    const double v[4] = {a.x, a.y, b.x, b.y};
+    const uint32_t c[4] = {cc.x, cc.y, cc.z, cc.w};
+    if (cat == 3) {                                       // singles (Alg. 5)
+        const int4 o = reinterpret_cast<const int4*>(so)[lane];
+        const double* x = static_cast<const double*>(P.x);
+        store_y<0>(P, o.x, v[0] * gx(x, c[0]));
+        store_y<0>(P, o.y, v[1] * gx(x, c[1]));
+        store_y<0>(P, o.z, v[2] * gx(x, c[2]));
+        store_y<0>(P, o.w, v[3] * gx(x, c[3]));
+        return;
+    }
+    short_compute_f64<VAR>(P, cat, v, c, so[lane], cat == 1 ? -1 : so[32 + lane], lane);
+}
+
+template <int VAR>
+__device__ __forceinline__ void medium_stage_f64(const MainParams& P, const uint8_t* st, int lane) {
+    const int64_t* h = reinterpret_cast<const int64_t*>(st);
+    const int g = lane >> 2, t = lane & 3;
+    const int nreg = static_cast<int>(h[2]);
+    const int64_t ivb = h[3], icb = h[4];
+    const double* siv = reinterpret_cast<const double*>(st + h[5]);
+    const int32_t* sic = reinterpret_cast<const int32_t*>(st + h[6]);
+    const int64_t* sip = reinterpret_cast<const int64_t*>(st + HDR);
+    const int32_t orow = reinterpret_cast<const int32_t*>(st + HDR + 80)[g];
+    const double* srv = reinterpret_cast<const double*>(st + HDR + 112);
+    const int32_t* src = reinterpret_cast<const int32_t*>(st + HDR + 112 + nreg * 256);
+    const double* x = static_cast<const double*>(P.x);
+    const int nfull = nreg >> 2, rem = nreg & 3;
+    double c0 = 0.0, c1 = 0.0, part = 0.0;
+    for (int ch = 0; ch < nfull; ++ch) {
+        const double2 a = reinterpret_cast<const double2*>(srv + ch * 128 + lane * 4)[0];
+        const double2 b = reinterpret_cast<const double2*>(srv + ch * 128 + lane * 4)[1];
+        const uint4 cc = reinterpret_cast<const uint4*>(src + ch * 128 + lane * 4)[0];
+        const double va[4] = {a.x, a.y, b.x, b.y};
+        const uint32_t ca[4] = {cc.x, cc.y, cc.z, cc.w};
+        double xv[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) xv[j] = gx(x, ca[j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, va[j], xv[j]);
+            else part = fma(va[j], xv[j], part);
+        }
+    }
+    const int rbase = nfull * 128 + lane * rem;
+#pragma unroll
+    for (int j = 0; j < 3; ++j) {
+        if (j < rem) {                                     // rem is warp-uniform
+            const double xv = gx(x, static_cast<uint32_t>(src[rbase + j]));
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, srv[rbase + j], xv);
+            else part = fma(srv[rbase + j], xv, part);
+        }
+    }
+    if constexpr (VAR == VAR_MMA) {
+        const double d = diag_to_quad(c0, c1, lane);
+        part = t == 0 ? d : 0.0;
+    }
+    const int64_t ie = sip[g + 1];
+    for (int64_t k = sip[g] + t; k < ie; k += 4) part = fma(siv[k - ivb], gx(x, static_cast<uint32_t>(sic[k - icb])), part);
+    part += __shfl_xor_sync(FULL, part, 1);
+    part += __shfl_xor_sync(FULL, part, 2);
+    if (t == 0) store_y<0>(P, orow, part);
+}
+
+// ---- consumers, FP16 ----
+template <int VAR>
+__device__ __forceinline__ void long_stage_f16(const MainParams& P, const uint8_t* st, int64_t u, int lane) {
+    // lane l takes halves 8l..8l+7 (group l/16) and 256+8l.. (group 2 + l/16)
+    const uint4* sv = reinterpret_cast<const uint4*>(st + HDR);
+    const uint4* sc = reinterpret_cast<const uint4*>(st + HDR + 1024);
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    float gs[2];
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+        const uint4 a = sv[lane + 32 * j];
+        const uint4 ca = sc[2 * lane + 64 * j], cb = sc[2 * lane + 64 * j + 1];
+        const uint32_t av[4] = {a.x, a.y, a.z, a.w};
+        const uint32_t cv[8] = {ca.x, ca.y, ca.z, ca.w, cb.x, cb.y, cb.z, cb.w};
+        uint16_t xh[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) xh[e] = gxh(x, cv[e]);
+        if constexpr (VAR == VAR_MMA) {
+            float c0 = 0.f, c1 = 0.f;
+#pragma unroll
+            for (int h = 0; h < 4; ++h) hmma(c0, c1, av[h], pack2(xh[2 * h], xh[2 * h + 1]));
+            gs[j] = is_diag_holder(lane) ? (((lane >> 2) & 1) ? c1 : c0) : 0.f;
+        } else {
+            float s = 0.f;
+#pragma unroll
+            for (int h = 0; h < 4; ++h) {
+                const float2 af = u2f2(av[h]);
+                s = fmaf(af.x, h2f(xh[2 * h]), s);
+                s = fmaf(af.y, h2f(xh[2 * h + 1]), s);
+            }
+            gs[j] = s;
+        }
+    }
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) {
+        gs[0] += __shfl_xor_sync(FULL, gs[0], o);
+        gs[1] += __shfl_xor_sync(FULL, gs[1], o);
+    }
+    if ((lane & 15) == 0) {
+        float* part = static_cast<float*>(P.partial) + u * 4 + (lane >> 4);
+        part[0] = gs[0];   // group lane/16
+        part[2] = gs[1];   // group 2 + lane/16
+    }
+}
+
+template <int VAR>
+__device__ __forceinline__ void short_stage_f16(const MainParams& P, const uint8_t* st, int cat, int lane) {
+    const uint2 a = reinterpret_cast<const uint2*>(st + HDR)[lane];
+    const uint4 cc = reinterpret_cast<const uint4*>(st + HDR + 256)[lane];
+    const int32_t* so = reinterpret_cast<const int32_t*>(st + HDR + 256 + 512);
+    const uint32_t c[4] = {cc.x, cc.y, cc.z, cc.w};
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    if (cat == 3) {
+        const int4 o = reinterpret_cast<const int4*>(so)[lane];
+        const float2 lo = u2f2(a.x), hi = u2f2(a.y);
+        store_y<1>(P, o.x, lo.x * h2f(gxh(x, c[0])));
+        store_y<1>(P, o.y, lo.y * h2f(gxh(x, c[1])));
+        store_y<1>(P, o.z, hi.x * h2f(gxh(x, c[2])));
+        store_y<1>(P, o.w, hi.y * h2f(gxh(x, c[3])));
+        return;
+    }
+    short_compute_f16<VAR>(P, cat, a.x, a.y, c, so[lane], cat == 1 ? -1 : so[32 + lane], lane);
+}
+
+template <int VAR>
+__device__ __forceinline__ void medium_stage_f16(const MainParams& P, const uint8_t* st, int lane) {
+    const int64_t* h = reinterpret_cast<const int64_t*>(st);
+    const int g = lane >> 2, t = lane & 3;
+    const int nreg = static_cast<int>(h[2]);
+    const int64_t ivb = h[3], icb = h[4];
+    const unsigned short* siv = reinterpret_cast<const unsigned short*>(st + h[5]);
+    const int32_t* sic = reinterpret_cast<const int32_t*>(st + h[6]);
+    const int64_t* sip = reinterpret_cast<const int64_t*>(st + HDR);
+    const int32_t orow = reinterpret_cast<const int32_t*>(st + HDR + 80)[g];
+    const uint32_t* srv = reinterpret_cast<const uint32_t*>(st + HDR + 112);      // half pairs
+    const int32_t* src = reinterpret_cast<const int32_t*>(st + HDR + 112 + nreg * 128);
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    float c0 = 0.f, c1 = 0.f, part = 0.f;
+    auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) {
+        const uint16_t xa = gxh(x, ca), xb = gxh(x, cb);
+        if constexpr (VAR == VAR_MMA) {
+            hmma(c0, c1, a, pack2(xa, xb));
+        } else {
+            const float2 av = u2f2(a);
+            part = fmaf(av.x, h2f(xa), part);
+            part = fmaf(av.y, h2f(xb), part);
+        }
+    };
+    const int nfull = nreg >> 2, rem = nreg & 3;
+    for (int ch = 0; ch < nfull; ++ch) {             // chunk: lane holds 4 half pairs + 8 columns
+        const uint4 a = reinterpret_cast<const uint4*>(srv + ch * 128 + lane * 4)[0];
+        const uint4 ca = reinterpret_cast<const uint4*>(src + ch * 256 + lane * 8)[0];
+        const uint4 cb = reinterpret_cast<const uint4*>(src + ch * 256 + lane * 8)[1];
+        block(a.x, ca.x, ca.y);
+        block(a.y, ca.z, ca.w);
+        block(a.z, cb.x, cb.y);
+        block(a.w, cb.z, cb.w);
+    }
+#pragma unroll
+    for (int j = 0; j < 3; ++j) {
+        if (j < rem) {
+            const int e = nfull * 128 + lane * rem + j;    // half-pair index
+            block(srv[e], static_cast<uint32_t>(src[2 * e]), static_cast<uint32_t>(src[2 * e + 1]));
+        }
+    }
+    if constexpr (VAR == VAR_MMA) {
+        const float d = diag_to_quad(c0, c1, lane);
+        part = t == 0 ? d : 0.f;
+    }
+    const int64_t ie = sip[g + 1];
+    for (int64_t k = sip[g] + t; k < ie; k += 4)
+        part = fmaf(h2f(siv[k - ivb]), h2f(gxh(x, static_cast<uint32_t>(sic[k - icb]))), part);
+    part += __shfl_xor_sync(FULL, part, 1);
+    part += __shfl_xor_sync(FULL, part, 2);
+    if (t == 0) store_y<1>(P, orow, part);
+}
+
+#ifndef DASP_PIPE_WARPS
+#define DASP_PIPE_WARPS 8
+#endif
+constexpr int PW = DASP_PIPE_WARPS;
+
+template <int DT, int VAR>
+__global__ void __launch_bounds__(PW * 32) dasp_pipe_kernel(const MainParams P, const uint64_t* __restrict__ items,
+                                                           int64_t n_items) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint8_t* stages = smem + warp * NSTAGE * STAGE;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + PW * NSTAGE * STAGE) + warp * NSTAGE;
+    const int64_t NW = static_cast<int64_t>(gridDim.x) * PW;
+    const int64_t w0 = static_cast<int64_t>(blockIdx.x) * PW + warp;
+    const uint64_t pol = stream_policy();
+    if (w0 >= n_items) return;
+
+    // producer state (lane 0): item words and medium pointers, one item of look-ahead
+    uint64_t wa = 0, wb = 0;
+    MedPtr ma{0, 0, 0, 0}, mb{0, 0, 0, 0};
+    auto load_ptrs = [&](uint64_t w, MedPtr& m) {
+        if (item_kind(w) == IT_MED) {
+            const int64_t rb = static_cast<int64_t>(w & ((1ull << 62) - 1));
+            m.base = __ldg(P.rb_ptr + rb); m.end = __ldg(P.rb_ptr + rb + 1);
+            m.irr0 = __ldg(P.irr_ptr + rb * 8); m.irr1 = __ldg(P.irr_ptr + rb * 8 + 8);
+        }
+    };
+    if (lane == 0) {
+        for (int s = 0; s < NSTAGE; ++s) mbar_init(&bars[s], 1);
+        fence_mbar_init();
+        fence_proxy_async();
+        for (int s = 0; s < NSTAGE; ++s) {
+            const int64_t i = w0 + s * NW;
+            if (i < n_items) {
+                uint64_t w = __ldg(items + i);
+                MedPtr m{0, 0, 0, 0};
+                load_ptrs(w, m);
+                produce<DT>(P, w, m, stages + s * STAGE, &bars[s], pol);
+            }
+        }
+        const int64_t ia = w0 + NSTAGE * NW, ib = ia + NW;
+        if (ia < n_items) { wa = __ldg(items + ia); load_ptrs(wa, ma); }
+        if (ib < n_items) wb = __ldg(items + ib);
+    }
+    __syncwarp();
+    for (int64_t k = 0;; ++k) {
+        const int64_t i = w0 + k * NW;
+        if (i >= n_items) break;
+        const int s = static_cast<int>(k % NSTAGE);
+        uint8_t* st = stages + s * STAGE;
+        mbar_wait(&bars[s], static_cast<uint32_t>((k / NSTAGE) & 1));
+        const int64_t* h = reinterpret_cast<const int64_t*>(st);
+        const int kind = static_cast<int>(h[0]);
+        if (kind == IT_LONG) {
+            if constexpr (DT == 0) long_stage_f64<VAR>(P, st, h[1], lane);
+            else long_stage_f16<VAR>(P, st, h[1], lane);
+        } else if (kind == IT_SHORT) {
+            if constexpr (DT == 0) short_stage_f64<VAR>(P, st, static_cast<int>(h[3]), lane);
+            else short_stage_f16<VAR>(P, st, static_cast<int>(h[3]), lane);
+        } else if (kind == IT_MED) {
+            if constexpr (DT == 0) medium_stage_f64<VAR>(P, st, lane);
+            else medium_stage_f16<VAR>(P, st, lane);
+        } else {                                          // row-block larger than a stage
+            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb_meta(P, h[1], lane), lane, pol);
+            else medium_rb_f16<VAR>(P, rb_meta(P, h[1], lane), lane, pol);
+        }
+        __syncwarp();
+        if (lane == 0) {
+            const int64_t inext = i + NSTAGE * NW;
+            if (inext < n_items) {
+                fence_proxy_async();                      // our generic reads of the stage precede the refill
+                produce<DT>(P, wa, ma, st, &bars[s], pol);
+                wa = wb;
+                ma = MedPtr{0, 0, 0, 0};
+                load_ptrs(wa, ma);
+                const int64_t ic = inext + 2 * NW;
+                wb = ic < n_items ? __ldg(items + ic) : 0;
+            }
+        }
+        __syncwarp();
+    }
+}
+
 }  // namespace
 
 template <typename Kern>
@@ -584,6 +1090,38 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
         else e = launch_ex(dasp_main_kernel<1, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
     }
     if (e != cudaSuccess) return e;
+    return cudaGetLastError();
+}
+
+template <int DT, int VAR>
+static cudaError_t pipe_setup(int* blocks_per_sm) {
+    const size_t smem = pipe_smem_bytes();
+    cudaError_t e = cudaFuncSetAttribute(dasp_pipe_kernel<DT, VAR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         static_cast<int>(smem));
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, dasp_pipe_kernel<DT, VAR>, PW * 32, smem);
+}
+
+size_t pipe_smem_bytes() { return static_cast<size_t>(PW) * NSTAGE * (STAGE + 8); }
+int pipe_warps_per_block() { return PW; }
+
+cudaError_t pipe_occupancy(int dtype, int variant, int* blocks_per_sm) {
+    if (dtype == 0) return variant == VAR_MMA ? pipe_setup<0, VAR_MMA>(blocks_per_sm) : pipe_setup<0, VAR_CUDACORE>(blocks_per_sm);
+    return variant == VAR_MMA ? pipe_setup<1, VAR_MMA>(blocks_per_sm) : pipe_setup<1, VAR_CUDACORE>(blocks_per_sm);
+}
+
+cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint64_t* items, int64_t n_items,
+                        int64_t blocks, cudaStream_t s) {
+    if (n_items <= 0 || blocks <= 0) return cudaSuccess;
+    const size_t smem = pipe_smem_bytes();
+    dim3 grid(static_cast<unsigned>(blocks)), block(PW * 32);
+    if (dtype == 0) {
+        if (variant == VAR_MMA) dasp_pipe_kernel<0, VAR_MMA><<<grid, block, smem, s>>>(p, items, n_items);
+        else dasp_pipe_kernel<0, VAR_CUDACORE><<<grid, block, smem, s>>>(p, items, n_items);
+    } else {
+        if (variant == VAR_MMA) dasp_pipe_kernel<1, VAR_MMA><<<grid, block, smem, s>>>(p, items, n_items);
+        else dasp_pipe_kernel<1, VAR_CUDACORE><<<grid, block, smem, s>>>(p, items, n_items);
+    }
     return cudaGetLastError();
 }
 

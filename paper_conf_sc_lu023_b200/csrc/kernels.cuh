@@ -60,6 +60,14 @@ struct FinishParams {
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s);
+
+// Persistent TMA-staged pipeline kernel (kernels.cu): items are 64-bit words
+// (kind<<62 | payload; see kernels.cu item_kind / produce).
+size_t pipe_smem_bytes();
+int pipe_warps_per_block();
+cudaError_t pipe_occupancy(int dtype, int variant, int* blocks_per_sm);   // also sets the smem attribute
+cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint64_t* items, int64_t n_items,
+                        int64_t blocks, cudaStream_t s);
 cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s);
 
 }  // namespace dasp

@@ -271,3 +271,26 @@ def test_long_unit_order_is_result_neutral(monkeypatch):
     assert np.array_equal(ys[0], ys[2]) and np.array_equal(ys[1], ys[3])
     y_ref, s = oracle_ref(A, x, "f64")
     assert oracle.tolerance_ok(ys[0], y_ref, s).all()
+
+
+# the TMA-staged persistent kernel (dasp_options_t.pipeline): same bits as the direct kernel on
+# integer inputs, every class, both dtypes and variants, several panel sizes
+@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("name,gen", CASES, ids=[c[0] for c in CASES])
+def test_pipeline_kernel_parity(name, gen, dt, variant):
+    A = gen(synth.VAL_INT)
+    x = synth.vector(41, A.n, synth.VAL_INT)
+    y0 = synth.vector(42, A.m, synth.VAL_INT)
+    for panel in [-1, 700]:
+        plan = make(A, dt, pipeline=True, panel_rows=panel)
+        assert plan.info["pipeline"] == 1
+        y = run(plan, x, dt, 2.0, -1.0, y0, variant=variant)
+        y_ref, _ = oracle_ref(A, x, dt, 2.0, -1.0, y0)
+        assert np.array_equal(y, y_ref)
+    A = gen(synth.VAL_UNIFORM)
+    x = synth.vector(43, A.n)
+    plan = make(A, dt, pipeline=True)
+    y = run(plan, x, dt, variant=variant)
+    y_ref, s = oracle_ref(A, x, dt)
+    assert oracle.tolerance_ok(y, y_ref, s, dt).all()
