@@ -47,12 +47,16 @@ def parse():
     ap.add_argument("--config", default="c2")            # configs[1]: 27-point stencil 128^3, FP64
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--dtype", default="f64", choices=["f64", "f16"])
-    ap.add_argument("--variant", default="mma", choices=["mma", "cudacore"])
+    ap.add_argument("--variant", default="cudacore", choices=["mma", "cudacore"])
+    ap.add_argument("--no-compare", action="store_true", help="skip timing the other compute variant")
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--pipeline", action="store_true", help="use the TMA-staged persistent kernel")
     ap.add_argument("--panel-rows", type=int, default=0, help="rows per panel (0 auto, -1 one global panel)")
     ap.add_argument("--no-triad", action="store_true")
+    ap.add_argument("--iterate", action="store_true", help="N=1: run the row-slab iteration (x <- alpha*A*x)")
+    ap.add_argument("--fused", action="store_true", help="slab mode: fuse the x all-gather into the SpMV "
+                    "epilogue (symmetric memory + dasp_spmv_scatter)")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=12.0)
@@ -265,7 +269,8 @@ def main():
     x_global = synth.vector(101, spec.n)
 
     t1 = time.perf_counter()
-    if world == 1:
+    use_slab = world > 1 or args.iterate
+    if not use_slab:
         # single GPU: plain SpMV over resident inputs, y overwritten every step
         plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
                                      device=local, variant=variant, medium_rb_per_warp=args.rbw,
@@ -280,7 +285,7 @@ def main():
         def step():
             dasp.dasp_spmv(plan, xd, yd, alpha, 0.0, stream, variant=variant, check=False)
     else:
-        it = SlabSpMV(slab, world, rank, dev, args.dtype, variant=variant)
+        it = SlabSpMV(slab, world, rank, dev, args.dtype, variant=variant, fused=args.fused)
         plan = it.plan
         it.set_x(x_global)
         alpha = 1.0 / max(slab.inf_norm, 1e-300)   # iterated SpMV stays bounded
@@ -317,6 +322,27 @@ def main():
     kern = dasp.dasp_plan_read_timing(plan)
     ms_step = ms_total / args.steps
 
+    # the other compute variant on the same plan and inputs (north_star: the MMA block-dot path
+    # is justified, or not, against the CUDA-core variant of the same format)
+    compare = None
+    if not use_slab and not args.no_compare:
+        other = dasp.DASP_VARIANT_CUDACORE if variant == dasp.DASP_VARIANT_MMA else dasp.DASP_VARIANT_MMA
+        vname = {dasp.DASP_VARIANT_MMA: "mma", dasp.DASP_VARIANT_CUDACORE: "cudacore"}
+        nrep = max(10, args.steps // 4)
+        for _ in range(5):
+            dasp.dasp_spmv(plan, xd, yd, 1.0, 0.0, stream, variant=other, check=False)
+        torch.cuda.synchronize(dev)
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        c0.record(stream)
+        for _ in range(nrep):
+            dasp.dasp_spmv(plan, xd, yd, 1.0, 0.0, stream, variant=other, check=False)
+        c1.record(stream)
+        torch.cuda.synchronize(dev)
+        oms = c0.elapsed_time(c1) / nrep
+        compare = {vname[variant]: {"GFLOPS": 2.0 * float(lens.sum()) / (ms_step * 1e-3) / 1e9, "ms_per_step": ms_step},
+                   vname[other]: {"GFLOPS": 2.0 * float(lens.sum()) / (oms * 1e-3) / 1e9, "ms_per_step": oms,
+                                  "steps": nrep}}
+
     nnz_total = int(lens.sum())
     flops_step = 2.0 * nnz_total
     gflops = flops_step / (ms_step * 1e-3) / 1e9
@@ -346,7 +372,34 @@ def main():
 
     # ---- e2e: the same metric through the C-ABI with HOST buffers (copies inside the timed region) ----
     e2e = None
-    if world == 1 and args.e2e_steps > 0:
+    if use_slab and args.e2e_steps > 0:
+        # per step: this rank's x slab host->device, assemble x (all-gather), SpMV, y slab device->host
+        S0 = slab.S
+        xh = torch.from_numpy(x_global[slab.row0:slab.row0 + slab.rows].copy()).pin_memory()
+        yh = torch.empty(slab.rows, dtype=torch.float64).pin_memory()
+        times = []
+        for k in range(args.e2e_steps + 1):
+            torch.cuda.synchronize(dev)
+            if world > 1:
+                dist.barrier()
+            t0 = time.perf_counter()
+            it.x[it.cur][rank * S0: rank * S0 + slab.rows].copy_(xh, non_blocking=True)
+            if world > 1 and not args.fused:
+                dist.all_gather_into_tensor(it.x[it.cur], it.x[it.cur][rank * S0:(rank + 1) * S0])
+            it.step(alpha)
+            yh.copy_(it.x[it.cur][rank * S0: rank * S0 + slab.rows], non_blocking=True)
+            torch.cuda.synchronize(dev)
+            if k:
+                times.append(time.perf_counter() - t0)
+        dt = max(times) if times else float("nan")
+        if world > 1:
+            t = torch.tensor([dt], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+        e2e = {"value": flops_step / dt / 1e9, "unit": "GFLOPS", "ms_per_step": dt * 1e3,
+               "h2d_bytes_per_step": int(xh.numel() * 8) * world, "d2h_bytes_per_step": int(yh.numel() * 8) * world,
+               "api": "dasp_spmv" + ("_scatter" if args.fused else "") + " (row-slab iteration)"}
+    if not use_slab and args.e2e_steps > 0:
         xdt_np = np.float64 if args.dtype == "f64" else np.float16
         xh = torch.from_numpy(x_global.astype(xdt_np)).pin_memory()
         yh = torch.empty(slab.rows, dtype=torch.float64 if args.dtype == "f64" else torch.float32).pin_memory()
@@ -381,13 +434,16 @@ def main():
             "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config),
                        "m": int(spec.m), "n": int(spec.n), "nnz": nnz_total, "variant": args.variant,
                        "kernel": "pipeline" if info.get("pipeline") else "direct", "panel_rows": info["panel_rows"],
-                       "parallelism": f"row-slab x{world}" + (" + NCCL all-gather of x" if world > 1 else ""),
+                       "parallelism": f"row-slab x{world}" + (
+                           (" + fused NVLink scatter of y into every rank's x" if args.fused else " + NCCL all-gather of x")
+                           if use_slab else ""),
                        "l2": "inputs larger than L2 (packed A streamed every step); x stays L2-resident "
                              "across steps as in the paper's averaged back-to-back runs"},
             "effective_gbs": eff_gbs, "effective_frac_of_peak": eff_gbs / peak,
             "alg_gbs_step": bm["total"] * world / (ms_step * 1e-3) / 1e9 if world == 1 else None,
             "gpu_launches": int(info["launches_per_spmv"]) * args.steps,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "variant_compare": compare,
             "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,
                      "rows": {"empty": info["n_empty"], "short": info["n_len1"] + info["n_len2"] + info["n_len3"]
                               + info["n_len4"], "medium": info["row_medium"], "long": info["row_long"]},

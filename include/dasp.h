@@ -59,7 +59,8 @@ typedef enum {
 
 typedef struct {
     int32_t device;             /* CUDA device ordinal; -1 = host-only plan (builder only)   */
-    int32_t variant;            /* default variant of dasp_spmv (DASP_VARIANT_MMA if 0)       */
+    int32_t variant;            /* default variant of dasp_spmv (0: DASP_VARIANT_CUDACORE, the
+                                   faster one on B200 in our measurements)      */
     int32_t validate;           /* 1: O(nnz) CSR validation (default); 0: skip               */
     int32_t keep_host;          /* 1: keep the host staging copy of the packed arrays        */
     int32_t medium_rb_per_warp; /* row-blocks per warp in the medium kernel (P:L271-273
@@ -75,8 +76,8 @@ typedef struct {
                                    registers (faster on B200 in our measurements) */
 } dasp_options_t;
 
-/* Fills `opts` with the defaults: device 0, MMA variant, validate, no keep_host, auto LOOP_NUM,
- * automatic panel size. */
+/* Fills `opts` with the defaults: device 0, CUDA-core variant, validate, no keep_host, auto
+ * LOOP_NUM, automatic panel size, direct (non-pipelined) kernel. */
 void dasp_options_default(dasp_options_t* opts);
 
 /* Plan statistics (Fig. 12's class shares; build cost). */
@@ -140,6 +141,20 @@ dasp_status_t dasp_spmv(dasp_plan_t plan, const void* x, void* y, double alpha, 
 /* As dasp_spmv with an explicit compute variant (dasp_variant_t). */
 dasp_status_t dasp_spmv_ex(dasp_plan_t plan, const void* x, void* y, double alpha, double beta,
                            void* stream, int32_t variant);
+
+/*
+ * dasp_spmv_scatter — dasp_spmv whose result is written to several buffers at once, the fused
+ * SpMV + all-gather of the row-slab multi-GPU mode:
+ *   y_dst[0]          this GPU's y (read if beta != 0), m elements;
+ *   y_dst[1..ndst-1]  further device-visible destinations that receive the same m values at the
+ *                     same offsets -- normally the peer GPUs' x buffers mapped into this process
+ *                     over NVLink (CUDA IPC / symmetric memory), so every rank's slab lands in every
+ *                     rank's next x directly from the epilogue, tile by tile, with no collective.
+ * 1 <= ndst <= 8.  The caller orders the peers' next reads after this call (e.g. a device-side
+ * barrier across ranks).  Returns INVALID_ARG for ndst out of range or a null destination.
+ */
+dasp_status_t dasp_spmv_scatter(dasp_plan_t plan, const void* x, void* const* y_dst, int32_t ndst,
+                                double alpha, double beta, void* stream);
 
 /*
  * dasp_spmv_host — end-to-end call with HOST buffers: copies x (and y if beta != 0) to

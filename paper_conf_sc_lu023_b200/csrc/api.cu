@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -21,7 +22,7 @@ struct TimingRec {
 };
 
 struct dasp_plan_s {
-    int dtype = 0, device = -1, variant = DASP_VARIANT_MMA, rbw = 1;
+    int dtype = 0, device = -1, variant = DASP_VARIANT_CUDACORE, rbw = 1;
     bool keep_host = false;
     HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
     void* d[DASP_ARR_COUNT] = {};
@@ -52,17 +53,23 @@ namespace {
 int sx(int dtype) { return dtype == DASP_R_64F ? 8 : 2; }
 int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
 
-// LOOP_NUM of P:L271-273 (R11): row-blocks per warp from the number of medium rows
 // automatic panel: ~1M rows keeps a panel's x window and y (8 B each per row) well inside the
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
 constexpr int64_t kAllocPad = 64;   // TMA windows may read up to 16 B past an array's end
 
-int auto_rbw(int64_t row_medium) {
+// LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
+// small matrices keep the paper's 1 / 2; for large ones, uniform medium rows (coefficient of
+// variation of the length < 0.5, e.g. stencils) run best with 8 row-blocks per warp, ragged
+// ones (power-law) with 4 -- more would leave warps with very unequal work.
+int auto_rbw(int64_t row_medium, int64_t nnz_medium, int64_t sumsq_medium) {
     if (row_medium < 59990) return 1;
     if (row_medium < 400000) return 2;
-    return 4;
+    const double mean = static_cast<double>(nnz_medium) / static_cast<double>(row_medium);
+    const double var = static_cast<double>(sumsq_medium) / static_cast<double>(row_medium) - mean * mean;
+    const double cv = var > 0 ? std::sqrt(var) / mean : 0.0;
+    return cv < 0.5 ? 8 : 4;
 }
 
 struct DeviceGuard {
@@ -141,7 +148,7 @@ const char* dasp_version(void) { return "dasp-b200 0.1 (sm_100a)"; }
 void dasp_options_default(dasp_options_t* o) {
     if (!o) return;
     o->device = 0;
-    o->variant = DASP_VARIANT_MMA;
+    o->variant = DASP_VARIANT_CUDACORE;   // measured >= the MMA variant on B200
     o->validate = 1;
     o->keep_host = 0;
     o->medium_rb_per_warp = 0;
@@ -173,7 +180,7 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     dasp_options_t o;
     dasp_options_default(&o);
     if (opts) o = *opts;
-    if (o.variant != DASP_VARIANT_MMA && o.variant != DASP_VARIANT_CUDACORE) o.variant = DASP_VARIANT_MMA;
+    if (o.variant != DASP_VARIANT_MMA && o.variant != DASP_VARIANT_CUDACORE) o.variant = DASP_VARIANT_CUDACORE;
     if (o.validate && row_ptr[m] != nnz) return DASP_ERR_INVALID_CSR;
 
     dasp_plan_s* p = new (std::nothrow) dasp_plan_s;
@@ -195,7 +202,7 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         return static_cast<dasp_status_t>(st);
     }
     HostFormat& f = p->host;
-    p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium);
+    p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
     // per-panel launch descriptors: warps = long units + medium warps + tiles
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<int32_t> blk_panel;
@@ -352,7 +359,29 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     return DASP_OK;
 }
 
+static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp::ExtraDst& extra, double alpha,
+                               double beta, void* stream, int32_t variant);
+
 dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, double beta, void* stream, int32_t variant) {
+    dasp::ExtraDst none{};
+    none.n = 0;
+    return spmv_impl(p, x, y, none, alpha, beta, stream, variant);
+}
+
+dasp_status_t dasp_spmv_scatter(dasp_plan_t p, const void* x, void* const* y_dst, int32_t ndst, double alpha,
+                                double beta, void* stream) {
+    if (!p || !y_dst || ndst < 1 || ndst > dasp::MAX_EXTRA_DST + 1) return DASP_ERR_INVALID_ARG;
+    dasp::ExtraDst ex{};
+    ex.n = ndst - 1;
+    for (int d = 1; d < ndst; ++d) {
+        if (!y_dst[d] || y_dst[d] == x) return DASP_ERR_INVALID_ARG;
+        ex.ptr[d - 1] = y_dst[d];
+    }
+    return spmv_impl(p, x, y_dst[0], ex, alpha, beta, stream, DASP_VARIANT_DEFAULT);
+}
+
+static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp::ExtraDst& extra, double alpha,
+                               double beta, void* stream, int32_t variant) {
     if (!p) return DASP_ERR_INVALID_ARG;
     if (p->device < 0) return DASP_ERR_UNSUPPORTED;
     const HostFormat& f = p->host;
@@ -367,8 +396,8 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
     if (on) ++p->timing_calls;
     cudaError_t e;
     if (alpha == 0.0) {  // quick path: y = beta*y
-        if (beta == 1.0) return DASP_OK;
-        e = timed(p, DASP_K_SCALE, s, on, [&] { return dasp::launch_scale(y, f.m, beta, p->dtype, s); });
+        if (beta == 1.0 && extra.n == 0) return DASP_OK;
+        e = timed(p, DASP_K_SCALE, s, on, [&] { return dasp::launch_scale(y, f.m, beta, p->dtype, s, extra); });
         return e == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
     }
     if (!x && f.n > 0) return DASP_ERR_INVALID_ARG;
@@ -395,6 +424,7 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
     mp.unit_order = static_cast<const int32_t*>(p->d_unit_order);
     mp.rbw = p->rbw;
     mp.class_mask = 7;
+    mp.extra = extra;
     // DASP_PROFILE_CLASS (profiling only; the other classes' rows are then NOT computed):
     // 1 = long units, 2 = medium warps, 3 = short tiles
     if (const char* pc = std::getenv("DASP_PROFILE_CLASS")) {
@@ -408,7 +438,7 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
         return dasp::launch_main(mp, p->dtype, variant, p->blocks, s, x, p->apw_bytes, p->apw_hit);
     });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
-    const int64_t n0 = beta == 1.0 ? 0 : f.n0;
+    const int64_t n0 = (beta == 1.0 && extra.n == 0) ? 0 : f.n0;   // scatter mode must still copy them
     if (f.row_long + n0 > 0) {
         dasp::FinishParams fp;
         fp.partial = p->d_partial;
@@ -420,6 +450,7 @@ dasp_status_t dasp_spmv_ex(dasp_plan_t p, const void* x, void* y, double alpha, 
         fp.beta = beta;
         fp.row_long = f.row_long;
         fp.n0 = n0;
+        fp.extra = extra;
         e = timed(p, DASP_K_FINISH, s, on, [&] { return dasp::launch_finish(fp, p->dtype, s); });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }

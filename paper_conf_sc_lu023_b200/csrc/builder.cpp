@@ -70,7 +70,7 @@ struct Panel {
     std::vector<int64_t> rows[C_NUM];   // class lists, ascending original order (global row ids)
     std::vector<int64_t> sorted;        // medium rows, stable by length desc, padded to 8 with -1
     std::vector<int64_t> nreg;          // regular blocks per row-block
-    int64_t nrb = 0, n_groups = 0, nnz_long = 0, nnz_med = 0, reg = 0, irr = 0;
+    int64_t nrb = 0, n_groups = 0, nnz_long = 0, nnz_med = 0, sq_med = 0, reg = 0, irr = 0;
     int64_t p13 = 0, p22 = 0, n3l = 0, n2l = 0, n4cat = 0, ns = 0, t13 = 0, t4 = 0, t22 = 0, ts = 0;
     // offsets into the concatenated arrays (set between the passes)
     int64_t o_long_row = 0, o_group = 0, o_rb = 0, o_reg = 0, o_irr = 0, o_tile = 0, o_out = 0, o_empty = 0;
@@ -129,14 +129,15 @@ void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
         for (int64_t r : MR) P.sorted[h[MAX_LEN - (rp[r + 1] - rp[r])]++] = r;
     }
     P.nreg.assign(static_cast<size_t>(P.nrb), 0);
-    int64_t reg = 0, irr = 0, nnz_med = 0;
-#pragma omp parallel for schedule(static) reduction(+ : reg, irr, nnz_med) if (par)
+    int64_t reg = 0, irr = 0, nnz_med = 0, sq_med = 0;
+#pragma omp parallel for schedule(static) reduction(+ : reg, irr, nnz_med, sq_med) if (par)
     for (int64_t rb = 0; rb < P.nrb; ++rb) {
         int64_t L[MMA_M];
         for (int g = 0; g < MMA_M; ++g) {
             const int64_t r = P.sorted[rb * MMA_M + g];
             L[g] = r < 0 ? 0 : rp[r + 1] - rp[r];
             nnz_med += L[g];
+            sq_med += L[g] * L[g];
         }
         // regular iff the 8 x K block holds more than tau * 8K real slots (tau = 0.75, strict R4);
         // the regular blocks form a prefix (R6)
@@ -150,7 +151,7 @@ void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
         reg += b * geo.BE;
         for (int g = 0; g < MMA_M; ++g) irr += std::max<int64_t>(0, L[g] - geo.K * b);
     }
-    P.reg = reg; P.irr = irr; P.nnz_med = nnz_med;
+    P.reg = reg; P.irr = irr; P.nnz_med = nnz_med; P.sq_med = sq_med;
     // a4: short piecing counts (R13)
     const int64_t n1 = P.rows[C_S1].size(), n2 = P.rows[C_S2].size(), n3 = P.rows[C_S3].size(), n4 = P.rows[C_S4].size();
     P.p13 = std::min(n1, n3); P.p22 = n2 / 2; P.n3l = n3 - P.p13; P.n2l = n2 % 2;
@@ -316,7 +317,7 @@ int build_impl(HostFormat& f, int64_t m, const int64_t* rp, const int32_t* col, 
         f.n3 += P.rows[C_S3].size(); f.n4 += P.rows[C_S4].size();
         f.row_medium += P.rows[C_MED].size();
         f.t13 += P.t13; f.t4 += P.t4; f.t22 += P.t22; f.ts += P.ts;
-        f.nnz_long += P.nnz_long; f.nnz_medium += P.nnz_med;
+        f.nnz_long += P.nnz_long; f.nnz_medium += P.nnz_med; f.sumsq_medium += P.sq_med;
     }
     f.n0 = emp;
     f.row_long = lr;

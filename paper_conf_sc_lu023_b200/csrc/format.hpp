@@ -44,6 +44,7 @@ struct HostFormat {
     int64_t nrb = 0, n_groups = 0, n_groups_padded = 0, t13 = 0, t4 = 0, t22 = 0, ts = 0;
     int64_t nnz_long_new = 0, nnz_reg_new = 0, nnz_irreg = 0, nnz_short_new = 0;
     int64_t nnz_long = 0, nnz_medium = 0, nnz_short = 0;
+    int64_t sumsq_medium = 0;  // sum of squared medium row lengths (launch tuning)
     int64_t panel_rows = 0;   // rows per panel (R28); >= m: one panel = the paper's global format
     int64_t n_panels = 0;
     HostBuf arr[DASP_ARR_COUNT];

@@ -125,6 +125,7 @@ __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typena
     Y r = static_cast<Y>(P.alpha) * acc;
     if (P.beta != 0.0) r += static_cast<Y>(P.beta) * y[row];
     y[row] = r;
+    for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;   // peers (scatter)
 }
 
 // ------------------------------------------------------------------------------------------
@@ -228,9 +229,8 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
 // medium rows (Alg. 3): row-block = 8 rows; regular 8 x K blocks in lane-interleaved chunks
 // of CW blocks (R18), then the irregular tails with 4 lanes per row, then y.
 // ------------------------------------------------------------------------------------------
-// A row-block's metadata: its regular range, this lane's row's irregular range and output row.
-// The warp loads the NEXT row-block's metadata before working on the current one, so every
-// row-block after the first costs one memory round trip (stream loads) plus the gathers.
+// A row-block's metadata: its regular range, this lane's row's irregular range and output row
+// (all five loads issued together, ahead of the stream loads that depend on them).
 struct RbMeta {
     int64_t base, ib;         // regular region start; this lane's row's irregular start
     int32_t nelem, ilen;      // regular elements (<= 64 blocks); irregular length (<= 256)
@@ -526,12 +526,11 @@ __global__ void __launch_bounds__(MAIN_THREADS, DASP_MIN_BLOCKS) dasp_main_kerne
         const int64_t rbp0 = __ldg(&D->rb0);
         const int64_t rb0 = rbp0 + w * P.rbw;
         const int64_t rb1 = min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb));
-        RbMeta cur = rb_meta(P, rb0, lane);
         for (int64_t rb = rb0; rb < rb1; ++rb) {
-            const RbMeta nxt = rb + 1 < rb1 ? rb_meta(P, rb + 1, lane) : cur;   // prefetch
-            if constexpr (DT == 0) medium_rb_f64<VAR>(P, cur, lane, pol);
-            else medium_rb_f16<VAR>(P, cur, lane, pol);
-            cur = nxt;
+            // (prefetching the next row-block's metadata here was measured: it costs registers
+            // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta.jsonl)
+            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb_meta(P, rb, lane), lane, pol);
+            else medium_rb_f16<VAR>(P, rb_meta(P, rb, lane), lane, pol);
         }
         return;
     }
@@ -574,23 +573,29 @@ __global__ void __launch_bounds__(256) dasp_finish_kernel(const FinishParams P) 
             Y r = static_cast<Y>(P.alpha) * s;
             if (P.beta != 0.0) r += static_cast<Y>(P.beta) * y[row];
             y[row] = r;
+            for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;
         }
         return;
     }
     const int64_t e = (w - P.row_long) * 32 + lane;
     if (e < P.n0) {
         const int32_t row = P.empty_rows[e];
-        y[row] = P.beta != 0.0 ? static_cast<Y>(P.beta) * y[row] : Y(0);
+        const Y r = P.beta != 0.0 ? static_cast<Y>(P.beta) * y[row] : Y(0);
+        y[row] = r;
+        for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;
     }
 }
 
 template <int DT>
-__global__ void dasp_scale_kernel(void* yv, int64_t m, double beta) {
+__global__ void dasp_scale_kernel(void* yv, int64_t m, double beta, const ExtraDst extra) {
     using Y = typename Tr<DT>::Y;
     Y* y = static_cast<Y*>(yv);
     for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < m;
-         i += static_cast<int64_t>(gridDim.x) * blockDim.x)
-        y[i] = beta != 0.0 ? static_cast<Y>(beta) * y[i] : Y(0);
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const Y r = beta != 0.0 ? static_cast<Y>(beta) * y[i] : Y(0);
+        y[i] = r;
+        for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[i] = r;
+    }
 }
 
 // ==========================================================================================
@@ -1134,12 +1139,12 @@ cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s) {
+cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s, const ExtraDst& extra) {
     if (m == 0) return cudaSuccess;
     int64_t blocks = (m + 255) / 256;
     if (blocks > 148 * 16) blocks = 148 * 16;
-    if (dtype == 0) dasp_scale_kernel<0><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta);
-    else dasp_scale_kernel<1><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta);
+    if (dtype == 0) dasp_scale_kernel<0><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
+    else dasp_scale_kernel<1><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
     return cudaGetLastError();
 }
 

@@ -7,6 +7,15 @@
 namespace dasp {
 
 constexpr int MAIN_THREADS = 256;
+constexpr int MAX_EXTRA_DST = 7;   // dasp_spmv_scatter: up to 8 destinations (this GPU + 7 peers)
+
+// Extra destinations of y (dasp_spmv_scatter): every value stored into y is also stored at the
+// same row offset of each extra[d] -- typically a peer GPU's x buffer mapped over NVLink, so
+// iterated SpMV needs no separate all-gather.
+struct ExtraDst {
+    void* ptr[MAX_EXTRA_DST];
+    int32_t n;
+};
 constexpr int WARPS_PER_BLOCK = MAIN_THREADS / 32;
 
 // One row panel (R28) as the fused kernel sees it.  A panel owns the blocks
@@ -43,6 +52,7 @@ struct MainParams {
     double alpha, beta;
     int32_t rbw;
     int32_t class_mask;       // bit 0 long, bit 1 medium, bit 2 short (profiling; 7 = all)
+    ExtraDst extra;
 };
 
 struct FinishParams {
@@ -53,6 +63,7 @@ struct FinishParams {
     void* y;
     double alpha, beta;
     int64_t row_long, n0;
+    ExtraDst extra;
 };
 
 // variant: 1 = MMA (DMMA/HMMA diagonal trick), 2 = CUDA-core.  dtype: 0 = FP64, 1 = FP16.
@@ -68,6 +79,6 @@ int pipe_warps_per_block();
 cudaError_t pipe_occupancy(int dtype, int variant, int* blocks_per_sm);   // also sets the smem attribute
 cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint64_t* items, int64_t n_items,
                         int64_t blocks, cudaStream_t s);
-cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s);
+cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s, const ExtraDst& extra);
 
 }  // namespace dasp

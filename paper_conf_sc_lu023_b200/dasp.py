@@ -26,7 +26,7 @@ STATUS = ["DASP_OK", "DASP_ERR_INVALID_ARG", "DASP_ERR_INVALID_CSR", "DASP_ERR_O
           "DASP_ERR_CUDA", "DASP_ERR_UNSUPPORTED", "DASP_ERR_INTERNAL"]
 
 # every symbol include/dasp.h declares (tests check the library exports all of them)
-EXPORTS = ["dasp_options_default", "dasp_plan_create", "dasp_spmv", "dasp_spmv_ex", "dasp_spmv_host",
+EXPORTS = ["dasp_options_default", "dasp_plan_create", "dasp_spmv", "dasp_spmv_ex", "dasp_spmv_scatter", "dasp_spmv_host",
            "dasp_plan_destroy", "dasp_status_string", "dasp_plan_get_info", "dasp_plan_copy_array",
            "dasp_partition_rows", "dasp_remap_columns", "dasp_plan_set_timing", "dasp_plan_read_timing",
            "dasp_version"]
@@ -74,6 +74,7 @@ def _load():
         "dasp_spmv": ([vp, vp, vp, d, d, vp], ctypes.c_int),
         "dasp_spmv_ex": ([vp, vp, vp, d, d, vp, i32], ctypes.c_int),
         "dasp_spmv_host": ([vp, vp, vp, d, d, vp], ctypes.c_int),
+        "dasp_spmv_scatter": ([vp, vp, ctypes.POINTER(vp), i32, d, d, vp], ctypes.c_int),
         "dasp_plan_destroy": ([vp], ctypes.c_int),
         "dasp_status_string": ([ctypes.c_int], ctypes.c_char_p),
         "dasp_plan_get_info": ([vp, ctypes.POINTER(PlanInfo)], ctypes.c_int),
@@ -150,7 +151,7 @@ class Plan:
 
 
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
-                     variant: int = DASP_VARIANT_MMA, validate: bool = True, keep_host: bool = False,
+                     variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, keep_host: bool = False,
                      medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0,
                      pipeline: bool = False) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
@@ -205,6 +206,14 @@ def dasp_spmv(plan: Plan, x, y, alpha: float = 1.0, beta: float = 0.0, stream=No
         _check_vec(y, plan.m, yd, "y", dev)
     st = _lib.dasp_spmv_ex(plan.handle, _ptr(x), _ptr(y), float(alpha), float(beta), _stream_ptr(stream), variant)
     _check(st, "dasp_spmv")
+
+
+def dasp_spmv_scatter(plan: Plan, x, dsts, alpha: float = 1.0, beta: float = 0.0, stream=None):
+    """y = alpha*A*x + beta*y written to every pointer of `dsts` (dsts[0] is this GPU's y; the rest
+    are raw device pointers or tensors, e.g. peer x buffers mapped over NVLink)."""
+    ptrs = (ctypes.c_void_p * len(dsts))(*[_ptr(d) for d in dsts])
+    st = _lib.dasp_spmv_scatter(plan.handle, _ptr(x), ptrs, len(dsts), float(alpha), float(beta), _stream_ptr(stream))
+    _check(st, "dasp_spmv_scatter")
 
 
 def dasp_spmv_host(plan: Plan, x: np.ndarray, y: np.ndarray, alpha: float = 1.0, beta: float = 0.0, stream=None):

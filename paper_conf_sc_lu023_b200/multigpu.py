@@ -14,6 +14,12 @@ torch.distributed is the plumbing (process group, NCCL all-gather); the SpMV is 
 
 The local SpMV is pluggable (``local_spmv``) so the partition / remap / all-gather logic
 is testable on CPU with the gloo backend (tests/test_multigpu.py).
+
+``fused=True`` replaces the all-gather by the SpMV epilogue itself: both x buffers live in
+torch symmetric memory (every rank maps every peer's buffers over NVLink), and
+``dasp_spmv_scatter`` stores each y value of this rank's slab into ALL ranks' next x buffer
+(P posted NVLink stores per row, overlapped with the rest of the SpMV), followed by one
+device-side barrier across ranks.  No NCCL call is left on the data path.
 """
 from __future__ import annotations
 
@@ -64,6 +70,14 @@ def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, re
     return Slab(A.row_ptr, col, A.val, r0, r1 - r0, starts, S, inf_norm)
 
 
+def scatter_destinations(peer_base, rank, world, buf_index, n_pad, S, elem_bytes):
+    """Device addresses that receive this rank's y slab: its own next-x slab first (the one
+    dasp_spmv_scatter treats as y), then the same slab in every peer's next x.  peer_base[q] is
+    rank q's symmetric buffer [x0 | x1] as mapped into this process."""
+    off = (buf_index * n_pad + rank * S) * elem_bytes
+    return [peer_base[rank] + off] + [peer_base[q] + off for q in range(world) if q != rank]
+
+
 class SlabSpMV:
     """Iterated SpMV over P ranks: x_{k+1} = alpha * A x_k, x all-gathered every step.
 
@@ -71,14 +85,25 @@ class SlabSpMV:
     alpha)`` computes the slab rows; the default calls libdasp on this rank's GPU."""
 
     def __init__(self, slab: Slab, world: int, rank: int, device, dtype="f64", group=None, local_spmv=None,
-                 variant=dasp.DASP_VARIANT_DEFAULT):
+                 variant=dasp.DASP_VARIANT_DEFAULT, fused=False):
         import torch
         self.slab, self.world, self.rank, self.group = slab, world, rank, group
         self.device = torch.device(device)
         self.dtype = dtype
+        self.fused = fused
         tdt = torch.float64
         n_pad = world * slab.S
-        self.x = [torch.zeros(n_pad, dtype=tdt, device=self.device) for _ in range(2)]
+        self.n_pad = n_pad
+        if fused:
+            import torch.distributed as dist
+            import torch.distributed._symmetric_memory as symm_mem
+            buf = symm_mem.empty(2 * n_pad, dtype=tdt, device=self.device)
+            buf.zero_()
+            self.hdl = symm_mem.rendezvous(buf, group if group is not None else dist.group.WORLD)
+            self.peer_base = [int(b) for b in self.hdl.buffer_ptrs]
+            self.x = [buf[:n_pad], buf[n_pad:]]
+        else:
+            self.x = [torch.zeros(n_pad, dtype=tdt, device=self.device) for _ in range(2)]
         self.cur = 0
         if local_spmv is None:
             if self.device.type != "cuda":
@@ -123,8 +148,19 @@ class SlabSpMV:
         self.cur = 1 - self.cur
 
     def step(self, alpha=1.0):
+        if self.fused:
+            return self.fused_step(alpha)
         self.spmv(alpha)
         self.exchange()
+
+    def fused_step(self, alpha=1.0):
+        """One iteration with the all-gather fused into the SpMV epilogue (see module doc)."""
+        import torch
+        nb = 1 - self.cur
+        dsts = scatter_destinations(self.peer_base, self.rank, self.world, nb, self.n_pad, self.slab.S, 8)
+        dasp.dasp_spmv_scatter(self.plan, self.x[self.cur], dsts, alpha, 0.0, torch.cuda.current_stream(self.device))
+        self.hdl.barrier(channel=0)          # every rank's stores have landed before x is read
+        self.cur = nb
 
     def x_global(self) -> np.ndarray:
         st, S = self.slab.starts, self.slab.S

@@ -294,3 +294,26 @@ def test_pipeline_kernel_parity(name, gen, dt, variant):
     y = run(plan, x, dt, variant=variant)
     y_ref, s = oracle_ref(A, x, dt)
     assert oracle.tolerance_ok(y, y_ref, s, dt).all()
+
+
+# dasp_spmv_scatter: the fused SpMV + all-gather epilogue writes the same values to every
+# destination (here several local buffers stand in for the peers' x buffers)
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("pipeline", [False, True])
+def test_scatter_epilogue_writes_every_destination(dt, pipeline):
+    A = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
+    x = synth.vector(51, A.n, synth.VAL_INT)
+    y0 = synth.vector(52, A.m, synth.VAL_INT)
+    plan = make(A, dt, pipeline=pipeline)
+    xd = torch.from_numpy(x.astype(np.float64 if dt == "f64" else np.float16)).cuda()
+    ydt = torch.float64 if dt == "f64" else torch.float32
+    for alpha, beta in [(1.0, 0.0), (2.0, -1.0), (1.0, 1.0), (0.0, 3.0)]:
+        dst = [torch.from_numpy(y0).to(ydt).cuda()] + [torch.full((A.m,), float("nan"), dtype=ydt, device="cuda")
+                                                        for _ in range(3)]
+        dasp.dasp_spmv_scatter(plan, xd, dst, alpha, beta)
+        torch.cuda.synchronize()
+        y_ref, _ = oracle_ref(A, x, dt, alpha, beta, y0)
+        for d in dst:
+            assert np.array_equal(d.cpu().numpy().astype(np.float64), y_ref), (alpha, beta)
+    with pytest.raises(dasp.DaspError):
+        dasp.dasp_spmv_scatter(plan, xd, [dst[0]] * 9)

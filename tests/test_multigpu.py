@@ -80,3 +80,12 @@ def test_slab_bounds_cover_and_balance():
         per = np.add.reduceat(lens, s[:-1]) if len(lens) else []
         assert s[0] == 0 and s[-1] == len(lens)
         assert max(per) <= lens.sum() / P + lens.max()   # balanced up to one row
+
+
+def test_scatter_destinations_layout():
+    from paper_conf_sc_lu023_b200.multigpu import scatter_destinations
+    bases = [1000, 5000, 9000, 13000]
+    d = scatter_destinations(bases, rank=2, world=4, buf_index=1, n_pad=40, S=10, elem_bytes=8)
+    off = (40 + 2 * 10) * 8
+    assert d == [9000 + off, 1000 + off, 5000 + off, 13000 + off]
+    assert scatter_destinations([7], 0, 1, 0, 5, 5, 8) == [7]
