@@ -74,6 +74,11 @@ typedef struct {
                                    packed arrays in shared memory with cp.async.bulk (TMA) and
                                    mbarriers; 0 (default): one warp per item, loads straight to
                                    registers (faster on B200 in our measurements) */
+    int32_t max_len;            /* MAX_LEN, "an adjustable parameter": long iff len >
+                                   max_len; 0 = 256; must be >= 4                             */
+    double threshold;           /* tau, "a customized parameter": an 8 x MMA_K block is
+                                   regular iff it holds more than 8*MMA_K*tau nonzeros;
+                                   0 = 0.75; must be <= 1                                     */
 } dasp_options_t;
 
 /* Fills `opts` with the defaults: device 0, CUDA-core variant, validate, no keep_host, auto
@@ -99,6 +104,8 @@ typedef struct {
     int32_t launches_per_spmv;                         /* kernels one dasp_spmv enqueues    */
     int64_t panel_rows, n_panels;                      /* resolved panel size and count     */
     int32_t pipeline;                                  /* 1 if the TMA-staged kernel is used */
+    int64_t max_len;                                   /* resolved MAX_LEN                   */
+    double threshold;                                  /* resolved tau                       */
     double build_ms, upload_ms;                        /* host build; host->device upload   */
 } dasp_plan_info_t;
 

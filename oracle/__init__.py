@@ -50,7 +50,7 @@ def _L():
         lib = ctypes.CDLL(_SO)
         vp, i64, d = ctypes.c_void_p, ctypes.c_int64, ctypes.c_double
         lib.oracle_spmv.argtypes = [i64, vp, vp, vp, vp, d, d, vp, vp, vp]
-        lib.oracle_build.argtypes = [ctypes.c_int, i64, i64, vp, vp, vp, i64]
+        lib.oracle_build.argtypes = [ctypes.c_int, i64, i64, vp, vp, vp, i64, i64, d]
         lib.oracle_build.restype = vp
         lib.oracle_free.argtypes = [vp]
         lib.oracle_fmt_count.argtypes = [vp, ctypes.c_char_p]
@@ -105,13 +105,13 @@ def tolerance_ok(y, y_ref, s, dtype="f64"):
 class Format:
     """The oracle builder's arrays (numpy copies) and counts."""
 
-    def __init__(self, A, dtype="f64", panel_rows=0):
+    def __init__(self, A, dtype="f64", panel_rows=0, max_len=256, tau=0.75):
         lib = _L()
         dt = 0 if dtype == "f64" else 1
         val = np.ascontiguousarray(A.val.astype(np.float64 if dt == 0 else np.float16))
         rp = np.ascontiguousarray(A.row_ptr, dtype=np.int64)
         col = np.ascontiguousarray(A.col, dtype=np.int32)
-        h = lib.oracle_build(dt, A.m, A.n, _p(rp), _p(col), _p(val), int(panel_rows))
+        h = lib.oracle_build(dt, A.m, A.n, _p(rp), _p(col), _p(val), int(panel_rows), int(max_len), float(tau))
         try:
             self.counts = {c: int(lib.oracle_fmt_count(h, c.encode())) for c in COUNTS}
             self.arrays = {}
@@ -133,6 +133,7 @@ class Format:
         return b.view(np.int32)
 
 
-def build(A, dtype="f64", panel_rows=0) -> Format:
-    """panel_rows <= 0: one panel (the paper's global format); else panels of that many rows."""
-    return Format(A, dtype, panel_rows)
+def build(A, dtype="f64", panel_rows=0, max_len=256, tau=0.75) -> Format:
+    """panel_rows <= 0: one panel (the paper's global format); else panels of that many rows.
+    max_len: MAX_LEN; tau: the regular-block threshold."""
+    return Format(A, dtype, panel_rows, max_len, tau)

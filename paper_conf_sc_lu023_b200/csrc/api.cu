@@ -155,6 +155,8 @@ void dasp_options_default(dasp_options_t* o) {
     o->num_threads = 0;
     o->panel_rows = 0;
     o->pipeline = 0;
+    o->max_len = 256;
+    o->threshold = 0.75;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -194,7 +196,8 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     // panel size (R28): -1 one panel (the paper's global format); 0 automatic; env override
     int64_t panel_rows = o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
     if (const char* pr = std::getenv("DASP_PANEL_ROWS")) panel_rows = std::atoll(pr);
-    int st = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0, panel_rows);
+    int st = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0, panel_rows,
+                                o.max_len, o.threshold);
     auto t1 = std::chrono::steady_clock::now();
     p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
     if (st != DASP_OK) {
@@ -513,6 +516,8 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
     o->pipeline = p->pipe ? 1 : 0;
+    o->max_len = f.max_len;
+    o->threshold = f.tau;
     o->build_ms = p->build_ms;
     o->upload_ms = p->upload_ms;
     return DASP_OK;

@@ -77,14 +77,14 @@ struct Panel {
     int64_t nout() const { return 64 * t13 + 32 * t4 + 64 * t22 + SHORT_TILE * ts; }
 };
 
-inline int class_of(int64_t L) { return L > MAX_LEN ? C_LONG : (L > 4 ? C_MED : static_cast<int>(L)); }
+inline int class_of(int64_t L, int64_t max_len) { return L > max_len ? C_LONG : (L > 4 ? C_MED : static_cast<int>(L)); }
 
 // ---- pass 1: classification, medium order, counts ----
-void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
+void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par, int64_t max_len, double tau) {
     const int64_t n = P.r1 - P.r0;
     // a1: classes (R1: empty rows are their own class), lists in ascending row order
     if (!par) {
-        for (int64_t i = P.r0; i < P.r1; ++i) P.rows[class_of(rp[i + 1] - rp[i])].push_back(i);
+        for (int64_t i = P.r0; i < P.r1; ++i) P.rows[class_of(rp[i + 1] - rp[i], max_len)].push_back(i);
     } else {  // stable parallel partition
         const int T = omp_get_max_threads();
         std::vector<int64_t> cnt(static_cast<size_t>(T) * C_NUM, 0), off(static_cast<size_t>(T) * C_NUM);
@@ -92,7 +92,7 @@ void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
         {
             const int tid = omp_get_thread_num();
             const int64_t lo = P.r0 + n * tid / T, hi = P.r0 + n * (tid + 1) / T;
-            for (int64_t i = lo; i < hi; ++i) cnt[static_cast<size_t>(tid) * C_NUM + class_of(rp[i + 1] - rp[i])]++;
+            for (int64_t i = lo; i < hi; ++i) cnt[static_cast<size_t>(tid) * C_NUM + class_of(rp[i + 1] - rp[i], max_len)]++;
         }
         int64_t total[C_NUM] = {0};
         for (int k = 0; k < C_NUM; ++k)
@@ -107,7 +107,7 @@ void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
             const int64_t lo = P.r0 + n * tid / T, hi = P.r0 + n * (tid + 1) / T;
             int64_t o[C_NUM];
             for (int k = 0; k < C_NUM; ++k) o[k] = off[static_cast<size_t>(tid) * C_NUM + k];
-            for (int64_t i = lo; i < hi; ++i) { const int c = class_of(rp[i + 1] - rp[i]); P.rows[c][o[c]++] = i; }
+            for (int64_t i = lo; i < hi; ++i) { const int c = class_of(rp[i + 1] - rp[i], max_len); P.rows[c][o[c]++] = i; }
         }
     }
     // a2: long groups
@@ -116,17 +116,17 @@ void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
         P.nnz_long += L;
         P.n_groups += (L + geo.G - 1) / geo.G;
     }
-    // a3: stable descending sort by length (R26): counting sort on MAX_LEN - len
+    // a3: stable descending sort by length (R26): counting sort on max_len - len
     const auto& MR = P.rows[C_MED];
     const int64_t nm = static_cast<int64_t>(MR.size());
     P.nrb = (nm + MMA_M - 1) / MMA_M;  // R7
     P.sorted.assign(static_cast<size_t>(P.nrb * MMA_M), -1);
     {
-        constexpr int NB = MAX_LEN + 1;
-        std::vector<int64_t> h(NB + 1, 0);
-        for (int64_t r : MR) h[MAX_LEN - (rp[r + 1] - rp[r]) + 1]++;
-        for (int b = 0; b < NB; ++b) h[b + 1] += h[b];
-        for (int64_t r : MR) P.sorted[h[MAX_LEN - (rp[r + 1] - rp[r])]++] = r;
+        const int64_t NB = max_len + 1;
+        std::vector<int64_t> h(static_cast<size_t>(NB + 1), 0);
+        for (int64_t r : MR) h[max_len - (rp[r + 1] - rp[r]) + 1]++;
+        for (int64_t b = 0; b < NB; ++b) h[b + 1] += h[b];
+        for (int64_t r : MR) P.sorted[h[max_len - (rp[r + 1] - rp[r])]++] = r;
     }
     P.nreg.assign(static_cast<size_t>(P.nrb), 0);
     int64_t reg = 0, irr = 0, nnz_med = 0, sq_med = 0;
@@ -139,13 +139,14 @@ void plan_panel(Panel& P, const Geometry& geo, const int64_t* rp, bool par) {
             nnz_med += L[g];
             sq_med += L[g] * L[g];
         }
-        // regular iff the 8 x K block holds more than tau * 8K real slots (tau = 0.75, strict R4);
-        // the regular blocks form a prefix (R6)
+        // regular iff the 8 x K block holds more than tau * 8K real slots (default tau = 0.75,
+        // strict R4); the regular blocks form a prefix (R6)
+        const double thr = static_cast<double>(geo.BE) * tau;
         int64_t b = 0;
         for (;;) {
             int64_t c = 0;
             for (int g = 0; g < MMA_M; ++g) c += std::clamp<int64_t>(L[g] - geo.K * b, 0, geo.K);
-            if (4 * c > 3 * static_cast<int64_t>(geo.BE)) ++b; else break;
+            if (static_cast<double>(c) > thr) ++b; else break;
         }
         P.nreg[rb] = b;
         reg += b * geo.BE;
@@ -304,7 +305,7 @@ int build_impl(HostFormat& f, int64_t m, const int64_t* rp, const int32_t* col, 
     // many panels: one thread per panel; few panels: threads inside each panel
     const bool outer = np >= 2 * T;
 #pragma omp parallel for schedule(dynamic, 1) if (outer)
-    for (int64_t q = 0; q < np; ++q) plan_panel(panels[q], geo, rp, !outer);
+    for (int64_t q = 0; q < np; ++q) plan_panel(panels[q], geo, rp, !outer, f.max_len, f.tau);
 
     // offsets of every panel in the concatenated arrays
     int64_t lr = 0, grp = 0, rb = 0, reg = 0, irr = 0, tile = 0, out = 0, emp = 0;
@@ -368,8 +369,11 @@ int build_impl(HostFormat& f, int64_t m, const int64_t* rp, const int32_t* col, 
 }  // namespace
 
 int build_format(HostFormat& f, int dtype, int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col,
-                 const void* val, int nthreads, bool validate, int64_t panel_rows) {
+                 const void* val, int nthreads, bool validate, int64_t panel_rows, int64_t max_len, double tau) {
     f = HostFormat{};
+    f.max_len = max_len > 0 ? max_len : MAX_LEN;
+    f.tau = tau > 0.0 ? tau : 0.75;
+    if (f.max_len < 4 || f.tau > 1.0) return DASP_ERR_INVALID_ARG;
     f.geo = geometry(dtype);
     f.dtype = dtype;
     f.m = m;

@@ -25,7 +25,7 @@ inline Geometry geometry(int dtype) {
     return Geometry{2, 8, 64, 2, 128, 4, 4};
 }
 
-constexpr int MAX_LEN = 256;
+constexpr int MAX_LEN = 256;     // P:L152 (default; plan option max_len)
 constexpr int MMA_M = 8;
 constexpr int32_t PAD_COL = -1;  // R12: sentinel column of pads (x read as 0)
 constexpr int SHORT_TILE = 128;  // elements per short tile (32 four-slot rows)
@@ -45,6 +45,8 @@ struct HostFormat {
     int64_t nnz_long_new = 0, nnz_reg_new = 0, nnz_irreg = 0, nnz_short_new = 0;
     int64_t nnz_long = 0, nnz_medium = 0, nnz_short = 0;
     int64_t sumsq_medium = 0;  // sum of squared medium row lengths (launch tuning)
+    int64_t max_len = MAX_LEN; // long iff len > max_len
+    double tau = 0.75;         // regular iff count > BE * tau
     int64_t panel_rows = 0;   // rows per panel (R28); >= m: one panel = the paper's global format
     int64_t n_panels = 0;
     HostBuf arr[DASP_ARR_COUNT];
@@ -53,6 +55,7 @@ struct HostFormat {
 
 // Builds the format on the host.  Returns a dasp_status_t.
 int build_format(HostFormat& f, int dtype, int64_t m, int64_t n, const int64_t* row_ptr,
-                 const int32_t* col, const void* val, int nthreads, bool validate, int64_t panel_rows);
+                 const int32_t* col, const void* val, int nthreads, bool validate, int64_t panel_rows,
+                 int64_t max_len, double tau);
 
 }  // namespace dasp

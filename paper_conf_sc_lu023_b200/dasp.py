@@ -42,7 +42,8 @@ class DaspError(RuntimeError):
 class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("variant", ctypes.c_int32), ("validate", ctypes.c_int32),
                 ("keep_host", ctypes.c_int32), ("medium_rb_per_warp", ctypes.c_int32),
-                ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64), ("pipeline", ctypes.c_int32)]
+                ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64), ("pipeline", ctypes.c_int32),
+                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -55,6 +56,7 @@ class PlanInfo(ctypes.Structure):
                    "nnz_short", "device_bytes", "alg_bytes_beta0", "alg_bytes_beta1")] + \
                [("medium_rb_per_warp", ctypes.c_int32), ("launches_per_spmv", ctypes.c_int32),
                 ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64), ("pipeline", ctypes.c_int32),
+                ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
                 ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double)]
 
     def as_dict(self):
@@ -153,7 +155,7 @@ class Plan:
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                      variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, keep_host: bool = False,
                      medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0,
-                     pipeline: bool = False) -> Plan:
+                     pipeline: bool = False, max_len: int = 256, threshold: float = 0.75) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
@@ -177,6 +179,7 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     opts.keep_host, opts.medium_rb_per_warp, opts.num_threads = int(keep_host), medium_rb_per_warp, num_threads
     opts.panel_rows = panel_rows
     opts.pipeline = int(pipeline)
+    opts.max_len, opts.threshold = int(max_len), float(threshold)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))

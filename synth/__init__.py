@@ -27,7 +27,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "libsynth.so")
 
 SYN_UNIFORM, SYN_MIX, SYN_STENCIL27, SYN_POWERLAW, SYN_MIXED64, SYN_SHORT, SYN_LENLIST = range(7)
-VAL_UNIFORM, VAL_INT, VAL_ONES = range(3)
+VAL_UNIFORM, VAL_INT, VAL_ONES, VAL_SPD = range(4)
 
 
 class _Params(ctypes.Structure):

@@ -31,7 +31,7 @@ enum {
     SYN_LENLIST = 6    /* lengths given by the caller (edge-case tests)        */
 };
 
-enum { VAL_UNIFORM = 0, VAL_INT = 1, VAL_ONES = 2 };
+enum { VAL_UNIFORM = 0, VAL_INT = 1, VAL_ONES = 2, VAL_SPD = 3 };
 
 typedef struct {
     int64_t m, n;
@@ -258,7 +258,10 @@ int synth_fill(int kind, const synth_params* p, int64_t row0, int64_t nrows, con
             row_cols(kind, p, row, L, buf);
             for (int64_t k = 0; k < L; ++k) {
                 col[b + k] = (int32_t)buf[k];
-                val[b + k] = gen_val(kind, p, row, k, L);
+                /* VAL_SPD: -1 off the diagonal, L + 0.5 on it: symmetric patterns (stencils) give a
+                   strictly diagonally dominant symmetric, hence SPD, matrix (solver consumer, f4) */
+                if (p->val_mode == VAL_SPD) val[b + k] = buf[k] == row ? (double)L + 0.5 : -1.0;
+                else val[b + k] = gen_val(kind, p, row, k, L);
             }
         }
         free(buf);

@@ -145,3 +145,35 @@ def test_remap_columns_padded_layout():
     assert S == np.diff(s).max()
     owner = np.searchsorted(s, A.col, side="right") - 1
     assert np.array_equal(col, owner * S + (A.col - s[owner]))
+
+
+# f3: MAX_LEN ("adjustable") and tau ("customized") as plan options
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("max_len,tau", [(16, 0.75), (64, 0.5), (1000, 0.9), (256, 1.0), (4, 0.75)])
+def test_builder_knobs_bit_exact(dt, max_len, tau):
+    A = synth.generate(synth.config("c1b"))
+    plan = host_plan(A, dt, max_len=max_len, threshold=tau, panel_rows=1500)
+    info = plan.info
+    assert info["max_len"] == max_len and info["threshold"] == tau
+    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt, panel_rows=1500, max_len=max_len, tau=tau)
+    for k, v in ref.counts.items():
+        assert info[COUNT_MAP[k]] == v, k
+    for arr in dasp.ARRAYS:
+        assert np.array_equal(dasp.dasp_plan_copy_array(plan, arr), ref.arrays[arr]), arr
+    lens = np.diff(A.row_ptr)
+    assert info["row_long"] == int((lens > max_len).sum())
+    assert info["row_medium"] == int(((lens > 4) & (lens <= max_len)).sum())
+
+
+def test_knob_closed_forms_on_stencil():
+    # 16^3 stencil: MAX_LEN = 20 turns every len-27 row long; tau = 1.0 leaves no regular block
+    from tests.test_oracle import stencil_hist
+    A = synth.generate(synth.config("c2", scale=16 / 128))
+    h = stencil_hist(16)
+    info = host_plan(A, "f64", max_len=20).info
+    assert info["row_long"] == h[27] and info["row_medium"] == h[18] + h[12] + h[8]
+    assert info["nnz_long_new"] == h[27] * 64          # one group of 64 per len-27 row
+    info = host_plan(A, "f64", threshold=1.0).info
+    assert info["nnz_reg_new"] == 0 and info["nnz_irreg"] == A.nnz
+    with pytest.raises(dasp.DaspError):
+        host_plan(A, "f64", max_len=3)

@@ -317,3 +317,16 @@ def test_scatter_epilogue_writes_every_destination(dt, pipeline):
             assert np.array_equal(d.cpu().numpy().astype(np.float64), y_ref), (alpha, beta)
     with pytest.raises(dasp.DaspError):
         dasp.dasp_spmv_scatter(plan, xd, [dst[0]] * 9)
+
+
+# f3 knobs: MAX_LEN and tau move rows between classes and slots between regular / irregular;
+# the result must not change (bit-exact on integers)
+@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("max_len,tau", [(16, 0.75), (64, 0.5), (1000, 0.9), (256, 1.0), (4, 0.3)])
+def test_parity_knobs(dt, max_len, tau):
+    A = synth.generate(synth.config("c3", scale=0.004, val_mode=synth.VAL_INT))
+    x = synth.vector(71, A.n, synth.VAL_INT)
+    y_ref, _ = oracle_ref(A, x, dt)
+    for v in VARIANTS:
+        plan = make(A, dt, max_len=max_len, threshold=tau)
+        assert np.array_equal(run(plan, x, dt, variant=v), y_ref)
