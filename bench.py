@@ -127,6 +127,7 @@ class ClockSampler:
 # bytes per launch: CSR-equivalent and algorithmic (what the DASP format moves)
 # ----------------------------------------------------------------------------------------------
 def byte_model(info, dtype, beta_nonzero=False):
+    """Algorithmic bytes per launch of each kernel."""
     sv, sx, sy = (8, 8, 8) if dtype == "f64" else (2, 2, 4)
     sa = sy
     b1 = 2 if beta_nonzero else 1
@@ -136,15 +137,16 @@ def byte_model(info, dtype, beta_nonzero=False):
     nrb = info["rowblocks"]
     nout = 64 * info["tiles_13"] + 32 * info["tiles_4"] + 64 * info["tiles_22"] + 128 * info["tiles_single"]
     n_short_rows = info["n_len1"] + info["n_len2"] + info["n_len3"] + info["n_len4"]
-    main = (ngp * G * (sv + 4) + ngp * sa
-            + (info["nnz_reg_new"] + info["nnz_irreg"]) * (sv + 4) + 8 * (nrb + 1) + 8 * (8 * nrb + 1) + 4 * 8 * nrb
+    long_ = ngp * G * (sv + 4) + ngp * sa + 4 * (ngp // 4)          # slots, group partials, unit order
+    main = ((info["nnz_reg_new"] + info["nnz_irreg"]) * (sv + 4) + 8 * (nrb + 1) + 8 * (8 * nrb + 1) + 4 * 8 * nrb
             + info["row_medium"] * sy * b1
             + info["nnz_short_new"] * (sv + 4) + 4 * nout + n_short_rows * sy * b1
-            + n * sx)
+            + n * sx)                                                   # x counted once, here
     finish = (ngp * sa + 8 * (info["row_long"] + 1) + 4 * info["row_long"] + info["row_long"] * sy * b1
               + info["n_empty"] * (4 + sy * b1))
     csr_equiv = nnz * (sv + 4) + (m + 1) * 8 + n * sx + m * sy * b1
-    return {"main": main, "finish": finish, "total": main + finish, "csr_equiv": csr_equiv}
+    return {"dasp_long_kernel": long_, "dasp_main_kernel": main, "dasp_finish_kernel": finish,
+            "total": long_ + main + finish, "csr_equiv": csr_equiv}
 
 
 def load_peaks():
@@ -179,12 +181,14 @@ def stream_triad(dev, n=1 << 28, reps=20):
     return 24.0 * n / (best * 1e-3) / 1e9
 
 
-def load_traffic(config, dtype, variant):
+def load_traffic(config, dtype, variant, kernel="dasp_main_kernel"):
+    """ncu DRAM bytes per launch recorded by scripts/ncu_summary.py (profiles/ncu_traffic.json)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        return d.get(f"{config}/{dtype}/{variant}")
+        return d.get(f"{config}/{dtype}/{variant}/{kernel}", d.get(f"{config}/{dtype}/{variant}")
+                     if kernel == "dasp_main_kernel" else None)
     except Exception:
         return None
 
@@ -260,7 +264,8 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    slab = build_slab(gen_rows, lens, rank, world, reduce_max)
+    use_slab = world > 1 or args.iterate
+    slab = build_slab(gen_rows, lens, rank, world, reduce_max, need_norm=use_slab)
     gen_s = time.perf_counter() - t0
     if args.dtype == "f16":
         if world > 1:
@@ -269,7 +274,6 @@ def main():
     x_global = synth.vector(101, spec.n)
 
     t1 = time.perf_counter()
-    use_slab = world > 1 or args.iterate
     if not use_slab:
         # single GPU: plain SpMV over resident inputs, y overwritten every step
         plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
@@ -355,20 +359,24 @@ def main():
         csr_bytes = float(t.item())
     eff_gbs = csr_bytes / (ms_step * 1e-3) / 1e9
 
-    # ---- roofline of the dominant kernel (the fused main kernel), per launch ----
+    # ---- roofline of the dominant kernel (largest share of the step), per launch ----
     peak, peak_src = load_peaks()
-    main_ms, main_n = kern["dasp_main_kernel"]
-    fin_ms, fin_n = kern["dasp_finish_kernel"]
-    main_avg = main_ms / max(main_n, 1)
-    achieved = bm["main"] / (main_avg * 1e-3) / 1e9 if main_n else None
-    traffic = load_traffic(workload, args.dtype, args.variant)
+    per_kernel = {k: (ms, nl) for k, (ms, nl) in kern.items() if nl}
+    dom = max(per_kernel, key=lambda k: per_kernel[k][0]) if per_kernel else "dasp_main_kernel"
+    dom_ms, dom_n = per_kernel.get(dom, (0.0, 0))
+    dom_avg = dom_ms / max(dom_n, 1)
+    dom_bytes = bm.get(dom, bm["total"])
+    achieved = dom_bytes / (dom_avg * 1e-3) / 1e9 if dom_n else None
+    traffic = load_traffic(workload, args.dtype, args.variant, dom)
     triad = None if args.no_triad else stream_triad(dev)
-    roofline = {"kernel": "dasp_main_kernel", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+    roofline = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak if achieved else None, "traffic": traffic,
-                "alg_bytes_per_launch": bm["main"], "avg_launch_ms": main_avg,
-                "share_of_step": (main_ms / max(main_n, 1)) / ms_step if main_n else None,
-                "finish_avg_ms": fin_ms / fin_n if fin_n else 0.0, "peak_source": peak_src,
-                "stream_triad_gbs": triad, "frac_of_triad": achieved / triad if (achieved and triad) else None}
+                "alg_bytes_per_launch": dom_bytes, "avg_launch_ms": dom_avg,
+                "share_of_step": dom_avg / ms_step if dom_n else None, "peak_source": peak_src,
+                "stream_triad_gbs": triad, "frac_of_triad": achieved / triad if (achieved and triad) else None,
+                "kernels": {k: {"avg_ms": ms / nl, "launches": nl, "alg_bytes": bm.get(k),
+                                "alg_gbs": bm[k] / (ms / nl * 1e-3) / 1e9 if k in bm and ms > 0 else None}
+                            for k, (ms, nl) in per_kernel.items()}}
 
     # ---- e2e: the same metric through the C-ABI with HOST buffers (copies inside the timed region) ----
     e2e = None
@@ -442,6 +450,7 @@ def main():
             "effective_gbs": eff_gbs, "effective_frac_of_peak": eff_gbs / peak,
             "alg_gbs_step": bm["total"] * world / (ms_step * 1e-3) / 1e9 if world == 1 else None,
             "gpu_launches": int(info["launches_per_spmv"]) * args.steps,
+            "gpu_launches_per_step": int(info["launches_per_spmv"]),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "variant_compare": compare,
             "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,

@@ -219,10 +219,12 @@ dasp_status_t dasp_remap_columns(int32_t* col, int64_t nnz, const int64_t* start
 
 /* Kernel ids of the per-kernel timing below. */
 typedef enum {
-    DASP_K_MAIN = 0,      /* fused long-phase-1 + medium + short/single kernel (Alg. 2 l.1-16, Alg. 3-5) */
+    DASP_K_MAIN = 0,      /* medium + short/single kernel, panel by panel (Alg. 3-5); with
+                             options.pipeline the persistent kernel that also does the long units */
     DASP_K_FINISH = 1,    /* long phase 2 (Alg. 2 l.17-25) + empty rows */
     DASP_K_SCALE = 2,     /* alpha == 0 quick path */
-    DASP_K_COUNT = 3
+    DASP_K_LONG = 3,      /* long phase 1 (Alg. 2 l.1-16) */
+    DASP_K_COUNT = 4
 } dasp_kernel_t;
 
 /*

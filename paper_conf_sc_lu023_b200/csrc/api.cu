@@ -32,7 +32,8 @@ struct dasp_plan_s {
     void* d_yh = nullptr;
     int64_t device_bytes = 0;
     double build_ms = 0, upload_ms = 0;
-    int64_t blocks = 0;                   // grid of the fused main kernel
+    int64_t blocks = 0;                   // grid of the medium/short kernel
+    int64_t n_units = 0;                  // long units (long kernel)
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
     void* d_blk_panel = nullptr;          // int32 panel of every block
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
@@ -218,12 +219,13 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
             d.blk0 = blk;
             d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5]; d.nmw = (e[5] + p->rbw - 1) / p->rbw;
             d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
-            const int64_t warps = d.nunits + d.nmw + d.t13 + d.t4 + d.t22 + d.ts;
+            const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
             const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
             blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
             blk += nb;
         }
         p->blocks = blk;
+        p->n_units = f.n_groups_padded / f.geo.UG;
     }
     // long-unit execution order (a launch schedule, not part of the format): inside each panel
     // the units run bucketed by the column of their first element, so that the warps in flight
@@ -434,6 +436,10 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
         const int c = std::atoi(pc);
         if (c >= 1 && c <= 3) mp.class_mask = 1 << (c - 1);
     }
+    if (!p->pipe && p->n_units > 0 && (mp.class_mask & 1)) {
+        e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s); });
+        if (e != cudaSuccess) return DASP_ERR_CUDA;
+    }
     e = timed(p, DASP_K_MAIN, s, on, [&] {
         if (p->pipe)
             return dasp::launch_pipe(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_items), p->n_items,
@@ -512,7 +518,8 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta0 = alg_bytes(p, false);
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
-    o->launches_per_spmv = (p->blocks > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
+    o->launches_per_spmv = p->pipe ? (p->n_items > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0)
+                                   : (p->n_units > 0 ? 1 : 0) + (p->blocks > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
     o->pipeline = p->pipe ? 1 : 0;

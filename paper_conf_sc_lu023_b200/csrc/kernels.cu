@@ -503,23 +503,40 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
 #ifndef DASP_MIN_BLOCKS
 #define DASP_MIN_BLOCKS 4   // caps registers at 64: >= 32 resident warps per SM, no spills
 #endif
+#ifndef DASP_MIN_BLOCKS_F16
+#define DASP_MIN_BLOCKS_F16 4
+#endif
+// long rows, phase 1 (Alg. 2 l.1-16), in their own launch: the unit path needs few registers
+// and is gather-latency bound, so it runs at higher occupancy (40 registers, 48 warps
+// per SM) than the medium path, which needs 64 (profiles/r01/long_kernel_occupancy.jsonl).  Units run in
+// the column-bucketed schedule `unit_order`.
+#ifndef DASP_LONG_MIN_BLOCKS
+#define DASP_LONG_MIN_BLOCKS 6
+#endif
+#ifndef DASP_LONG_MIN_BLOCKS_F16
+#define DASP_LONG_MIN_BLOCKS_F16 6
+#endif
 template <int DT, int VAR>
-__global__ void __launch_bounds__(MAIN_THREADS, DASP_MIN_BLOCKS) dasp_main_kernel(const MainParams P) {
+__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_LONG_MIN_BLOCKS : DASP_LONG_MIN_BLOCKS_F16)
+dasp_long_kernel(const MainParams P, int64_t n_units) {
+    const int64_t w = (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5;
+    if (w >= n_units) return;
+    const int lane = threadIdx.x & 31;
+    const uint64_t pol = stream_policy();
+    const int64_t u = __ldg(P.unit_order + w);
+    if constexpr (DT == 0) long_unit_f64<VAR>(P, u, lane, pol);
+    else long_unit_f16<VAR>(P, u, lane, pol);
+}
+
+// medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
+template <int DT, int VAR>
+__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : DASP_MIN_BLOCKS_F16) dasp_main_kernel(const MainParams P) {
     const int lane = threadIdx.x & 31;
     // role of this warp inside its panel; the descriptor fields are loaded only on the branch
     // that needs them so they do not stay live (register pressure = occupancy)
     const PanelDesc* D = P.panels + __ldg(P.blk_panel + blockIdx.x);
     int64_t w = (static_cast<int64_t>(blockIdx.x) - __ldg(&D->blk0)) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
     const uint64_t pol = stream_policy();
-    const int64_t nunits = __ldg(&D->nunits);
-    if (w < nunits) {                                    // long rows, phase 1
-        if (!(P.class_mask & 1)) return;
-        const int64_t u = __ldg(P.unit_order + __ldg(&D->unit0) + w);
-        if constexpr (DT == 0) long_unit_f64<VAR>(P, u, lane, pol);
-        else long_unit_f16<VAR>(P, u, lane, pol);
-        return;
-    }
-    w -= nunits;
     const int64_t nmw = __ldg(&D->nmw);
     if (w < nmw) {                                       // medium rows
         if (!(P.class_mask & 2)) return;
@@ -1126,6 +1143,21 @@ cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint6
     } else {
         if (variant == VAR_MMA) dasp_pipe_kernel<1, VAR_MMA><<<grid, block, smem, s>>>(p, items, n_items);
         else dasp_pipe_kernel<1, VAR_CUDACORE><<<grid, block, smem, s>>>(p, items, n_items);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s) {
+    if (n_units <= 0) return cudaSuccess;
+    const int64_t blocks = (n_units * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
+    if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
+    if (dtype == 0) {
+        if (variant == VAR_MMA) dasp_long_kernel<0, VAR_MMA><<<grid, block, 0, s>>>(p, n_units);
+        else dasp_long_kernel<0, VAR_CUDACORE><<<grid, block, 0, s>>>(p, n_units);
+    } else {
+        if (variant == VAR_MMA) dasp_long_kernel<1, VAR_MMA><<<grid, block, 0, s>>>(p, n_units);
+        else dasp_long_kernel<1, VAR_CUDACORE><<<grid, block, 0, s>>>(p, n_units);
     }
     return cudaGetLastError();
 }

@@ -18,10 +18,10 @@ struct ExtraDst {
 };
 constexpr int WARPS_PER_BLOCK = MAIN_THREADS / 32;
 
-// One row panel (R28) as the fused kernel sees it.  A panel owns the blocks
-// [blk0, blk0 + ceil(warps/8)); its warps are, in order:
-//   nunits long units (UG groups each; Alg. 2 l.1-16), nmw medium warps (rbw row-blocks each;
-//   Alg. 3, LOOP_NUM P:L271), then one warp per short tile (1&3 | len4 | 2&2 | singles).
+// One row panel (R28) as the medium/short kernel sees it.  A panel owns the blocks
+// [blk0, blk0 + ceil(warps/8)); its warps are, in order: nmw medium warps (rbw row-blocks each;
+// Alg. 3, LOOP_NUM P:L271), then one warp per short tile (1&3 | len4 | 2&2 | singles).  The long
+// units (unit0, nunits) run in their own kernel (dasp_long_kernel).
 struct PanelDesc {
     int64_t blk0;
     int64_t unit0, nunits;
@@ -70,6 +70,7 @@ struct FinishParams {
 // apw_bytes > 0: launch with an L2 access-policy window (persisting) over [apw_base, +apw_bytes)
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
+cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
 cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s);
 
 // Persistent TMA-staged pipeline kernel (kernels.cu): items are 64-bit words

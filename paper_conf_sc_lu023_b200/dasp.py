@@ -17,8 +17,8 @@ LIB_PATH = os.environ.get("DASP_LIB", os.path.join(_HERE, "libdasp.so"))   # ove
 
 DASP_R_64F, DASP_R_16F = 0, 1
 DASP_VARIANT_DEFAULT, DASP_VARIANT_MMA, DASP_VARIANT_CUDACORE = 0, 1, 2
-DASP_K_MAIN, DASP_K_FINISH, DASP_K_SCALE, DASP_K_COUNT = 0, 1, 2, 3
-KERNEL_NAMES = ["dasp_main_kernel", "dasp_finish_kernel", "dasp_scale_kernel"]
+DASP_K_MAIN, DASP_K_FINISH, DASP_K_SCALE, DASP_K_LONG, DASP_K_COUNT = 0, 1, 2, 3, 4
+KERNEL_NAMES = ["dasp_main_kernel", "dasp_finish_kernel", "dasp_scale_kernel", "dasp_long_kernel"]
 
 ARRAYS = ["long_val", "long_col", "group_ptr", "long_out", "rb_ptr", "reg_val", "reg_col", "irr_ptr",
           "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows", "panels"]

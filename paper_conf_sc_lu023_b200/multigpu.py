@@ -49,8 +49,10 @@ class Slab:
         return int(self.row_ptr[-1])
 
 
-def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, reduce_max=None) -> Slab:
-    """generate_rows(row0, nrows) -> CSR of those rows (global columns).  reduce_max(v) -> max over ranks."""
+def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, reduce_max=None,
+               need_norm: bool = True) -> Slab:
+    """generate_rows(row0, nrows) -> CSR of those rows (global columns).  reduce_max(v) -> max over ranks.
+    need_norm=False skips the infinity norm (only the iteration needs it)."""
     starts = slab_bounds(row_lengths, world)
     r0, r1 = int(starts[rank]), int(starts[rank + 1])
     A = generate_rows(r0, r1 - r0)
@@ -59,14 +61,16 @@ def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, re
     else:
         col = np.ascontiguousarray(A.col, dtype=np.int32).copy()
         S = dasp.dasp_remap_columns(col, starts)
-    absval = np.abs(A.val.astype(np.float64))
-    lens = np.diff(A.row_ptr)
-    rs = np.zeros(len(lens))
-    nz = lens > 0
-    if nz.any():
-        rs[nz] = np.add.reduceat(absval, A.row_ptr[:-1][nz])
-    local = float(rs.max()) if len(rs) else 0.0
-    inf_norm = reduce_max(local) if reduce_max else local
+    inf_norm = 1.0
+    if need_norm:
+        absval = np.abs(A.val.astype(np.float64))
+        lens = np.diff(A.row_ptr)
+        rs = np.zeros(len(lens))
+        nz = lens > 0
+        if nz.any():
+            rs[nz] = np.add.reduceat(absval, A.row_ptr[:-1][nz])
+        local = float(rs.max()) if len(rs) else 0.0
+        inf_norm = reduce_max(local) if reduce_max else local
     return Slab(A.row_ptr, col, A.val, r0, r1 - r0, starts, S, inf_norm)
 
 

@@ -3,7 +3,8 @@
 
     python scripts/ncu_summary.py OUT.md KEY=REPORT.ncu-rep [KEY=REPORT.ncu-rep ...]
 
-KEY is "<workload>/<dtype>/<variant>" (bench.py's lookup key for roofline.traffic).
+KEY is "<workload>/<dtype>/<variant>"; traffic is stored per "<KEY>/<kernel>" (bench.py's lookup
+key for roofline.traffic); every dasp_* kernel captured in the report is summarised.
 profiles/ncu_traffic.json receives dram__bytes_read.sum + dram__bytes_write.sum per launch.
 """
 import csv
@@ -59,9 +60,12 @@ def main():
     for arg in sys.argv[2:]:
         key, rep = arg.split("=", 1)
         for k, d in enumerate(raw(rep)):
-            if "dasp_main_kernel" not in d.get("Kernel Name", ("", ""))[1]:
+            kname = d.get("Kernel Name", ("", ""))[1]
+            kern = next((n for n in ("dasp_main_kernel", "dasp_long_kernel", "dasp_finish_kernel", "dasp_pipe_kernel")
+                         if n in kname), None)
+            if kern is None:
                 continue
-            lines.append(f"## {key}  ({os.path.basename(rep)})")
+            lines.append(f"## {key} — {kern}  ({os.path.basename(rep)})")
             lines.append("")
             lines.append("| metric | value |")
             lines.append("|---|---|")
@@ -74,9 +78,10 @@ def main():
             lines.append("| top stall samples | " + ", ".join(f"{m.split('stalled_')[1]} {int(c)}" for c, m in stalls) + " |")
             rd = to_bytes(*d["dram__bytes_read.sum"])
             wr = to_bytes(*d["dram__bytes_write.sum"])
-            traffic[key] = rd + wr
+            traffic[f"{key}/{kern}"] = rd + wr
+            if kern == "dasp_main_kernel":
+                traffic[key] = rd + wr
             lines.append("")
-            break
     with open(out_md, "w") as f:
         f.write("\n".join(lines) + "\n")
     with open(traffic_path, "w") as f:
