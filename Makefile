@@ -18,10 +18,13 @@ $(OBJ)/builder.o: $(SRC)/builder.cpp $(SRC)/format.hpp include/dasp.h | $(OBJ)
 $(OBJ)/kernels.o: $(SRC)/kernels.cu $(SRC)/kernels.cuh | $(OBJ)
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $(OBJ)/kernels.ptxas.txt || (cat $(OBJ)/kernels.ptxas.txt; false)
 
-$(OBJ)/api.o: $(SRC)/api.cu $(SRC)/kernels.cuh $(SRC)/format.hpp include/dasp.h | $(OBJ)
+$(OBJ)/api.o: $(SRC)/api.cu $(SRC)/kernels.cuh $(SRC)/gpu_builder.cuh $(SRC)/format.hpp include/dasp.h | $(OBJ)
 	$(NVCC) $(NVFLAGS) -c $< -o $@
 
-$(PKG)/libdasp.so: $(OBJ)/builder.o $(OBJ)/kernels.o $(OBJ)/api.o
+$(OBJ)/gpu_builder.o: $(SRC)/gpu_builder.cu $(SRC)/gpu_builder.cuh $(SRC)/format.hpp include/dasp.h | $(OBJ)
+	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $(OBJ)/gpu_builder.ptxas.txt || (cat $(OBJ)/gpu_builder.ptxas.txt; false)
+
+$(PKG)/libdasp.so: $(OBJ)/builder.o $(OBJ)/kernels.o $(OBJ)/gpu_builder.o $(OBJ)/api.o
 	$(NVCC) $(ARCH) -shared -o $@ $^ -Xcompiler -fopenmp -lgomp
 
 oracle/liboracle.so: oracle/oracle.c
@@ -37,8 +40,8 @@ clean:
 
 # experiment builds: one libdasp_<VAR=value>.so per -D setting in EXPVARS
 EXPVARS ?= DASP_NSTAGE=3 DASP_NSTAGE=4
-exp: $(OBJ)/builder.o $(OBJ)/api.o
+exp: $(OBJ)/builder.o $(OBJ)/api.o $(OBJ)/gpu_builder.o
 	for v in $(EXPVARS); do \
 	  $(NVCC) $(NVFLAGS) -D$$v -c $(SRC)/kernels.cu -o $(OBJ)/kernels_$$v.o 2> $(OBJ)/kernels_$$v.ptxas.txt && \
-	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$v.so $(OBJ)/builder.o $(OBJ)/kernels_$$v.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
+	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$v.so $(OBJ)/builder.o $(OBJ)/kernels_$$v.o $(OBJ)/gpu_builder.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
 	done

@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--panel-rows", type=int, default=0, help="rows per panel (0 auto, -1 one global panel)")
     ap.add_argument("--no-triad", action="store_true")
     ap.add_argument("--iterate", action="store_true", help="N=1: run the row-slab iteration (x <- alpha*A*x)")
+    ap.add_argument("--no-gpu-build", action="store_true", help="skip timing the device-side builder")
     ap.add_argument("--fused", action="store_true", help="slab mode: fuse the x all-gather into the SpMV "
                     "epilogue (symmetric memory + dasp_spmv_scatter)")
     ap.add_argument("--e2e-steps", type=int, default=10)
@@ -421,6 +422,29 @@ def main():
                "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
                "d2h_bytes_per_step": int(yh.numel() * yh.element_size()), "api": "dasp_spmv_host"}
 
+    # ---- preprocessing cost (Fig. 13): host builder vs the device builder (f2) ----
+    gpu_build = None
+    if not use_slab and not args.no_gpu_build:
+        try:
+            vdt = torch.float64 if args.dtype == "f64" else torch.float16
+            d_rp = torch.from_numpy(slab.row_ptr).to(dev)
+            d_col = torch.from_numpy(np.ascontiguousarray(slab.col)).to(dev)
+            d_val = torch.from_numpy(np.ascontiguousarray(slab.val)).to(vdt).to(dev)
+            torch.cuda.synchronize(dev)
+            t0 = time.perf_counter()
+            dplan = dasp.dasp_plan_create_device(d_rp, d_col, d_val, slab.rows, spec.n, args.dtype, device=local,
+                                                 panel_rows=args.panel_rows)
+            wall = (time.perf_counter() - t0) * 1e3
+            gpu_build = {"gpu_build_ms": dplan.info["build_ms"], "wall_ms": wall,
+                         "host_build_ms": info["build_ms"], "host_upload_ms": info["upload_ms"],
+                         "spmv_equivalents": dplan.info["build_ms"] / ms_step,
+                         "host_spmv_equivalents": (info["build_ms"] + info["upload_ms"]) / ms_step}
+            dplan.destroy()
+            del d_rp, d_col, d_val
+            torch.cuda.empty_cache()
+        except Exception as exc:   # reported, not fatal: the bench line is about the SpMV
+            gpu_build = {"error": str(exc)}
+
     # ---- CPU oracle on the host cores (rank 0, N = 1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -452,7 +476,7 @@ def main():
             "gpu_launches": int(info["launches_per_spmv"]) * args.steps,
             "gpu_launches_per_step": int(info["launches_per_spmv"]),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-            "variant_compare": compare,
+            "variant_compare": compare, "preprocessing": gpu_build,
             "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,
                      "rows": {"empty": info["n_empty"], "short": info["n_len1"] + info["n_len2"] + info["n_len3"]
                               + info["n_len4"], "medium": info["row_medium"], "long": info["row_long"]},

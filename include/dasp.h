@@ -130,6 +130,18 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
                                dasp_dtype_t dtype, const dasp_options_t* opts);
 
 /*
+ * dasp_plan_create_device — the same plan built ON THE GPU: the CSR is
+ * given as DEVICE pointers on opts->device (d_row_ptr int64[m+1], d_col_idx int32[nnz], d_val
+ * double or binary16 [nnz]); classification, sorts, scans and scatters run as kernels on `stream`
+ * (cudaStream_t as void*), the packed arrays are written in place in device memory and are
+ * byte-identical to dasp_plan_create's.  Synchronises `stream`.  opts->device must be >= 0;
+ * keep_host is ignored.  Errors as dasp_plan_create.
+ */
+dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz,
+                                      const int64_t* d_row_ptr, const int32_t* d_col_idx, const void* d_val,
+                                      dasp_dtype_t dtype, const dasp_options_t* opts, void* stream);
+
+/*
  * dasp_spmv — the hot path (§3.3, Alg. 2-5):  y = alpha*A*x + beta*y.
  *
  *   x : DEVICE pointer on the plan's device, n elements (f64, or f16 bits for DASP_R_16F).

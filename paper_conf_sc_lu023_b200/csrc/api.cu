@@ -8,10 +8,12 @@
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <memory>
 #include <new>
 #include <vector>
 
 #include "format.hpp"
+#include "gpu_builder.cuh"
 #include "kernels.cuh"
 
 using dasp::HostFormat;
@@ -58,7 +60,7 @@ int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
-constexpr int64_t kAllocPad = 64;   // TMA windows may read up to 16 B past an array's end
+constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // TMA windows may read up to 16 B past an array's end
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
 // small matrices keep the paper's 1 / 2; for large ones, uniform medium rows (coefficient of
@@ -173,75 +175,47 @@ const char* dasp_status_string(dasp_status_t s) {
     return "DASP_ERR_UNKNOWN";
 }
 
-dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr,
-                               const int32_t* col_idx, const void* val, dasp_dtype_t dtype, const dasp_options_t* opts) {
-    if (!plan_out) return DASP_ERR_INVALID_ARG;
-    *plan_out = nullptr;
-    if (m < 0 || n < 0 || nnz < 0 || n > 0x7fffffffLL || m > 0x7fffffffLL) return DASP_ERR_INVALID_ARG;
-    if (dtype != DASP_R_64F && dtype != DASP_R_16F) return DASP_ERR_INVALID_ARG;
-    if (!row_ptr || (nnz > 0 && (!col_idx || !val))) return DASP_ERR_INVALID_ARG;
-    dasp_options_t o;
-    dasp_options_default(&o);
-    if (opts) o = *opts;
-    if (o.variant != DASP_VARIANT_MMA && o.variant != DASP_VARIANT_CUDACORE) o.variant = DASP_VARIANT_CUDACORE;
-    if (o.validate && row_ptr[m] != nnz) return DASP_ERR_INVALID_CSR;
+}  // extern "C"
 
-    dasp_plan_s* p = new (std::nothrow) dasp_plan_s;
-    if (!p) return DASP_ERR_OUT_OF_MEMORY;
-    p->dtype = dtype;
-    p->device = o.device;
-    p->variant = o.variant;
-    p->keep_host = o.keep_host != 0 || o.device < 0;
+namespace {
 
-    auto t0 = std::chrono::steady_clock::now();
-    // panel size (R28): -1 one panel (the paper's global format); 0 automatic; env override
-    int64_t panel_rows = o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
-    if (const char* pr = std::getenv("DASP_PANEL_ROWS")) panel_rows = std::atoll(pr);
-    int st = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0, panel_rows,
-                                o.max_len, o.threshold);
-    auto t1 = std::chrono::steady_clock::now();
-    p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
-    if (st != DASP_OK) {
-        delete p;
-        return static_cast<dasp_status_t>(st);
-    }
+// Launch metadata shared by host- and device-built plans: LOOP_NUM, the per-panel descriptors of
+// the medium/short kernel, the long-unit schedule, the pipelined kernel's item words, and their
+// device copies.  `panel_table` (host) is the DASP_ARR_PANELS content; `unit_first_col[u]` the
+// column of the first element of long unit u (for the column-bucket schedule).
+dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_t* panel_table,
+                           const std::vector<int32_t>& unit_first_col) {
     HostFormat& f = p->host;
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
-    // per-panel launch descriptors: warps = long units + medium warps + tiles
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<int32_t> blk_panel;
-    {
-        const int64_t* pt = static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr);
-        int64_t blk = 0;
-        for (int64_t q = 0; q < f.n_panels; ++q) {
-            const int64_t* e = pt + q * dasp::PANEL_FIELDS;
-            dasp::PanelDesc& d = desc[q];
-            d.blk0 = blk;
-            d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5]; d.nmw = (e[5] + p->rbw - 1) / p->rbw;
-            d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
-            const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
-            const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
-            blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
-            blk += nb;
-        }
-        p->blocks = blk;
-        p->n_units = f.n_groups_padded / f.geo.UG;
+    int64_t blk = 0;
+    for (int64_t q = 0; q < f.n_panels; ++q) {
+        const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
+        dasp::PanelDesc& d = desc[q];
+        d.blk0 = blk;
+        d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5]; d.nmw = (e[5] + p->rbw - 1) / p->rbw;
+        d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
+        const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
+        const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
+        blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
+        blk += nb;
     }
+    p->blocks = blk;
+    p->n_units = f.n_groups_padded / f.geo.UG;
     // long-unit execution order (a launch schedule, not part of the format): inside each panel
     // the units run bucketed by the column of their first element, so that the warps in flight
     // gather from ~1/kColBuckets of x at a time instead of all of it (long rows' columns are
     // sorted, so a unit covers a narrow column range).  Partials are per group and summed in
     // group order by the finish kernel: the result is bitwise independent of this order.
-    std::vector<int32_t> unit_order(static_cast<size_t>(f.n_groups_padded / f.geo.UG));
+    std::vector<int32_t> unit_order(static_cast<size_t>(p->n_units));
     {
-        const int32_t* lc = static_cast<const int32_t*>(f.arr[DASP_ARR_LONG_COL].ptr);
-        const int64_t ue = static_cast<int64_t>(f.geo.UG) * f.geo.G;
         const char* lo_env = std::getenv("DASP_LONG_ORDER");
         const bool bucketed = !(lo_env && std::atoi(lo_env) == 0) && f.n > 0;
         for (const auto& d : desc) {
             std::vector<int32_t> cnt(kColBuckets + 1, 0);
             auto bucket = [&](int64_t u) {
-                const int32_t c = lc[u * ue];
+                const int32_t c = unit_first_col[u];
                 return c < 0 ? kColBuckets - 1 : static_cast<int>(static_cast<int64_t>(c) * kColBuckets / f.n);
             };
             if (!bucketed) {
@@ -257,109 +231,203 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     // row-blocks, short tiles (kind<<62 | payload; kernels.cu produce())
     std::vector<uint64_t> items;
     bool items_ok = true;
-    for (const auto& d : desc) {
-        for (int64_t w = 0; w < d.nunits; ++w) items.push_back((1ull << 62) | static_cast<uint64_t>(unit_order[d.unit0 + w]));
-        for (int64_t r = 0; r < d.nrb; ++r) items.push_back((2ull << 62) | static_cast<uint64_t>(d.rb0 + r));
-        const int64_t nt = d.t13 + d.t4 + d.t22 + d.ts;
-        for (int64_t t = 0; t < nt; ++t) {
-            int64_t cat, ob;
-            if (t < d.t13) { cat = 0; ob = d.out0 + t * 64; }
-            else if (t < d.t13 + d.t4) { cat = 1; ob = d.out0 + 64 * d.t13 + (t - d.t13) * 32; }
-            else if (t < d.t13 + d.t4 + d.t22) { cat = 2; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + (t - d.t13 - d.t4) * 64; }
-            else { cat = 3; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + 64 * d.t22 + (t - d.t13 - d.t4 - d.t22) * 128; }
-            const int64_t tile = d.tile0 + t;
-            if (tile >= (int64_t(1) << 27) || ob >= (int64_t(1) << 33)) items_ok = false;
-            items.push_back((3ull << 62) | (static_cast<uint64_t>(cat) << 60) | (static_cast<uint64_t>(tile) << 33) |
-                            static_cast<uint64_t>(ob));
+    const char* pe = std::getenv("DASP_PIPE");   // overrides the option (experiments)
+    const bool want_pipe = pe ? std::atoi(pe) != 0 : o.pipeline != 0;
+    if (want_pipe) {
+        for (const auto& d : desc) {
+            for (int64_t w = 0; w < d.nunits; ++w) items.push_back((1ull << 62) | static_cast<uint64_t>(unit_order[d.unit0 + w]));
+            for (int64_t r = 0; r < d.nrb; ++r) items.push_back((2ull << 62) | static_cast<uint64_t>(d.rb0 + r));
+            const int64_t nt = d.t13 + d.t4 + d.t22 + d.ts;
+            for (int64_t t = 0; t < nt; ++t) {
+                int64_t cat, ob;
+                if (t < d.t13) { cat = 0; ob = d.out0 + t * 64; }
+                else if (t < d.t13 + d.t4) { cat = 1; ob = d.out0 + 64 * d.t13 + (t - d.t13) * 32; }
+                else if (t < d.t13 + d.t4 + d.t22) { cat = 2; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + (t - d.t13 - d.t4) * 64; }
+                else { cat = 3; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + 64 * d.t22 + (t - d.t13 - d.t4 - d.t22) * 128; }
+                const int64_t tile = d.tile0 + t;
+                if (tile >= (int64_t(1) << 27) || ob >= (int64_t(1) << 33)) items_ok = false;
+                items.push_back((3ull << 62) | (static_cast<uint64_t>(cat) << 60) | (static_cast<uint64_t>(tile) << 33) |
+                                static_cast<uint64_t>(ob));
+            }
         }
     }
     p->n_items = static_cast<int64_t>(items.size());
-    {
-        // DASP_PIPE overrides the option (experiments)
-        const char* pe = std::getenv("DASP_PIPE");
-        p->pipe = items_ok && (pe ? std::atoi(pe) != 0 : o.pipeline != 0);
-    }
-    for (int a = 0; a < DASP_ARR_COUNT; ++a) p->bytes[a] = f.arr[a].bytes;
+    p->pipe = want_pipe && items_ok;
+    if (p->device < 0) return DASP_OK;
 
+    auto upload = [&](void** dst, const void* src, size_t bytes) -> dasp_status_t {
+        if (cudaMalloc(dst, std::max<size_t>(bytes, 16)) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
+        p->device_bytes += static_cast<int64_t>(bytes);
+        if (bytes && cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice) != cudaSuccess) return DASP_ERR_CUDA;
+        return DASP_OK;
+    };
+    const int64_t pb = std::max<int64_t>(f.n_groups_padded, 1) * sy(p->dtype);
+    if (cudaMalloc(&p->d_partial, static_cast<size_t>(pb)) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
+    p->device_bytes += pb;
+    dasp_status_t st;
+    if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
+    if ((st = upload(&p->d_blk_panel, blk_panel.data(), blk_panel.size() * 4)) != DASP_OK) return st;
+    if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
+    if (p->pipe) {
+        int bps = 0, nsm = 0;
+        if ((st = upload(&p->d_items, items.data(), items.size() * 8)) != DASP_OK) return st;
+        if (dasp::pipe_occupancy(p->dtype, DASP_VARIANT_CUDACORE, &bps) != cudaSuccess ||   // sets both kernels'
+            dasp::pipe_occupancy(p->dtype, DASP_VARIANT_MMA, &bps) != cudaSuccess ||        // smem attribute
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess)
+            return DASP_ERR_CUDA;
+        // persistent grid: every SM full, never more warps than items
+        const int64_t wpb = dasp::pipe_warps_per_block();
+        p->pipe_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->n_items + wpb - 1) / wpb);
+    }
+    // optional persisting L2 access-policy window over x (DASP_X_APW=1; measured slower on C3,
+    // profiles/r01, so off by default)
+    const char* apw = std::getenv("DASP_X_APW");
+    if (apw && std::atoi(apw) > 0) {
+        cudaDeviceProp prop;
+        if (cudaGetDeviceProperties(&prop, p->device) == cudaSuccess && prop.persistingL2CacheMaxSize > 0) {
+            const size_t xb = static_cast<size_t>(f.n) * sx(p->dtype);
+            size_t lim = std::min<size_t>(static_cast<size_t>(prop.persistingL2CacheMaxSize), xb);
+            size_t win = std::min<size_t>(static_cast<size_t>(prop.accessPolicyMaxWindowSize), xb);
+            if (lim > 0 && win > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim) == cudaSuccess) {
+                p->apw_bytes = win;
+                p->apw_hit = std::min(1.0f, static_cast<float>(lim) / static_cast<float>(win));
+            }
+        }
+        cudaGetLastError();
+    }
+    return DASP_OK;
+}
+
+dasp_status_t check_create_args(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz, const void* row_ptr,
+                                const void* col_idx, const void* val, dasp_dtype_t dtype, const dasp_options_t* opts,
+                                dasp_options_t& o) {
+    if (!plan_out) return DASP_ERR_INVALID_ARG;
+    *plan_out = nullptr;
+    if (m < 0 || n < 0 || nnz < 0 || n > 0x7fffffffLL || m > 0x7fffffffLL) return DASP_ERR_INVALID_ARG;
+    if (dtype != DASP_R_64F && dtype != DASP_R_16F) return DASP_ERR_INVALID_ARG;
+    if (!row_ptr || (nnz > 0 && (!col_idx || !val))) return DASP_ERR_INVALID_ARG;
+    dasp_options_default(&o);
+    if (opts) o = *opts;
+    if (o.variant != DASP_VARIANT_MMA && o.variant != DASP_VARIANT_CUDACORE) o.variant = DASP_VARIANT_CUDACORE;
+    return DASP_OK;
+}
+
+int64_t resolve_panel_rows(const dasp_options_t& o) {
+    // panel size (R28): -1 one panel (the paper's global format); 0 automatic; env override
+    int64_t panel_rows = o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
+    if (const char* pr = std::getenv("DASP_PANEL_ROWS")) panel_rows = std::atoll(pr);
+    return panel_rows;
+}
+
+dasp_status_t fail(dasp_plan_s* p, dasp_status_t st) {
     if (p->device >= 0) {
         DeviceGuard guard(p->device);
+        free_device(p);
+    }
+    p->host.release();
+    delete p;
+    return st;
+}
+
+}  // namespace
+
+extern "C" {
+
+dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz, const int64_t* row_ptr,
+                               const int32_t* col_idx, const void* val, dasp_dtype_t dtype, const dasp_options_t* opts) {
+    dasp_options_t o;
+    dasp_status_t st = check_create_args(plan_out, m, n, nnz, row_ptr, col_idx, val, dtype, opts, o);
+    if (st != DASP_OK) return st;
+    if (o.validate && row_ptr[m] != nnz) return DASP_ERR_INVALID_CSR;
+
+    dasp_plan_s* p = new (std::nothrow) dasp_plan_s;
+    if (!p) return DASP_ERR_OUT_OF_MEMORY;
+    p->dtype = dtype;
+    p->device = o.device;
+    p->variant = o.variant;
+    p->keep_host = o.keep_host != 0 || o.device < 0;
+
+    auto t0 = std::chrono::steady_clock::now();
+    int bst = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0,
+                                 resolve_panel_rows(o), o.max_len, o.threshold);
+    auto t1 = std::chrono::steady_clock::now();
+    p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    if (bst != DASP_OK) {
+        delete p;
+        return static_cast<dasp_status_t>(bst);
+    }
+    HostFormat& f = p->host;
+    for (int a = 0; a < DASP_ARR_COUNT; ++a) p->bytes[a] = f.arr[a].bytes;
+    std::vector<int32_t> first_col(static_cast<size_t>(f.n_groups_padded / f.geo.UG));
+    {
+        const int32_t* lc = static_cast<const int32_t*>(f.arr[DASP_ARR_LONG_COL].ptr);
+        const int64_t ue = static_cast<int64_t>(f.geo.UG) * f.geo.G;
+        for (size_t u = 0; u < first_col.size(); ++u) first_col[u] = lc[u * ue];
+    }
+    std::unique_ptr<DeviceGuard> guard;
+    if (p->device >= 0) guard.reset(new DeviceGuard(p->device));
+    st = setup_launch(p, o, static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr), first_col);
+    if (st != DASP_OK) return fail(p, st);
+    if (p->device >= 0) {
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
             if (p->bytes[a] == 0) continue;
             // 256 B alignment from cudaMalloc keeps every lane's 16/32 B vector load aligned
-            if (cudaMalloc(&p->d[a], static_cast<size_t>(p->bytes[a] + kAllocPad)) != cudaSuccess) {
-                free_device(p); f.release(); delete p;
-                return DASP_ERR_OUT_OF_MEMORY;
-            }
+            if (cudaMalloc(&p->d[a], static_cast<size_t>(p->bytes[a] + kAllocPad)) != cudaSuccess)
+                return fail(p, DASP_ERR_OUT_OF_MEMORY);
             p->device_bytes += p->bytes[a];
-        }
-        const int64_t pb = std::max<int64_t>(f.n_groups_padded, 1) * sy(dtype);
-        if (cudaMalloc(&p->d_partial, static_cast<size_t>(pb)) != cudaSuccess) {
-            free_device(p); f.release(); delete p;
-            return DASP_ERR_OUT_OF_MEMORY;
-        }
-        p->device_bytes += pb;
-        const size_t db = desc.size() * sizeof(dasp::PanelDesc), bb = std::max<size_t>(blk_panel.size(), 1) * 4;
-        if (cudaMalloc(&p->d_panels, std::max<size_t>(db, 1)) != cudaSuccess || cudaMalloc(&p->d_blk_panel, bb) != cudaSuccess) {
-            free_device(p); f.release(); delete p;
-            return DASP_ERR_OUT_OF_MEMORY;
-        }
-        if ((db && cudaMemcpy(p->d_panels, desc.data(), db, cudaMemcpyHostToDevice) != cudaSuccess) ||
-            (!blk_panel.empty() && cudaMemcpy(p->d_blk_panel, blk_panel.data(), blk_panel.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)) {
-            free_device(p); f.release(); delete p;
-            return DASP_ERR_CUDA;
-        }
-        p->device_bytes += db + bb;
-        const size_t ub = std::max<size_t>(unit_order.size(), 1) * 4;
-        if (cudaMalloc(&p->d_unit_order, ub) != cudaSuccess) { free_device(p); f.release(); delete p; return DASP_ERR_OUT_OF_MEMORY; }
-        if (!unit_order.empty() && cudaMemcpy(p->d_unit_order, unit_order.data(), unit_order.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) {
-            free_device(p); f.release(); delete p;
-            return DASP_ERR_CUDA;
-        }
-        p->device_bytes += ub;
-        if (p->pipe) {
-            const size_t ib = std::max<size_t>(items.size(), 1) * 8;
-            int bps = 0, nsm = 0;
-            if (cudaMalloc(&p->d_items, ib) != cudaSuccess) { free_device(p); f.release(); delete p; return DASP_ERR_OUT_OF_MEMORY; }
-            if ((!items.empty() && cudaMemcpy(p->d_items, items.data(), items.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess) ||
-                dasp::pipe_occupancy(p->dtype, DASP_VARIANT_CUDACORE, &bps) != cudaSuccess ||   // sets both kernels'
-                dasp::pipe_occupancy(p->dtype, DASP_VARIANT_MMA, &bps) != cudaSuccess ||        // smem attribute
-                cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess) {
-                free_device(p); f.release(); delete p;
-                return DASP_ERR_CUDA;
-            }
-            // persistent grid: every SM full, never more warps than items
-            const int64_t wpb = dasp::pipe_warps_per_block();
-            p->pipe_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->n_items + wpb - 1) / wpb);
-            p->device_bytes += ib;
-        }
-        // optional persisting L2 access-policy window over x (DASP_X_APW=1; measured slower on
-        // C3, profiles/r01, so off by default)
-        const char* apw = std::getenv("DASP_X_APW");
-        if (apw && std::atoi(apw) > 0) {
-            cudaDeviceProp prop;
-            if (cudaGetDeviceProperties(&prop, p->device) == cudaSuccess && prop.persistingL2CacheMaxSize > 0) {
-                const size_t xb = static_cast<size_t>(f.n) * sx(dtype);
-                size_t lim = std::min<size_t>(static_cast<size_t>(prop.persistingL2CacheMaxSize), xb);
-                size_t win = std::min<size_t>(static_cast<size_t>(prop.accessPolicyMaxWindowSize), xb);
-                if (lim > 0 && win > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim) == cudaSuccess) {
-                    p->apw_bytes = win;
-                    p->apw_hit = std::min(1.0f, static_cast<float>(lim) / static_cast<float>(win));
-                }
-            }
-            cudaGetLastError();
         }
         auto u0 = std::chrono::steady_clock::now();
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
             if (p->bytes[a] == 0) continue;
-            if (cudaMemcpy(p->d[a], f.arr[a].ptr, static_cast<size_t>(p->bytes[a]), cudaMemcpyHostToDevice) != cudaSuccess) {
-                free_device(p); f.release(); delete p;
-                return DASP_ERR_CUDA;
-            }
+            if (cudaMemcpy(p->d[a], f.arr[a].ptr, static_cast<size_t>(p->bytes[a]), cudaMemcpyHostToDevice) != cudaSuccess)
+                return fail(p, DASP_ERR_CUDA);
         }
         auto u1 = std::chrono::steady_clock::now();
         p->upload_ms = std::chrono::duration<double, std::milli>(u1 - u0).count();
         if (!p->keep_host) f.release();
     }
+    *plan_out = p;
+    return DASP_OK;
+}
+
+dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz,
+                                      const int64_t* d_row_ptr, const int32_t* d_col_idx, const void* d_val,
+                                      dasp_dtype_t dtype, const dasp_options_t* opts, void* stream) {
+    dasp_options_t o;
+    dasp_status_t st = check_create_args(plan_out, m, n, nnz, d_row_ptr, d_col_idx, d_val, dtype, opts, o);
+    if (st != DASP_OK) return st;
+    if (o.device < 0) return DASP_ERR_INVALID_ARG;
+    dasp_plan_s* p = new (std::nothrow) dasp_plan_s;
+    if (!p) return DASP_ERR_OUT_OF_MEMORY;
+    p->dtype = dtype;
+    p->device = o.device;
+    p->variant = o.variant;
+    p->keep_host = false;
+    DeviceGuard guard(p->device);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    auto t0 = std::chrono::steady_clock::now();
+    int bst = dasp::build_format_device(p->host, p->d, dtype, m, n, d_row_ptr, d_col_idx, d_val, o.validate != 0,
+                                        resolve_panel_rows(o), o.max_len, o.threshold, s);
+    auto t1 = std::chrono::steady_clock::now();
+    p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    if (bst != DASP_OK) {
+        delete p;
+        return static_cast<dasp_status_t>(bst);
+    }
+    HostFormat& f = p->host;
+    if (f.nnz != nnz) return fail(p, DASP_ERR_INVALID_CSR);
+    for (int a = 0; a < DASP_ARR_COUNT; ++a) {
+        p->bytes[a] = f.arr[a].bytes;
+        p->device_bytes += p->bytes[a];
+    }
+    // first column of every long unit, gathered on the device
+    std::vector<int32_t> first_col(static_cast<size_t>(f.n_groups_padded / f.geo.UG));
+    if (!first_col.empty() &&
+        dasp::gather_unit_first_col(static_cast<const int32_t*>(p->d[DASP_ARR_LONG_COL]), f.geo.UG * f.geo.G,
+                                    static_cast<int64_t>(first_col.size()), first_col.data(), s) != cudaSuccess)
+        return fail(p, DASP_ERR_CUDA);
+    st = setup_launch(p, o, f.panel_table.data(), first_col);
+    if (st != DASP_OK) return fail(p, st);
     *plan_out = p;
     return DASP_OK;
 }

@@ -3,6 +3,7 @@
 #pragma once
 #include <cstddef>
 #include <cstdint>
+#include <vector>
 
 #include "../../include/dasp.h"
 
@@ -47,6 +48,7 @@ struct HostFormat {
     int64_t sumsq_medium = 0;  // sum of squared medium row lengths (launch tuning)
     int64_t max_len = MAX_LEN; // long iff len > max_len
     double tau = 0.75;         // regular iff count > BE * tau
+    std::vector<int64_t> panel_table;   // device-built plans: host copy of the panel table
     int64_t panel_rows = 0;   // rows per panel (R28); >= m: one panel = the paper's global format
     int64_t n_panels = 0;
     HostBuf arr[DASP_ARR_COUNT];

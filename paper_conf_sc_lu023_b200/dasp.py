@@ -26,7 +26,7 @@ STATUS = ["DASP_OK", "DASP_ERR_INVALID_ARG", "DASP_ERR_INVALID_CSR", "DASP_ERR_O
           "DASP_ERR_CUDA", "DASP_ERR_UNSUPPORTED", "DASP_ERR_INTERNAL"]
 
 # every symbol include/dasp.h declares (tests check the library exports all of them)
-EXPORTS = ["dasp_options_default", "dasp_plan_create", "dasp_spmv", "dasp_spmv_ex", "dasp_spmv_scatter", "dasp_spmv_host",
+EXPORTS = ["dasp_options_default", "dasp_plan_create", "dasp_plan_create_device", "dasp_spmv", "dasp_spmv_ex", "dasp_spmv_scatter", "dasp_spmv_host",
            "dasp_plan_destroy", "dasp_status_string", "dasp_plan_get_info", "dasp_plan_copy_array",
            "dasp_partition_rows", "dasp_remap_columns", "dasp_plan_set_timing", "dasp_plan_read_timing",
            "dasp_version"]
@@ -73,6 +73,8 @@ def _load():
         "dasp_options_default": ([ctypes.POINTER(Options)], None),
         "dasp_plan_create": ([ctypes.POINTER(vp), i64, i64, i64, vp, vp, vp, ctypes.c_int, ctypes.POINTER(Options)],
                              ctypes.c_int),
+        "dasp_plan_create_device": ([ctypes.POINTER(vp), i64, i64, i64, vp, vp, vp, ctypes.c_int,
+                                     ctypes.POINTER(Options), vp], ctypes.c_int),
         "dasp_spmv": ([vp, vp, vp, d, d, vp], ctypes.c_int),
         "dasp_spmv_ex": ([vp, vp, vp, d, d, vp, i32], ctypes.c_int),
         "dasp_spmv_host": ([vp, vp, vp, d, d, vp], ctypes.c_int),
@@ -184,6 +186,32 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))
     _check(st, "dasp_plan_create")
+    return Plan(h, dtype, m, n)
+
+
+def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
+                            variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, medium_rb_per_warp: int = 0,
+                            panel_rows: int = 0, pipeline: bool = False, max_len: int = 256, threshold: float = 0.75,
+                            stream=None) -> Plan:
+    """Build the plan on the GPU from a device CSR (torch CUDA tensors: int64 row_ptr, int32
+    col_idx, float64 / float16 val) -- SURVEY.md §8(f) f2."""
+    import torch
+    want = torch.float64 if dtype == "f64" else torch.float16
+    for t, dt_ in ((row_ptr, torch.int64), (col_idx, torch.int32), (val, want)):
+        if not isinstance(t, torch.Tensor) or not t.is_cuda or t.dtype != dt_ or not t.is_contiguous():
+            raise ValueError("dasp_plan_create_device needs contiguous CUDA tensors (int64, int32, value dtype)")
+    if row_ptr.numel() != m + 1:
+        raise ValueError("row_ptr must have m+1 entries")
+    opts = Options()
+    _lib.dasp_options_default(ctypes.byref(opts))
+    opts.device, opts.variant, opts.validate = device, variant, int(validate)
+    opts.medium_rb_per_warp, opts.panel_rows, opts.pipeline = medium_rb_per_warp, panel_rows, int(pipeline)
+    opts.max_len, opts.threshold = int(max_len), float(threshold)
+    h = ctypes.c_void_p()
+    st = _lib.dasp_plan_create_device(ctypes.byref(h), m, n, int(col_idx.numel()), _ptr(row_ptr), _ptr(col_idx),
+                                      _ptr(val), DASP_R_64F if dtype == "f64" else DASP_R_16F, ctypes.byref(opts),
+                                      _stream_ptr(stream))
+    _check(st, "dasp_plan_create_device")
     return Plan(h, dtype, m, n)
 
 
