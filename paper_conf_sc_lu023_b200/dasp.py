@@ -140,7 +140,7 @@ class Plan:
         self.m, self.n = m, n
 
     def __del__(self):
-        if getattr(self, "handle", None):
+        if getattr(self, "handle", None) and _lib is not None:   # _lib is None at interpreter exit
             _lib.dasp_plan_destroy(self.handle)
             self.handle = None
 

@@ -15,4 +15,4 @@ for name in ["c3", "c2"]:
     h = dasp.dasp_plan_create(A.row_ptr, A.col, A.val, A.m, A.n, "f64")
     print(name, "host build", h.info["build_ms"], "upload", h.info["upload_ms"], "wall", (time.perf_counter() - t) * 1e3, flush=True)
 PY
-DASP_GB_TRACE=1 timeout 600 python /tmp/gbt.py > gpurun_out/gbt.log 2>&1; tail -40 gpurun_out/gbt.log
+DASP_GB_TRACE=1 PYTHONPATH=$PWD timeout 600 python /tmp/gbt.py > gpurun_out/gbt.log 2>&1; tail -40 gpurun_out/gbt.log
