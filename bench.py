@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--config", default="c2")            # configs[1]: 27-point stencil 128^3, FP64
     ap.add_argument("--scale", type=float, default=1.0)
-    ap.add_argument("--dtype", default="f64", choices=["f64", "f16"])
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f16", "f32"])
     ap.add_argument("--variant", default="cudacore", choices=["mma", "cudacore"])
     ap.add_argument("--no-compare", action="store_true", help="skip timing the other compute variant")
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
@@ -127,27 +127,31 @@ class ClockSampler:
 # ----------------------------------------------------------------------------------------------
 # bytes per launch: CSR-equivalent and algorithmic (what the DASP format moves)
 # ----------------------------------------------------------------------------------------------
-def byte_model(info, dtype, beta_nonzero=False):
+def byte_model(info, dtype, beta_nonzero=False, split_short=False):
     """Algorithmic bytes per launch of each kernel."""
-    sv, sx, sy = (8, 8, 8) if dtype == "f64" else (2, 2, 4)
-    sa = sy
+    sv, sx, sy = {"f64": (8, 8, 8), "f16": (2, 2, 4), "f32": (4, 4, 4)}[dtype]
+    sa = 4 if dtype == "f16" else 8
     b1 = 2 if beta_nonzero else 1
     m, n, nnz = info["m"], info["n"], info["nnz"]
-    G = 64 if dtype == "f64" else 128
+    G = 128 if dtype == "f16" else 64
     ngp = info["n_groups_padded"]
     nrb = info["rowblocks"]
     nout = 64 * info["tiles_13"] + 32 * info["tiles_4"] + 64 * info["tiles_22"] + 128 * info["tiles_single"]
     n_short_rows = info["n_len1"] + info["n_len2"] + info["n_len3"] + info["n_len4"]
     long_ = ngp * G * (sv + 4) + ngp * sa + 4 * (ngp // 4)          # slots, group partials, unit order
-    main = ((info["nnz_reg_new"] + info["nnz_irreg"]) * (sv + 4) + 8 * (nrb + 1) + 8 * (8 * nrb + 1) + 4 * 8 * nrb
-            + info["row_medium"] * sy * b1
-            + info["nnz_short_new"] * (sv + 4) + 4 * nout + n_short_rows * sy * b1
-            + n * sx)                                                   # x counted once, here
+    medium = ((info["nnz_reg_new"] + info["nnz_irreg"]) * (sv + 4) + 8 * (nrb + 1) + 8 * (8 * nrb + 1)
+              + 4 * 8 * nrb + info["row_medium"] * sy * b1)
+    short = info["nnz_short_new"] * (sv + 4) + 4 * nout + n_short_rows * sy * b1
+    main = medium + (0 if split_short else short) + n * sx           # x counted once, here
     finish = (ngp * sa + 8 * (info["row_long"] + 1) + 4 * info["row_long"] + info["row_long"] * sy * b1
               + info["n_empty"] * (4 + sy * b1))
     csr_equiv = nnz * (sv + 4) + (m + 1) * 8 + n * sx + m * sy * b1
-    return {"dasp_long_kernel": long_, "dasp_main_kernel": main, "dasp_finish_kernel": finish,
-            "total": long_ + main + finish, "csr_equiv": csr_equiv}
+    out = {"dasp_long_kernel": long_, "dasp_main_kernel": main, "dasp_finish_kernel": finish,
+           "total": long_ + main + finish + (short if split_short else 0), "csr_equiv": csr_equiv}
+    if split_short:
+        out["dasp_short_kernel"] = short + 8 * info["tiles_13"] + 8 * info["tiles_4"] + 8 * info["tiles_22"] \
+            + 8 * info["tiles_single"]                                    # + per-tile metadata
+    return out
 
 
 def load_peaks():
@@ -213,8 +217,9 @@ def row_sample(A, target_nnz):
 
 def time_oracle(A, x, dtype, budget_s):
     import oracle
-    val = A.val if dtype == "f64" else A.val.astype(np.float16).astype(np.float64)
-    xv = x if dtype == "f64" else x.astype(np.float16).astype(np.float64)
+    narrow = {"f64": np.float64, "f16": np.float16, "f32": np.float32}[dtype]
+    val = A.val.astype(narrow).astype(np.float64)
+    xv = x.astype(narrow).astype(np.float64)
     oracle.spmv(A.row_ptr[:2], A.col[:1], val[:1], xv)  # load the library
     reps, t_total = 0, 0.0
     while t_total < budget_s and reps < 50:
@@ -268,10 +273,10 @@ def main():
     use_slab = world > 1 or args.iterate
     slab = build_slab(gen_rows, lens, rank, world, reduce_max, need_norm=use_slab)
     gen_s = time.perf_counter() - t0
-    if args.dtype == "f16":
+    if args.dtype != "f64":
         if world > 1:
-            raise SystemExit("FP16 multi-GPU is not part of the north star (x f16 vs y f32)")
-        slab.val = slab.val.astype(np.float16)
+            raise SystemExit("FP16 / FP32 multi-GPU is not part of the north star")
+        slab.val = slab.val.astype(np.float16 if args.dtype == "f16" else np.float32)
     x_global = synth.vector(101, spec.n)
 
     t1 = time.perf_counter()
@@ -280,7 +285,7 @@ def main():
         plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
                                      device=local, variant=variant, medium_rb_per_warp=args.rbw,
                                      pipeline=args.pipeline, panel_rows=args.panel_rows)
-        xdt = torch.float64 if args.dtype == "f64" else torch.float16
+        xdt = {"f64": torch.float64, "f16": torch.float16, "f32": torch.float32}[args.dtype]
         ydt = torch.float64 if args.dtype == "f64" else torch.float32
         xd = torch.from_numpy(x_global).to(xdt).to(dev)
         yd = torch.zeros(slab.rows, dtype=ydt, device=dev)
@@ -351,7 +356,7 @@ def main():
     nnz_total = int(lens.sum())
     flops_step = 2.0 * nnz_total
     gflops = flops_step / (ms_step * 1e-3) / 1e9
-    bm = byte_model(info, args.dtype)
+    bm = byte_model(info, args.dtype, split_short=kern.get("dasp_short_kernel", (0, 0))[1] > 0)
     # whole-job CSR-equivalent bytes: sum over ranks (slab models), else the local one
     csr_bytes = bm["csr_equiv"]
     if world > 1:
@@ -409,7 +414,7 @@ def main():
                "h2d_bytes_per_step": int(xh.numel() * 8) * world, "d2h_bytes_per_step": int(yh.numel() * 8) * world,
                "api": "dasp_spmv" + ("_scatter" if args.fused else "") + " (row-slab iteration)"}
     if not use_slab and args.e2e_steps > 0:
-        xdt_np = np.float64 if args.dtype == "f64" else np.float16
+        xdt_np = {"f64": np.float64, "f16": np.float16, "f32": np.float32}[args.dtype]
         xh = torch.from_numpy(x_global.astype(xdt_np)).pin_memory()
         yh = torch.empty(slab.rows, dtype=torch.float64 if args.dtype == "f64" else torch.float32).pin_memory()
         dasp.dasp_spmv_host(plan, xh.data_ptr(), yh.data_ptr(), 1.0, 0.0, stream)
@@ -426,7 +431,7 @@ def main():
     gpu_build = None
     if not use_slab and not args.no_gpu_build:
         try:
-            vdt = torch.float64 if args.dtype == "f64" else torch.float16
+            vdt = {"f64": torch.float64, "f16": torch.float16, "f32": torch.float32}[args.dtype]
             d_rp = torch.from_numpy(slab.row_ptr).to(dev)
             d_col = torch.from_numpy(np.ascontiguousarray(slab.col)).to(dev)
             d_val = torch.from_numpy(np.ascontiguousarray(slab.val)).to(vdt).to(dev)
@@ -448,8 +453,7 @@ def main():
     # ---- CPU oracle on the host cores (rank 0, N = 1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        A = synth.CSR(slab.rows, spec.n, slab.row_ptr, slab.col,
-                      slab.val.astype(np.float64) if args.dtype == "f16" else slab.val)
+        A = synth.CSR(slab.rows, spec.n, slab.row_ptr, slab.col, slab.val.astype(np.float64))
         target = max(1, int(min(A.nnz, 1.5e8)))
         S, stride = row_sample(A, target)
         per, reps = time_oracle(S, x_global, args.dtype, args.cpu_budget_s)
@@ -498,14 +502,14 @@ def run_reference(args, spec, workload, metric, rank, world):
     lens = synth.row_lengths(spec)
     nnz = int(lens.sum())
     A = synth.generate(spec)
-    if args.dtype == "f16":
-        A.val = A.val.astype(np.float16).astype(np.float64)
+    narrow = {"f64": np.float64, "f16": np.float16, "f32": np.float32}[args.dtype]
+    A.val = A.val.astype(narrow).astype(np.float64)
     x = synth.vector(101, spec.n)
     total = args.steps + max(args.warmup, 3)
     per_step_nnz = int(np.clip(90.0 * 2.5e8 / total, 2e5, nnz))   # ~90 s of oracle work in all
     S, stride = row_sample(A, per_step_nnz)
     import oracle
-    xv = x.astype(np.float16).astype(np.float64) if args.dtype == "f16" else x
+    xv = x.astype(narrow).astype(np.float64)
     for _ in range(max(args.warmup, 3)):
         oracle.spmv(S.row_ptr, S.col, S.val, xv)
     t0 = time.perf_counter()

@@ -36,7 +36,7 @@ extern "C" {
 
 typedef struct dasp_plan_s* dasp_plan_t;
 
-typedef enum { DASP_R_64F = 0, DASP_R_16F = 1 } dasp_dtype_t;
+typedef enum { DASP_R_64F = 0, DASP_R_16F = 1, DASP_R_32F = 2 } dasp_dtype_t;
 
 typedef enum {
     DASP_OK = 0,
@@ -116,7 +116,8 @@ typedef struct {
  *   row_ptr   : HOST int64[m+1], row_ptr[0] = 0, non-decreasing, row_ptr[m] = nnz.
  *   col_idx   : HOST int32[nnz], 0 <= col < n.  Unsorted columns and duplicates are allowed
  *               (duplicates are summed like any other entry).
- *   val       : HOST double[nnz] (DASP_R_64F) or uint16_t[nnz] binary16 bits (DASP_R_16F).
+ *   val       : HOST double[nnz] (DASP_R_64F), uint16_t[nnz] binary16 bits (DASP_R_16F) or
+ *               float[nnz] (DASP_R_32F).
  *   opts      : NULL for defaults.
  *
  * Copies everything it needs (the caller may free the CSR on return), builds the DASP
@@ -144,8 +145,8 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
 /*
  * dasp_spmv — the hot path (§3.3, Alg. 2-5):  y = alpha*A*x + beta*y.
  *
- *   x : DEVICE pointer on the plan's device, n elements (f64, or f16 bits for DASP_R_16F).
- *   y : DEVICE pointer, m elements (f64, or f32 for DASP_R_16F).  Read only if beta != 0
+ *   x : DEVICE pointer on the plan's device, n elements (f64 / f16 bits / f32 by dtype).
+ *   y : DEVICE pointer, m elements (f64 / f32 / f32 by dtype).  Read only if beta != 0
  *       (BLAS convention: beta == 0 overwrites y, NaNs in y do not propagate).
  *   stream : cudaStream_t as void* (NULL = default stream).  Enqueue only; no host sync.
  *
@@ -236,7 +237,8 @@ typedef enum {
     DASP_K_FINISH = 1,    /* long phase 2 (Alg. 2 l.17-25) + empty rows */
     DASP_K_SCALE = 2,     /* alpha == 0 quick path */
     DASP_K_LONG = 3,      /* long phase 1 (Alg. 2 l.1-16) */
-    DASP_K_COUNT = 4
+    DASP_K_SHORT = 4,     /* short tiles when they run in their own kernel (DASP_SPLIT_SHORT) */
+    DASP_K_COUNT = 5
 } dasp_kernel_t;
 
 /*

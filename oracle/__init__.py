@@ -90,7 +90,8 @@ def tolerance_ok(y, y_ref, s, dtype="f64"):
 
     Rows with s == 0 must match exactly; NaN must match NaN; Inf must match sign."""
     y = np.asarray(y, dtype=np.float64)
-    tol = 1e-12 if dtype == "f64" else 2e-3
+    # FP32 (R29): f64 arithmetic then one rounding to f32 -> |err| <= 2^-24 |y| + tiny <= 1e-7 s
+    tol = {"f64": 1e-12, "f32": 1e-7}.get(dtype, 2e-3)
     nan_ref, nan_y = np.isnan(y_ref), np.isnan(y)
     inf_ref = np.isinf(y_ref)
     fin = ~(nan_ref | inf_ref)
@@ -107,8 +108,8 @@ class Format:
 
     def __init__(self, A, dtype="f64", panel_rows=0, max_len=256, tau=0.75):
         lib = _L()
-        dt = 0 if dtype == "f64" else 1
-        val = np.ascontiguousarray(A.val.astype(np.float64 if dt == 0 else np.float16))
+        dt = {"f64": 0, "f16": 1, "f32": 2}[dtype]
+        val = np.ascontiguousarray(A.val.astype({0: np.float64, 1: np.float16, 2: np.float32}[dt]))
         rp = np.ascontiguousarray(A.row_ptr, dtype=np.int64)
         col = np.ascontiguousarray(A.col, dtype=np.int32)
         h = lib.oracle_build(dt, A.m, A.n, _p(rp), _p(col), _p(val), int(panel_rows), int(max_len), float(tau))
@@ -127,7 +128,7 @@ class Format:
     def view(self, name):
         b = self.arrays[name]
         if name.endswith("_val"):
-            return b.view(np.float64 if self.dtype == "f64" else np.float16)
+            return b.view({"f64": np.float64, "f16": np.float16, "f32": np.float32}[self.dtype])
         if name in ("group_ptr", "rb_ptr", "irr_ptr", "panels"):
             return b.view(np.int64)
         return b.view(np.int32)

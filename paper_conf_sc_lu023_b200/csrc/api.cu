@@ -36,6 +36,9 @@ struct dasp_plan_s {
     double build_ms = 0, upload_ms = 0;
     int64_t blocks = 0;                   // grid of the medium/short kernel
     int64_t n_units = 0;                  // long units (long kernel)
+    bool split_short = false;             // short tiles in their own kernel (else in the main kernel)
+    int64_t n_tiles = 0;
+    void* d_tile_meta = nullptr;          // uint64 cat << 62 | output base, per tile (split mode)
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
     void* d_blk_panel = nullptr;          // int32 panel of every block
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
@@ -53,13 +56,15 @@ struct dasp_plan_s {
 
 namespace {
 
-int sx(int dtype) { return dtype == DASP_R_64F ? 8 : 2; }
+int sx(int dtype) { return dtype == DASP_R_64F ? 8 : (dtype == DASP_R_32F ? 4 : 2); }
 int sy(int dtype) { return dtype == DASP_R_64F ? 8 : 4; }
+int sa(int dtype) { return dtype == DASP_R_16F ? 4 : 8; }   // long-group partials: f32 (FP16) / f64
 
 // automatic panel: ~1M rows keeps a panel's x window and y (8 B each per row) well inside the
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
+constexpr bool kSplitShortDefault = false;
 constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // TMA windows may read up to 16 B past an array's end
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
@@ -97,7 +102,8 @@ void free_device(dasp_plan_s* p) {
     if (p->d_blk_panel) cudaFree(p->d_blk_panel);
     if (p->d_unit_order) cudaFree(p->d_unit_order);
     if (p->d_items) cudaFree(p->d_items);
-    p->d_panels = p->d_blk_panel = p->d_unit_order = p->d_items = nullptr;
+    if (p->d_tile_meta) cudaFree(p->d_tile_meta);
+    p->d_panels = p->d_blk_panel = p->d_unit_order = p->d_items = p->d_tile_meta = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -130,7 +136,7 @@ cudaError_t timed(dasp_plan_s* p, int kernel, cudaStream_t s, bool on, F&& launc
 
 int64_t alg_bytes(const dasp_plan_s* p, bool beta) {
     const HostFormat& f = p->host;
-    const int64_t s_v = f.geo.sv, s_x = sx(p->dtype), s_y = sy(p->dtype), s_a = s_y;
+    const int64_t s_v = f.geo.sv, s_x = sx(p->dtype), s_y = sy(p->dtype), s_a = sa(p->dtype);
     const int64_t nmp = f.nrb * 8;
     const int64_t nout = 64 * f.t13 + 32 * f.t4 + 64 * f.t22 + 128 * f.ts;
     int64_t b = 0;
@@ -189,6 +195,11 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<int32_t> blk_panel;
+    std::vector<uint64_t> tile_meta;
+    {
+        const char* ss = std::getenv("DASP_SPLIT_SHORT");
+        p->split_short = ss ? std::atoi(ss) != 0 : kSplitShortDefault;
+    }
     int64_t blk = 0;
     for (int64_t q = 0; q < f.n_panels; ++q) {
         const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
@@ -196,6 +207,18 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         d.blk0 = blk;
         d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5]; d.nmw = (e[5] + p->rbw - 1) / p->rbw;
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
+        if (p->split_short) {   // tiles leave the main kernel; per-tile metadata for the short kernel
+            for (int64_t t = 0; t < d.t13 + d.t4 + d.t22 + d.ts; ++t) {
+                uint64_t cat;
+                int64_t ob;
+                if (t < d.t13) { cat = 0; ob = d.out0 + t * 64; }
+                else if (t < d.t13 + d.t4) { cat = 1; ob = d.out0 + 64 * d.t13 + (t - d.t13) * 32; }
+                else if (t < d.t13 + d.t4 + d.t22) { cat = 2; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + (t - d.t13 - d.t4) * 64; }
+                else { cat = 3; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + 64 * d.t22 + (t - d.t13 - d.t4 - d.t22) * 128; }
+                tile_meta.push_back((cat << 62) | static_cast<uint64_t>(ob));
+            }
+            d.t13 = d.t4 = d.t22 = d.ts = 0;
+        }
         const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
         const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
         blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
@@ -203,6 +226,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     }
     p->blocks = blk;
     p->n_units = f.n_groups_padded / f.geo.UG;
+    p->n_tiles = static_cast<int64_t>(tile_meta.size());
     // long-unit execution order (a launch schedule, not part of the format): inside each panel
     // the units run bucketed by the column of their first element, so that the warps in flight
     // gather from ~1/kColBuckets of x at a time instead of all of it (long rows' columns are
@@ -252,7 +276,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         }
     }
     p->n_items = static_cast<int64_t>(items.size());
-    p->pipe = want_pipe && items_ok;
+    p->pipe = want_pipe && items_ok && p->dtype != DASP_R_32F;   // the staged kernel covers FP64 / FP16
     if (p->device < 0) return DASP_OK;
 
     auto upload = [&](void** dst, const void* src, size_t bytes) -> dasp_status_t {
@@ -261,13 +285,14 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         if (bytes && cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice) != cudaSuccess) return DASP_ERR_CUDA;
         return DASP_OK;
     };
-    const int64_t pb = std::max<int64_t>(f.n_groups_padded, 1) * sy(p->dtype);
+    const int64_t pb = std::max<int64_t>(f.n_groups_padded, 1) * sa(p->dtype);
     if (cudaMalloc(&p->d_partial, static_cast<size_t>(pb)) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
     p->device_bytes += pb;
     dasp_status_t st;
     if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
     if ((st = upload(&p->d_blk_panel, blk_panel.data(), blk_panel.size() * 4)) != DASP_OK) return st;
     if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
+    if (p->split_short && (st = upload(&p->d_tile_meta, tile_meta.data(), tile_meta.size() * 8)) != DASP_OK) return st;
     if (p->pipe) {
         int bps = 0, nsm = 0;
         if ((st = upload(&p->d_items, items.data(), items.size() * 8)) != DASP_OK) return st;
@@ -304,7 +329,7 @@ dasp_status_t check_create_args(dasp_plan_t* plan_out, int64_t m, int64_t n, int
     if (!plan_out) return DASP_ERR_INVALID_ARG;
     *plan_out = nullptr;
     if (m < 0 || n < 0 || nnz < 0 || n > 0x7fffffffLL || m > 0x7fffffffLL) return DASP_ERR_INVALID_ARG;
-    if (dtype != DASP_R_64F && dtype != DASP_R_16F) return DASP_ERR_INVALID_ARG;
+    if (dtype != DASP_R_64F && dtype != DASP_R_16F && dtype != DASP_R_32F) return DASP_ERR_INVALID_ARG;
     if (!row_ptr || (nnz > 0 && (!col_idx || !val))) return DASP_ERR_INVALID_ARG;
     dasp_options_default(&o);
     if (opts) o = *opts;
@@ -508,6 +533,12 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
         e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s); });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }
+    if (!p->pipe && p->split_short && p->n_tiles > 0 && (mp.class_mask & 4)) {
+        e = timed(p, DASP_K_SHORT, s, on, [&] {
+            return dasp::launch_short(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_tile_meta), p->n_tiles, s);
+        });
+        if (e != cudaSuccess) return DASP_ERR_CUDA;
+    }
     e = timed(p, DASP_K_MAIN, s, on, [&] {
         if (p->pipe)
             return dasp::launch_pipe(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_items), p->n_items,
@@ -587,7 +618,8 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
     o->launches_per_spmv = p->pipe ? (p->n_items > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0)
-                                   : (p->n_units > 0 ? 1 : 0) + (p->blocks > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0);
+                                   : (p->n_units > 0 ? 1 : 0) + (p->blocks > 0 ? 1 : 0) + (p->n_tiles > 0 ? 1 : 0) +
+                                         (f.row_long + f.n0 > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
     o->pipeline = p->pipe ? 1 : 0;

@@ -56,8 +56,8 @@ inline int64_t reg_pos(const Geometry& geo, int64_t nreg, int g, int64_t s) {
 }
 
 // position of (4-slot row r in [0,32), inner slot c in [0,4)) inside a short tile
-inline int short_pos(int sv, int r, int c) {
-    if (sv == 8) return 4 * (4 * (r & 7) + c) + (r >> 3);      // lane (g=r&7, t=c), j = r>>3
+inline int short_pos(int K, int r, int c) {
+    if (K == 4) return 4 * (4 * (r & 7) + c) + (r >> 3);       // m8n8k4: lane (g=r&7, t=c), j = r>>3
     int q = r >> 3, g = r & 7;
     int t = ((q & 1) << 1) | (c >> 1);
     int j = ((q >> 1) << 1) | (c & 1);
@@ -245,9 +245,9 @@ void fill_panel(HostFormat& f, const Panel& P, const int64_t* rp, const int32_t*
         auto put_row4 = [&](int64_t tile, int r, int64_t ra, int la, int64_t rb_, int lb) {
             V* tv = sv + tile * SHORT_TILE;
             int32_t* tc = sc + tile * SHORT_TILE;
-            for (int k = 0; k < la; ++k) { const int p = short_pos(geo.sv, r, k); tv[p] = val[rp[ra] + k]; tc[p] = col[rp[ra] + k]; }
+            for (int k = 0; k < la; ++k) { const int p = short_pos(geo.K, r, k); tv[p] = val[rp[ra] + k]; tc[p] = col[rp[ra] + k]; }
             if (rb_ >= 0)
-                for (int k = 0; k < lb; ++k) { const int p = short_pos(geo.sv, r, la + k); tv[p] = val[rp[rb_] + k]; tc[p] = col[rp[rb_] + k]; }
+                for (int k = 0; k < lb; ++k) { const int p = short_pos(geo.K, r, la + k); tv[p] = val[rp[rb_] + k]; tc[p] = col[rp[rb_] + k]; }
         };
         // 1&3: slot 0 = len-1 row, slots 1-3 = len-3 row (Alg. 4 masks)
 #pragma omp parallel for schedule(static) if (par)
@@ -398,6 +398,7 @@ int build_format(HostFormat& f, int dtype, int64_t m, int64_t n, const int64_t* 
     }
     int st;
     if (dtype == DASP_R_64F) st = build_impl<uint64_t>(f, m, row_ptr, col, static_cast<const uint64_t*>(val));
+    else if (dtype == DASP_R_32F) st = build_impl<uint32_t>(f, m, row_ptr, col, static_cast<const uint32_t*>(val));
     else st = build_impl<uint16_t>(f, m, row_ptr, col, static_cast<const uint16_t*>(val));
     if (st != DASP_OK) f.release();
     return st;

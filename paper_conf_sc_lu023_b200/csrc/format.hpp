@@ -23,6 +23,7 @@ struct Geometry {
 
 inline Geometry geometry(int dtype) {
     if (dtype == DASP_R_64F) return Geometry{8, 4, 32, 1, 64, 4, 4};
+    if (dtype == DASP_R_32F) return Geometry{4, 4, 32, 1, 64, 4, 4};   // FP64 blocks, 4-byte values (R29)
     return Geometry{2, 8, 64, 2, 128, 4, 4};
 }
 

@@ -218,8 +218,8 @@ struct ShortPanel {      // per panel, built on the host from the class counts
     int64_t q13, q4, q22, qs;   // prefix offsets of the flattened per-category index spaces
 };
 
-__device__ __forceinline__ int short_pos(int sv, int r, int c) {
-    if (sv == 8) return 4 * (4 * (r & 7) + c) + (r >> 3);
+__device__ __forceinline__ int short_pos(int K, int r, int c) {
+    if (K == 4) return 4 * (4 * (r & 7) + c) + (r >> 3);
     const int q = r >> 3, g = r & 7;
     const int t = ((q & 1) << 1) | (c >> 1);
     const int j = ((q >> 1) << 1) | (c & 1);
@@ -237,16 +237,16 @@ __device__ __forceinline__ int64_t panel_of(const ShortPanel* sp, int64_t np, in
 }
 
 template <typename V>
-__device__ __forceinline__ void put_row4(const int64_t* rp, const int32_t* col, const V* val, V* tv, int32_t* tc, int sv,
+__device__ __forceinline__ void put_row4(const int64_t* rp, const int32_t* col, const V* val, V* tv, int32_t* tc, int K,
                                          int r, int64_t ra, int la, int64_t rb_, int lb) {
-    for (int k = 0; k < la; ++k) { const int p = short_pos(sv, r, k); tv[p] = val[rp[ra] + k]; tc[p] = col[rp[ra] + k]; }
+    for (int k = 0; k < la; ++k) { const int p = short_pos(K, r, k); tv[p] = val[rp[ra] + k]; tc[p] = col[rp[ra] + k]; }
     if (rb_ >= 0)
-        for (int k = 0; k < lb; ++k) { const int p = short_pos(sv, r, la + k); tv[p] = val[rp[rb_] + k]; tc[p] = col[rp[rb_] + k]; }
+        for (int k = 0; k < lb; ++k) { const int p = short_pos(K, r, la + k); tv[p] = val[rp[rb_] + k]; tc[p] = col[rp[rb_] + k]; }
 }
 
 template <typename V>
 __global__ void k_short(const int64_t* rp, const int32_t* col, const V* val, const int32_t* order, const ShortPanel* sp,
-                        int64_t np, int cat, int64_t total, int sv, V* sval, int32_t* scol, int32_t* sout) {
+                        int64_t np, int cat, int64_t total, int K, V* sval, int32_t* scol, int32_t* sout) {
     const int64_t j = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
     if (j >= total) return;
     const int64_t p = panel_of(sp, np, j, cat);
@@ -256,7 +256,7 @@ __global__ void k_short(const int64_t* rp, const int32_t* col, const V* val, con
         const int r = static_cast<int>(q % 32);
         const int64_t a = order[P.s[1] + q], b = order[P.s[3] + q];
         const int64_t tile = P.tile0 + q / 32;
-        put_row4(rp, col, val, sval + tile * 128, scol + tile * 128, sv, r, a, 1, b, 3);
+        put_row4(rp, col, val, sval + tile * 128, scol + tile * 128, K, r, a, 1, b, 3);
         const int64_t o = P.out0 + (q / 32) * 64 + 16 * (r >> 3) + (r & 7);
         sout[o] = static_cast<int32_t>(a);
         sout[o + 8] = static_cast<int32_t>(b);
@@ -268,14 +268,14 @@ __global__ void k_short(const int64_t* rp, const int32_t* col, const V* val, con
         else if (q < P.n[4] + P.n3l) { row = order[P.s[3] + P.p13 + q - P.n[4]]; len = 3; }
         else { row = order[P.s[2] + P.n[2] - 1]; len = 2; }
         const int64_t tile = P.tile0 + P.t13 + q / 32;
-        put_row4(rp, col, val, sval + tile * 128, scol + tile * 128, sv, static_cast<int>(q % 32), row, len, -1, 0);
+        put_row4(rp, col, val, sval + tile * 128, scol + tile * 128, K, static_cast<int>(q % 32), row, len, -1, 0);
         sout[P.out0 + 64 * P.t13 + q] = static_cast<int32_t>(row);
     } else if (cat == 2) {                            // 2&2
         const int64_t q = j - P.q22;
         const int r = static_cast<int>(q % 32);
         const int64_t a = order[P.s[2] + 2 * q], b = order[P.s[2] + 2 * q + 1];
         const int64_t tile = P.tile0 + P.t13 + P.t4 + q / 32;
-        put_row4(rp, col, val, sval + tile * 128, scol + tile * 128, sv, r, a, 2, b, 2);
+        put_row4(rp, col, val, sval + tile * 128, scol + tile * 128, K, r, a, 2, b, 2);
         const int64_t o = P.out0 + 64 * P.t13 + 32 * P.t4 + (q / 32) * 64 + 16 * (r >> 3) + (r & 7);
         sout[o] = static_cast<int32_t>(a);
         sout[o + 8] = static_cast<int32_t>(b);
@@ -512,7 +512,7 @@ int build_impl(HostFormat& f, void** d, const int64_t* rp, const int32_t* col, c
     for (int c = 0; c < 4; ++c)
         if (tot[c] > 0)
             k_short<V><<<nblk(tot[c]), 256, 0, s>>>(rp, col, val, order.as<int32_t>(), dsp.as<ShortPanel>(), np, c, tot[c],
-                                                    geo.sv, static_cast<V*>(d[DASP_ARR_SHORT_VAL]),
+                                                    geo.K, static_cast<V*>(d[DASP_ARR_SHORT_VAL]),
                                                     static_cast<int32_t*>(d[DASP_ARR_SHORT_COL]),
                                                     static_cast<int32_t*>(d[DASP_ARR_SHORT_OUT]));
 
@@ -578,9 +578,9 @@ int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, in
         if (hb) return DASP_ERR_INVALID_CSR;
     }
     for (int a = 0; a < DASP_ARR_COUNT; ++a) d_arrays[a] = nullptr;
-    int st = dtype == DASP_R_64F
-                 ? build_impl<uint64_t>(f, d_arrays, d_row_ptr, d_col, static_cast<const uint64_t*>(d_val), s)
-                 : build_impl<uint16_t>(f, d_arrays, d_row_ptr, d_col, static_cast<const uint16_t*>(d_val), s);
+    int st = dtype == DASP_R_64F   ? build_impl<uint64_t>(f, d_arrays, d_row_ptr, d_col, static_cast<const uint64_t*>(d_val), s)
+             : dtype == DASP_R_32F ? build_impl<uint32_t>(f, d_arrays, d_row_ptr, d_col, static_cast<const uint32_t*>(d_val), s)
+                                   : build_impl<uint16_t>(f, d_arrays, d_row_ptr, d_col, static_cast<const uint16_t*>(d_val), s);
     if (st != DASP_OK) {
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
             if (d_arrays[a]) cudaFree(d_arrays[a]);

@@ -67,10 +67,42 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
 __device__ __forceinline__ double gx(const double* x, uint32_t c) {
     return static_cast<int32_t>(c) >= 0 ? __ldg(x + static_cast<int32_t>(c)) : 0.0;
 }
+__device__ __forceinline__ double gx_f64(const double* x, uint32_t c) { return gx(x, c); }
 __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
     return static_cast<int32_t>(c) >= 0 ? __ldg(reinterpret_cast<const unsigned short*>(x) + static_cast<int32_t>(c))
                                         : static_cast<uint16_t>(0);
 }
+// Value streams of the m8n8k4-geometry paths: FP64 (DT 0) and FP32 storage (DT 2, computed in
+// FP64: every float converts exactly, so the DMMA / FMA arithmetic is the FP64 path's).
+template <int DT> struct ValIO;
+template <> struct ValIO<0> {
+    using T = double;
+    static __device__ __forceinline__ void ld2(const T* p, uint64_t pol, double& a, double& b) { ld2_f64(p, pol, a, b); }
+    static __device__ __forceinline__ void ld4(const T* p, uint64_t pol, double (&v)[4]) { ld4_f64(p, pol, v); }
+    static __device__ __forceinline__ double ld1(const T* p, uint64_t pol) { return ld1_f64(p, pol); }
+    static __device__ __forceinline__ double gx(const T* x, uint32_t c) { return gx_f64(x, c); }
+};
+template <> struct ValIO<2> {
+    using T = float;
+    static __device__ __forceinline__ void ld2(const T* p, uint64_t pol, double& a, double& b) {
+        uint32_t u0, u1;
+        ld2_b32(p, pol, u0, u1);
+        a = static_cast<double>(__uint_as_float(u0));
+        b = static_cast<double>(__uint_as_float(u1));
+    }
+    static __device__ __forceinline__ void ld4(const T* p, uint64_t pol, double (&v)[4]) {
+        uint32_t u[4];
+        ld4_b32(p, pol, u);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) v[j] = static_cast<double>(__uint_as_float(u[j]));
+    }
+    static __device__ __forceinline__ double ld1(const T* p, uint64_t pol) {
+        return static_cast<double>(__uint_as_float(ld1_b32(p, pol)));
+    }
+    static __device__ __forceinline__ double gx(const T* x, uint32_t c) {
+        return static_cast<int32_t>(c) >= 0 ? static_cast<double>(__ldg(x + static_cast<int32_t>(c))) : 0.0;
+    }
+};
 __device__ __forceinline__ float h2f(uint16_t h) { return __half2float(__ushort_as_half(h)); }
 __device__ __forceinline__ float2 u2f2(uint32_t u) {  // two packed binary16 -> two f32 (exact)
     return make_float2(h2f(static_cast<uint16_t>(u & 0xffffu)), h2f(static_cast<uint16_t>(u >> 16)));
@@ -115,6 +147,10 @@ template <> struct Tr<1> {  // FP16 storage, FP32 accumulate
     using V = uint16_t; using Y = float; using A = float; using X = uint16_t;
     static constexpr int K = 8, BE = 64, EPL = 2, G = 128, UG = 4, CW = 4;
 };
+template <> struct Tr<2> {  // FP32 storage, FP64 accumulate (R29), FP64 geometry
+    using V = float; using Y = float; using A = double; using X = float;
+    static constexpr int K = 4, BE = 32, EPL = 1, G = 64, UG = 4, CW = 4;
+};
 
 // y[row] = alpha*acc + beta*y[row] (beta == 0: y not read, R16)
 template <int DT>
@@ -136,21 +172,22 @@ __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typena
 // span, and the 32 gathers of one instruction hit 64 consecutive, column-sorted elements of a
 // long row, so they share sectors in L1.  Group j is accumulated separately (4 accumulators)
 // and reduced over the warp.
-template <int VAR>
+template <int DT, int VAR>
 __device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, int lane, uint64_t pol) {
-    const double* lv = static_cast<const double*>(P.long_val) + u * 256;
+    using IO = ValIO<DT>;
+    const typename IO::T* lv = static_cast<const typename IO::T*>(P.long_val) + u * 256;
     const int32_t* lc = P.long_col + u * 256;
-    const double* x = static_cast<const double*>(P.x);
+    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
     double v[8];
     uint32_t c[8];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-        ld2_f64(lv + 2 * (lane + 32 * j), pol, v[2 * j], v[2 * j + 1]);
+        IO::ld2(lv + 2 * (lane + 32 * j), pol, v[2 * j], v[2 * j + 1]);
         ld2_b32(lc + 2 * (lane + 32 * j), pol, c[2 * j], c[2 * j + 1]);
     }
     double xv[8];
 #pragma unroll
-    for (int e = 0; e < 8; ++e) xv[e] = gx(x, c[e]);
+    for (int e = 0; e < 8; ++e) xv[e] = IO::gx(x, c[e]);
     double gsum[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
@@ -243,38 +280,39 @@ __device__ __forceinline__ RbMeta rb_meta(const MainParams& P, int64_t rb, int l
                   static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i)};
 }
 
-template <int VAR>
+template <int DT, int VAR>
 __device__ __forceinline__ void medium_rb_f64(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
     const int t = lane & 3;
     const int64_t base = M.base, ib = M.ib, ie = M.ib + M.ilen;
     const int32_t orow = M.orow;
     const int nreg = M.nelem >> 5;
     const int nfull = nreg >> 2, rem = nreg & 3;
-    const double* rv = static_cast<const double*>(P.reg_val) + base;
+    using IO = ValIO<DT>;
+    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + base;
     const int32_t* rc = P.reg_col + base;
-    const double* iv = static_cast<const double*>(P.irr_val);
-    const double* x = static_cast<const double*>(P.x);
+    const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
     // round 1: first chunk (4 blocks, 256-bit value load), the ragged last chunk and the
     // first irregular element of this lane, all in flight together
     double va[4] = {0.0, 0.0, 0.0, 0.0};
     uint32_t ca[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
-    if (nfull > 0) { ld4_f64(rv + lane * 4, pol, va); ld4_b32(rc + lane * 4, pol, ca); }
+    if (nfull > 0) { IO::ld4(rv + lane * 4, pol, va); ld4_b32(rc + lane * 4, pol, ca); }
     double vr[3] = {0.0, 0.0, 0.0};
     uint32_t cr[3] = {0xffffffffu, 0xffffffffu, 0xffffffffu};
     const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane * rem;
 #pragma unroll
     for (int j = 0; j < 3; ++j)
-        if (j < rem) { vr[j] = ld1_f64(rv + rbase + j, pol); cr[j] = ld1_b32(rc + rbase + j, pol); }
+        if (j < rem) { vr[j] = IO::ld1(rv + rbase + j, pol); cr[j] = ld1_b32(rc + rbase + j, pol); }
     int64_t k = ib + t;
     double vi = 0.0;
     uint32_t ci = 0xffffffffu;
-    if (k < ie) { vi = ld1_f64(iv + k, pol); ci = ld1_b32(P.irr_col + k, pol); }
+    if (k < ie) { vi = IO::ld1(iv + k, pol); ci = ld1_b32(P.irr_col + k, pol); }
     double c0 = 0.0, c1 = 0.0, part = 0.0;
     for (int ch = 0; ch < nfull; ++ch) {
-        if (ch > 0) { ld4_f64(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
+        if (ch > 0) { IO::ld4(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
         double xv[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) xv[j] = gx(x, ca[j]);
+        for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
             if constexpr (VAR == VAR_MMA) dmma(c0, c1, va[j], xv[j]);
@@ -283,8 +321,8 @@ __device__ __forceinline__ void medium_rb_f64(const MainParams& P, const RbMeta&
     }
     double xr[3];
 #pragma unroll
-    for (int j = 0; j < 3; ++j) xr[j] = gx(x, cr[j]);     // pads / unused slots read 0
-    const double xi = gx(x, ci);
+    for (int j = 0; j < 3; ++j) xr[j] = IO::gx(x, cr[j]);     // pads / unused slots read 0
+    const double xi = IO::gx(x, ci);
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
         if (j < rem) {                                     // rem is warp-uniform
@@ -297,10 +335,10 @@ __device__ __forceinline__ void medium_rb_f64(const MainParams& P, const RbMeta&
         part = t == 0 ? d : 0.0;
     }
     part = fma(vi, xi, part);                              // Alg. 3 l.20-24: irregular part
-    for (k += 4; k < ie; k += 4) part = fma(ld1_f64(iv + k, pol), gx(x, ld1_b32(P.irr_col + k, pol)), part);
+    for (k += 4; k < ie; k += 4) part = fma(IO::ld1(iv + k, pol), IO::gx(x, ld1_b32(P.irr_col + k, pol)), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
-    if (t == 0) store_y<0>(P, orow, part);                 // Alg. 3 l.25 through the output map (R9)
+    if (t == 0) store_y<DT>(P, orow, part);                 // Alg. 3 l.25 through the output map (R9)
 }
 
 template <int VAR>
@@ -371,21 +409,22 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta&
 // cat 0 = 1&3 (seg0 = slot 0, seg1 = slots 1-3), 1 = len-4, 2 = 2&2 (slots 0-1 | 2-3)
 __device__ __forceinline__ int seg_of(int cat, int slot) { return cat == 0 ? (slot > 0) : (cat == 2 ? (slot >> 1) : 0); }
 
-template <int VAR>
+template <int DT, int VAR>
 __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
                                                uint64_t pol) {
     const int g = lane >> 2, t = lane & 3;
     const int nseg = cat == 1 ? 1 : 2;
     double v[4];
     uint32_t c[4];
-    ld4_f64(static_cast<const double*>(P.short_val) + tile * 128 + lane * 4, pol, v);
+    using IO = ValIO<DT>;
+    IO::ld4(static_cast<const typename IO::T*>(P.short_val) + tile * 128 + lane * 4, pol, v);
     ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
     const int32_t o0 = __ldg(P.short_out + obase + lane);                        // outputs L, L+32
     const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
-    const double* x = static_cast<const double*>(P.x);
+    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
     double xv[4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) xv[j] = gx(x, c[j]);
+    for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, c[j]);
     const int myseg = seg_of(cat, t);
     // output o = 16j + 8s + g (two outputs per four-slot row) or 8j + g (len-4)
     const int src = 4 * (lane & 7);                      // quad of row g' = lane & 7
@@ -409,8 +448,8 @@ __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int
             if ((lane >> 3) == blk - 4) r1 = val;
         }
     }
-    store_y<0>(P, o0, r0);
-    if (nseg == 2) store_y<0>(P, o1, r1);
+    store_y<DT>(P, o0, r0);
+    if (nseg == 2) store_y<DT>(P, o1, r1);
 }
 
 template <int VAR>
@@ -480,11 +519,13 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
     uint32_t c[4], o[4];
     ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
     ld4_b32(P.short_out + obase + lane * 4, pol, o);
-    if constexpr (DT == 0) {
+    if constexpr (DT != 1) {
+        using IO = ValIO<DT>;
         double v[4];
-        ld4_f64(static_cast<const double*>(P.short_val) + tile * 128 + lane * 4, pol, v);
+        IO::ld4(static_cast<const typename IO::T*>(P.short_val) + tile * 128 + lane * 4, pol, v);
 #pragma unroll
-        for (int j = 0; j < 4; ++j) store_y<0>(P, static_cast<int32_t>(o[j]), v[j] * gx(static_cast<const double*>(P.x), c[j]));
+        for (int j = 0; j < 4; ++j)
+            store_y<DT>(P, static_cast<int32_t>(o[j]), v[j] * IO::gx(static_cast<const typename IO::T*>(P.x), c[j]));
     } else {
         uint32_t a0, a2;
         ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
@@ -524,8 +565,8 @@ dasp_long_kernel(const MainParams P, int64_t n_units) {
     const int lane = threadIdx.x & 31;
     const uint64_t pol = stream_policy();
     const int64_t u = __ldg(P.unit_order + w);
-    if constexpr (DT == 0) long_unit_f64<VAR>(P, u, lane, pol);
-    else long_unit_f16<VAR>(P, u, lane, pol);
+    if constexpr (DT == 1) long_unit_f16<VAR>(P, u, lane, pol);
+    else long_unit_f64<DT, VAR>(P, u, lane, pol);
 }
 
 // medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
@@ -546,8 +587,8 @@ __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : DASP
         for (int64_t rb = rb0; rb < rb1; ++rb) {
             // (prefetching the next row-block's metadata here was measured: it costs registers
             // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta.jsonl)
-            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb_meta(P, rb, lane), lane, pol);
-            else medium_rb_f16<VAR>(P, rb_meta(P, rb, lane), lane, pol);
+            if constexpr (DT == 1) medium_rb_f16<VAR>(P, rb_meta(P, rb, lane), lane, pol);
+            else medium_rb_f64<DT, VAR>(P, rb_meta(P, rb, lane), lane, pol);
         }
         return;
     }
@@ -566,8 +607,27 @@ __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : DASP
         singles_tile<DT>(P, tile, obase, lane, pol);
         return;
     }
-    if constexpr (DT == 0) short_tile_f64<VAR>(P, cat, tile, obase, lane, pol);
-    else short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
+    if constexpr (DT == 1) short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
+    else short_tile_f64<DT, VAR>(P, cat, tile, obase, lane, pol);
+}
+
+// short tiles in their own launch (split mode): tile_meta[t] = cat << 62 | output base
+#ifndef DASP_SHORT_MIN_BLOCKS
+#define DASP_SHORT_MIN_BLOCKS 6
+#endif
+template <int DT, int VAR>
+__global__ void __launch_bounds__(MAIN_THREADS, DASP_SHORT_MIN_BLOCKS)
+dasp_short_kernel(const MainParams P, const uint64_t* __restrict__ tile_meta, int64_t n_tiles) {
+    const int64_t t = (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5;
+    if (t >= n_tiles) return;
+    const int lane = threadIdx.x & 31;
+    const uint64_t pol = stream_policy();
+    const uint64_t meta = __ldg(tile_meta + t);
+    const int cat = static_cast<int>(meta >> 62);
+    const int64_t obase = static_cast<int64_t>(meta & ((1ull << 62) - 1));
+    if (cat == 3) { singles_tile<DT>(P, t, obase, lane, pol); return; }
+    if constexpr (DT == 1) short_tile_f16<VAR>(P, cat, t, obase, lane, pol);
+    else short_tile_f64<DT, VAR>(P, cat, t, obase, lane, pol);
 }
 
 // long phase 2 (Alg. 2 l.17-25): one warp per long row, lane-strided sum of the group partials
@@ -1055,7 +1115,7 @@ __global__ void __launch_bounds__(PW * 32) dasp_pipe_kernel(const MainParams P, 
             if constexpr (DT == 0) medium_stage_f64<VAR>(P, st, lane);
             else medium_stage_f16<VAR>(P, st, lane);
         } else {                                          // row-block larger than a stage
-            if constexpr (DT == 0) medium_rb_f64<VAR>(P, rb_meta(P, h[1], lane), lane, pol);
+            if constexpr (DT == 0) medium_rb_f64<0, VAR>(P, rb_meta(P, h[1], lane), lane, pol);
             else medium_rb_f16<VAR>(P, rb_meta(P, h[1], lane), lane, pol);
         }
         __syncwarp();
@@ -1104,13 +1164,10 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     const unsigned nb = static_cast<unsigned>(blocks);
     cudaError_t e;
-    if (dtype == 0) {
-        if (variant == VAR_MMA) e = launch_ex(dasp_main_kernel<0, VAR_MMA>, nb, s, apw_base, apw_bytes, apw_hit, p);
-        else e = launch_ex(dasp_main_kernel<0, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
-    } else {
-        if (variant == VAR_MMA) e = launch_ex(dasp_main_kernel<1, VAR_MMA>, nb, s, apw_base, apw_bytes, apw_hit, p);
-        else e = launch_ex(dasp_main_kernel<1, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
-    }
+    const bool mma = variant == VAR_MMA;
+    if (dtype == 0) e = launch_ex(mma ? dasp_main_kernel<0, VAR_MMA> : dasp_main_kernel<0, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
+    else if (dtype == 1) e = launch_ex(mma ? dasp_main_kernel<1, VAR_MMA> : dasp_main_kernel<1, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
+    else e = launch_ex(mma ? dasp_main_kernel<2, VAR_MMA> : dasp_main_kernel<2, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
@@ -1152,13 +1209,25 @@ cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_u
     const int64_t blocks = (n_units * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
-    if (dtype == 0) {
-        if (variant == VAR_MMA) dasp_long_kernel<0, VAR_MMA><<<grid, block, 0, s>>>(p, n_units);
-        else dasp_long_kernel<0, VAR_CUDACORE><<<grid, block, 0, s>>>(p, n_units);
-    } else {
-        if (variant == VAR_MMA) dasp_long_kernel<1, VAR_MMA><<<grid, block, 0, s>>>(p, n_units);
-        else dasp_long_kernel<1, VAR_CUDACORE><<<grid, block, 0, s>>>(p, n_units);
-    }
+    const bool mma = variant == VAR_MMA;
+    auto k = dtype == 0 ? (mma ? dasp_long_kernel<0, VAR_MMA> : dasp_long_kernel<0, VAR_CUDACORE>)
+           : dtype == 1 ? (mma ? dasp_long_kernel<1, VAR_MMA> : dasp_long_kernel<1, VAR_CUDACORE>)
+                        : (mma ? dasp_long_kernel<2, VAR_MMA> : dasp_long_kernel<2, VAR_CUDACORE>);
+    k<<<grid, block, 0, s>>>(p, n_units);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_short(const MainParams& p, int dtype, int variant, const uint64_t* tile_meta, int64_t n_tiles,
+                         cudaStream_t s) {
+    if (n_tiles <= 0) return cudaSuccess;
+    const int64_t blocks = (n_tiles * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
+    if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
+    const bool mma = variant == VAR_MMA;
+    auto k = dtype == 0 ? (mma ? dasp_short_kernel<0, VAR_MMA> : dasp_short_kernel<0, VAR_CUDACORE>)
+           : dtype == 1 ? (mma ? dasp_short_kernel<1, VAR_MMA> : dasp_short_kernel<1, VAR_CUDACORE>)
+                        : (mma ? dasp_short_kernel<2, VAR_MMA> : dasp_short_kernel<2, VAR_CUDACORE>);
+    k<<<grid, block, 0, s>>>(p, tile_meta, n_tiles);
     return cudaGetLastError();
 }
 
@@ -1167,7 +1236,8 @@ cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s) {
     if (warps == 0) return cudaSuccess;
     dim3 grid(static_cast<unsigned>((warps * 32 + 255) / 256)), block(256);
     if (dtype == 0) dasp_finish_kernel<0><<<grid, block, 0, s>>>(p);
-    else dasp_finish_kernel<1><<<grid, block, 0, s>>>(p);
+    else if (dtype == 1) dasp_finish_kernel<1><<<grid, block, 0, s>>>(p);
+    else dasp_finish_kernel<2><<<grid, block, 0, s>>>(p);
     return cudaGetLastError();
 }
 
@@ -1176,7 +1246,8 @@ cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_
     int64_t blocks = (m + 255) / 256;
     if (blocks > 148 * 16) blocks = 148 * 16;
     if (dtype == 0) dasp_scale_kernel<0><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
-    else dasp_scale_kernel<1><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
+    else if (dtype == 1) dasp_scale_kernel<1><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
+    else dasp_scale_kernel<2><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
     return cudaGetLastError();
 }
 

@@ -71,6 +71,8 @@ struct FinishParams {
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
+cudaError_t launch_short(const MainParams& p, int dtype, int variant, const uint64_t* tile_meta, int64_t n_tiles,
+                         cudaStream_t s);
 cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s);
 
 // Persistent TMA-staged pipeline kernel (kernels.cu): items are 64-bit words

@@ -15,10 +15,10 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("DASP_LIB", os.path.join(_HERE, "libdasp.so"))   # override: experiment builds
 
-DASP_R_64F, DASP_R_16F = 0, 1
+DASP_R_64F, DASP_R_16F, DASP_R_32F = 0, 1, 2
 DASP_VARIANT_DEFAULT, DASP_VARIANT_MMA, DASP_VARIANT_CUDACORE = 0, 1, 2
-DASP_K_MAIN, DASP_K_FINISH, DASP_K_SCALE, DASP_K_LONG, DASP_K_COUNT = 0, 1, 2, 3, 4
-KERNEL_NAMES = ["dasp_main_kernel", "dasp_finish_kernel", "dasp_scale_kernel", "dasp_long_kernel"]
+DASP_K_MAIN, DASP_K_FINISH, DASP_K_SCALE, DASP_K_LONG, DASP_K_SHORT, DASP_K_COUNT = 0, 1, 2, 3, 4, 5
+KERNEL_NAMES = ["dasp_main_kernel", "dasp_finish_kernel", "dasp_scale_kernel", "dasp_long_kernel", "dasp_short_kernel"]
 
 ARRAYS = ["long_val", "long_col", "group_ptr", "long_out", "rb_ptr", "reg_val", "reg_col", "irr_ptr",
           "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows", "panels"]
@@ -161,7 +161,8 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
-    (dtype "f16"; passed as binary16 bits).  panel_rows: 0 automatic, -1 one global panel."""
+    (dtype "f16"; passed as binary16 bits) or float32[nnz] (dtype "f32").  panel_rows: 0 automatic,
+    -1 one global panel."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     if dtype == "f64":
@@ -170,6 +171,9 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     elif dtype == "f16":
         val = np.ascontiguousarray(val, dtype=np.float16)
         dt = DASP_R_16F
+    elif dtype == "f32":
+        val = np.ascontiguousarray(val, dtype=np.float32)
+        dt = DASP_R_32F
     else:
         raise ValueError(dtype)
     if len(row_ptr) != m + 1:
@@ -196,7 +200,7 @@ def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = 
     """Build the plan on the GPU from a device CSR (torch CUDA tensors: int64 row_ptr, int32
     col_idx, float64 / float16 val) -- SURVEY.md §8(f) f2."""
     import torch
-    want = torch.float64 if dtype == "f64" else torch.float16
+    want = {"f64": torch.float64, "f16": torch.float16, "f32": torch.float32}[dtype]
     for t, dt_ in ((row_ptr, torch.int64), (col_idx, torch.int32), (val, want)):
         if not isinstance(t, torch.Tensor) or not t.is_cuda or t.dtype != dt_ or not t.is_contiguous():
             raise ValueError("dasp_plan_create_device needs contiguous CUDA tensors (int64, int32, value dtype)")
@@ -209,7 +213,8 @@ def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = 
     opts.max_len, opts.threshold = int(max_len), float(threshold)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create_device(ctypes.byref(h), m, n, int(col_idx.numel()), _ptr(row_ptr), _ptr(col_idx),
-                                      _ptr(val), DASP_R_64F if dtype == "f64" else DASP_R_16F, ctypes.byref(opts),
+                                      _ptr(val), {"f64": DASP_R_64F, "f16": DASP_R_16F, "f32": DASP_R_32F}[dtype],
+                                      ctypes.byref(opts),
                                       _stream_ptr(stream))
     _check(st, "dasp_plan_create_device")
     return Plan(h, dtype, m, n)
@@ -232,7 +237,8 @@ def dasp_spmv(plan: Plan, x, y, alpha: float = 1.0, beta: float = 0.0, stream=No
         import torch
         dev = plan.info["device"] if not hasattr(plan, "_dev") else plan._dev
         plan._dev = dev
-        xd, yd = (torch.float64, torch.float64) if plan.dtype == "f64" else (torch.float16, torch.float32)
+        xd, yd = {"f64": (torch.float64, torch.float64), "f16": (torch.float16, torch.float32),
+                  "f32": (torch.float32, torch.float32)}[plan.dtype]
         _check_vec(x, plan.n, xd, "x", dev)
         _check_vec(y, plan.m, yd, "y", dev)
     st = _lib.dasp_spmv_ex(plan.handle, _ptr(x), _ptr(y), float(alpha), float(beta), _stream_ptr(stream), variant)

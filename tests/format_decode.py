@@ -13,13 +13,13 @@ PAD = -1
 
 
 def params(dtype):
-    if dtype == "f64":
+    if dtype in ("f64", "f32"):
         return dict(K=4, BE=32, EPL=1, G=64, UG=4, CW=4)
     return dict(K=8, BE=64, EPL=2, G=128, UG=4, CW=4)
 
 
 def _bits(vals):
-    return vals.view(np.uint64) if vals.dtype == np.float64 else vals.view(np.uint16)
+    return vals.view({8: np.uint64, 4: np.uint32, 2: np.uint16}[vals.dtype.itemsize])
 
 
 def decode(F, get, dtype):
@@ -95,7 +95,7 @@ def decode(F, get, dtype):
                 for lane in range(32):
                     g, t = lane >> 2, lane & 3
                     for j in range(4):
-                        if dtype == "f64":
+                        if dtype in ("f64", "f32"):
                             r, c = 8 * j + g, t
                         else:
                             r = 8 * ((t >> 1) + (0 if j < 2 else 2)) + g
@@ -142,7 +142,7 @@ def check_roundtrip(A, F, get, dtype):
     for c, v in pads:
         assert c == PAD and v == 0, "pads must be exactly (+0, -1)"
     assert sorted(rows) == list(range(A.m)), "every row exactly once"
-    vals = A.val if dtype == "f64" else A.val.astype(np.float16)
+    vals = {"f64": A.val, "f32": A.val.astype(np.float32), "f16": A.val.astype(np.float16)}[dtype]
     bits = _bits(np.ascontiguousarray(vals))
     for i in range(A.m):
         a, b = A.row_ptr[i], A.row_ptr[i + 1]

@@ -20,7 +20,7 @@ COUNT_MAP = {"n0": "n_empty", "n1": "n_len1", "n2": "n_len2", "n3": "n_len3", "n
 
 
 def host_plan(A, dt, **kw):
-    val = A.val if dt == "f64" else A.val.astype(np.float16)
+    val = {"f64": A.val, "f16": A.val.astype(np.float16), "f32": A.val.astype(np.float32)}[dt]
     return dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dt, device=-1, **kw)
 
 
@@ -39,13 +39,13 @@ CASES = list(matrices())
 
 
 @pytest.mark.parametrize("panel", [0, -1, 1, 97, 1000])
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", ["f64", "f16", "f32"])
 @pytest.mark.parametrize("name,A", CASES, ids=[c[0] for c in CASES])
 def test_builder_bit_exact_vs_oracle(name, A, dt, panel):
     if panel in (1, 97) and A.m > 20000:
         pytest.skip("tiny panels on the small matrices only")
     plan = host_plan(A, dt, panel_rows=panel)
-    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt, panel_rows=plan.info["panel_rows"])
+    ref = oracle.build(A, dt, panel_rows=plan.info["panel_rows"])
     info = plan.info
     for k, v in ref.counts.items():
         assert info[COUNT_MAP[k]] == v, k
@@ -56,7 +56,7 @@ def test_builder_bit_exact_vs_oracle(name, A, dt, panel):
         assert np.array_equal(got, want), arr
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", ["f64", "f16", "f32"])
 @pytest.mark.parametrize("panel", [-1, 333])
 def test_builder_roundtrip_via_abi(dt, panel):
     A = synth.generate(synth.config("c1b"))
@@ -67,7 +67,7 @@ def test_builder_roundtrip_via_abi(dt, panel):
     def get(name):
         b = dasp.dasp_plan_copy_array(plan, name)
         if name.endswith("_val"):
-            return b.view(np.float64 if dt == "f64" else np.float16)
+            return b.view({"f64": np.float64, "f16": np.float16, "f32": np.float32}[dt])
         if name in ("group_ptr", "rb_ptr", "irr_ptr", "panels"):
             return b.view(np.int64)
         return b.view(np.int32)

@@ -20,7 +20,7 @@ def _cuda():
 
 
 def device_plan(A, dt, **kw):
-    val = A.val if dt == "f64" else A.val.astype(np.float16)
+    val = A.val.astype({"f64": np.float64, "f16": np.float16, "f32": np.float32}[dt])
     return dasp.dasp_plan_create_device(torch.from_numpy(A.row_ptr).cuda(), torch.from_numpy(A.col).cuda(),
                                         torch.from_numpy(np.ascontiguousarray(val)).cuda(), A.m, A.n, dt, **kw)
 
@@ -39,15 +39,14 @@ def cases():
 CASES = list(cases())
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", ["f64", "f16", "f32"])
 @pytest.mark.parametrize("panel", [-1, 97, 1000])
 @pytest.mark.parametrize("name,A", CASES, ids=[c[0] for c in CASES])
 def test_device_builder_bytes(name, A, dt, panel):
     dplan = device_plan(A, dt, panel_rows=panel)
     info = dplan.info
-    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt, panel_rows=info["panel_rows"])
-    hplan = dasp.dasp_plan_create(A.row_ptr, A.col, A.val if dt == "f64" else A.val.astype(np.float16), A.m, A.n, dt,
-                                  device=-1, panel_rows=panel)
+    ref = oracle.build(A, dt, panel_rows=info["panel_rows"])
+    hplan = dasp.dasp_plan_create(A.row_ptr, A.col, A.val, A.m, A.n, dt, device=-1, panel_rows=panel)
     hinfo = hplan.info
     for k in ["n_empty", "n_len1", "n_len2", "n_len3", "n_len4", "row_medium", "row_long", "rowblocks", "n_groups",
               "n_groups_padded", "tiles_13", "tiles_4", "tiles_22", "tiles_single", "nnz_long_new", "nnz_reg_new",

@@ -17,6 +17,8 @@ pytestmark = pytest.mark.gpu
 from paper_conf_sc_lu023_b200 import dasp  # noqa: E402
 
 VARIANTS = [dasp.DASP_VARIANT_MMA, dasp.DASP_VARIANT_CUDACORE]
+DTYPES = ["f64", "f16", "f32"]
+NP_VAL = {"f64": np.float64, "f16": np.float16, "f32": np.float32}
 VNAME = {dasp.DASP_VARIANT_MMA: "mma", dasp.DASP_VARIANT_CUDACORE: "cudacore"}
 
 
@@ -28,12 +30,12 @@ def _cuda():
 
 
 def make(A, dt, **kw):
-    val = A.val if dt == "f64" else A.val.astype(np.float16)
+    val = A.val.astype(NP_VAL[dt])
     return dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dt, device=0, **kw)
 
 
 def run(plan, x_np, dt, alpha=1.0, beta=0.0, y0=None, variant=0):
-    xd = torch.from_numpy(np.ascontiguousarray(x_np.astype(np.float64 if dt == "f64" else np.float16))).cuda()
+    xd = torch.from_numpy(np.ascontiguousarray(x_np.astype(NP_VAL[dt]))).cuda()
     ydt = torch.float64 if dt == "f64" else torch.float32
     if y0 is None:
         y = torch.full((plan.m,), float("nan"), dtype=ydt, device="cuda")
@@ -45,9 +47,9 @@ def run(plan, x_np, dt, alpha=1.0, beta=0.0, y0=None, variant=0):
 
 
 def oracle_ref(A, x, dt, alpha=1.0, beta=0.0, y0=None):
-    if dt == "f16":
-        val = A.val.astype(np.float16).astype(np.float64)
-        x = x.astype(np.float16).astype(np.float64)
+    if dt != "f64":   # the oracle is fed the same stored values (exactly widened to f64)
+        val = A.val.astype(NP_VAL[dt]).astype(np.float64)
+        x = x.astype(NP_VAL[dt]).astype(np.float64)
         if y0 is not None:
             y0 = y0.astype(np.float32).astype(np.float64)
     else:
@@ -70,7 +72,7 @@ CASES = list(cases())
 
 
 @pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("name,gen", CASES, ids=[c[0] for c in CASES])
 def test_parity_random_values(name, gen, dt, variant):
     A = gen(synth.VAL_UNIFORM)
@@ -86,7 +88,7 @@ def test_parity_random_values(name, gen, dt, variant):
 # P5: small-integer values make every summation order exact -> bit-exact in both dtypes,
 # which also pins the MMA fragment layout and the diagonal lanes (Fig. 4).
 @pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("name,gen", CASES, ids=[c[0] for c in CASES])
 def test_parity_integer_bit_exact(name, gen, dt, variant):
     A = gen(synth.VAL_INT)
@@ -99,7 +101,7 @@ def test_parity_integer_bit_exact(name, gen, dt, variant):
 
 # R28 panels: every panel size gives the same exact integer results (and parity on reals)
 @pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("panel", [-1, 1, 97, 1000, 50000])
 def test_parity_panels(panel, dt, variant):
     A = synth.generate(synth.config("c3", scale=0.01, val_mode=synth.VAL_INT))
@@ -117,7 +119,7 @@ def test_parity_panels(panel, dt, variant):
     assert np.array_equal(y, y_ref)
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 def test_identity_diagonal_permutation_exact(dt):
     n = 5003
     rng = np.random.default_rng(3)
@@ -129,12 +131,12 @@ def test_identity_diagonal_permutation_exact(dt):
         for v in VARIANTS:
             y = run(make(A, dt), x, dt, variant=v)
             y_ref, _ = oracle_ref(A, x, dt)
-            if dt == "f16":   # one fp16 x fp16 product is exact in fp32, then rounded to y's fp32
+            if dt != "f64":   # one product is exact in the wide type, then rounded to y's fp32
                 y_ref = y_ref.astype(np.float32).astype(np.float64)
             assert np.array_equal(y, y_ref)
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 def test_alpha_beta(dt):
     A = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
     x = synth.vector(1, A.n, synth.VAL_INT)
@@ -151,7 +153,7 @@ def test_alpha_beta(dt):
 
 
 # P11: pads carry a sentinel column, so an Inf in x only reaches rows that store that column
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 def test_inf_in_x_only_reaches_referencing_rows(dt):
     A = synth.generate(synth.config("c1b"))
     x = synth.vector(4, A.n)
@@ -169,12 +171,12 @@ def test_inf_in_x_only_reaches_referencing_rows(dt):
     assert np.isfinite(base).all()
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("panel", [-1, 500])
 def test_device_arrays_match_oracle_builder(dt, panel):
     A = synth.generate(synth.config("c1b"))
     plan = make(A, dt, panel_rows=panel)   # keep_host off: copy_array reads back the device buffers
-    ref = oracle.build(A if dt == "f64" else A.to_fp16(), dt, panel_rows=plan.info["panel_rows"])
+    ref = oracle.build(A, dt, panel_rows=plan.info["panel_rows"])
     for arr in dasp.ARRAYS:
         assert np.array_equal(dasp.dasp_plan_copy_array(plan, arr), ref.arrays[arr]), arr
 
@@ -247,13 +249,13 @@ def _sampled_parity(A, dt, nsample=20000, seed=0):
     return plan
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 def test_full_size_stencil_sampled(dt):
     A = synth.generate(synth.config("c2"))
     _sampled_parity(A, dt)
 
 
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 def test_full_size_powerlaw_sampled(dt):
     A = synth.generate(synth.config("c3"))
     _sampled_parity(A, dt)
@@ -298,14 +300,14 @@ def test_pipeline_kernel_parity(name, gen, dt, variant):
 
 # dasp_spmv_scatter: the fused SpMV + all-gather epilogue writes the same values to every
 # destination (here several local buffers stand in for the peers' x buffers)
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("pipeline", [False, True])
 def test_scatter_epilogue_writes_every_destination(dt, pipeline):
     A = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
     x = synth.vector(51, A.n, synth.VAL_INT)
     y0 = synth.vector(52, A.m, synth.VAL_INT)
     plan = make(A, dt, pipeline=pipeline)
-    xd = torch.from_numpy(x.astype(np.float64 if dt == "f64" else np.float16)).cuda()
+    xd = torch.from_numpy(x.astype(NP_VAL[dt])).cuda()
     ydt = torch.float64 if dt == "f64" else torch.float32
     for alpha, beta in [(1.0, 0.0), (2.0, -1.0), (1.0, 1.0), (0.0, 3.0)]:
         dst = [torch.from_numpy(y0).to(ydt).cuda()] + [torch.full((A.m,), float("nan"), dtype=ydt, device="cuda")
@@ -321,7 +323,7 @@ def test_scatter_epilogue_writes_every_destination(dt, pipeline):
 
 # f3 knobs: MAX_LEN and tau move rows between classes and slots between regular / irregular;
 # the result must not change (bit-exact on integers)
-@pytest.mark.parametrize("dt", ["f64", "f16"])
+@pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("max_len,tau", [(16, 0.75), (64, 0.5), (1000, 0.9), (256, 1.0), (4, 0.3)])
 def test_parity_knobs(dt, max_len, tau):
     A = synth.generate(synth.config("c3", scale=0.004, val_mode=synth.VAL_INT))
@@ -330,3 +332,16 @@ def test_parity_knobs(dt, max_len, tau):
     for v in VARIANTS:
         plan = make(A, dt, max_len=max_len, threshold=tau)
         assert np.array_equal(run(plan, x, dt, variant=v), y_ref)
+
+
+# short tiles in their own launch (DASP_SPLIT_SHORT=1): same bits as the fused main kernel
+@pytest.mark.parametrize("dt", DTYPES)
+def test_split_short_kernel_parity(dt, monkeypatch):
+    monkeypatch.setenv("DASP_SPLIT_SHORT", "1")
+    for name, gen in CASES:
+        A = gen(synth.VAL_INT)
+        x = synth.vector(101, A.n, synth.VAL_INT)
+        y_ref, _ = oracle_ref(A, x, dt)
+        for v in VARIANTS:
+            plan = make(A, dt, panel_rows=900)
+            assert np.array_equal(run(plan, x, dt, variant=v), y_ref), name
