@@ -38,10 +38,10 @@ clean:
 
 .PHONY: all clean
 
-# experiment builds: one libdasp_<VAR=value>.so per -D setting in EXPVARS
+# experiment builds: one libdasp_<VAR=value[+VAR=value]>.so per EXPVARS entry (comma-separated -D settings)
 EXPVARS ?= DASP_NSTAGE=3 DASP_NSTAGE=4
 exp: $(OBJ)/builder.o $(OBJ)/api.o $(OBJ)/gpu_builder.o
 	for v in $(EXPVARS); do \
-	  $(NVCC) $(NVFLAGS) -D$$v -c $(SRC)/kernels.cu -o $(OBJ)/kernels_$$v.o 2> $(OBJ)/kernels_$$v.ptxas.txt && \
-	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$v.so $(OBJ)/builder.o $(OBJ)/kernels_$$v.o $(OBJ)/gpu_builder.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
+	  $(NVCC) $(NVFLAGS) -D$$(echo $$v | sed 's/,/ -D/g') -c $(SRC)/kernels.cu -o $(OBJ)/kernels_$$(echo $$v | tr , +).o 2> $(OBJ)/kernels_$$(echo $$v | tr , +).ptxas.txt && \
+	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$(echo $$v | tr , +).so $(OBJ)/builder.o $(OBJ)/kernels_$$(echo $$v | tr , +).o $(OBJ)/gpu_builder.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
 	done

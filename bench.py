@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--no-triad", action="store_true")
     ap.add_argument("--iterate", action="store_true", help="N=1: run the row-slab iteration (x <- alpha*A*x)")
     ap.add_argument("--no-gpu-build", action="store_true", help="skip timing the device-side builder")
+    ap.add_argument("--halo", action="store_true", help="slab mode: sparse halo exchange (all_to_all of the referenced "
+                    "remote x only) overlapped with the local sub-matrix SpMV (SURVEY.md 8(f) f1)")
     ap.add_argument("--fused", action="store_true", help="slab mode: fuse the x all-gather into the SpMV "
                     "epilogue (symmetric memory + dasp_spmv_scatter)")
     ap.add_argument("--e2e-steps", type=int, default=10)
@@ -248,7 +250,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_lu023_b200 import dasp
-    from paper_conf_sc_lu023_b200.multigpu import SlabSpMV, build_slab
+    from paper_conf_sc_lu023_b200.multigpu import HaloSlabSpMV, SlabSpMV, build_slab
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -271,7 +273,7 @@ def main():
         return float(t.item())
 
     use_slab = world > 1 or args.iterate
-    slab = build_slab(gen_rows, lens, rank, world, reduce_max, need_norm=use_slab)
+    slab = build_slab(gen_rows, lens, rank, world, reduce_max, need_norm=use_slab, remap=not args.halo)
     gen_s = time.perf_counter() - t0
     if args.dtype != "f64":
         if world > 1:
@@ -295,7 +297,10 @@ def main():
         def step():
             dasp.dasp_spmv(plan, xd, yd, alpha, 0.0, stream, variant=variant, check=False)
     else:
-        it = SlabSpMV(slab, world, rank, dev, args.dtype, variant=variant, fused=args.fused)
+        if args.halo:
+            it = HaloSlabSpMV(slab, world, rank, dev, args.dtype, variant=variant)
+        else:
+            it = SlabSpMV(slab, world, rank, dev, args.dtype, variant=variant, fused=args.fused)
         plan = it.plan
         it.set_x(x_global)
         alpha = 1.0 / max(slab.inf_norm, 1e-300)   # iterated SpMV stays bounded
@@ -305,6 +310,9 @@ def main():
             it.step(alpha)
     plan_s = time.perf_counter() - t1
     info = plan.info
+    launches_step = int(info["launches_per_spmv"])
+    if use_slab and args.halo and it.plan_rem is not None:   # remote sub-matrix SpMV + halo pack
+        launches_step += int(it.plan_rem.info["launches_per_spmv"]) + 1
 
     # ---- warm-up, then K timed steps (barrier + synchronize on both sides, CUDA events) ----
     for _ in range(max(args.warmup, 3)):
@@ -397,11 +405,16 @@ def main():
             if world > 1:
                 dist.barrier()
             t0 = time.perf_counter()
-            it.x[it.cur][rank * S0: rank * S0 + slab.rows].copy_(xh, non_blocking=True)
-            if world > 1 and not args.fused:
-                dist.all_gather_into_tensor(it.x[it.cur], it.x[it.cur][rank * S0:(rank + 1) * S0])
-            it.step(alpha)
-            yh.copy_(it.x[it.cur][rank * S0: rank * S0 + slab.rows], non_blocking=True)
+            if args.halo:
+                it.my_x().copy_(xh, non_blocking=True)
+                it.step(alpha)
+                yh.copy_(it.my_x(), non_blocking=True)
+            else:
+                it.x[it.cur][rank * S0: rank * S0 + slab.rows].copy_(xh, non_blocking=True)
+                if world > 1 and not args.fused:
+                    dist.all_gather_into_tensor(it.x[it.cur], it.x[it.cur][rank * S0:(rank + 1) * S0])
+                it.step(alpha)
+                yh.copy_(it.x[it.cur][rank * S0: rank * S0 + slab.rows], non_blocking=True)
             torch.cuda.synchronize(dev)
             if k:
                 times.append(time.perf_counter() - t0)
@@ -412,7 +425,8 @@ def main():
             dt = float(t.item())
         e2e = {"value": flops_step / dt / 1e9, "unit": "GFLOPS", "ms_per_step": dt * 1e3,
                "h2d_bytes_per_step": int(xh.numel() * 8) * world, "d2h_bytes_per_step": int(yh.numel() * 8) * world,
-               "api": "dasp_spmv" + ("_scatter" if args.fused else "") + " (row-slab iteration)"}
+               "api": "dasp_spmv" + ("_scatter" if args.fused else "") + (" + dasp_gather_halo" if args.halo else "")
+                      + " (row-slab iteration)"}
     if not use_slab and args.e2e_steps > 0:
         xdt_np = {"f64": np.float64, "f16": np.float16, "f32": np.float32}[args.dtype]
         xh = torch.from_numpy(x_global.astype(xdt_np)).pin_memory()
@@ -471,14 +485,15 @@ def main():
                        "m": int(spec.m), "n": int(spec.n), "nnz": nnz_total, "variant": args.variant,
                        "kernel": "pipeline" if info.get("pipeline") else "direct", "panel_rows": info["panel_rows"],
                        "parallelism": f"row-slab x{world}" + (
-                           (" + fused NVLink scatter of y into every rank's x" if args.fused else " + NCCL all-gather of x")
-                           if use_slab else ""),
+                           (" + fused NVLink scatter of y into every rank's x" if args.fused else
+                            " + sparse halo all_to_all overlapped with the local sub-matrix" if args.halo else
+                            " + NCCL all-gather of x") if use_slab else ""),
                        "l2": "inputs larger than L2 (packed A streamed every step); x stays L2-resident "
                              "across steps as in the paper's averaged back-to-back runs"},
             "effective_gbs": eff_gbs, "effective_frac_of_peak": eff_gbs / peak,
             "alg_gbs_step": bm["total"] * world / (ms_step * 1e-3) / 1e9 if world == 1 else None,
-            "gpu_launches": int(info["launches_per_spmv"]) * args.steps,
-            "gpu_launches_per_step": int(info["launches_per_spmv"]),
+            "gpu_launches": launches_step * args.steps,
+            "gpu_launches_per_step": launches_step,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "variant_compare": compare, "preprocessing": gpu_build,
             "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,

@@ -230,6 +230,16 @@ dasp_status_t dasp_partition_rows(const int64_t* row_ptr, int64_t m, int32_t npa
 dasp_status_t dasp_remap_columns(int32_t* col, int64_t nnz, const int64_t* starts, int32_t nparts,
                                  int64_t* stride);
 
+/*
+ * dasp_gather_halo — the pack step of the sparse x exchange:
+ * dst[k] = src[idx[k]] for 0 <= k < n, on DEVICE arrays, enqueued on `stream`.  elem_bytes is the
+ * x element size (8 = f64, 4 = f32, 2 = f16 bits); values are copied bit for bit.  idx[k] must be
+ * in [0, len(src)) (not checked on the device).  n == 0 is a no-op.  Errors: DASP_ERR_INVALID_ARG
+ * (null pointer with n > 0, n < 0, elem_bytes not 2/4/8), DASP_ERR_CUDA (launch failure).
+ */
+dasp_status_t dasp_gather_halo(const void* src, const int32_t* idx, int64_t n, void* dst, int32_t elem_bytes,
+                               void* stream);
+
 /* Kernel ids of the per-kernel timing below. */
 typedef enum {
     DASP_K_MAIN = 0,      /* medium + short/single kernel, panel by panel (Alg. 3-5); with

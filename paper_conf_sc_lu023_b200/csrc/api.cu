@@ -45,6 +45,10 @@ struct dasp_plan_s {
     void* d_items = nullptr;              // uint64 item words of the pipelined kernel
     int64_t n_items = 0, pipe_blocks = 0;
     bool pipe = false;                    // persistent TMA-staged kernel (else the one-warp-per-item kernel)
+    bool dyn = false;                     // persistent main kernel with the dynamic (atomic) schedule
+    void* d_item_start = nullptr;         // int64 [n_panels + 1] first work item of every panel
+    void* d_sched = nullptr;              // 2 x u64 counters of the dynamic schedule (self-resetting)
+    int64_t dyn_items = 0, dyn_blocks = 0;
     size_t apw_bytes = 0;                 // L2 persisting access-policy window over x (0 = off)
     float apw_hit = 1.0f;
     // timing
@@ -65,6 +69,7 @@ int sa(int dtype) { return dtype == DASP_R_16F ? 4 : 8; }   // long-group partia
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
 constexpr bool kSplitShortDefault = false;
+constexpr bool kDynSchedDefault = false;
 constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // TMA windows may read up to 16 B past an array's end
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
@@ -103,7 +108,10 @@ void free_device(dasp_plan_s* p) {
     if (p->d_unit_order) cudaFree(p->d_unit_order);
     if (p->d_items) cudaFree(p->d_items);
     if (p->d_tile_meta) cudaFree(p->d_tile_meta);
+    if (p->d_item_start) cudaFree(p->d_item_start);
+    if (p->d_sched) cudaFree(p->d_sched);
     p->d_panels = p->d_blk_panel = p->d_unit_order = p->d_items = p->d_tile_meta = nullptr;
+    p->d_item_start = p->d_sched = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -201,6 +209,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         p->split_short = ss ? std::atoi(ss) != 0 : kSplitShortDefault;
     }
     int64_t blk = 0;
+    std::vector<int64_t> item_start(1, 0);
     for (int64_t q = 0; q < f.n_panels; ++q) {
         const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
         dasp::PanelDesc& d = desc[q];
@@ -220,6 +229,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
             d.t13 = d.t4 = d.t22 = d.ts = 0;
         }
         const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
+        item_start.push_back(item_start.back() + warps);
         const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
         blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
         blk += nb;
@@ -303,6 +313,25 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         // persistent grid: every SM full, never more warps than items
         const int64_t wpb = dasp::pipe_warps_per_block();
         p->pipe_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->n_items + wpb - 1) / wpb);
+    }
+    // dynamic schedule of the main kernel (DASP_SCHED=1 / options)
+    {
+        const char* se = std::getenv("DASP_SCHED");
+        p->dyn = se ? std::atoi(se) == 1 : kDynSchedDefault;
+        p->dyn_items = item_start.back();
+        if (p->dyn && !p->pipe && p->dyn_items > 0) {
+            int bps = 0, nsm = 0;
+            if (dasp::main_dyn_occupancy(p->dtype, p->variant, &bps) != cudaSuccess ||
+                cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess)
+                return DASP_ERR_CUDA;
+            const int64_t wpb = dasp::WARPS_PER_BLOCK;
+            p->dyn_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->dyn_items + wpb - 1) / wpb);
+            if ((st = upload(&p->d_item_start, item_start.data(), item_start.size() * 8)) != DASP_OK) return st;
+            const uint64_t zero[2] = {0, 0};
+            if ((st = upload(&p->d_sched, zero, sizeof(zero))) != DASP_OK) return st;
+        } else {
+            p->dyn = false;
+        }
     }
     // optional persisting L2 access-policy window over x (DASP_X_APW=1; measured slower on C3,
     // profiles/r01, so off by default)
@@ -523,6 +552,8 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.rbw = p->rbw;
     mp.class_mask = 7;
     mp.extra = extra;
+    mp.item_start = static_cast<const int64_t*>(p->d_item_start);
+    mp.sched = static_cast<unsigned long long*>(p->d_sched);
     // DASP_PROFILE_CLASS (profiling only; the other classes' rows are then NOT computed):
     // 1 = long units, 2 = medium warps, 3 = short tiles
     if (const char* pc = std::getenv("DASP_PROFILE_CLASS")) {
@@ -543,6 +574,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
         if (p->pipe)
             return dasp::launch_pipe(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_items), p->n_items,
                                      p->pipe_blocks, s);
+        if (p->dyn) return dasp::launch_main_dyn(mp, p->dtype, variant, p->dyn_blocks, p->dyn_items, s);
         return dasp::launch_main(mp, p->dtype, variant, p->blocks, s, x, p->apw_bytes, p->apw_hit);
     });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
@@ -677,6 +709,14 @@ dasp_status_t dasp_remap_columns(int32_t* col, int64_t nnz, const int64_t* start
         col[k] = static_cast<int32_t>(q * S + (c - starts[q]));
     }
     return bad ? DASP_ERR_INVALID_ARG : DASP_OK;
+}
+
+dasp_status_t dasp_gather_halo(const void* src, const int32_t* idx, int64_t n, void* dst, int32_t elem_bytes,
+                               void* stream) {
+    if (n < 0 || (n > 0 && (!src || !idx || !dst)) || (elem_bytes != 2 && elem_bytes != 4 && elem_bytes != 8))
+        return DASP_ERR_INVALID_ARG;
+    return dasp::launch_gather(src, idx, n, dst, elem_bytes, static_cast<cudaStream_t>(stream)) == cudaSuccess
+               ? DASP_OK : DASP_ERR_CUDA;
 }
 
 dasp_status_t dasp_plan_set_timing(dasp_plan_t p, int32_t capacity) {

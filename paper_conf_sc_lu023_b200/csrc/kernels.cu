@@ -77,6 +77,10 @@ __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
 template <int DT> struct ValIO;
 template <> struct ValIO<0> {
     using T = double;
+    using R = double;   // register image of one value while its load is in flight
+    static __device__ __forceinline__ double cv(R r) { return r; }
+    static __device__ __forceinline__ void ld4r(const T* p, uint64_t pol, R (&v)[4]) { ld4_f64(p, pol, v); }
+    static __device__ __forceinline__ R ld1r(const T* p, uint64_t pol) { return ld1_f64(p, pol); }
     static __device__ __forceinline__ void ld2(const T* p, uint64_t pol, double& a, double& b) { ld2_f64(p, pol, a, b); }
     static __device__ __forceinline__ void ld4(const T* p, uint64_t pol, double (&v)[4]) { ld4_f64(p, pol, v); }
     static __device__ __forceinline__ double ld1(const T* p, uint64_t pol) { return ld1_f64(p, pol); }
@@ -84,6 +88,10 @@ template <> struct ValIO<0> {
 };
 template <> struct ValIO<2> {
     using T = float;
+    using R = uint32_t; // the float's bits: converted at use, one register per value in flight
+    static __device__ __forceinline__ double cv(R r) { return static_cast<double>(__uint_as_float(r)); }
+    static __device__ __forceinline__ void ld4r(const T* p, uint64_t pol, R (&v)[4]) { ld4_b32(p, pol, v); }
+    static __device__ __forceinline__ R ld1r(const T* p, uint64_t pol) { return ld1_b32(p, pol); }
     static __device__ __forceinline__ void ld2(const T* p, uint64_t pol, double& a, double& b) {
         uint32_t u0, u1;
         ld2_b32(p, pol, u0, u1);
@@ -280,76 +288,118 @@ __device__ __forceinline__ RbMeta rb_meta(const MainParams& P, int64_t rb, int l
                   static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i)};
 }
 
-template <int DT, int VAR>
-__device__ __forceinline__ void medium_rb_f64(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
-    const int t = lane & 3;
-    const int64_t base = M.base, ib = M.ib, ie = M.ib + M.ilen;
-    const int32_t orow = M.orow;
+// A row-block is processed in two halves so that a warp can keep the round-1 loads of two
+// row-blocks in flight before it gathers x for the first (DASP_PAIR_*; the loads of a
+// row-block depend on nothing but its metadata, R18):
+//   medium_load_*   round 1: the first 4-block chunk (256/128-bit loads), the ragged last chunk
+//                   and this lane's first irregular element;
+//   medium_finish_* the gathers, the remaining chunks, the irregular tail and the y store.
+// A row-block with nelem = ilen = 0 and orow = -1 issues no load and stores nothing.
+template <int DT> struct MedLd {
+    typename ValIO<DT>::R va[4], vr[3], vi;
+    uint32_t ca[4], cr[3], ci;
+};
+template <int DT>
+__device__ __forceinline__ void medium_load_f64(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, MedLd<DT>& L) {
+    using IO = ValIO<DT>;
     const int nreg = M.nelem >> 5;
     const int nfull = nreg >> 2, rem = nreg & 3;
-    using IO = ValIO<DT>;
-    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + base;
-    const int32_t* rc = P.reg_col + base;
-    const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
-    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
-    // round 1: first chunk (4 blocks, 256-bit value load), the ragged last chunk and the
-    // first irregular element of this lane, all in flight together
-    double va[4] = {0.0, 0.0, 0.0, 0.0};
-    uint32_t ca[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
-    if (nfull > 0) { IO::ld4(rv + lane * 4, pol, va); ld4_b32(rc + lane * 4, pol, ca); }
-    double vr[3] = {0.0, 0.0, 0.0};
-    uint32_t cr[3] = {0xffffffffu, 0xffffffffu, 0xffffffffu};
+    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
+    const int32_t* rc = P.reg_col + M.base;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { L.va[j] = 0; L.ca[j] = 0xffffffffu; }
+    if (nfull > 0) { IO::ld4r(rv + lane * 4, pol, L.va); ld4_b32(rc + lane * 4, pol, L.ca); }
     const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane * rem;
 #pragma unroll
-    for (int j = 0; j < 3; ++j)
-        if (j < rem) { vr[j] = IO::ld1(rv + rbase + j, pol); cr[j] = ld1_b32(rc + rbase + j, pol); }
-    int64_t k = ib + t;
-    double vi = 0.0;
-    uint32_t ci = 0xffffffffu;
-    if (k < ie) { vi = IO::ld1(iv + k, pol); ci = ld1_b32(P.irr_col + k, pol); }
+    for (int j = 0; j < 3; ++j) {
+        L.vr[j] = 0; L.cr[j] = 0xffffffffu;
+        if (j < rem) { L.vr[j] = IO::ld1r(rv + rbase + j, pol); L.cr[j] = ld1_b32(rc + rbase + j, pol); }
+    }
+    const int64_t k = M.ib + (lane & 3);
+    L.vi = 0; L.ci = 0xffffffffu;
+    if (k < M.ib + M.ilen) { L.vi = IO::ld1r(static_cast<const typename IO::T*>(P.irr_val) + k, pol); L.ci = ld1_b32(P.irr_col + k, pol); }
+}
+template <int DT, int VAR>
+__device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbMeta& M, const MedLd<DT>& L, int lane,
+                                                  uint64_t pol) {
+    using IO = ValIO<DT>;
+    const int t = lane & 3;
+    const int nreg = M.nelem >> 5;
+    const int nfull = nreg >> 2, rem = nreg & 3;
+    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
+    const int32_t* rc = P.reg_col + M.base;
+    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
     double c0 = 0.0, c1 = 0.0, part = 0.0;
+    typename IO::R va[4];
+    uint32_t ca[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { va[j] = L.va[j]; ca[j] = L.ca[j]; }
     for (int ch = 0; ch < nfull; ++ch) {
-        if (ch > 0) { IO::ld4(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
+        if (ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
         double xv[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
-            if constexpr (VAR == VAR_MMA) dmma(c0, c1, va[j], xv[j]);
-            else part = fma(va[j], xv[j], part);
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, IO::cv(va[j]), xv[j]);
+            else part = fma(IO::cv(va[j]), xv[j], part);
         }
     }
     double xr[3];
 #pragma unroll
-    for (int j = 0; j < 3; ++j) xr[j] = IO::gx(x, cr[j]);     // pads / unused slots read 0
-    const double xi = IO::gx(x, ci);
+    for (int j = 0; j < 3; ++j) xr[j] = IO::gx(x, L.cr[j]);   // pads / unused slots read 0
+    const double xi = IO::gx(x, L.ci);
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
         if (j < rem) {                                     // rem is warp-uniform
-            if constexpr (VAR == VAR_MMA) dmma(c0, c1, vr[j], xr[j]);
-            else part = fma(vr[j], xr[j], part);
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, IO::cv(L.vr[j]), xr[j]);
+            else part = fma(IO::cv(L.vr[j]), xr[j], part);
         }
     }
     if constexpr (VAR == VAR_MMA) {                        // Alg. 3 l.13-17: diagonal -> quad g
         const double d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.0;
     }
-    part = fma(vi, xi, part);                              // Alg. 3 l.20-24: irregular part
-    for (k += 4; k < ie; k += 4) part = fma(IO::ld1(iv + k, pol), IO::gx(x, ld1_b32(P.irr_col + k, pol)), part);
+    part = fma(IO::cv(L.vi), xi, part);                    // Alg. 3 l.20-24: irregular part
+    const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+    for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
+        part = fma(IO::ld1(iv + k, pol), IO::gx(x, ld1_b32(P.irr_col + k, pol)), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
-    if (t == 0) store_y<DT>(P, orow, part);                 // Alg. 3 l.25 through the output map (R9)
+    if (t == 0) store_y<DT>(P, M.orow, part);              // Alg. 3 l.25 through the output map (R9)
 }
 
-template <int VAR>
-__device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
-    const int t = lane & 3;
-    const int64_t base = M.base, ib = M.ib, ie = M.ib + M.ilen;
-    const int32_t orow = M.orow;
+struct MedLdH {
+    uint32_t va[4], ca[8], vr[3], cr[6], ci;
+    uint16_t vi;
+};
+__device__ __forceinline__ void medium_load_f16(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, MedLdH& L) {
     const int nreg = M.nelem >> 6;
     const int nfull = nreg >> 2, rem = nreg & 3;
-    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + base;
-    const int32_t* rc = P.reg_col + base;
+    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
+    const int32_t* rc = P.reg_col + M.base;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) L.va[j] = 0u;
+#pragma unroll
+    for (int e = 0; e < 8; ++e) L.ca[e] = 0xffffffffu;
+    if (nfull > 0) { ld4_b32(rv + lane * 8, pol, L.va); ld8_b32(rc + lane * 8, pol, L.ca); }
+    const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2 * rem;
+#pragma unroll
+    for (int j = 0; j < 3; ++j) {
+        L.vr[j] = 0u; L.cr[2 * j] = L.cr[2 * j + 1] = 0xffffffffu;
+        if (j < rem) { L.vr[j] = ld1_b32(rv + rbase + 2 * j, pol); ld2_b32(rc + rbase + 2 * j, pol, L.cr[2 * j], L.cr[2 * j + 1]); }
+    }
+    const int64_t k = M.ib + (lane & 3);
+    L.vi = 0; L.ci = 0xffffffffu;
+    if (k < M.ib + M.ilen) { L.vi = __ldg(static_cast<const unsigned short*>(P.irr_val) + k); L.ci = ld1_b32(P.irr_col + k, pol); }
+}
+template <int VAR>
+__device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbMeta& M, const MedLdH& L, int lane, uint64_t pol) {
+    const int t = lane & 3;
+    const int nreg = M.nelem >> 6;
+    const int nfull = nreg >> 2, rem = nreg & 3;
+    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
+    const int32_t* rc = P.reg_col + M.base;
     const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
     float c0 = 0.f, c1 = 0.f, part = 0.f;
@@ -364,23 +414,11 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta&
             part = fmaf(av.y, h2f(xb), part);
         }
     };
-    // round 1: first chunk (4 blocks: 16 B values, 32 B columns), the ragged last chunk and
-    // the first irregular element
-    uint32_t va[4] = {0u, 0u, 0u, 0u}, ca[8];
+    uint32_t va[4], ca[8];
 #pragma unroll
-    for (int e = 0; e < 8; ++e) ca[e] = 0xffffffffu;
-    if (nfull > 0) { ld4_b32(rv + lane * 8, pol, va); ld8_b32(rc + lane * 8, pol, ca); }
-    uint32_t vr[3] = {0u, 0u, 0u}, cr[6];
+    for (int j = 0; j < 4; ++j) va[j] = L.va[j];
 #pragma unroll
-    for (int e = 0; e < 6; ++e) cr[e] = 0xffffffffu;
-    const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2 * rem;
-#pragma unroll
-    for (int j = 0; j < 3; ++j)
-        if (j < rem) { vr[j] = ld1_b32(rv + rbase + 2 * j, pol); ld2_b32(rc + rbase + 2 * j, pol, cr[2 * j], cr[2 * j + 1]); }
-    int64_t k = ib + t;
-    uint16_t vi = 0;
-    uint32_t ci = 0xffffffffu;
-    if (k < ie) { vi = __ldg(iv + k); ci = ld1_b32(P.irr_col + k, pol); }
+    for (int e = 0; e < 8; ++e) ca[e] = L.ca[e];
     for (int ch = 0; ch < nfull; ++ch) {
         if (ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
 #pragma unroll
@@ -388,17 +426,72 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta&
     }
 #pragma unroll
     for (int j = 0; j < 3; ++j)
-        if (j < rem) block(vr[j], cr[2 * j], cr[2 * j + 1]);   // rem is warp-uniform
+        if (j < rem) block(L.vr[j], L.cr[2 * j], L.cr[2 * j + 1]);   // rem is warp-uniform
     if constexpr (VAR == VAR_MMA) {
         const float d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.f;
     }
-    part = fmaf(h2f(vi), h2f(gxh(x, ci)), part);
-    for (k += 4; k < ie; k += 4)
+    part = fmaf(h2f(L.vi), h2f(gxh(x, L.ci)), part);
+    for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
         part = fmaf(h2f(__ldg(iv + k)), h2f(gxh(x, ld1_b32(P.irr_col + k, pol))), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
-    if (t == 0) store_y<1>(P, orow, part);
+    if (t == 0) store_y<1>(P, M.orow, part);
+}
+
+template <int DT, int VAR>
+__device__ __forceinline__ void medium_rb_f64(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
+    MedLd<DT> L;
+    medium_load_f64<DT>(P, M, lane, pol, L);
+    medium_finish_f64<DT, VAR>(P, M, L, lane, pol);
+}
+template <int VAR>
+__device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta& M, int lane, uint64_t pol) {
+    MedLdH L;
+    medium_load_f16(P, M, lane, pol, L);
+    medium_finish_f16<VAR>(P, M, L, lane, pol);
+}
+
+// row-blocks in flight per warp step (1 or 2), per value type
+#ifndef DASP_PAIR_F64
+#define DASP_PAIR_F64 1
+#endif
+#ifndef DASP_PAIR_F16
+#define DASP_PAIR_F16 1
+#endif
+#ifndef DASP_PAIR_F32
+#define DASP_PAIR_F32 1
+#endif
+template <int DT> __host__ __device__ constexpr int med_pair() { return DT == 0 ? DASP_PAIR_F64 : (DT == 1 ? DASP_PAIR_F16 : DASP_PAIR_F32); }
+
+template <int DT, int VAR>
+__device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int64_t rb1, int lane, uint64_t pol) {
+    if constexpr (med_pair<DT>() == 2) {
+        for (int64_t rb = rb0; rb < rb1; rb += 2) {
+            const RbMeta MA = rb_meta(P, rb, lane);
+            const RbMeta MB = rb + 1 < rb1 ? rb_meta(P, rb + 1, lane) : RbMeta{0, 0, 0, 0, -1};
+            if constexpr (DT == 1) {
+                MedLdH LA, LB;
+                medium_load_f16(P, MA, lane, pol, LA);
+                medium_load_f16(P, MB, lane, pol, LB);
+                medium_finish_f16<VAR>(P, MA, LA, lane, pol);
+                medium_finish_f16<VAR>(P, MB, LB, lane, pol);
+            } else {
+                MedLd<DT> LA, LB;
+                medium_load_f64<DT>(P, MA, lane, pol, LA);
+                medium_load_f64<DT>(P, MB, lane, pol, LB);
+                medium_finish_f64<DT, VAR>(P, MA, LA, lane, pol);
+                medium_finish_f64<DT, VAR>(P, MB, LB, lane, pol);
+            }
+        }
+    } else {
+        for (int64_t rb = rb0; rb < rb1; ++rb) {
+            // (prefetching the next row-block's metadata here was measured: it costs registers
+            // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta_prefetch_rbw.jsonl)
+            if constexpr (DT == 1) medium_rb_f16<VAR>(P, rb_meta(P, rb, lane), lane, pol);
+            else medium_rb_f64<DT, VAR>(P, rb_meta(P, rb, lane), lane, pol);
+        }
+    }
 }
 
 // ------------------------------------------------------------------------------------------
@@ -538,6 +631,27 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
     }
 }
 
+// short tile t of panel D (tiles [1&3][len4][2&2][singles], Alg. 4-5)
+template <int DT, int VAR>
+__device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc* D, int64_t t, int lane, uint64_t pol) {
+    const int64_t t13 = __ldg(&D->t13), t4 = __ldg(&D->t4), t22 = __ldg(&D->t22);
+    if (t >= t13 + t4 + t22 + __ldg(&D->ts) || !(P.class_mask & 4)) return;
+    const int64_t tile = __ldg(&D->tile0) + t;
+    const int64_t out0 = __ldg(&D->out0);
+    int cat;
+    int64_t obase;
+    if (t < t13) { cat = 0; obase = out0 + t * 64; }
+    else if (t < t13 + t4) { cat = 1; obase = out0 + 64 * t13 + (t - t13) * 32; }
+    else if (t < t13 + t4 + t22) { cat = 2; obase = out0 + 64 * t13 + 32 * t4 + (t - t13 - t4) * 64; }
+    else {
+        obase = out0 + 64 * t13 + 32 * t4 + 64 * t22 + (t - t13 - t4 - t22) * 128;
+        singles_tile<DT>(P, tile, obase, lane, pol);
+        return;
+    }
+    if constexpr (DT == 1) short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
+    else short_tile_f64<DT, VAR>(P, cat, tile, obase, lane, pol);
+}
+
 // ------------------------------------------------------------------------------------------
 // the fused main kernel
 // ------------------------------------------------------------------------------------------
@@ -546,6 +660,9 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
 #endif
 #ifndef DASP_MIN_BLOCKS_F16
 #define DASP_MIN_BLOCKS_F16 4
+#endif
+#ifndef DASP_MIN_BLOCKS_F32
+#define DASP_MIN_BLOCKS_F32 4
 #endif
 // long rows, phase 1 (Alg. 2 l.1-16), in their own launch: the unit path needs few registers
 // and is gather-latency bound, so it runs at higher occupancy (40 registers, 48 warps
@@ -571,7 +688,8 @@ dasp_long_kernel(const MainParams P, int64_t n_units) {
 
 // medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
 template <int DT, int VAR>
-__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : DASP_MIN_BLOCKS_F16) dasp_main_kernel(const MainParams P) {
+__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32))
+dasp_main_kernel(const MainParams P) {
     const int lane = threadIdx.x & 31;
     // role of this warp inside its panel; the descriptor fields are loaded only on the branch
     // that needs them so they do not stay live (register pressure = occupancy)
@@ -584,31 +702,51 @@ __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : DASP
         const int64_t rbp0 = __ldg(&D->rb0);
         const int64_t rb0 = rbp0 + w * P.rbw;
         const int64_t rb1 = min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb));
-        for (int64_t rb = rb0; rb < rb1; ++rb) {
-            // (prefetching the next row-block's metadata here was measured: it costs registers
-            // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta.jsonl)
-            if constexpr (DT == 1) medium_rb_f16<VAR>(P, rb_meta(P, rb, lane), lane, pol);
-            else medium_rb_f64<DT, VAR>(P, rb_meta(P, rb, lane), lane, pol);
+        medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);
+        return;
+    }
+    short_item<DT, VAR>(P, D, w - nmw, lane, pol);
+}
+
+// persistent variant with a dynamic schedule: every warp takes the next work item from a
+// global counter (prefetching the following one while it works), walks the panel table
+// forward, and runs the same medium chunk / short tile code.  Removes the last-wave tail and
+// the per-block straggler slots of the static grid; the last warp to finish resets the
+// counters for the next launch.
+template <int DT, int VAR>
+__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32))
+dasp_main_dyn_kernel(const MainParams P, int64_t n_items) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t pol = stream_policy();
+    unsigned long long* ctr = P.sched;
+    long long c = lane == 0 ? static_cast<long long>(atomicAdd(ctr, 1ull)) : 0;
+    c = __shfl_sync(FULL, c, 0);
+    int q = 0;
+    while (c < n_items) {
+        const long long nxt = lane == 0 ? static_cast<long long>(atomicAdd(ctr, 1ull)) : 0;
+        while (c >= __ldg(P.item_start + q + 1)) ++q;
+        const PanelDesc* D = P.panels + q;
+        const int64_t local = c - __ldg(P.item_start + q);
+        const int64_t nmw = __ldg(&D->nmw);
+        if (local < nmw) {
+            if (P.class_mask & 2) {
+                const int64_t rbp0 = __ldg(&D->rb0);
+                const int64_t rb0 = rbp0 + local * P.rbw;
+                medium_rbs<DT, VAR>(P, rb0, min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb)), lane, pol);
+            }
+        } else {
+            short_item<DT, VAR>(P, D, local - nmw, lane, pol);
         }
-        return;
+        c = __shfl_sync(FULL, nxt, 0);
     }
-    const int64_t t = w - nmw;                           // short tiles: [1&3][len4][2&2][singles]
-    const int64_t t13 = __ldg(&D->t13), t4 = __ldg(&D->t4), t22 = __ldg(&D->t22);
-    if (t >= t13 + t4 + t22 + __ldg(&D->ts) || !(P.class_mask & 4)) return;
-    const int64_t tile = __ldg(&D->tile0) + t;
-    const int64_t out0 = __ldg(&D->out0);
-    int cat;
-    int64_t obase;
-    if (t < t13) { cat = 0; obase = out0 + t * 64; }
-    else if (t < t13 + t4) { cat = 1; obase = out0 + 64 * t13 + (t - t13) * 32; }
-    else if (t < t13 + t4 + t22) { cat = 2; obase = out0 + 64 * t13 + 32 * t4 + (t - t13 - t4) * 64; }
-    else {
-        obase = out0 + 64 * t13 + 32 * t4 + 64 * t22 + (t - t13 - t4 - t22) * 128;
-        singles_tile<DT>(P, tile, obase, lane, pol);
-        return;
+    if (lane == 0) {
+        __threadfence();
+        const unsigned long long total = static_cast<unsigned long long>(gridDim.x) * (MAIN_THREADS / 32);
+        if (atomicAdd(ctr + 1, 1ull) == total - 1) {   // every warp has made its last grab
+            atomicExch(ctr, 0ull);
+            atomicExch(ctr + 1, 0ull);
+        }
     }
-    if constexpr (DT == 1) short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
-    else short_tile_f64<DT, VAR>(P, cat, tile, obase, lane, pol);
 }
 
 // short tiles in their own launch (split mode): tile_meta[t] = cat << 62 | output base
@@ -1135,6 +1273,15 @@ __global__ void __launch_bounds__(PW * 32) dasp_pipe_kernel(const MainParams P, 
     }
 }
 
+// halo pack for the sparse x exchange: dst[k] = src[idx[k]], elements of
+// E bytes moved as raw words (no arithmetic)
+template <typename W>
+__global__ void __launch_bounds__(256) dasp_gather_kernel(const W* __restrict__ src, const int32_t* __restrict__ idx,
+                                                          int64_t n, W* __restrict__ dst) {
+    for (int64_t k = static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x; k < n; k += static_cast<int64_t>(gridDim.x) * 256)
+        dst[k] = src[__ldg(idx + k)];
+}
+
 }  // namespace
 
 template <typename Kern>
@@ -1170,6 +1317,25 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
     else e = launch_ex(mma ? dasp_main_kernel<2, VAR_MMA> : dasp_main_kernel<2, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
+}
+
+cudaError_t launch_main_dyn(const MainParams& p, int dtype, int variant, int64_t blocks, int64_t n_items, cudaStream_t s) {
+    if (blocks <= 0 || n_items <= 0) return cudaSuccess;
+    const unsigned nb = static_cast<unsigned>(blocks);
+    const bool mma = variant == VAR_MMA;
+    if (dtype == 0) (mma ? dasp_main_dyn_kernel<0, VAR_MMA> : dasp_main_dyn_kernel<0, VAR_CUDACORE>)<<<nb, MAIN_THREADS, 0, s>>>(p, n_items);
+    else if (dtype == 1) (mma ? dasp_main_dyn_kernel<1, VAR_MMA> : dasp_main_dyn_kernel<1, VAR_CUDACORE>)<<<nb, MAIN_THREADS, 0, s>>>(p, n_items);
+    else (mma ? dasp_main_dyn_kernel<2, VAR_MMA> : dasp_main_dyn_kernel<2, VAR_CUDACORE>)<<<nb, MAIN_THREADS, 0, s>>>(p, n_items);
+    return cudaGetLastError();
+}
+
+cudaError_t main_dyn_occupancy(int dtype, int variant, int* bps) {
+    const bool mma = variant == VAR_MMA;
+    if (dtype == 0)
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, mma ? dasp_main_dyn_kernel<0, VAR_MMA> : dasp_main_dyn_kernel<0, VAR_CUDACORE>, MAIN_THREADS, 0);
+    if (dtype == 1)
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, mma ? dasp_main_dyn_kernel<1, VAR_MMA> : dasp_main_dyn_kernel<1, VAR_CUDACORE>, MAIN_THREADS, 0);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, mma ? dasp_main_dyn_kernel<2, VAR_MMA> : dasp_main_dyn_kernel<2, VAR_CUDACORE>, MAIN_THREADS, 0);
 }
 
 template <int DT, int VAR>
@@ -1248,6 +1414,20 @@ cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_
     if (dtype == 0) dasp_scale_kernel<0><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
     else if (dtype == 1) dasp_scale_kernel<1><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
     else dasp_scale_kernel<2><<<static_cast<unsigned>(blocks), 256, 0, s>>>(y, m, beta, extra);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gather(const void* src, const int32_t* idx, int64_t n, void* dst, int elem_bytes, cudaStream_t s) {
+    if (n == 0) return cudaSuccess;
+    int64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    const unsigned b = static_cast<unsigned>(blocks);
+    if (elem_bytes == 8)
+        dasp_gather_kernel<uint64_t><<<b, 256, 0, s>>>(static_cast<const uint64_t*>(src), idx, n, static_cast<uint64_t*>(dst));
+    else if (elem_bytes == 4)
+        dasp_gather_kernel<uint32_t><<<b, 256, 0, s>>>(static_cast<const uint32_t*>(src), idx, n, static_cast<uint32_t*>(dst));
+    else
+        dasp_gather_kernel<uint16_t><<<b, 256, 0, s>>>(static_cast<const uint16_t*>(src), idx, n, static_cast<uint16_t*>(dst));
     return cudaGetLastError();
 }
 

@@ -53,6 +53,10 @@ struct MainParams {
     int32_t rbw;
     int32_t class_mask;       // bit 0 long, bit 1 medium, bit 2 short (profiling; 7 = all)
     ExtraDst extra;
+    // dynamic schedule of the main kernel (launch_main_dyn): panel q's work items are
+    // [item_start[q], item_start[q+1]) = its medium warps' row-block chunks, then its short tiles
+    const int64_t* item_start;
+    unsigned long long* sched;  // [0] next item, [1] finished warps; both 0 between launches
 };
 
 struct FinishParams {
@@ -71,6 +75,10 @@ struct FinishParams {
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
+// persistent main kernel with dynamic (atomic counter) work distribution over the items of
+// MainParams::item_start; blocks = resident blocks (main_dyn_occupancy x SMs) or fewer
+cudaError_t launch_main_dyn(const MainParams& p, int dtype, int variant, int64_t blocks, int64_t n_items, cudaStream_t s);
+cudaError_t main_dyn_occupancy(int dtype, int variant, int* blocks_per_sm);
 cudaError_t launch_short(const MainParams& p, int dtype, int variant, const uint64_t* tile_meta, int64_t n_tiles,
                          cudaStream_t s);
 cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s);
@@ -83,5 +91,7 @@ cudaError_t pipe_occupancy(int dtype, int variant, int* blocks_per_sm);   // als
 cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint64_t* items, int64_t n_items,
                         int64_t blocks, cudaStream_t s);
 cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s, const ExtraDst& extra);
+// dst[k] = src[idx[k]] for k < n, elements of elem_bytes (2, 4 or 8) bytes
+cudaError_t launch_gather(const void* src, const int32_t* idx, int64_t n, void* dst, int elem_bytes, cudaStream_t s);
 
 }  // namespace dasp

@@ -28,7 +28,7 @@ STATUS = ["DASP_OK", "DASP_ERR_INVALID_ARG", "DASP_ERR_INVALID_CSR", "DASP_ERR_O
 # every symbol include/dasp.h declares (tests check the library exports all of them)
 EXPORTS = ["dasp_options_default", "dasp_plan_create", "dasp_plan_create_device", "dasp_spmv", "dasp_spmv_ex", "dasp_spmv_scatter", "dasp_spmv_host",
            "dasp_plan_destroy", "dasp_status_string", "dasp_plan_get_info", "dasp_plan_copy_array",
-           "dasp_partition_rows", "dasp_remap_columns", "dasp_plan_set_timing", "dasp_plan_read_timing",
+           "dasp_partition_rows", "dasp_remap_columns", "dasp_gather_halo", "dasp_plan_set_timing", "dasp_plan_read_timing",
            "dasp_version"]
 
 
@@ -85,6 +85,7 @@ def _load():
         "dasp_plan_copy_array": ([vp, i32, vp, ctypes.POINTER(i64)], ctypes.c_int),
         "dasp_partition_rows": ([vp, i64, i32, vp], ctypes.c_int),
         "dasp_remap_columns": ([vp, i64, vp, i32, ctypes.POINTER(i64)], ctypes.c_int),
+        "dasp_gather_halo": ([vp, vp, i64, vp, i32, vp], ctypes.c_int),
         "dasp_plan_set_timing": ([vp, i32], ctypes.c_int),
         "dasp_plan_read_timing": ([vp, vp, vp], ctypes.c_int),
         "dasp_version": ([], ctypes.c_char_p),
@@ -296,6 +297,16 @@ def dasp_remap_columns(col: np.ndarray, starts: np.ndarray) -> int:
     _check(_lib.dasp_remap_columns(_ptr(col), len(col), starts.ctypes.data, len(starts) - 1, ctypes.byref(S)),
            "dasp_remap_columns")
     return int(S.value)
+
+
+def dasp_gather_halo(src, idx, dst, stream=None):
+    """dst[k] = src[idx[k]] on the device (the halo pack of the sparse x exchange).  src / dst are
+    CUDA tensors of the same element size (2, 4 or 8 bytes), idx an int32 CUDA tensor."""
+    n = idx.numel()
+    if dst.numel() < n or src.element_size() != dst.element_size():
+        raise ValueError("dasp_gather_halo: dst too small or element sizes differ")
+    _check(_lib.dasp_gather_halo(_ptr(src), _ptr(idx), n, _ptr(dst), src.element_size(), _stream_ptr(stream)),
+           "dasp_gather_halo")
 
 
 def dasp_plan_set_timing(plan: Plan, capacity: int):

@@ -20,6 +20,18 @@ torch symmetric memory (every rank maps every peer's buffers over NVLink), and
 ``dasp_spmv_scatter`` stores each y value of this rank's slab into ALL ranks' next x buffer
 (P posted NVLink stores per row, overlapped with the rest of the SpMV), followed by one
 device-side barrier across ranks.  No NCCL call is left on the data path.
+
+``HaloSlabSpMV`` shrinks and hides the exchange instead: each slab is split
+by column owner into a LOCAL sub-matrix (columns inside the slab, indexed 0..rows_p-1, so it
+reads this rank's x slab directly) and a REMOTE sub-matrix whose columns are renumbered
+0..R-1 over the sorted set of remote columns it references (its halo).  One step is
+
+    side stream:  dasp_gather_halo(x_p -> send)  ;  all_to_all_single(recv <- send)   (NCCL)
+    main stream:  dasp_spmv(local, x_p -> y_p, alpha, 0)        (overlaps the exchange)
+                  wait(side) ; dasp_spmv(remote, recv -> y_p, alpha, 1)
+
+so only referenced x values move (a stencil slab exchanges two planes instead of all of x) and
+the local part computes while they move.  x_p is the slab alone (no padded global x).
 """
 from __future__ import annotations
 
@@ -50,13 +62,14 @@ class Slab:
 
 
 def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, reduce_max=None,
-               need_norm: bool = True) -> Slab:
+               need_norm: bool = True, remap: bool = True) -> Slab:
     """generate_rows(row0, nrows) -> CSR of those rows (global columns).  reduce_max(v) -> max over ranks.
-    need_norm=False skips the infinity norm (only the iteration needs it)."""
+    need_norm=False skips the infinity norm (only the iteration needs it); remap=False keeps
+    global columns (the halo mode splits them itself)."""
     starts = slab_bounds(row_lengths, world)
     r0, r1 = int(starts[rank]), int(starts[rank + 1])
     A = generate_rows(r0, r1 - r0)
-    if world == 1:                      # one slab: no remap (also valid for rectangular matrices)
+    if world == 1 or not remap:         # one slab: no remap (also valid for rectangular matrices)
         col, S = np.ascontiguousarray(A.col, dtype=np.int32), A.n
     else:
         col = np.ascontiguousarray(A.col, dtype=np.int32).copy()
@@ -71,7 +84,9 @@ def build_slab(generate_rows, row_lengths: np.ndarray, rank: int, world: int, re
             rs[nz] = np.add.reduceat(absval, A.row_ptr[:-1][nz])
         local = float(rs.max()) if len(rs) else 0.0
         inf_norm = reduce_max(local) if reduce_max else local
-    return Slab(A.row_ptr, col, A.val, r0, r1 - r0, starts, S, inf_norm)
+    slab = Slab(A.row_ptr, col, A.val, r0, r1 - r0, starts, S, inf_norm)
+    slab.remapped = world > 1 and remap
+    return slab
 
 
 def scatter_destinations(peer_base, rank, world, buf_index, n_pad, S, elem_bytes):
@@ -170,3 +185,174 @@ class SlabSpMV:
         st, S = self.slab.starts, self.slab.S
         b = self.x[self.cur].cpu().numpy()
         return np.concatenate([b[q * S: q * S + st[q + 1] - st[q]] for q in range(self.world)])
+
+
+# ------------------------------------------------------------------------------------------
+# sparse halo exchange (f1)
+# ------------------------------------------------------------------------------------------
+class HaloSplit:
+    """A slab split by column owner.  loc_*: CSR over local columns (c - starts[rank]);
+    rem_*: CSR over halo positions; halo: the sorted global columns the slab references outside
+    itself; recv_counts[q]: how many of them rank q owns (halo is grouped by owner because it is
+    sorted and owners are contiguous column ranges)."""
+
+    def __init__(self, loc, rem, halo, recv_counts):
+        (self.loc_row_ptr, self.loc_col, self.loc_val) = loc
+        (self.rem_row_ptr, self.rem_col, self.rem_val) = rem
+        self.halo = halo
+        self.recv_counts = recv_counts
+
+
+def split_halo(row_ptr, col, val, starts, rank) -> HaloSplit:
+    """Split a slab CSR (global columns, square matrix partitioned like its rows) into its local
+    and remote sub-matrices; the per-row order of the nonzeros is kept in both."""
+    starts = np.asarray(starts, dtype=np.int64)
+    n = int(starts[-1])
+    r0, r1 = int(starts[rank]), int(starts[rank + 1])
+    rows = len(row_ptr) - 1
+    c = np.asarray(col, dtype=np.int64)
+    if len(c) and (c.min() < 0 or c.max() >= n):
+        raise ValueError("split_halo: column out of range")
+    own = (c >= r0) & (c < r1)
+    row_of = np.repeat(np.arange(rows, dtype=np.int64), np.diff(row_ptr))
+
+    def sub(mask, newcol):
+        rp = np.zeros(rows + 1, dtype=np.int64)
+        np.cumsum(np.bincount(row_of[mask], minlength=rows), out=rp[1:])
+        return rp, np.ascontiguousarray(newcol, dtype=np.int32), np.ascontiguousarray(val[mask])
+
+    loc = sub(own, c[own] - r0)
+    rc = c[~own]
+    mark = np.zeros(n, dtype=bool)
+    mark[rc] = True
+    halo = np.flatnonzero(mark).astype(np.int64)
+    pos = np.cumsum(mark, dtype=np.int64) - 1
+    rem = sub(~own, pos[rc])
+    recv_counts = (np.searchsorted(halo, starts[1:]) - np.searchsorted(halo, starts[:-1])).astype(np.int64)
+    return HaloSplit(loc, rem, halo, recv_counts)
+
+
+def exchange_lists(split: HaloSplit, starts, rank, world, group=None, device="cpu"):
+    """Setup-time exchange of the halo requests: returns (send_idx int32 local positions, grouped
+    by destination rank, send_counts[q]).  One all_to_all of counts and one of indices."""
+    import torch
+    import torch.distributed as dist
+    dev = torch.device(device)
+    rc = torch.from_numpy(split.recv_counts.copy()).to(dev)
+    sc = torch.empty_like(rc)
+    dist.all_to_all_single(sc, rc, group=group)
+    send_counts = sc.cpu().numpy().astype(np.int64)
+    req = torch.from_numpy(split.halo.copy()).to(dev)
+    got = torch.empty(int(send_counts.sum()), dtype=torch.int64, device=dev)
+    dist.all_to_all_single(got, req, output_split_sizes=send_counts.tolist(),
+                           input_split_sizes=split.recv_counts.tolist(), group=group)
+    send_idx = got.cpu().numpy() - int(np.asarray(starts)[rank])
+    rows = int(np.asarray(starts)[rank + 1] - np.asarray(starts)[rank])
+    if len(send_idx) and (send_idx.min() < 0 or send_idx.max() >= rows):
+        raise RuntimeError("exchange_lists: a peer requested a column this rank does not own")
+    return send_idx.astype(np.int32), send_counts
+
+
+class HaloSlabSpMV:
+    """Iterated SpMV x_{k+1} = alpha*A*x_k with the sparse halo exchange overlapped with the
+    local part (module doc).  ``spmv_local(x, y, alpha)``, ``spmv_remote(h, y, alpha)`` (y +=)
+    and ``pack(x, idx, out)`` are pluggable for the CPU tests; the defaults are libdasp calls."""
+
+    def __init__(self, slab: Slab, world: int, rank: int, device, dtype="f64", group=None,
+                 variant=dasp.DASP_VARIANT_DEFAULT, spmv_local=None, spmv_remote=None, pack=None):
+        import torch
+        if getattr(slab, "remapped", False):
+            raise ValueError("HaloSlabSpMV needs a slab with global columns (build_slab(remap=False))")
+        self.slab, self.world, self.rank, self.group = slab, world, rank, group
+        self.device = torch.device(device)
+        self.split = split_halo(slab.row_ptr, slab.col, slab.val, slab.starts, rank)
+        if world > 1:
+            send_idx, self.send_counts = exchange_lists(self.split, slab.starts, rank, world, group,
+                                                        self.device if self.device.type == "cuda" else "cpu")
+        else:
+            send_idx, self.send_counts = np.zeros(0, np.int32), np.zeros(1, np.int64)
+        tdt = torch.float64
+        self.x = [torch.zeros(slab.rows, dtype=tdt, device=self.device) for _ in range(2)]
+        self.cur = 0
+        self.send_idx = torch.from_numpy(send_idx).to(self.device)
+        self.send = torch.zeros(len(send_idx), dtype=tdt, device=self.device)
+        self.recv = torch.zeros(len(self.split.halo), dtype=tdt, device=self.device)
+        self.n_halo = len(self.split.halo)
+        self.plan = self.plan_rem = None
+        sp = self.split
+        if spmv_local is None:
+            if self.device.type != "cuda":
+                raise RuntimeError("the libdasp slab SpMV needs a CUDA device (no CPU fallback)")
+            dev = self.device.index or 0
+            self.plan = dasp.dasp_plan_create(sp.loc_row_ptr, sp.loc_col, sp.loc_val, slab.rows, slab.rows, dtype,
+                                              device=dev)
+            if self.n_halo:
+                self.plan_rem = dasp.dasp_plan_create(sp.rem_row_ptr, sp.rem_col, sp.rem_val, slab.rows, self.n_halo,
+                                                      dtype, device=dev)
+
+            def _loc(x, y, alpha):
+                dasp.dasp_spmv(self.plan, x, y, alpha, 0.0, torch.cuda.current_stream(self.device), variant=variant,
+                               check=False)
+
+            def _rem(h, y, alpha):
+                dasp.dasp_spmv(self.plan_rem, h, y, alpha, 1.0, torch.cuda.current_stream(self.device),
+                               variant=variant, check=False)
+
+            def _pack(x, idx, out):
+                dasp.dasp_gather_halo(x, idx, out, torch.cuda.current_stream(self.device))
+            spmv_local, spmv_remote, pack = _loc, _rem, _pack
+            self.side = torch.cuda.Stream(self.device)
+        else:
+            self.side = None
+        self.spmv_local, self.spmv_remote, self.pack = spmv_local, spmv_remote, pack
+
+    @property
+    def halo_bytes(self) -> int:
+        """x bytes this rank receives per step (an all-gather would receive (n - rows)*8)."""
+        return self.n_halo * 8
+
+    def set_x(self, x_global: np.ndarray):
+        import torch
+        r0 = self.slab.row0
+        self.x[self.cur].copy_(torch.from_numpy(np.ascontiguousarray(x_global[r0:r0 + self.slab.rows], dtype=np.float64)))
+
+    def my_x(self):
+        return self.x[self.cur]
+
+    def _exchange(self):
+        import torch.distributed as dist
+        if self.world > 1:
+            self.pack(self.x[self.cur], self.send_idx, self.send)
+            dist.all_to_all_single(self.recv, self.send, output_split_sizes=self.split.recv_counts.tolist(),
+                                   input_split_sizes=self.send_counts.tolist(), group=self.group)
+
+    def step(self, alpha=1.0):
+        import torch
+        nxt = self.x[1 - self.cur]
+        if self.side is not None:
+            main = torch.cuda.current_stream(self.device)
+            self.side.wait_stream(main)            # x_cur is final; the last remote SpMV read recv
+            with torch.cuda.stream(self.side):
+                self._exchange()
+            self.spmv_local(self.x[self.cur], nxt, alpha)
+            main.wait_stream(self.side)
+        else:
+            self._exchange()
+            self.spmv_local(self.x[self.cur], nxt, alpha)
+        if self.n_halo:
+            self.spmv_remote(self.recv, nxt, alpha)
+        self.cur = 1 - self.cur
+
+    def x_global(self) -> np.ndarray:
+        """The whole current x on every rank (test / readback helper, one all_gather)."""
+        import torch
+        import torch.distributed as dist
+        st = self.slab.starts
+        if self.world == 1:
+            return self.x[self.cur].cpu().numpy().copy()
+        S = int(max(np.diff(st)))
+        buf = torch.zeros(S, dtype=torch.float64, device=self.device)
+        buf[:self.slab.rows] = self.x[self.cur]
+        parts = [torch.empty_like(buf) for _ in range(self.world)]
+        dist.all_gather(parts, buf, group=self.group)
+        return np.concatenate([parts[q].cpu().numpy()[: st[q + 1] - st[q]] for q in range(self.world)])
