@@ -129,8 +129,10 @@ class ClockSampler:
 # ----------------------------------------------------------------------------------------------
 # bytes per launch: CSR-equivalent and algorithmic (what the DASP format moves)
 # ----------------------------------------------------------------------------------------------
-def byte_model(info, dtype, beta_nonzero=False, split_short=False):
-    """Algorithmic bytes per launch of each kernel."""
+def byte_model(info, dtype, beta_nonzero=False, split_short=False, fused_finish=True):
+    """Algorithmic bytes per launch of each kernel.  fused_finish: the long-row
+    phase 2 and the empty rows run inside dasp_main_kernel (the default; a separate
+    dasp_finish_kernel only with the pipelined kernel)."""
     sv, sx, sy = {"f64": (8, 8, 8), "f16": (2, 2, 4), "f32": (4, 4, 4)}[dtype]
     sa = 4 if dtype == "f16" else 8
     b1 = 2 if beta_nonzero else 1
@@ -148,8 +150,11 @@ def byte_model(info, dtype, beta_nonzero=False, split_short=False):
     finish = (ngp * sa + 8 * (info["row_long"] + 1) + 4 * info["row_long"] + info["row_long"] * sy * b1
               + info["n_empty"] * (4 + sy * b1))
     csr_equiv = nnz * (sv + 4) + (m + 1) * 8 + n * sx + m * sy * b1
-    out = {"dasp_long_kernel": long_, "dasp_main_kernel": main, "dasp_finish_kernel": finish,
-           "total": long_ + main + finish + (short if split_short else 0), "csr_equiv": csr_equiv}
+    if fused_finish:
+        main += finish
+    out = {"dasp_long_kernel": long_, "dasp_main_kernel": main, "dasp_finish_kernel": 0 if fused_finish else finish,
+           "total": long_ + main + (0 if fused_finish else finish) + (short if split_short else 0),
+           "csr_equiv": csr_equiv}
     if split_short:
         out["dasp_short_kernel"] = short + 8 * info["tiles_13"] + 8 * info["tiles_4"] + 8 * info["tiles_22"] \
             + 8 * info["tiles_single"]                                    # + per-tile metadata
@@ -364,7 +369,8 @@ def main():
     nnz_total = int(lens.sum())
     flops_step = 2.0 * nnz_total
     gflops = flops_step / (ms_step * 1e-3) / 1e9
-    bm = byte_model(info, args.dtype, split_short=kern.get("dasp_short_kernel", (0, 0))[1] > 0)
+    bm = byte_model(info, args.dtype, split_short=kern.get("dasp_short_kernel", (0, 0))[1] > 0,
+                    fused_finish=kern.get("dasp_finish_kernel", (0, 0))[1] == 0)
     # whole-job CSR-equivalent bytes: sum over ranks (slab models), else the local one
     csr_bytes = bm["csr_equiv"]
     if world > 1:

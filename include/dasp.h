@@ -244,7 +244,8 @@ dasp_status_t dasp_gather_halo(const void* src, const int32_t* idx, int64_t n, v
 typedef enum {
     DASP_K_MAIN = 0,      /* medium + short/single kernel, panel by panel (Alg. 3-5); with
                              options.pipeline the persistent kernel that also does the long units */
-    DASP_K_FINISH = 1,    /* long phase 2 (Alg. 2 l.17-25) + empty rows */
+    DASP_K_FINISH = 1,    /* long phase 2 (Alg. 2 l.17-25) + empty rows: only with options.pipeline; otherwise
+                             they are the first warps of DASP_K_MAIN */
     DASP_K_SCALE = 2,     /* alpha == 0 quick path */
     DASP_K_LONG = 3,      /* long phase 1 (Alg. 2 l.1-16) */
     DASP_K_SHORT = 4,     /* short tiles when they run in their own kernel (DASP_SPLIT_SHORT) */

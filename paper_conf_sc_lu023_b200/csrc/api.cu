@@ -319,13 +319,14 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         const char* se = std::getenv("DASP_SCHED");
         p->dyn = se ? std::atoi(se) == 1 : kDynSchedDefault;
         p->dyn_items = item_start.back();
-        if (p->dyn && !p->pipe && p->dyn_items > 0) {
+        const int64_t all_items = p->dyn_items + dasp::finish_warps(f.row_long, f.n0);
+        if (p->dyn && !p->pipe && all_items > 0) {
             int bps = 0, nsm = 0;
             if (dasp::main_dyn_occupancy(p->dtype, p->variant, &bps) != cudaSuccess ||
                 cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess)
                 return DASP_ERR_CUDA;
             const int64_t wpb = dasp::WARPS_PER_BLOCK;
-            p->dyn_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->dyn_items + wpb - 1) / wpb);
+            p->dyn_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (all_items + wpb - 1) / wpb);
             if ((st = upload(&p->d_item_start, item_start.data(), item_start.size() * 8)) != DASP_OK) return st;
             const uint64_t zero[2] = {0, 0};
             if ((st = upload(&p->d_sched, zero, sizeof(zero))) != DASP_OK) return st;
@@ -570,16 +571,25 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
         });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }
+    const int64_t n0 = (beta == 1.0 && extra.n == 0) ? 0 : f.n0;   // scatter mode must still copy them
+    // long-row phase 2 and the empty rows run as the first warps of the main kernel (the long
+    // kernel before it has written every partial); only the pipelined kernel keeps a finish launch
+    mp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
+    mp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
+    mp.empty_rows = static_cast<const int32_t*>(p->d[DASP_ARR_EMPTY_ROWS]);
+    mp.row_long = f.row_long;
+    mp.n0 = n0;
+    mp.fin_warps = (!p->pipe && (mp.class_mask & 1)) ? dasp::finish_warps(f.row_long, n0) : 0;
+    const int64_t fin_blocks = (mp.fin_warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
     e = timed(p, DASP_K_MAIN, s, on, [&] {
         if (p->pipe)
             return dasp::launch_pipe(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_items), p->n_items,
                                      p->pipe_blocks, s);
-        if (p->dyn) return dasp::launch_main_dyn(mp, p->dtype, variant, p->dyn_blocks, p->dyn_items, s);
-        return dasp::launch_main(mp, p->dtype, variant, p->blocks, s, x, p->apw_bytes, p->apw_hit);
+        if (p->dyn) return dasp::launch_main_dyn(mp, p->dtype, variant, p->dyn_blocks, mp.fin_warps + p->dyn_items, s);
+        return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s, x, p->apw_bytes, p->apw_hit);
     });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
-    const int64_t n0 = (beta == 1.0 && extra.n == 0) ? 0 : f.n0;   // scatter mode must still copy them
-    if (f.row_long + n0 > 0) {
+    if (p->pipe && f.row_long + n0 > 0) {
         dasp::FinishParams fp;
         fp.partial = p->d_partial;
         fp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
@@ -650,8 +660,8 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
     o->launches_per_spmv = p->pipe ? (p->n_items > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0)
-                                   : (p->n_units > 0 ? 1 : 0) + (p->blocks > 0 ? 1 : 0) + (p->n_tiles > 0 ? 1 : 0) +
-                                         (f.row_long + f.n0 > 0 ? 1 : 0);
+                                   : (p->n_units > 0 ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0) +
+                                         (p->n_tiles > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
     o->pipeline = p->pipe ? 1 : 0;

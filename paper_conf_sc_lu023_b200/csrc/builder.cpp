@@ -42,7 +42,7 @@ template <typename T>
 T* as(HostBuf& b) { return static_cast<T*>(b.ptr); }
 
 // position of slot s (0 <= s < K*nreg) of row g of a row-block, inside the row-block's
-// regular region: lane-interleaved chunks of CW blocks (R18).
+// regular region: lane-interleaved chunks of CW blocks, the ragged last chunk block by block (R18).
 inline int64_t reg_pos(const Geometry& geo, int64_t nreg, int g, int64_t s) {
     int64_t b = s / geo.K;
     int k = static_cast<int>(s % geo.K);
@@ -52,7 +52,8 @@ inline int64_t reg_pos(const Geometry& geo, int64_t nreg, int g, int64_t s) {
     int lane = 4 * g + t;
     int64_t c = b / geo.CW, jb = b % geo.CW;
     int64_t w = std::min<int64_t>(geo.CW, nreg - c * geo.CW);
-    return c * geo.CW * geo.BE + lane * w * geo.EPL + jb * geo.EPL + e;
+    if (w == geo.CW) return c * geo.CW * geo.BE + lane * w * geo.EPL + jb * geo.EPL + e;   // full chunk
+    return c * geo.CW * geo.BE + jb * geo.BE + lane * geo.EPL + e;                          // ragged tail
 }
 
 // position of (4-slot row r in [0,32), inner slot c in [0,4)) inside a short tile

@@ -199,7 +199,8 @@ __global__ void k_med_fill(const int64_t* rp, const int32_t* col, const V* val, 
         const int lane = 4 * g + t;
         const int64_t c = b / CW, jb = b % CW;
         const int64_t w = min(static_cast<int64_t>(CW), nr - c * CW);
-        const int64_t at = base + c * CW * BE + lane * w * EPL + jb * EPL + e;
+        const int64_t at = w == CW ? base + c * CW * BE + lane * w * EPL + jb * EPL + e    // full chunk (R18)
+                                   : base + c * CW * BE + jb * BE + lane * EPL + e;        // ragged tail
         if (s < L) { rv[at] = val[src + s]; rc[at] = col[src + s]; }
         else { rv[at] = V(0); rc[at] = PAD_COL; }
     }

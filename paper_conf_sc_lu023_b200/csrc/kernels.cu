@@ -309,11 +309,11 @@ __device__ __forceinline__ void medium_load_f64(const MainParams& P, const RbMet
 #pragma unroll
     for (int j = 0; j < 4; ++j) { L.va[j] = 0; L.ca[j] = 0xffffffffu; }
     if (nfull > 0) { IO::ld4r(rv + lane * 4, pol, L.va); ld4_b32(rc + lane * 4, pol, L.ca); }
-    const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane * rem;
+    const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane;   // ragged chunk: block j at 32j (R18)
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
         L.vr[j] = 0; L.cr[j] = 0xffffffffu;
-        if (j < rem) { L.vr[j] = IO::ld1r(rv + rbase + j, pol); L.cr[j] = ld1_b32(rc + rbase + j, pol); }
+        if (j < rem) { L.vr[j] = IO::ld1r(rv + rbase + 32 * j, pol); L.cr[j] = ld1_b32(rc + rbase + 32 * j, pol); }
     }
     const int64_t k = M.ib + (lane & 3);
     L.vi = 0; L.ci = 0xffffffffu;
@@ -383,11 +383,11 @@ __device__ __forceinline__ void medium_load_f16(const MainParams& P, const RbMet
 #pragma unroll
     for (int e = 0; e < 8; ++e) L.ca[e] = 0xffffffffu;
     if (nfull > 0) { ld4_b32(rv + lane * 8, pol, L.va); ld8_b32(rc + lane * 8, pol, L.ca); }
-    const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2 * rem;
+    const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2;   // ragged chunk: block j at 64j (R18)
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
         L.vr[j] = 0u; L.cr[2 * j] = L.cr[2 * j + 1] = 0xffffffffu;
-        if (j < rem) { L.vr[j] = ld1_b32(rv + rbase + 2 * j, pol); ld2_b32(rc + rbase + 2 * j, pol, L.cr[2 * j], L.cr[2 * j + 1]); }
+        if (j < rem) { L.vr[j] = ld1_b32(rv + rbase + 64 * j, pol); ld2_b32(rc + rbase + 64 * j, pol, L.cr[2 * j], L.cr[2 * j + 1]); }
     }
     const int64_t k = M.ib + (lane & 3);
     L.vi = 0; L.ci = 0xffffffffu;
@@ -631,6 +631,54 @@ __device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, 
     }
 }
 
+// long-row phase 2 (Alg. 2 l.17-25): 8 lanes per long row (4 rows per warp), each lane sums
+// the partials g0 + sl + 8j with four independent accumulators (loads in flight), then a
+// 3-step shuffle tree.  The order is fixed, so results are deterministic; both the fused main
+// kernel and the separate finish kernel use this routine.
+template <int DT>
+__device__ __forceinline__ typename Tr<DT>::A long_row_sum(const void* partial, const int64_t* group_ptr, int64_t r,
+                                                           int64_t row_long, int lane) {
+    using A = typename Tr<DT>::A;
+    const A* part = static_cast<const A*>(partial);
+    const int sl = lane & 7;
+    A s0 = 0, s1 = 0, s2 = 0, s3 = 0;
+    if (r < row_long) {
+        const int64_t g0 = __ldg(group_ptr + r), g1 = __ldg(group_ptr + r + 1);
+        int64_t k = g0 + sl;
+        for (; k + 24 < g1; k += 32) { s0 += part[k]; s1 += part[k + 8]; s2 += part[k + 16]; s3 += part[k + 24]; }
+        for (; k < g1; k += 8) s0 += part[k];
+    }
+    A s = (s0 + s1) + (s2 + s3);
+    s += __shfl_xor_sync(FULL, s, 1);
+    s += __shfl_xor_sync(FULL, s, 2);
+    s += __shfl_xor_sync(FULL, s, 4);
+    return s;
+}
+// empty rows (R1): y = beta*y (0 when beta == 0, y not read)
+template <int DT>
+__device__ __forceinline__ void empty_row(void* yv, int32_t row, double beta, const ExtraDst& extra) {
+    using Y = typename Tr<DT>::Y;
+    Y* y = static_cast<Y*>(yv);
+    const Y r = beta != 0.0 ? static_cast<Y>(beta) * y[row] : Y(0);
+    y[row] = r;
+    for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[row] = r;
+}
+// finish warp fw of the fused main kernel: long rows 4fw..4fw+3, or empty rows (4 per lane)
+template <int DT>
+__device__ __forceinline__ void finish_warp(const MainParams& P, int64_t fw, int lane) {
+    const int64_t lw = (P.row_long + 3) / 4;
+    if (fw < lw) {
+        const int64_t r = fw * 4 + (lane >> 3);
+        const auto s = long_row_sum<DT>(P.partial, P.group_ptr, r, P.row_long, lane);
+        if ((lane & 7) == 0 && r < P.row_long) store_y<DT>(P, __ldg(P.long_out + r), s);
+        return;
+    }
+    const int64_t e0 = (fw - lw) * 128 + lane * 4;
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+        if (e0 + j < P.n0) empty_row<DT>(P.y, __ldg(P.empty_rows + e0 + j), P.beta, P.extra);
+}
+
 // short tile t of panel D (tiles [1&3][len4][2&2][singles], Alg. 4-5)
 template <int DT, int VAR>
 __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc* D, int64_t t, int lane, uint64_t pol) {
@@ -691,10 +739,17 @@ template <int DT, int VAR>
 __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32))
 dasp_main_kernel(const MainParams P) {
     const int lane = threadIdx.x & 31;
+    const int64_t fin_blocks = (P.fin_warps + WARPS_PER_BLOCK - 1) / WARPS_PER_BLOCK;
+    if (blockIdx.x < fin_blocks) {                       // long-row phase 2 + empty rows
+        const int64_t fw = static_cast<int64_t>(blockIdx.x) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+        if (fw < P.fin_warps) finish_warp<DT>(P, fw, lane);
+        return;
+    }
+    const int64_t b = static_cast<int64_t>(blockIdx.x) - fin_blocks;
     // role of this warp inside its panel; the descriptor fields are loaded only on the branch
     // that needs them so they do not stay live (register pressure = occupancy)
-    const PanelDesc* D = P.panels + __ldg(P.blk_panel + blockIdx.x);
-    int64_t w = (static_cast<int64_t>(blockIdx.x) - __ldg(&D->blk0)) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+    const PanelDesc* D = P.panels + __ldg(P.blk_panel + b);
+    int64_t w = (b - __ldg(&D->blk0)) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
     const uint64_t pol = stream_policy();
     const int64_t nmw = __ldg(&D->nmw);
     if (w < nmw) {                                       // medium rows
@@ -724,9 +779,15 @@ dasp_main_dyn_kernel(const MainParams P, int64_t n_items) {
     int q = 0;
     while (c < n_items) {
         const long long nxt = lane == 0 ? static_cast<long long>(atomicAdd(ctr, 1ull)) : 0;
-        while (c >= __ldg(P.item_start + q + 1)) ++q;
+        if (c < P.fin_warps) {                           // long-row phase 2 + empty rows first
+            finish_warp<DT>(P, c, lane);
+            c = __shfl_sync(FULL, nxt, 0);
+            continue;
+        }
+        const int64_t ci = c - P.fin_warps;
+        while (ci >= __ldg(P.item_start + q + 1)) ++q;
         const PanelDesc* D = P.panels + q;
-        const int64_t local = c - __ldg(P.item_start + q);
+        const int64_t local = ci - __ldg(P.item_start + q);
         const int64_t nmw = __ldg(&D->nmw);
         if (local < nmw) {
             if (P.class_mask & 2) {
@@ -772,33 +833,27 @@ dasp_short_kernel(const MainParams P, const uint64_t* __restrict__ tile_meta, in
 // in a fixed order, butterfly reduction (deterministic, R19); then the empty rows (R1).
 template <int DT>
 __global__ void __launch_bounds__(256) dasp_finish_kernel(const FinishParams P) {
-    using A = typename Tr<DT>::A;
-    using Y = typename Tr<DT>::Y;
     const int lane = threadIdx.x & 31;
     const int64_t w = (static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x) / 32;
-    Y* y = static_cast<Y*>(P.y);
-    if (w < P.row_long) {
-        const A* part = static_cast<const A*>(P.partial);
-        A s = 0;
-        for (int64_t k = P.group_ptr[w] + lane; k < P.group_ptr[w + 1]; k += 32) s += part[k];
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
-        if (lane == 0) {
-            const int32_t row = P.long_out[w];
-            Y r = static_cast<Y>(P.alpha) * s;
-            if (P.beta != 0.0) r += static_cast<Y>(P.beta) * y[row];
-            y[row] = r;
-            for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;
+    const int64_t lw = (P.row_long + 3) / 4;
+    if (w < lw) {
+        using Y = typename Tr<DT>::Y;
+        const int64_t r = w * 4 + (lane >> 3);
+        const auto s = long_row_sum<DT>(P.partial, P.group_ptr, r, P.row_long, lane);
+        if ((lane & 7) == 0 && r < P.row_long) {
+            Y* y = static_cast<Y*>(P.y);
+            const int32_t row = __ldg(P.long_out + r);
+            Y v = static_cast<Y>(P.alpha) * s;
+            if (P.beta != 0.0) v += static_cast<Y>(P.beta) * y[row];
+            y[row] = v;
+            for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = v;
         }
         return;
     }
-    const int64_t e = (w - P.row_long) * 32 + lane;
-    if (e < P.n0) {
-        const int32_t row = P.empty_rows[e];
-        const Y r = P.beta != 0.0 ? static_cast<Y>(P.beta) * y[row] : Y(0);
-        y[row] = r;
-        for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;
-    }
+    const int64_t e0 = (w - lw) * 128 + lane * 4;
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+        if (e0 + j < P.n0) empty_row<DT>(P.y, __ldg(P.empty_rows + e0 + j), P.beta, P.extra);
 }
 
 template <int DT>
@@ -1053,13 +1108,13 @@ __device__ __forceinline__ void medium_stage_f64(const MainParams& P, const uint
             else part = fma(va[j], xv[j], part);
         }
     }
-    const int rbase = nfull * 128 + lane * rem;
+    const int rbase = nfull * 128 + lane;                // ragged chunk: block j at 32j (R18)
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
         if (j < rem) {                                     // rem is warp-uniform
-            const double xv = gx(x, static_cast<uint32_t>(src[rbase + j]));
-            if constexpr (VAR == VAR_MMA) dmma(c0, c1, srv[rbase + j], xv);
-            else part = fma(srv[rbase + j], xv, part);
+            const double xv = gx(x, static_cast<uint32_t>(src[rbase + 32 * j]));
+            if constexpr (VAR == VAR_MMA) dmma(c0, c1, srv[rbase + 32 * j], xv);
+            else part = fma(srv[rbase + 32 * j], xv, part);
         }
     }
     if constexpr (VAR == VAR_MMA) {
@@ -1174,7 +1229,7 @@ __device__ __forceinline__ void medium_stage_f16(const MainParams& P, const uint
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
         if (j < rem) {
-            const int e = nfull * 128 + lane * rem + j;    // half-pair index
+            const int e = nfull * 128 + 32 * j + lane;     // half-pair index (ragged chunk, R18)
             block(srv[e], static_cast<uint32_t>(src[2 * e]), static_cast<uint32_t>(src[2 * e + 1]));
         }
     }
@@ -1398,7 +1453,7 @@ cudaError_t launch_short(const MainParams& p, int dtype, int variant, const uint
 }
 
 cudaError_t launch_finish(const FinishParams& p, int dtype, cudaStream_t s) {
-    const int64_t warps = p.row_long + (p.n0 + 31) / 32;
+    const int64_t warps = finish_warps(p.row_long, p.n0);
     if (warps == 0) return cudaSuccess;
     dim3 grid(static_cast<unsigned>((warps * 32 + 255) / 256)), block(256);
     if (dtype == 0) dasp_finish_kernel<0><<<grid, block, 0, s>>>(p);

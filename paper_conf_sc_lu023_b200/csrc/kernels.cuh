@@ -57,7 +57,15 @@ struct MainParams {
     // [item_start[q], item_start[q+1]) = its medium warps' row-block chunks, then its short tiles
     const int64_t* item_start;
     unsigned long long* sched;  // [0] next item, [1] finished warps; both 0 between launches
+    // long-row phase 2 + empty rows fused into the main kernel (its first fin_warps warps / items;
+    // the long kernel has completed, so every group partial is final)
+    const int64_t* group_ptr;
+    const int32_t* long_out;
+    const int32_t* empty_rows;
+    int64_t row_long, n0, fin_warps;
 };
+// finish work of the fused main kernel: 4 long rows per warp, then 128 empty rows per warp
+inline int64_t finish_warps(int64_t row_long, int64_t n0) { return (row_long + 3) / 4 + (n0 + 127) / 128; }
 
 struct FinishParams {
     const void* partial;
