@@ -64,7 +64,8 @@ def decode(F, get, dtype):
                 g, t = lane >> 2, lane & 3
                 for e in range(EPL):
                     slot = K * b + (t if EPL == 1 else 2 * t + e)
-                    at = base + lane * w * EPL + jb * EPL + e
+                    # R18: full chunks lane-interleaved, the ragged last chunk block by block
+                    at = base + (lane * w * EPL + jb * EPL + e if w == CW else jb * BE + lane * EPL + e)
                     slots[g][slot] = (rc[at], rv[at])
         for g in range(8):
             i = rb * 8 + g
