@@ -1,23 +1,29 @@
 #!/bin/bash
-# Round check: build, smoke, GPU tests, default bench line, config sweep, ncu evidence.
+# Round check: build, smoke, GPU tests, default bench line, reference arm, config sweep, ncu evidence.
 mkdir -p gpurun_out
 make -j8 all > gpurun_out/make.log 2>&1 || { tail -30 gpurun_out/make.log; exit 1; }
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
 timeout 900 python bench.py > gpurun_out/bench.log 2> gpurun_out/bench.err; echo "bench rc=$?"; cat gpurun_out/bench.log
 timeout 900 python bench.py --impl reference --steps 5 --warmup 3 > gpurun_out/bench_ref.log 2> gpurun_out/bench_ref.err; echo "ref rc=$?"; cat gpurun_out/bench_ref.log
-B="python bench.py --steps 500 --warmup 10 --e2e-steps 0 --no-cpu-baseline --no-triad"
+B="python bench.py --steps 500 --warmup 10 --e2e-steps 0 --no-cpu-baseline --no-triad --no-gpu-build"
 : > gpurun_out/sweep.jsonl
-for cfg in "c2" "c3" "c2big" "c7" "c6 --scale 20" "c1a" "c1b"; do for dt in f64 f16; do
+for cfg in "c2" "c2big" "c3" "c7" "c6 --scale 20" "c5 --scale 0.05" "c1a" "c1b"; do for dt in f64 f16 f32; do
   timeout 300 $B --config $cfg --dtype $dt >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err
 done; done
 timeout 300 python bench.py --steps 200 --warmup 5 --e2e-steps 3 --no-cpu-baseline --no-triad --iterate --config c5 --scale 0.05 >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err
-S="python bench.py --steps 3 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-triad --no-compare"
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_c2.csv $S > /dev/null 2>&1
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_c3.csv $S --config c3 > /dev/null 2>&1
-for v in mma cudacore; do
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:dasp_main -s 3 -c 1 -o gpurun_out/prof_c2_f64_$v $S --variant $v > /dev/null 2>&1
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:dasp_main -s 3 -c 1 -o gpurun_out/prof_c3_f64_$v $S --variant $v --config c3 > /dev/null 2>&1
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:dasp_main -s 3 -c 1 -o gpurun_out/prof_c2_f16_$v $S --variant $v --dtype f16 > /dev/null 2>&1
+timeout 300 python bench.py --steps 200 --warmup 5 --e2e-steps 3 --no-cpu-baseline --no-triad --iterate --halo --config c2 >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err
+S="python bench.py --steps 3 --warmup 3 --e2e-steps 0 --no-cpu-baseline --no-triad --no-compare --no-gpu-build"
+for cfg in c2 c3; do
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$cfg.csv $S --config $cfg > /dev/null 2>&1
 done
+P="ncu --set full --clock-control none --import-source on -k regex:dasp_(main|long) -s 3 -c 2"
+timeout 900 $P -o gpurun_out/prof_c2_f64_cudacore $S > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c2_f64_mma $S --variant mma > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c2big_f64_cudacore $S --config c2big > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c3_f64_cudacore $S --config c3 > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c3_f64_mma $S --config c3 --variant mma > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c2_f16_cudacore $S --dtype f16 > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c2_f32_cudacore $S --dtype f32 > /dev/null 2>&1
+timeout 900 $P -o gpurun_out/prof_c3_f16_cudacore $S --config c3 --dtype f16 > /dev/null 2>&1
 echo done

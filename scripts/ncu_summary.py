@@ -56,7 +56,7 @@ def main():
     out_md = sys.argv[1]
     traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
-    lines = ["# ncu summaries (dasp_main_kernel, `--set full --clock-control none`, one launch each)", ""]
+    lines = ["# ncu summaries (dasp_main_kernel / dasp_long_kernel, `--set full --clock-control none`, one launch each)", ""]
     for arg in sys.argv[2:]:
         key, rep = arg.split("=", 1)
         for k, d in enumerate(raw(rep)):
