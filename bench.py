@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f16", "f32"])
     ap.add_argument("--variant", default="cudacore", choices=["mma", "cudacore"])
     ap.add_argument("--no-compare", action="store_true", help="skip timing the other compute variant")
+    ap.add_argument("--no-graph", action="store_true", help="skip the CUDA-graph replay measurement (N=1 SpMV)")
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--pipeline", action="store_true", help="use the TMA-staged persistent kernel")
@@ -366,6 +367,35 @@ def main():
                    vname[other]: {"GFLOPS": 2.0 * float(lens.sum()) / (oms * 1e-3) / 1e9, "ms_per_step": oms,
                                   "steps": nrep}}
 
+    # the same K SpMVs captured once into a CUDA graph and replayed (launch overhead removed; what an
+    # iterative caller gets by capturing its loop).  Reported beside the eager number, not instead.
+    graph = None
+    if not use_slab and not args.no_graph:
+        try:
+            dasp.dasp_plan_set_timing(plan, 0)
+            gs = torch.cuda.Stream(dev)
+            gs.wait_stream(stream)
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.stream(gs):
+                dasp.dasp_spmv(plan, xd, yd, alpha, 0.0, gs, variant=variant, check=False)   # warm, outside
+                with torch.cuda.graph(g, stream=gs):
+                    for _ in range(args.steps):
+                        dasp.dasp_spmv(plan, xd, yd, alpha, 0.0, gs, variant=variant, check=False)
+            torch.cuda.synchronize(dev)
+            g.replay()
+            torch.cuda.synchronize(dev)
+            g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            g0.record(stream)
+            g.replay()
+            g1.record(stream)
+            torch.cuda.synchronize(dev)
+            gms = g0.elapsed_time(g1) / args.steps
+            graph = {"ms_per_step": gms, "GFLOPS": 2.0 * float(lens.sum()) / (gms * 1e-3) / 1e9,
+                     "kernel_nodes": int(info["launches_per_spmv"]) * args.steps}
+            del g
+        except Exception as exc:   # reported, not fatal
+            graph = {"error": str(exc)}
+
     nnz_total = int(lens.sum())
     flops_step = 2.0 * nnz_total
     gflops = flops_step / (ms_step * 1e-3) / 1e9
@@ -501,7 +531,7 @@ def main():
             "gpu_launches": launches_step * args.steps,
             "gpu_launches_per_step": launches_step,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-            "variant_compare": compare, "preprocessing": gpu_build,
+            "variant_compare": compare, "cuda_graph": graph, "preprocessing": gpu_build,
             "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,
                      "rows": {"empty": info["n_empty"], "short": info["n_len1"] + info["n_len2"] + info["n_len3"]
                               + info["n_len4"], "medium": info["row_medium"], "long": info["row_long"]},

@@ -452,6 +452,221 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta&
     medium_finish_f16<VAR>(P, M, L, lane, pol);
 }
 
+// ------------------------------------------------------------------------------------------
+// medium row-blocks with cp.async staging (DASP_MED_ASYNC): the round-1 stream data of the next
+// TWO row-blocks is copied into a per-warp shared-memory double buffer (LDGSTS, each lane its
+// own bytes, so no cross-lane synchronisation) while the current one gathers x and reduces; the
+// metadata runs two row-blocks ahead.  Bytes in flight no longer cost registers.
+// Stage layout (3072 B per warp per stage, structure of arrays):
+//   m8n8k4 (FP64/FP32, value size sv): VA[32][4 sv] @0, CA[32][16] @1024, VR[3][32][sv] @1536,
+//                                      CR[3][32][4] @2304, VI[32][8] @2688, CI[32][4] @2944
+//   FP16:                              VA[32][16] @0, CA[32][32] @512, VR[3][32][4] @1536,
+//                                      CR[3][32][8] @1920, VI[32][4] @2688, CI[32][4] @2816
+// ------------------------------------------------------------------------------------------
+#ifndef DASP_MED_ASYNC
+#define DASP_MED_ASYNC 0
+#endif
+constexpr int MED_STAGE = 3072;
+__device__ __forceinline__ void cpa16(uint32_t dst, const void* src, uint64_t pol) {
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void cpa8(uint32_t dst, const void* src, uint64_t pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;" ::"r"(dst), "l"(src), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void cpa4(uint32_t dst, const void* src, uint64_t pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(dst), "l"(src), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cpa_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <int DT>
+__device__ __forceinline__ void med_issue(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, uint32_t st) {
+    constexpr int SH = DT == 1 ? 6 : 5;
+    const int nreg = M.nelem >> SH;
+    const int nfull = nreg >> 2, rem = nreg & 3;
+    const int32_t* rc = P.reg_col + M.base;
+    if constexpr (DT == 1) {
+        const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
+        if (nfull > 0) {
+            cpa16(st + lane * 16, rv + lane * 8, pol);
+            cpa16(st + 512 + lane * 32, rc + lane * 8, pol);
+            cpa16(st + 512 + lane * 32 + 16, rc + lane * 8 + 4, pol);
+        }
+        const int64_t rb = static_cast<int64_t>(nfull) * 256 + lane * 2;
+        for (int j = 0; j < rem; ++j) {
+            cpa4(st + 1536 + j * 128 + lane * 4, rv + rb + 64 * j, pol);
+            cpa8(st + 1920 + j * 256 + lane * 8, rc + rb + 64 * j, pol);
+        }
+        const int64_t k = M.ib + (lane & 3);
+        if (k < M.ib + M.ilen) {   // the aligned 4-B word holding half k (arrays carry a tail pad)
+            const uint16_t* iv = static_cast<const uint16_t*>(P.irr_val);
+            cpa4(st + 2688 + lane * 4, iv + (k & ~int64_t(1)), pol);
+            cpa4(st + 2816 + lane * 4, P.irr_col + k, pol);
+        }
+    } else {
+        using IO = ValIO<DT>;
+        constexpr int SV = sizeof(typename IO::T);
+        const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
+        if (nfull > 0) {
+            cpa16(st + lane * 4 * SV, rv + lane * 4, pol);
+            if constexpr (SV == 8) cpa16(st + lane * 32 + 16, rv + lane * 4 + 2, pol);
+            cpa16(st + 1024 + lane * 16, rc + lane * 4, pol);
+        }
+        const int64_t rb = static_cast<int64_t>(nfull) * 128 + lane;
+        for (int j = 0; j < rem; ++j) {
+            if constexpr (SV == 8) cpa8(st + 1536 + j * 256 + lane * 8, rv + rb + 32 * j, pol);
+            else cpa4(st + 1536 + j * 256 + lane * 4, rv + rb + 32 * j, pol);
+            cpa4(st + 2304 + j * 128 + lane * 4, rc + rb + 32 * j, pol);
+        }
+        const int64_t k = M.ib + (lane & 3);
+        if (k < M.ib + M.ilen) {
+            const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+            if constexpr (SV == 8) cpa8(st + 2688 + lane * 8, iv + k, pol);
+            else cpa4(st + 2688 + lane * 8, iv + k, pol);
+            cpa4(st + 2944 + lane * 4, P.irr_col + k, pol);
+        }
+    }
+    cpa_commit();
+}
+
+template <int DT, int VAR>
+__device__ __forceinline__ void med_compute(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, const uint8_t* st) {
+    const int t = lane & 3;
+    constexpr int SH = DT == 1 ? 6 : 5;
+    const int nreg = M.nelem >> SH;
+    const int nfull = nreg >> 2, rem = nreg & 3;
+    const int32_t* rc = P.reg_col + M.base;
+    const bool has_i = M.ib + t < M.ib + M.ilen;
+    if constexpr (DT == 1) {
+        const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
+        const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
+        const uint16_t* x = static_cast<const uint16_t*>(P.x);
+        float c0 = 0.f, c1 = 0.f, part = 0.f;
+        auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) {
+            const uint16_t xa = gxh(x, ca), xb = gxh(x, cb);
+            if constexpr (VAR == VAR_MMA) {
+                hmma(c0, c1, a, pack2(xa, xb));
+            } else {
+                const float2 av = u2f2(a);
+                part = fmaf(av.x, h2f(xa), part);
+                part = fmaf(av.y, h2f(xb), part);
+            }
+        };
+        for (int ch = 0; ch < nfull; ++ch) {
+            uint32_t va[4], ca[8];
+            if (ch == 0) {
+                const uint4 a = *reinterpret_cast<const uint4*>(st + lane * 16);
+                const uint4 c0v = *reinterpret_cast<const uint4*>(st + 512 + lane * 32);
+                const uint4 c1v = *reinterpret_cast<const uint4*>(st + 512 + lane * 32 + 16);
+                va[0] = a.x; va[1] = a.y; va[2] = a.z; va[3] = a.w;
+                ca[0] = c0v.x; ca[1] = c0v.y; ca[2] = c0v.z; ca[3] = c0v.w;
+                ca[4] = c1v.x; ca[5] = c1v.y; ca[6] = c1v.z; ca[7] = c1v.w;
+            } else {
+                ld4_b32(rv + ch * 256 + lane * 8, pol, va);
+                ld8_b32(rc + ch * 256 + lane * 8, pol, ca);
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) block(va[j], ca[2 * j], ca[2 * j + 1]);
+        }
+#pragma unroll
+        for (int j = 0; j < 3; ++j) {
+            if (j < rem) {
+                const uint2 cc = *reinterpret_cast<const uint2*>(st + 1920 + j * 256 + lane * 8);
+                block(*reinterpret_cast<const uint32_t*>(st + 1536 + j * 128 + lane * 4), cc.x, cc.y);
+            }
+        }
+        if constexpr (VAR == VAR_MMA) {
+            const float d = diag_to_quad(c0, c1, lane);
+            part = t == 0 ? d : 0.f;
+        }
+        if (has_i) {
+            const int64_t k = M.ib + t;
+            const uint32_t wv = *reinterpret_cast<const uint32_t*>(st + 2688 + lane * 4);
+            const uint16_t h = static_cast<uint16_t>((k & 1) ? (wv >> 16) : (wv & 0xffffu));
+            part = fmaf(h2f(h), h2f(gxh(x, *reinterpret_cast<const uint32_t*>(st + 2816 + lane * 4))), part);
+        }
+        for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
+            part = fmaf(h2f(__ldg(iv + k)), h2f(gxh(x, ld1_b32(P.irr_col + k, pol))), part);
+        part += __shfl_xor_sync(FULL, part, 1);
+        part += __shfl_xor_sync(FULL, part, 2);
+        if (t == 0) store_y<1>(P, M.orow, part);
+    } else {
+        using IO = ValIO<DT>;
+        constexpr int SV = sizeof(typename IO::T);
+        const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
+        const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
+        double c0 = 0.0, c1 = 0.0, part = 0.0;
+        for (int ch = 0; ch < nfull; ++ch) {
+            double va[4];
+            uint32_t ca[4];
+            if (ch == 0) {
+                const typename IO::T* sv = reinterpret_cast<const typename IO::T*>(st + lane * 4 * SV);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) va[j] = static_cast<double>(sv[j]);
+                const uint4 cc = *reinterpret_cast<const uint4*>(st + 1024 + lane * 16);
+                ca[0] = cc.x; ca[1] = cc.y; ca[2] = cc.z; ca[3] = cc.w;
+            } else {
+                IO::ld4(rv + ch * 128 + lane * 4, pol, va);
+                ld4_b32(rc + ch * 128 + lane * 4, pol, ca);
+            }
+            double xv[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                if constexpr (VAR == VAR_MMA) dmma(c0, c1, va[j], xv[j]);
+                else part = fma(va[j], xv[j], part);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < 3; ++j) {
+            if (j < rem) {
+                const double v = static_cast<double>(*reinterpret_cast<const typename IO::T*>(st + 1536 + j * 256 + lane * SV));
+                const double xv = IO::gx(x, *reinterpret_cast<const uint32_t*>(st + 2304 + j * 128 + lane * 4));
+                if constexpr (VAR == VAR_MMA) dmma(c0, c1, v, xv);
+                else part = fma(v, xv, part);
+            }
+        }
+        if constexpr (VAR == VAR_MMA) {
+            const double d = diag_to_quad(c0, c1, lane);
+            part = t == 0 ? d : 0.0;
+        }
+        if (has_i) {
+            const double v = static_cast<double>(*reinterpret_cast<const typename IO::T*>(st + 2688 + lane * 8));
+            part = fma(v, IO::gx(x, *reinterpret_cast<const uint32_t*>(st + 2944 + lane * 4)), part);
+        }
+        const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+        for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
+            part = fma(IO::ld1(iv + k, pol), IO::gx(x, ld1_b32(P.irr_col + k, pol)), part);
+        part += __shfl_xor_sync(FULL, part, 1);
+        part += __shfl_xor_sync(FULL, part, 2);
+        if (t == 0) store_y<DT>(P, M.orow, part);
+    }
+}
+
+template <int DT, int VAR>
+__device__ __forceinline__ void medium_rbs_async(const MainParams& P, int64_t rb0, int64_t rb1, int lane, uint64_t pol,
+                                                 uint8_t* wsm) {
+    const RbMeta E{0, 0, 0, 0, -1};
+    const uint32_t s0 = static_cast<uint32_t>(__cvta_generic_to_shared(wsm));
+    RbMeta Ma = rb_meta(P, rb0, lane);
+    RbMeta Mb = rb0 + 1 < rb1 ? rb_meta(P, rb0 + 1, lane) : E;
+    med_issue<DT>(P, Ma, lane, pol, s0);
+    med_issue<DT>(P, Mb, lane, pol, s0 + MED_STAGE);
+    int sb = 0;
+    for (int64_t rb = rb0; rb < rb1; ++rb) {
+        const RbMeta Mc = rb + 2 < rb1 ? rb_meta(P, rb + 2, lane) : E;
+        cpa_wait<1>();
+        med_compute<DT, VAR>(P, Ma, lane, pol, wsm + sb * MED_STAGE);
+        med_issue<DT>(P, Mc, lane, pol, s0 + sb * MED_STAGE);
+        sb ^= 1;
+        Ma = Mb;
+        Mb = Mc;
+    }
+    cpa_wait<0>();
+}
+
 // row-blocks in flight per warp step (1 or 2), per value type
 #ifndef DASP_PAIR_F64
 #define DASP_PAIR_F64 1
@@ -757,7 +972,12 @@ dasp_main_kernel(const MainParams P) {
         const int64_t rbp0 = __ldg(&D->rb0);
         const int64_t rb0 = rbp0 + w * P.rbw;
         const int64_t rb1 = min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb));
+#if DASP_MED_ASYNC
+        __shared__ __align__(16) uint8_t med_smem[WARPS_PER_BLOCK * 2 * MED_STAGE];
+        medium_rbs_async<DT, VAR>(P, rb0, rb1, lane, pol, med_smem + (threadIdx.x >> 5) * 2 * MED_STAGE);
+#else
         medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);
+#endif
         return;
     }
     short_item<DT, VAR>(P, D, w - nmw, lane, pol);
@@ -1367,6 +1587,16 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
     const unsigned nb = static_cast<unsigned>(blocks);
     cudaError_t e;
     const bool mma = variant == VAR_MMA;
+#if DASP_MED_ASYNC
+    static bool carve[3][2] = {};                      // 4 blocks x 48 KB staging per SM
+    if (!carve[dtype][mma]) {
+        const void* k = dtype == 0 ? (mma ? (const void*)dasp_main_kernel<0, VAR_MMA> : (const void*)dasp_main_kernel<0, VAR_CUDACORE>)
+                      : dtype == 1 ? (mma ? (const void*)dasp_main_kernel<1, VAR_MMA> : (const void*)dasp_main_kernel<1, VAR_CUDACORE>)
+                                   : (mma ? (const void*)dasp_main_kernel<2, VAR_MMA> : (const void*)dasp_main_kernel<2, VAR_CUDACORE>);
+        cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
+        carve[dtype][mma] = true;
+    }
+#endif
     if (dtype == 0) e = launch_ex(mma ? dasp_main_kernel<0, VAR_MMA> : dasp_main_kernel<0, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
     else if (dtype == 1) e = launch_ex(mma ? dasp_main_kernel<1, VAR_MMA> : dasp_main_kernel<1, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
     else e = launch_ex(mma ? dasp_main_kernel<2, VAR_MMA> : dasp_main_kernel<2, VAR_CUDACORE>, nb, s, apw_base, apw_bytes, apw_hit, p);
