@@ -15,8 +15,10 @@
  * Precisions (north_star):
  *   DASP_R_64F : val f64, x f64, y f64; products and sums in f64 (DMMA m8n8k4).
  *   DASP_R_16F : val f16 (IEEE binary16 bits), x f16, y f32; products exact in f32 and sums
- *                in f32 (HMMA m16n8k16 f16->f32, R14/R15).  alpha/beta are applied
+ *                in f32 (HMMA m16n8k8 f16->f32, R14/R15).  alpha/beta are applied
  *                in f32.
+ *   DASP_R_32F : val f32, x f32, y f32 (R29): operands widened
+ *                exactly to f64, products and sums in f64 (FP64 block geometry), y rounded once.
  *
  * No torch or CUDA types cross this boundary: device pointers are plain pointers, the CUDA
  * stream is passed as `void*` (a cudaStream_t, NULL = legacy default stream).
@@ -52,7 +54,7 @@ typedef enum {
  * read either way; only the arithmetic differs.                                            */
 typedef enum {
     DASP_VARIANT_DEFAULT = 0,   /* the plan's default (options.variant)                       */
-    DASP_VARIANT_MMA = 1,       /* DMMA m8n8k4 (FP64) / HMMA m16n8k16 (FP16) + diagonal
+    DASP_VARIANT_MMA = 1,       /* DMMA m8n8k4 (FP64, FP32) / HMMA m16n8k8 (FP16) + diagonal
                                    extraction by shuffles (Alg. 2-4)              */
     DASP_VARIANT_CUDACORE = 2   /* per-lane FMA + warp-shuffle segmented reduction            */
 } dasp_variant_t;

@@ -1,10 +1,11 @@
 // kernels.cu — sm_100a kernels of the DASP SpMV hot path (§3.3, Alg. 2-5).
 //
-// One fused launch covers the three row classes (warp-uniform dispatch on the global warp
-// index), plus a small "finish" launch for long-row phase 2 (Alg. 2 l.17-25)
-// and empty rows.  Every block inner product is computed by one of two variants that read
-// the SAME packed arrays (north_star (3)):
-//   VAR_MMA      legacy warp MMA: DMMA m8n8k4 f64 (Listing 1) / HMMA m16n8k16
+// Two launches per SpMV: the long-row phase-1 kernel (Alg. 2 l.1-16), then the
+// main kernel, whose warps are (warp-uniform dispatch on the global warp index) long-row
+// phase 2 + empty rows first (Alg. 2 l.17-25), then per row panel the medium row-blocks
+// (Alg. 3) and short tiles (Alg. 4-5).  Every block inner product is computed by one of two
+// variants that read the SAME packed arrays (north_star (3)):
+//   VAR_MMA      legacy warp MMA: DMMA m8n8k4 f64 (Listing 1) / HMMA m16n8k8
 //                f16->f32; the block dot products sit on the diagonal of C (Fig. 4)
 //                and are extracted with shuffles (Alg. 2 l.10-13, Alg. 3 l.13-17).
 //   VAR_CUDACORE per-lane FMA and a warp-shuffle segmented reduction.
