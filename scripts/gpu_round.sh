@@ -26,4 +26,19 @@ timeout 900 $P -o gpurun_out/prof_c3_f64_mma $S --config c3 --variant mma > /dev
 timeout 900 $P -o gpurun_out/prof_c2_f16_cudacore $S --dtype f16 > /dev/null 2>&1
 timeout 900 $P -o gpurun_out/prof_c2_f32_cudacore $S --dtype f32 > /dev/null 2>&1
 timeout 900 $P -o gpurun_out/prof_c3_f16_cudacore $S --config c3 --dtype f16 > /dev/null 2>&1
+# summaries on the box (the reports themselves are too large to bring back, except two)
+echo '{}' > gpurun_out/ncu_traffic.json
+NCU_TRAFFIC=gpurun_out/ncu_traffic.json python scripts/ncu_summary.py gpurun_out/ncu_summary.md \
+  c2/f64/cudacore=gpurun_out/prof_c2_f64_cudacore.ncu-rep c2/f64/mma=gpurun_out/prof_c2_f64_mma.ncu-rep \
+  c2big/f64/cudacore=gpurun_out/prof_c2big_f64_cudacore.ncu-rep c3/f64/cudacore=gpurun_out/prof_c3_f64_cudacore.ncu-rep \
+  c3/f64/mma=gpurun_out/prof_c3_f64_mma.ncu-rep c2/f16/cudacore=gpurun_out/prof_c2_f16_cudacore.ncu-rep \
+  c2/f32/cudacore=gpurun_out/prof_c2_f32_cudacore.ncu-rep c3/f16/cudacore=gpurun_out/prof_c3_f16_cudacore.ncu-rep \
+  > gpurun_out/ncu_summary.log 2>&1
+for r in gpurun_out/*.ncu-rep; do
+  case $r in *prof_c2_f64_cudacore*|*prof_c3_f64_cudacore*) ;; *) rm -f $r ;; esac
+done
+[ "$(du -sm gpurun_out | cut -f1)" -gt 55 ] && rm -f gpurun_out/prof_c3_f64_cudacore.ncu-rep
+[ "$(du -sm gpurun_out | cut -f1)" -gt 55 ] && rm -f gpurun_out/prof_c2_f64_cudacore.ncu-rep
+du -sh gpurun_out
+timeout 600 python scripts/cg_bench.py > gpurun_out/cg.jsonl 2> gpurun_out/cg.err; echo "cg rc=$?"; cat gpurun_out/cg.jsonl
 echo done

@@ -2,6 +2,7 @@
 """Summarise Nsight Compute reports of dasp_main_kernel into profiles/ (markdown + traffic JSON).
 
     python scripts/ncu_summary.py OUT.md KEY=REPORT.ncu-rep [KEY=REPORT.ncu-rep ...]
+    NCU_TRAFFIC=path  overrides where the traffic JSON is merged (default profiles/ncu_traffic.json)
 
 KEY is "<workload>/<dtype>/<variant>"; traffic is stored per "<KEY>/<kernel>" (bench.py's lookup
 key for roofline.traffic); every dasp_* kernel captured in the report is summarised.
@@ -54,7 +55,7 @@ def to_bytes(unit, v):
 
 def main():
     out_md = sys.argv[1]
-    traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    traffic_path = os.environ.get("NCU_TRAFFIC", os.path.join(ROOT, "profiles", "ncu_traffic.json"))
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
     lines = ["# ncu summaries (dasp_main_kernel / dasp_long_kernel, `--set full --clock-control none`, one launch each)", ""]
     for arg in sys.argv[2:]:
