@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--pipeline", action="store_true", help="use the TMA-staged persistent kernel")
     ap.add_argument("--panel-rows", type=int, default=0, help="rows per panel (0 auto, -1 one global panel)")
+    ap.add_argument("--co-schedule", type=int, default=-1, choices=[-1, 0, 1],
+                    help="long-row units inside the medium/short kernel (1), in their own launch (0), auto (-1)")
     ap.add_argument("--no-triad", action="store_true")
     ap.add_argument("--iterate", action="store_true", help="N=1: run the row-slab iteration (x <- alpha*A*x)")
     ap.add_argument("--no-gpu-build", action="store_true", help="skip timing the device-side builder")
@@ -153,6 +155,9 @@ def byte_model(info, dtype, beta_nonzero=False, split_short=False, fused_finish=
     csr_equiv = nnz * (sv + 4) + (m + 1) * 8 + n * sx + m * sy * b1
     if fused_finish:
         main += finish
+    if info.get("co_scheduled"):          # long units run inside dasp_main_kernel (+ group_row)
+        main += long_ + 4 * ngp
+        long_ = 0
     out = {"dasp_long_kernel": long_, "dasp_main_kernel": main, "dasp_finish_kernel": 0 if fused_finish else finish,
            "total": long_ + main + (0 if fused_finish else finish) + (short if split_short else 0),
            "csr_equiv": csr_equiv}
@@ -292,7 +297,8 @@ def main():
         # single GPU: plain SpMV over resident inputs, y overwritten every step
         plan = dasp.dasp_plan_create(slab.row_ptr, slab.col, slab.val, slab.rows, spec.n, args.dtype,
                                      device=local, variant=variant, medium_rb_per_warp=args.rbw,
-                                     pipeline=args.pipeline, panel_rows=args.panel_rows)
+                                     pipeline=args.pipeline, panel_rows=args.panel_rows,
+                                     co_schedule=args.co_schedule)
         xdt = {"f64": torch.float64, "f16": torch.float16, "f32": torch.float32}[args.dtype]
         ydt = torch.float64 if args.dtype == "f64" else torch.float32
         xd = torch.from_numpy(x_global).to(xdt).to(dev)
@@ -520,6 +526,7 @@ def main():
             "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config),
                        "m": int(spec.m), "n": int(spec.n), "nnz": nnz_total, "variant": args.variant,
                        "kernel": "pipeline" if info.get("pipeline") else "direct", "panel_rows": info["panel_rows"],
+                       "co_scheduled": bool(info.get("co_scheduled")),
                        "parallelism": f"row-slab x{world}" + (
                            (" + fused NVLink scatter of y into every rank's x" if args.fused else
                             " + sparse halo all_to_all overlapped with the local sub-matrix" if args.halo else

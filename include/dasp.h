@@ -81,6 +81,11 @@ typedef struct {
     double threshold;           /* tau, "a customized parameter": an 8 x MMA_K block is
                                    regular iff it holds more than 8*MMA_K*tau nonzeros;
                                    0 = 0.75; must be <= 1                                     */
+    int32_t co_schedule;        /* 1: the long-row units run as blocks of the medium/short
+                                   kernel, interleaved with each panel's medium/short blocks,
+                                   and the warp that completes a long row runs its phase 2
+                                   (Alg. 2 l.17-25) -- one launch per SpMV; 0: long units in
+                                   their own launch before it; -1 (default): automatic (0)    */
 } dasp_options_t;
 
 /* Fills `opts` with the defaults: device 0, CUDA-core variant, validate, no keep_host, auto
@@ -109,6 +114,7 @@ typedef struct {
     int64_t max_len;                                   /* resolved MAX_LEN                   */
     double threshold;                                  /* resolved tau                       */
     double build_ms, upload_ms;                        /* host build; host->device upload   */
+    int32_t co_scheduled;                              /* 1 if long units run co-scheduled   */
 } dasp_plan_info_t;
 
 /*

@@ -40,7 +40,10 @@ struct dasp_plan_s {
     int64_t n_tiles = 0;
     void* d_tile_meta = nullptr;          // uint64 cat << 62 | output base, per tile (split mode)
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
-    void* d_blk_panel = nullptr;          // int32 panel of every block
+    void* d_blk_word = nullptr;           // uint64 role of every main-kernel block (kernels.cuh)
+    bool cosched = false;                 // long units co-scheduled inside the main kernel
+    void* d_long_cnt = nullptr;           // int32 per long row: groups not yet summed (co-scheduled)
+    void* d_group_row = nullptr;          // int32 per group: its long row, -1 for pad groups
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
     void* d_items = nullptr;              // uint64 item words of the pipelined kernel
     int64_t n_items = 0, pipe_blocks = 0;
@@ -70,6 +73,7 @@ constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
 constexpr bool kSplitShortDefault = false;
 constexpr bool kDynSchedDefault = false;
+constexpr bool kCoschedDefault = false;  // long units inside the main kernel: measured slower
 constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // TMA windows may read up to 16 B past an array's end
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
@@ -104,13 +108,16 @@ void free_device(dasp_plan_s* p) {
     }
     if (p->d_partial) cudaFree(p->d_partial);
     if (p->d_panels) cudaFree(p->d_panels);
-    if (p->d_blk_panel) cudaFree(p->d_blk_panel);
+    if (p->d_blk_word) cudaFree(p->d_blk_word);
+    if (p->d_long_cnt) cudaFree(p->d_long_cnt);
+    if (p->d_group_row) cudaFree(p->d_group_row);
+    p->d_long_cnt = p->d_group_row = nullptr;
     if (p->d_unit_order) cudaFree(p->d_unit_order);
     if (p->d_items) cudaFree(p->d_items);
     if (p->d_tile_meta) cudaFree(p->d_tile_meta);
     if (p->d_item_start) cudaFree(p->d_item_start);
     if (p->d_sched) cudaFree(p->d_sched);
-    p->d_panels = p->d_blk_panel = p->d_unit_order = p->d_items = p->d_tile_meta = nullptr;
+    p->d_panels = p->d_blk_word = p->d_unit_order = p->d_items = p->d_tile_meta = nullptr;
     p->d_item_start = p->d_sched = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
@@ -149,6 +156,7 @@ int64_t alg_bytes(const dasp_plan_s* p, bool beta) {
     const int64_t nout = 64 * f.t13 + 32 * f.t4 + 64 * f.t22 + 128 * f.ts;
     int64_t b = 0;
     b += f.n_groups_padded * f.geo.G * (s_v + 4) + 2 * f.n_groups_padded * s_a + 8 * (f.row_long + 1) + 4 * f.row_long;
+    if (p->cosched) b += 4 * f.n_groups_padded;   // group_row (co-scheduled phase 2)
     b += (f.nnz_reg_new + f.nnz_irreg) * (s_v + 4) + 8 * (f.nrb + 1) + 8 * (nmp + 1) + 4 * nmp;
     b += f.nnz_short_new * (s_v + 4) + 4 * nout;
     b += 4 * f.n0;
@@ -174,6 +182,7 @@ void dasp_options_default(dasp_options_t* o) {
     o->pipeline = 0;
     o->max_len = 256;
     o->threshold = 0.75;
+    o->co_schedule = -1;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -202,11 +211,16 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     HostFormat& f = p->host;
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
-    std::vector<int32_t> blk_panel;
+    std::vector<uint64_t> blk_word;
     std::vector<uint64_t> tile_meta;
     {
         const char* ss = std::getenv("DASP_SPLIT_SHORT");
         p->split_short = ss ? std::atoi(ss) != 0 : kSplitShortDefault;
+        const char* cs = std::getenv("DASP_COSCHED");
+        const char* pe = std::getenv("DASP_PIPE");
+        const bool pipe_wanted = pe ? std::atoi(pe) != 0 : o.pipeline != 0;
+        p->cosched = (cs ? std::atoi(cs) != 0 : (o.co_schedule < 0 ? kCoschedDefault : o.co_schedule != 0)) &&
+                     f.n_groups_padded > 0 && !pipe_wanted;
     }
     int64_t blk = 0;
     std::vector<int64_t> item_start(1, 0);
@@ -231,8 +245,16 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
         item_start.push_back(item_start.back() + warps);
         const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
-        blk_panel.insert(blk_panel.end(), static_cast<size_t>(nb), static_cast<int32_t>(q));
-        blk += nb;
+        // co-scheduled: the panel's long blocks are spread evenly among its main blocks, so the
+        // SMs always hold a mix of HBM-streaming long units and latency-bound medium/short warps
+        const int64_t nl = p->cosched ? (d.nunits + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK : 0;
+        int64_t il = 0, im = 0;
+        for (int64_t i = 0; i < nl + nb; ++i) {
+            const bool is_long = (i + 1) * nl / (nl + nb) > i * nl / (nl + nb);
+            const uint64_t idx = static_cast<uint64_t>(is_long ? il++ : im++);
+            blk_word.push_back((is_long ? (1ull << 63) : 0ull) | (static_cast<uint64_t>(q) << 32) | idx);
+        }
+        blk += nb + nl;
     }
     p->blocks = blk;
     p->n_units = f.n_groups_padded / f.geo.UG;
@@ -300,7 +322,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     p->device_bytes += pb;
     dasp_status_t st;
     if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
-    if ((st = upload(&p->d_blk_panel, blk_panel.data(), blk_panel.size() * 4)) != DASP_OK) return st;
+    if ((st = upload(&p->d_blk_word, blk_word.data(), blk_word.size() * 8)) != DASP_OK) return st;
     if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
     if (p->split_short && (st = upload(&p->d_tile_meta, tile_meta.data(), tile_meta.size() * 8)) != DASP_OK) return st;
     if (p->pipe) {
@@ -317,7 +339,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     // dynamic schedule of the main kernel (DASP_SCHED=1 / options)
     {
         const char* se = std::getenv("DASP_SCHED");
-        p->dyn = se ? std::atoi(se) == 1 : kDynSchedDefault;
+        p->dyn = (se ? std::atoi(se) == 1 : kDynSchedDefault) && !p->cosched;
         p->dyn_items = item_start.back();
         const int64_t all_items = p->dyn_items + dasp::finish_warps(f.row_long, f.n0);
         if (p->dyn && !p->pipe && all_items > 0) {
@@ -351,6 +373,22 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         cudaGetLastError();
     }
     return DASP_OK;
+}
+
+// co-scheduled mode: per-row group counters and per-group rows, from the device group_ptr
+dasp_status_t init_cosched(dasp_plan_s* p) {
+    const HostFormat& f = p->host;
+    if (!p->cosched || p->device < 0) return DASP_OK;
+    const size_t cb = static_cast<size_t>(std::max<int64_t>(f.row_long, 1)) * 4;
+    const size_t gb = static_cast<size_t>(std::max<int64_t>(f.n_groups_padded, 1)) * 4;
+    if (cudaMalloc(&p->d_long_cnt, cb) != cudaSuccess || cudaMalloc(&p->d_group_row, gb) != cudaSuccess)
+        return DASP_ERR_OUT_OF_MEMORY;
+    p->device_bytes += static_cast<int64_t>(cb + gb);
+    if (cudaMemset(p->d_group_row, 0xff, gb) != cudaSuccess) return DASP_ERR_CUDA;
+    if (dasp::launch_long_meta(static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]), f.row_long,
+                               static_cast<int32_t*>(p->d_long_cnt), static_cast<int32_t*>(p->d_group_row), nullptr) != cudaSuccess)
+        return DASP_ERR_CUDA;
+    return cudaDeviceSynchronize() == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
 }
 
 dasp_status_t check_create_args(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz, const void* row_ptr,
@@ -440,6 +478,7 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         auto u1 = std::chrono::steady_clock::now();
         p->upload_ms = std::chrono::duration<double, std::milli>(u1 - u0).count();
         if (!p->keep_host) f.release();
+        if ((st = init_cosched(p)) != DASP_OK) return fail(p, st);
     }
     *plan_out = p;
     return DASP_OK;
@@ -483,6 +522,7 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
         return fail(p, DASP_ERR_CUDA);
     st = setup_launch(p, o, f.panel_table.data(), first_col);
     if (st != DASP_OK) return fail(p, st);
+    if ((st = init_cosched(p)) != DASP_OK) return fail(p, st);
     *plan_out = p;
     return DASP_OK;
 }
@@ -529,7 +569,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
         return e == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
     }
     if (!x && f.n > 0) return DASP_ERR_INVALID_ARG;
-    dasp::MainParams mp;
+    dasp::MainParams mp{};
     mp.long_val = p->d[DASP_ARR_LONG_VAL];
     mp.long_col = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_COL]);
     mp.partial = p->d_partial;
@@ -548,20 +588,22 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.alpha = alpha;
     mp.beta = beta;
     mp.panels = static_cast<const dasp::PanelDesc*>(p->d_panels);
-    mp.blk_panel = static_cast<const int32_t*>(p->d_blk_panel);
+    mp.blk_word = static_cast<const uint64_t*>(p->d_blk_word);
     mp.unit_order = static_cast<const int32_t*>(p->d_unit_order);
     mp.rbw = p->rbw;
     mp.class_mask = 7;
     mp.extra = extra;
     mp.item_start = static_cast<const int64_t*>(p->d_item_start);
     mp.sched = static_cast<unsigned long long*>(p->d_sched);
+    mp.group_row = static_cast<const int32_t*>(p->d_group_row);
+    mp.long_cnt = p->cosched ? static_cast<int32_t*>(p->d_long_cnt) : nullptr;   // null: no phase 2 in the units
     // DASP_PROFILE_CLASS (profiling only; the other classes' rows are then NOT computed):
     // 1 = long units, 2 = medium warps, 3 = short tiles
     if (const char* pc = std::getenv("DASP_PROFILE_CLASS")) {
         const int c = std::atoi(pc);
         if (c >= 1 && c <= 3) mp.class_mask = 1 << (c - 1);
     }
-    if (!p->pipe && p->n_units > 0 && (mp.class_mask & 1)) {
+    if (!p->pipe && !p->cosched && p->n_units > 0 && (mp.class_mask & 1)) {
         e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s); });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }
@@ -577,9 +619,11 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
     mp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
     mp.empty_rows = static_cast<const int32_t*>(p->d[DASP_ARR_EMPTY_ROWS]);
-    mp.row_long = f.row_long;
+    // co-scheduled: phase 2 runs in the long units' completion (kernels.cu long_unit_complete),
+    // so the fin warps only write the empty rows
+    mp.row_long = p->cosched ? 0 : f.row_long;
     mp.n0 = n0;
-    mp.fin_warps = (!p->pipe && (mp.class_mask & 1)) ? dasp::finish_warps(f.row_long, n0) : 0;
+    mp.fin_warps = (!p->pipe && (mp.class_mask & 1)) ? dasp::finish_warps(mp.row_long, n0) : 0;
     const int64_t fin_blocks = (mp.fin_warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
     e = timed(p, DASP_K_MAIN, s, on, [&] {
         if (p->pipe)
@@ -660,11 +704,12 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
     o->launches_per_spmv = p->pipe ? (p->n_items > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0)
-                                   : (p->n_units > 0 ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0) +
+                                   : (p->n_units > 0 && !p->cosched ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0) +
                                          (p->n_tiles > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
     o->pipeline = p->pipe ? 1 : 0;
+    o->co_scheduled = p->cosched ? 1 : 0;
     o->max_len = f.max_len;
     o->threshold = f.tau;
     o->build_ms = p->build_ms;

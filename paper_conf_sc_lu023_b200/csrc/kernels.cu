@@ -165,12 +165,66 @@ template <> struct Tr<2> {  // FP32 storage, FP64 accumulate (R29), FP64 geometr
 template <int DT>
 __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typename Tr<DT>::A acc) {
     using Y = typename Tr<DT>::Y;
+    using A = typename Tr<DT>::A;
     if (row < 0) return;
     Y* y = static_cast<Y*>(P.y);
-    Y r = static_cast<Y>(P.alpha) * acc;
-    if (P.beta != 0.0) r += static_cast<Y>(P.beta) * y[row];
+    A ra = static_cast<A>(P.alpha) * acc;                // in the accumulator type, one final rounding
+    if (P.beta != 0.0) ra += static_cast<A>(P.beta) * static_cast<A>(y[row]);   // (FP32 variant, R29)
+    const Y r = static_cast<Y>(ra);
     y[row] = r;
     for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;   // peers (scatter)
+}
+
+// ------------------------------------------------------------------------------------------
+// co-scheduled long rows: long units run as blocks of the main kernel, so phase 2
+// (Alg. 2 l.17-25) cannot wait for a kernel boundary.  A unit counts its groups off its rows'
+// counters after its partials are visible; the warp that brings a row's counter to zero sums
+// that row's partials.  The sum is the fixed lane-strided order of long_row_sum_warp whichever
+// warp runs it, so results do not depend on the schedule (R19).
+// ------------------------------------------------------------------------------------------
+template <int DT>
+__device__ __forceinline__ typename Tr<DT>::A long_row_sum_warp(const void* partial, int64_t g0, int64_t g1, int lane) {
+    using A = typename Tr<DT>::A;
+    const A* part = static_cast<const A*>(partial);
+    A s0 = 0, s1 = 0, s2 = 0, s3 = 0;
+    int64_t k = g0 + lane;                               // L2 reads: written by other SMs in this launch
+    for (; k + 96 < g1; k += 128) { s0 += __ldcg(part + k); s1 += __ldcg(part + k + 32); s2 += __ldcg(part + k + 64); s3 += __ldcg(part + k + 96); }
+    for (; k < g1; k += 32) s0 += __ldcg(part + k);
+    A s = (s0 + s1) + (s2 + s3);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+    return s;
+}
+template <int DT>
+__device__ __forceinline__ void long_unit_complete(const MainParams& P, int64_t u, int lane) {
+    __threadfence();                                     // this lane's partial store, device-wide ...
+    __syncwarp();                                        // ... before any lane's counter update
+    const int32_t gr = lane < 4 ? __ldg(P.group_row + u * 4 + lane) : -1;
+    int32_t rr[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) rr[j] = __shfl_sync(FULL, gr, j);   // rows of groups 0..3 (non-decreasing)
+    const int32_t prev = __shfl_up_sync(FULL, gr, 1);
+    bool fin = false;
+    if (lane < 4 && gr >= 0 && (lane == 0 || prev != gr)) {   // first group of its row in this unit
+        int cnt = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) cnt += rr[j] == gr;
+        fin = atomicSub(P.long_cnt + gr, cnt) == cnt;
+    }
+    unsigned done = __ballot_sync(FULL, fin);
+    if (!done) return;
+    __threadfence();                                     // acquire: other warps' partials of the row
+    while (done) {
+        const int j = __ffs(done) - 1;
+        done &= done - 1;
+        const int32_t r = __shfl_sync(FULL, gr, j);
+        const int64_t g0 = __ldg(P.group_ptr + r), g1 = __ldg(P.group_ptr + r + 1);
+        const auto sum = long_row_sum_warp<DT>(P.partial, g0, g1, lane);
+        if (lane == 0) {
+            store_y<DT>(P, __ldg(P.long_out + r), sum);
+            P.long_cnt[r] = static_cast<int32_t>(g1 - g0);   // ready for the next launch
+        }
+    }
 }
 
 // ------------------------------------------------------------------------------------------
@@ -222,7 +276,7 @@ __device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, in
         kk += __shfl_xor_sync(FULL, kk, 2);
         kk += __shfl_xor_sync(FULL, kk, 1);
         if ((lane & 7) == 0) static_cast<double*>(P.partial)[u * 4 + 2 * (lane >> 4) + ((lane >> 3) & 1)] = kk;
-    }
+    }    if (P.long_cnt) long_unit_complete<DT>(P, u, lane);
 }
 
 // FP16: lane l reads 8-B value chunks l + 32j (j = 0..3): halves 4(l+32j)..+3, all in group j
@@ -268,7 +322,7 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
         kk += __shfl_xor_sync(FULL, kk, 2);
         kk += __shfl_xor_sync(FULL, kk, 1);
         if ((lane & 7) == 0) static_cast<float*>(P.partial)[u * 4 + 2 * (lane >> 4) + ((lane >> 3) & 1)] = kk;
-    }
+    }    if (P.long_cnt) long_unit_complete<1>(P, u, lane);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -874,8 +928,9 @@ __device__ __forceinline__ typename Tr<DT>::A long_row_sum(const void* partial, 
 template <int DT>
 __device__ __forceinline__ void empty_row(void* yv, int32_t row, double beta, const ExtraDst& extra) {
     using Y = typename Tr<DT>::Y;
+    using A = typename Tr<DT>::A;
     Y* y = static_cast<Y*>(yv);
-    const Y r = beta != 0.0 ? static_cast<Y>(beta) * y[row] : Y(0);
+    const Y r = beta != 0.0 ? static_cast<Y>(static_cast<A>(beta) * static_cast<A>(y[row])) : Y(0);
     y[row] = r;
     for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[row] = r;
 }
@@ -961,12 +1016,20 @@ dasp_main_kernel(const MainParams P) {
         if (fw < P.fin_warps) finish_warp<DT>(P, fw, lane);
         return;
     }
-    const int64_t b = static_cast<int64_t>(blockIdx.x) - fin_blocks;
     // role of this warp inside its panel; the descriptor fields are loaded only on the branch
     // that needs them so they do not stay live (register pressure = occupancy)
-    const PanelDesc* D = P.panels + __ldg(P.blk_panel + b);
-    int64_t w = (b - __ldg(&D->blk0)) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+    const uint64_t bw = __ldg(P.blk_word + (static_cast<int64_t>(blockIdx.x) - fin_blocks));
+    const PanelDesc* D = P.panels + static_cast<int32_t>((bw >> 32) & 0x7fffffffu);
+    int64_t w = static_cast<int64_t>(bw & 0xffffffffu) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
     const uint64_t pol = stream_policy();
+    if (bw >> 63) {                                      // co-scheduled long units (Alg. 2)
+        if (w < __ldg(&D->nunits)) {
+            const int64_t u = __ldg(P.unit_order + __ldg(&D->unit0) + w);
+            if constexpr (DT == 1) long_unit_f16<VAR>(P, u, lane, pol);
+            else long_unit_f64<DT, VAR>(P, u, lane, pol);
+        }
+        return;
+    }
     const int64_t nmw = __ldg(&D->nmw);
     if (w < nmw) {                                       // medium rows
         if (!(P.class_mask & 2)) return;
@@ -1064,8 +1127,10 @@ __global__ void __launch_bounds__(256) dasp_finish_kernel(const FinishParams P) 
         if ((lane & 7) == 0 && r < P.row_long) {
             Y* y = static_cast<Y*>(P.y);
             const int32_t row = __ldg(P.long_out + r);
-            Y v = static_cast<Y>(P.alpha) * s;
-            if (P.beta != 0.0) v += static_cast<Y>(P.beta) * y[row];
+            using A = typename Tr<DT>::A;
+            A va = static_cast<A>(P.alpha) * s;
+            if (P.beta != 0.0) va += static_cast<A>(P.beta) * static_cast<A>(y[row]);
+            const Y v = static_cast<Y>(va);
             y[row] = v;
             for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = v;
         }
@@ -1083,7 +1148,8 @@ __global__ void dasp_scale_kernel(void* yv, int64_t m, double beta, const ExtraD
     Y* y = static_cast<Y*>(yv);
     for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < m;
          i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
-        const Y r = beta != 0.0 ? static_cast<Y>(beta) * y[i] : Y(0);
+        using A = typename Tr<DT>::A;
+        const Y r = beta != 0.0 ? static_cast<Y>(static_cast<A>(beta) * static_cast<A>(y[i])) : Y(0);
         y[i] = r;
         for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[i] = r;
     }
@@ -1579,6 +1645,28 @@ static cudaError_t launch_ex(Kern kernel, unsigned blocks, cudaStream_t s, const
         cfg.numAttrs = 1;
     }
     return cudaLaunchKernelEx(&cfg, kernel, p);
+}
+
+namespace {
+// one warp per long row: its group count and the row index of each of its groups
+__global__ void __launch_bounds__(256) dasp_long_meta_kernel(const int64_t* __restrict__ group_ptr, int64_t row_long,
+                                                             int32_t* __restrict__ long_cnt, int32_t* __restrict__ group_row) {
+    const int64_t r = (static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x) >> 5;
+    if (r >= row_long) return;
+    const int lane = threadIdx.x & 31;
+    const int64_t g0 = group_ptr[r], g1 = group_ptr[r + 1];
+    if (lane == 0) long_cnt[r] = static_cast<int32_t>(g1 - g0);
+    for (int64_t g = g0 + lane; g < g1; g += 32) group_row[g] = static_cast<int32_t>(r);
+}
+}  // namespace
+
+cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,
+                             cudaStream_t s) {
+    if (row_long <= 0) return cudaSuccess;
+    const int64_t blocks = (row_long * 32 + 255) / 256;
+    if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    dasp_long_meta_kernel<<<static_cast<unsigned>(blocks), 256, 0, s>>>(group_ptr, row_long, long_cnt, group_row);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,

@@ -18,10 +18,11 @@ struct ExtraDst {
 };
 constexpr int WARPS_PER_BLOCK = MAIN_THREADS / 32;
 
-// One row panel (R28) as the medium/short kernel sees it.  A panel owns the blocks
-// [blk0, blk0 + ceil(warps/8)); its warps are, in order: nmw medium warps (rbw row-blocks each;
-// Alg. 3, LOOP_NUM P:L271), then one warp per short tile (1&3 | len4 | 2&2 | singles).  The long
-// units (unit0, nunits) run in their own kernel (dasp_long_kernel).
+// One row panel (R28) as the medium/short kernel sees it.  Its main warps are, in
+// order: nmw medium warps (rbw row-blocks each; Alg. 3, LOOP_NUM P:L271), then one warp per short
+// tile (1&3 | len4 | 2&2 | singles).  Its long units (unit0, nunits) run either in their own kernel
+// (dasp_long_kernel) or, co-scheduled, as long blocks of the main kernel interleaved with the
+// panel's main blocks (MainParams::blk_word).
 struct PanelDesc {
     int64_t blk0;
     int64_t unit0, nunits;
@@ -45,7 +46,10 @@ struct MainParams {
     const int32_t* short_col;
     const int32_t* short_out;
     const PanelDesc* panels;
-    const int32_t* blk_panel; // panel of every block
+    // role of every block after the fin blocks: bit 63 = long block (8 long units of the panel,
+    // co-scheduled mode), bits 32..62 = panel, bits 0..31 = block index among the panel's blocks
+    // of that kind
+    const uint64_t* blk_word;
     const int32_t* unit_order;// long units in execution order (column-bucketed per panel)
     const void* x;
     void* y;
@@ -63,6 +67,11 @@ struct MainParams {
     const int32_t* long_out;
     const int32_t* empty_rows;
     int64_t row_long, n0, fin_warps;
+    // co-scheduled long units (blk_word long blocks): group_row[g] = long row of group g (-1 for
+    // the pad groups); long_cnt[r] = groups of row r not yet summed in this launch (reset to the
+    // row's group count by the warp that completes the row, which then runs phase 2 for it)
+    const int32_t* group_row;
+    int32_t* long_cnt;
 };
 // finish work of the fused main kernel: 4 long rows per warp, then 128 empty rows per warp
 inline int64_t finish_warps(int64_t row_long, int64_t n0) { return (row_long + 3) / 4 + (n0 + 127) / 128; }
@@ -83,6 +92,10 @@ struct FinishParams {
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
+// co-scheduled mode metadata from group_ptr: long_cnt[r] = groups of row r, group_row[g] = row
+// (group_row must be pre-filled with -1 for the pad groups)
+cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,
+                             cudaStream_t s);
 // persistent main kernel with dynamic (atomic counter) work distribution over the items of
 // MainParams::item_start; blocks = resident blocks (main_dyn_occupancy x SMs) or fewer
 cudaError_t launch_main_dyn(const MainParams& p, int dtype, int variant, int64_t blocks, int64_t n_items, cudaStream_t s);

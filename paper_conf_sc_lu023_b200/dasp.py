@@ -43,7 +43,7 @@ class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("variant", ctypes.c_int32), ("validate", ctypes.c_int32),
                 ("keep_host", ctypes.c_int32), ("medium_rb_per_warp", ctypes.c_int32),
                 ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64), ("pipeline", ctypes.c_int32),
-                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double)]
+                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double), ("co_schedule", ctypes.c_int32)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -57,7 +57,7 @@ class PlanInfo(ctypes.Structure):
                [("medium_rb_per_warp", ctypes.c_int32), ("launches_per_spmv", ctypes.c_int32),
                 ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64), ("pipeline", ctypes.c_int32),
                 ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
-                ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double)]
+                ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double), ("co_scheduled", ctypes.c_int32)]
 
     def as_dict(self):
         return {name: getattr(self, name) for name, _ in self._fields_}
@@ -158,12 +158,14 @@ class Plan:
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                      variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, keep_host: bool = False,
                      medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0,
-                     pipeline: bool = False, max_len: int = 256, threshold: float = 0.75) -> Plan:
+                     pipeline: bool = False, max_len: int = 256, threshold: float = 0.75,
+                     co_schedule: int = -1) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
     (dtype "f16"; passed as binary16 bits) or float32[nnz] (dtype "f32").  panel_rows: 0 automatic,
-    -1 one global panel."""
+    -1 one global panel.  co_schedule: 1 long-row units inside the medium/short kernel (one
+    launch), 0 in their own launch, -1 automatic."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     if dtype == "f64":
@@ -187,6 +189,7 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     opts.panel_rows = panel_rows
     opts.pipeline = int(pipeline)
     opts.max_len, opts.threshold = int(max_len), float(threshold)
+    opts.co_schedule = int(co_schedule)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))
@@ -197,7 +200,7 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
 def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                             variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, medium_rb_per_warp: int = 0,
                             panel_rows: int = 0, pipeline: bool = False, max_len: int = 256, threshold: float = 0.75,
-                            stream=None) -> Plan:
+                            stream=None, co_schedule: int = -1) -> Plan:
     """Build the plan on the GPU from a device CSR (torch CUDA tensors: int64 row_ptr, int32
     col_idx, float64 / float16 val) -- SURVEY.md §8(f) f2."""
     import torch
@@ -212,6 +215,7 @@ def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = 
     opts.device, opts.variant, opts.validate = device, variant, int(validate)
     opts.medium_rb_per_warp, opts.panel_rows, opts.pipeline = medium_rb_per_warp, panel_rows, int(pipeline)
     opts.max_len, opts.threshold = int(max_len), float(threshold)
+    opts.co_schedule = int(co_schedule)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create_device(ctypes.byref(h), m, n, int(col_idx.numel()), _ptr(row_ptr), _ptr(col_idx),
                                       _ptr(val), {"f64": DASP_R_64F, "f16": DASP_R_16F, "f32": DASP_R_32F}[dtype],

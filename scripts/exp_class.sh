@@ -1,18 +1,14 @@
 #!/bin/bash
+# Per-class timing of the main kernel (DASP_PROFILE_CLASS: 2 = medium only, 3 = short only, 1 = long only)
+# plus the co-scheduled vs separate comparison and the GPU test suite.
 mkdir -p gpurun_out
 make -j8 all > gpurun_out/make.log 2>&1 || { tail -30 gpurun_out/make.log; exit 1; }
-timeout 300 python scripts/l2_probe.py > gpurun_out/l2_probe.txt 2>&1
-B="python bench.py --steps 100 --warmup 5 --e2e-steps 0 --no-cpu-baseline --config c3"
-: > gpurun_out/cls.jsonl
-for pr in 0 65536 262144 1048576; do
- for cls in 0 1 2 3; do
-  echo "{\"panel\": $pr, \"cls\": $cls}" >> gpurun_out/cls.jsonl
-  DASP_PANEL_ROWS=$pr DASP_PROFILE_CLASS=$cls timeout 300 $B >> gpurun_out/cls.jsonl 2>> gpurun_out/cls.err
- done
-done
-S="python bench.py --steps 2 --warmup 3 --e2e-steps 0 --no-cpu-baseline --config c3"
-for cls in 1 2 3; do
- DASP_PROFILE_CLASS=$cls timeout 600 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,lts__t_sector_hit_rate.pct,l1tex__t_sector_hit_rate.pct,sm__warps_active.avg.pct_of_peak_sustained_active --clock-control none -k regex:dasp_main -s 3 -c 1 --csv $S > gpurun_out/ncu_cls$cls.csv 2>/dev/null
- DASP_PANEL_ROWS=262144 DASP_PROFILE_CLASS=$cls timeout 600 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,lts__t_sector_hit_rate.pct,l1tex__t_sector_hit_rate.pct --clock-control none -k regex:dasp_main -s 3 -c 1 --csv $S > gpurun_out/ncu_cls${cls}_p.csv 2>/dev/null
-done
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "co_schedule" > gpurun_out/pytest_cosched.log 2>&1; echo "pytest cosched rc=$?"; tail -3 gpurun_out/pytest_cosched.log
+B="python bench.py --steps 300 --warmup 10 --e2e-steps 0 --no-cpu-baseline --no-triad --no-gpu-build --no-compare --no-graph"
+: > gpurun_out/class.jsonl
+for cfg in "c3" "c5 --scale 0.05"; do for dt in f64 f16; do
+  for pc in 1 2 3; do DASP_PROFILE_CLASS=$pc timeout 300 $B --config $cfg --dtype $dt >> gpurun_out/class.jsonl 2>> gpurun_out/class.err; echo "# class $pc" >> gpurun_out/class.jsonl; done
+  for cs in 0 1; do timeout 300 $B --config $cfg --dtype $dt --co-schedule $cs >> gpurun_out/class.jsonl 2>> gpurun_out/class.err; done
+done; done
+timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
 echo done

@@ -369,3 +369,47 @@ def test_cuda_graph_capture_replay(dt):
     g.replay()
     torch.cuda.synchronize()
     assert np.array_equal(yd.cpu().numpy().astype(np.float64), eager.astype(np.float64))
+
+
+# co-scheduled long rows (dasp_options_t.co_schedule): the long units run inside the
+# main kernel and the warp that completes a row's group counter runs its phase 2.  Both modes on
+# every long-row case; repeated launches check that the counters reset themselves (a stale
+# counter would skip or double a row's phase 2), and the two latest launches must be bitwise equal
+# (the phase-2 order is fixed whichever warp runs it).
+@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("cs", [0, 1])
+def test_co_schedule_parity_repeated(cs, dt, variant):
+    for name, gen in CASES:
+        for vm, seed in ((synth.VAL_UNIFORM, 41), (synth.VAL_INT, 42)):
+            A = gen(vm)
+            x = synth.vector(seed, A.n, vm)
+            plan = make(A, dt, co_schedule=cs, panel_rows=700)
+            assert plan.info["co_scheduled"] == (1 if cs and plan.info["row_long"] > 0 else 0), name
+            y_ref, s = oracle_ref(A, x, dt)
+            ys = [run(plan, x, dt, variant=variant) for _ in range(3)]
+            for y in ys:
+                if vm == synth.VAL_INT:
+                    assert np.array_equal(y, y_ref), name
+                else:
+                    assert oracle.tolerance_ok(y, y_ref, s, dt).all(), name
+            assert np.array_equal(ys[1], ys[2]), name
+            y0 = synth.vector(seed + 1, A.m, vm)
+            y = run(plan, x, dt, -0.5, 2.0, y0, variant=variant)
+            y_ref, s = oracle_ref(A, x, dt, -0.5, 2.0, y0)
+            assert oracle.tolerance_ok(y, y_ref, s, dt).all(), name
+
+
+def test_co_schedule_many_long_rows_one_launch_each():
+    """Rows of 257..20000 nonzeros (5..313 groups), so units straddle row ends and several rows
+    complete inside one unit; 20 launches, every one compared with the oracle."""
+    lens = list(np.random.default_rng(5).integers(257, 20000, size=300)) + [257] * 40 + [300, 5, 3, 0] * 10
+    A = synth.from_lengths(lens, n=60000, val_mode=synth.VAL_INT)
+    x = synth.vector(51, A.n, synth.VAL_INT)
+    y_ref, _ = oracle_ref(A, x, "f64")
+    for dt in DTYPES:
+        plan = make(A, dt, co_schedule=1)
+        assert plan.info["co_scheduled"] == 1
+        y_ref_dt, _ = oracle_ref(A, x, dt)
+        for _ in range(20):
+            assert np.array_equal(run(plan, x, dt), y_ref_dt), dt
