@@ -242,7 +242,8 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
             }
             d.t13 = d.t4 = d.t22 = d.ts = 0;
         }
-        const int64_t warps = d.nmw + d.t13 + d.t4 + d.t22 + d.ts;   // long units: own kernel
+        const int64_t tpw = dasp::short_tiles_per_warp(p->dtype);
+        const int64_t warps = d.nmw + (d.t13 + d.t4 + d.t22 + d.ts + tpw - 1) / tpw;   // long units: own kernel
         item_start.push_back(item_start.back() + warps);
         const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
         // co-scheduled: the panel's long blocks are spread evenly among its main blocks, so the

@@ -19,6 +19,41 @@
 
 #include "kernels.cuh"
 
+// build knobs of the medium path (experiments: make exp EXPVARS=...)
+// (per value type: the register allocation of the fused kernel, and with it the measured best
+// setting, differs between the FP64, FP16 and FP32 instantiations; profiles/r01b/knobs*.jsonl)
+//   SMALL_PAIR: two row-blocks without a full chunk loaded together
+//   CHUNK_PIPE: chunk c+1's stream loads issued while chunk c's gathers are in flight
+//   SHORT_TPW : short tiles per warp (1 or 2)
+#ifndef DASP_SMALL_PAIR_F64
+#define DASP_SMALL_PAIR_F64 0
+#endif
+#ifndef DASP_SMALL_PAIR_F16
+#define DASP_SMALL_PAIR_F16 1
+#endif
+#ifndef DASP_SMALL_PAIR_F32
+#define DASP_SMALL_PAIR_F32 0
+#endif
+#ifndef DASP_CHUNK_PIPE_F64
+#define DASP_CHUNK_PIPE_F64 0
+#endif
+#ifndef DASP_CHUNK_PIPE_F16
+#define DASP_CHUNK_PIPE_F16 1
+#endif
+#ifndef DASP_CHUNK_PIPE_F32
+#define DASP_CHUNK_PIPE_F32 0
+#endif
+#ifndef DASP_SHORT_TPW_F64
+#define DASP_SHORT_TPW_F64 2
+#endif
+#ifndef DASP_SHORT_TPW_F16
+#define DASP_SHORT_TPW_F16 2
+#endif
+#ifndef DASP_SHORT_TPW_F32
+#define DASP_SHORT_TPW_F32 2
+#endif
+#define DASP_BY_DT(DT, K) ((DT) == 0 ? K##_F64 : ((DT) == 1 ? K##_F16 : K##_F32))
+
 namespace dasp {
 namespace {
 
@@ -354,16 +389,20 @@ template <int DT> struct MedLd {
     typename ValIO<DT>::R va[4], vr[3], vi;
     uint32_t ca[4], cr[3], ci;
 };
-template <int DT>
+// FULL = false: the row-block is known to have no full chunk (nreg < CW), so the chunk state is
+// dead code and two such row-blocks fit in the registers of one (the small-pair path).
+template <int DT, bool FULL = true>
 __device__ __forceinline__ void medium_load_f64(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, MedLd<DT>& L) {
     using IO = ValIO<DT>;
     const int nreg = M.nelem >> 5;
-    const int nfull = nreg >> 2, rem = nreg & 3;
+    const int nfull = FULL ? nreg >> 2 : 0, rem = nreg & 3;
     const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
+    if constexpr (FULL) {
 #pragma unroll
-    for (int j = 0; j < 4; ++j) { L.va[j] = 0; L.ca[j] = 0xffffffffu; }
-    if (nfull > 0) { IO::ld4r(rv + lane * 4, pol, L.va); ld4_b32(rc + lane * 4, pol, L.ca); }
+        for (int j = 0; j < 4; ++j) { L.va[j] = 0; L.ca[j] = 0xffffffffu; }
+        if (nfull > 0) { IO::ld4r(rv + lane * 4, pol, L.va); ld4_b32(rc + lane * 4, pol, L.ca); }
+    }
     const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane;   // ragged chunk: block j at 32j (R18)
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
@@ -374,30 +413,44 @@ __device__ __forceinline__ void medium_load_f64(const MainParams& P, const RbMet
     L.vi = 0; L.ci = 0xffffffffu;
     if (k < M.ib + M.ilen) { L.vi = IO::ld1r(static_cast<const typename IO::T*>(P.irr_val) + k, pol); L.ci = ld1_b32(P.irr_col + k, pol); }
 }
-template <int DT, int VAR>
+template <int DT, int VAR, bool FULL = true>
 __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbMeta& M, const MedLd<DT>& L, int lane,
                                                   uint64_t pol) {
     using IO = ValIO<DT>;
     const int t = lane & 3;
     const int nreg = M.nelem >> 5;
-    const int nfull = nreg >> 2, rem = nreg & 3;
+    const int nfull = FULL ? nreg >> 2 : 0, rem = nreg & 3;
     const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
     const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
     double c0 = 0.0, c1 = 0.0, part = 0.0;
-    typename IO::R va[4];
-    uint32_t ca[4];
+    if constexpr (FULL) {
+        typename IO::R va[4];
+        uint32_t ca[4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) { va[j] = L.va[j]; ca[j] = L.ca[j]; }
-    for (int ch = 0; ch < nfull; ++ch) {
-        if (ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
-        double xv[4];
+        for (int j = 0; j < 4; ++j) { va[j] = L.va[j]; ca[j] = L.ca[j]; }
+        // software pipeline: chunk ch+1's stream loads are issued while chunk ch's gathers are
+        // in flight (one memory round trip per chunk instead of two)
+        for (int ch = 0; ch < nfull; ++ch) {
+            if (!DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
+            double xv[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
+            for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
+            typename IO::R vn[4];
+            uint32_t cn[4];
+            if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nfull) {
+                IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vn);
+                ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cn);
+            }
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            if constexpr (VAR == VAR_MMA) dmma(c0, c1, IO::cv(va[j]), xv[j]);
-            else part = fma(IO::cv(va[j]), xv[j], part);
+            for (int j = 0; j < 4; ++j) {
+                if constexpr (VAR == VAR_MMA) dmma(c0, c1, IO::cv(va[j]), xv[j]);
+                else part = fma(IO::cv(va[j]), xv[j], part);
+            }
+            if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nfull) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) { va[j] = vn[j]; ca[j] = cn[j]; }
+            }
         }
     }
     double xr[3];
@@ -428,16 +481,19 @@ struct MedLdH {
     uint32_t va[4], ca[8], vr[3], cr[6], ci;
     uint16_t vi;
 };
+template <bool FULL = true>
 __device__ __forceinline__ void medium_load_f16(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, MedLdH& L) {
     const int nreg = M.nelem >> 6;
-    const int nfull = nreg >> 2, rem = nreg & 3;
+    const int nfull = FULL ? nreg >> 2 : 0, rem = nreg & 3;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
+    if constexpr (FULL) {
 #pragma unroll
-    for (int j = 0; j < 4; ++j) L.va[j] = 0u;
+        for (int j = 0; j < 4; ++j) L.va[j] = 0u;
 #pragma unroll
-    for (int e = 0; e < 8; ++e) L.ca[e] = 0xffffffffu;
-    if (nfull > 0) { ld4_b32(rv + lane * 8, pol, L.va); ld8_b32(rc + lane * 8, pol, L.ca); }
+        for (int e = 0; e < 8; ++e) L.ca[e] = 0xffffffffu;
+        if (nfull > 0) { ld4_b32(rv + lane * 8, pol, L.va); ld8_b32(rc + lane * 8, pol, L.ca); }
+    }
     const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2;   // ragged chunk: block j at 64j (R18)
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
@@ -448,19 +504,18 @@ __device__ __forceinline__ void medium_load_f16(const MainParams& P, const RbMet
     L.vi = 0; L.ci = 0xffffffffu;
     if (k < M.ib + M.ilen) { L.vi = __ldg(static_cast<const unsigned short*>(P.irr_val) + k); L.ci = ld1_b32(P.irr_col + k, pol); }
 }
-template <int VAR>
+template <int VAR, bool FULL = true>
 __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbMeta& M, const MedLdH& L, int lane, uint64_t pol) {
     const int t = lane & 3;
     const int nreg = M.nelem >> 6;
-    const int nfull = nreg >> 2, rem = nreg & 3;
+    const int nfull = FULL ? nreg >> 2 : 0, rem = nreg & 3;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
     const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
     float c0 = 0.f, c1 = 0.f, part = 0.f;
     // one 8x8 block: this lane's two slots 2t, 2t+1 of row g
-    auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) {
-        const uint16_t xa = gxh(x, ca), xb = gxh(x, cb);
+    auto blockx = [&](uint32_t a, uint16_t xa, uint16_t xb) {
         if constexpr (VAR == VAR_MMA) {
             hmma(c0, c1, a, pack2(xa, xb));
         } else {
@@ -469,15 +524,29 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
             part = fmaf(av.y, h2f(xb), part);
         }
     };
-    uint32_t va[4], ca[8];
+    auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) { blockx(a, gxh(x, ca), gxh(x, cb)); };
+    if constexpr (FULL) {
+        uint32_t va[4], ca[8];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) va[j] = L.va[j];
+        for (int j = 0; j < 4; ++j) va[j] = L.va[j];
 #pragma unroll
-    for (int e = 0; e < 8; ++e) ca[e] = L.ca[e];
-    for (int ch = 0; ch < nfull; ++ch) {
-        if (ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
+        for (int e = 0; e < 8; ++e) ca[e] = L.ca[e];
+        for (int ch = 0; ch < nfull; ++ch) {   // chunk ch+1's loads overlap chunk ch's gathers
+            if (!DASP_CHUNK_PIPE_F16 && ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
+            uint16_t xh[8];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) block(va[j], ca[2 * j], ca[2 * j + 1]);
+            for (int e = 0; e < 8; ++e) xh[e] = gxh(x, ca[e]);
+            uint32_t vn[4], cn[8];
+            if (DASP_CHUNK_PIPE_F16 && ch + 1 < nfull) { ld4_b32(rv + (ch + 1) * 256 + lane * 8, pol, vn); ld8_b32(rc + (ch + 1) * 256 + lane * 8, pol, cn); }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) blockx(va[j], xh[2 * j], xh[2 * j + 1]);
+            if (DASP_CHUNK_PIPE_F16 && ch + 1 < nfull) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) va[j] = vn[j];
+#pragma unroll
+                for (int e = 0; e < 8; ++e) ca[e] = cn[e];
+            }
+        }
     }
 #pragma unroll
     for (int j = 0; j < 3; ++j)
@@ -754,6 +823,38 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
                 medium_finish_f64<DT, VAR>(P, MB, LB, lane, pol);
             }
         }
+    } else if constexpr (DASP_BY_DT(DT, DASP_SMALL_PAIR) != 0) {
+        // small-pair path: two consecutive row-blocks without a full chunk (nreg < CW: rows of
+        // up to ~15 nonzeros, most medium rows of a power-law matrix) load together, so a warp
+        // keeps two row-blocks' streams and gathers in flight; others take the single path.
+        constexpr int FULL_ELEMS = DT == 1 ? 256 : 128;   // elements of one CW-block chunk
+        int64_t rb = rb0;
+        while (rb < rb1) {
+            const RbMeta MA = rb_meta(P, rb, lane);     // both metadata rounds issued together
+            const RbMeta MB = rb + 1 < rb1 ? rb_meta(P, rb + 1, lane) : RbMeta{0, 0, FULL_ELEMS, 0, -1};
+            {
+                if (MA.nelem < FULL_ELEMS && MB.nelem < FULL_ELEMS) {
+                    if constexpr (DT == 1) {
+                        MedLdH LA, LB;
+                        medium_load_f16<false>(P, MA, lane, pol, LA);
+                        medium_load_f16<false>(P, MB, lane, pol, LB);
+                        medium_finish_f16<VAR, false>(P, MA, LA, lane, pol);
+                        medium_finish_f16<VAR, false>(P, MB, LB, lane, pol);
+                    } else {
+                        MedLd<DT> LA, LB;
+                        medium_load_f64<DT, false>(P, MA, lane, pol, LA);
+                        medium_load_f64<DT, false>(P, MB, lane, pol, LB);
+                        medium_finish_f64<DT, VAR, false>(P, MA, LA, lane, pol);
+                        medium_finish_f64<DT, VAR, false>(P, MB, LB, lane, pol);
+                    }
+                    rb += 2;
+                    continue;
+                }
+            }
+            if constexpr (DT == 1) medium_rb_f16<VAR>(P, MA, lane, pol);
+            else medium_rb_f64<DT, VAR>(P, MA, lane, pol);
+            ++rb;
+        }
     } else {
         for (int64_t rb = rb0; rb < rb1; ++rb) {
             // (prefetching the next row-block's metadata here was measured: it costs registers
@@ -765,29 +866,73 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
 }
 
 // ------------------------------------------------------------------------------------------
-// short rows (Alg. 4) and singles (Alg. 5): one tile of 32 four-slot rows.
-// Results are transposed with shuffles so that lane L writes outputs L and L+32 of the tile:
-// the output map is read with two coalesced loads issued at the start of the tile.
+// short rows (Alg. 4) and singles (Alg. 5): tiles of 32 four-slot rows.
+// One tile is processed in three steps so that a warp can hold TPW tiles' loads and gathers in
+// flight together (DASP_SHORT_TPW): short_load_* (values, columns and the output map, issued
+// together), short_gather_* (x), short_math_* (block dots, segment masks, y).  Results are
+// transposed with shuffles so that lane L writes outputs L and L+32 of a tile: the output map is
+// read with coalesced loads.
 // ------------------------------------------------------------------------------------------
-// cat 0 = 1&3 (seg0 = slot 0, seg1 = slots 1-3), 1 = len-4, 2 = 2&2 (slots 0-1 | 2-3)
+// cat 0 = 1&3 (seg0 = slot 0, seg1 = slots 1-3), 1 = len-4, 2 = 2&2 (slots 0-1 | 2-3), 3 = singles
 __device__ __forceinline__ int seg_of(int cat, int slot) { return cat == 0 ? (slot > 0) : (cat == 2 ? (slot >> 1) : 0); }
 
+struct ShortRef {
+    int cat;
+    int64_t tile, obase;
+};
+// tile t of panel D: category and output base (tiles [1&3][len4][2&2][singles])
+__device__ __forceinline__ ShortRef short_ref(const PanelDesc* D, int64_t t) {
+    const int64_t t13 = __ldg(&D->t13), t4 = __ldg(&D->t4), t22 = __ldg(&D->t22);
+    const int64_t out0 = __ldg(&D->out0);
+    ShortRef r;
+    r.tile = __ldg(&D->tile0) + t;
+    if (t < t13) { r.cat = 0; r.obase = out0 + t * 64; }
+    else if (t < t13 + t4) { r.cat = 1; r.obase = out0 + 64 * t13 + (t - t13) * 32; }
+    else if (t < t13 + t4 + t22) { r.cat = 2; r.obase = out0 + 64 * t13 + 32 * t4 + (t - t13 - t4) * 64; }
+    else { r.cat = 3; r.obase = out0 + 64 * t13 + 32 * t4 + 64 * t22 + (t - t13 - t4 - t22) * 128; }
+    return r;
+}
+// the output map: singles 4 consecutive outputs per lane; two-output tiles L and L+32; len-4 L
+__device__ __forceinline__ void short_load_out(const MainParams& P, const ShortRef& T, int lane, uint64_t pol,
+                                               int32_t (&o)[4]) {
+    if (T.cat == 3) {
+        ld4_b32(P.short_out + T.obase + lane * 4, pol, *reinterpret_cast<uint32_t(*)[4]>(&o));
+    } else {
+        o[0] = __ldg(P.short_out + T.obase + lane);
+        o[1] = T.cat != 1 ? __ldg(P.short_out + T.obase + 32 + lane) : -1;
+        o[2] = o[3] = -1;
+    }
+}
+
+template <int DT> struct ShortLd {          // FP64 / FP32 (m8n8k4 geometry)
+    typename ValIO<DT>::R v[4];
+    uint32_t c[4];
+    int32_t o[4];
+};
+template <int DT>
+__device__ __forceinline__ void short_load_f64(const MainParams& P, const ShortRef& T, int lane, uint64_t pol, ShortLd<DT>& L) {
+    using IO = ValIO<DT>;
+    IO::ld4r(static_cast<const typename IO::T*>(P.short_val) + T.tile * 128 + lane * 4, pol, L.v);
+    ld4_b32(P.short_col + T.tile * 128 + lane * 4, pol, L.c);
+    short_load_out(P, T, lane, pol, L.o);
+}
+template <int DT>
+__device__ __forceinline__ void short_gather_f64(const MainParams& P, const ShortLd<DT>& L, double (&xv)[4]) {
+    using IO = ValIO<DT>;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) xv[j] = IO::gx(static_cast<const typename IO::T*>(P.x), L.c[j]);
+}
 template <int DT, int VAR>
-__device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol) {
+__device__ __forceinline__ void short_math_f64(const MainParams& P, int cat, const ShortLd<DT>& L, const double (&xv)[4],
+                                               int lane) {
+    using IO = ValIO<DT>;
+    if (cat == 3) {                                      // singles (Alg. 5): 4 consecutive len-1 rows
+#pragma unroll
+        for (int j = 0; j < 4; ++j) store_y<DT>(P, L.o[j], IO::cv(L.v[j]) * xv[j]);
+        return;
+    }
     const int g = lane >> 2, t = lane & 3;
     const int nseg = cat == 1 ? 1 : 2;
-    double v[4];
-    uint32_t c[4];
-    using IO = ValIO<DT>;
-    IO::ld4(static_cast<const typename IO::T*>(P.short_val) + tile * 128 + lane * 4, pol, v);
-    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
-    const int32_t o0 = __ldg(P.short_out + obase + lane);                        // outputs L, L+32
-    const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
-    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
-    double xv[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, c[j]);
     const int myseg = seg_of(cat, t);
     // output o = 16j + 8s + g (two outputs per four-slot row) or 8j + g (len-4)
     const int src = 4 * (lane & 7);                      // quad of row g' = lane & 7
@@ -798,10 +943,10 @@ __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int
             double val;
             if constexpr (VAR == VAR_MMA) {              // x masked to the segment (Alg. 4 l.7-11)
                 double cc0 = 0.0, cc1 = 0.0;
-                dmma(cc0, cc1, v[j], myseg == s ? xv[j] : 0.0);
+                dmma(cc0, cc1, IO::cv(L.v[j]), myseg == s ? xv[j] : 0.0);
                 val = __shfl_sync(FULL, (g & 1) ? cc1 : cc0, src + ((lane & 7) >> 1));
             } else {
-                double p = myseg == s ? v[j] * xv[j] : 0.0;
+                double p = myseg == s ? IO::cv(L.v[j]) * xv[j] : 0.0;
                 p += __shfl_xor_sync(FULL, p, 1);
                 p += __shfl_xor_sync(FULL, p, 2);
                 val = __shfl_sync(FULL, p, src);
@@ -811,19 +956,36 @@ __device__ __forceinline__ void short_tile_f64(const MainParams& P, int cat, int
             if ((lane >> 3) == blk - 4) r1 = val;
         }
     }
-    store_y<DT>(P, o0, r0);
-    if (nseg == 2) store_y<DT>(P, o1, r1);
+    store_y<DT>(P, L.o[0], r0);
+    if (nseg == 2) store_y<DT>(P, L.o[1], r1);
 }
 
+struct ShortLdH {                                    // FP16 (two m16n8k8 blocks per tile)
+    uint32_t a0, a2, c[4];
+    int32_t o[4];
+};
+__device__ __forceinline__ void short_load_f16(const MainParams& P, const ShortRef& T, int lane, uint64_t pol, ShortLdH& L) {
+    ld2_b32(static_cast<const uint16_t*>(P.short_val) + T.tile * 128 + lane * 4, pol, L.a0, L.a2);
+    ld4_b32(P.short_col + T.tile * 128 + lane * 4, pol, L.c);
+    short_load_out(P, T, lane, pol, L.o);
+}
+__device__ __forceinline__ void short_gather_f16(const MainParams& P, const ShortLdH& L, uint16_t (&xh)[4]) {
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) xh[e] = gxh(x, L.c[e]);
+}
 template <int VAR>
-__device__ __forceinline__ void short_compute_f16(const MainParams& P, int cat, uint32_t a0, uint32_t a2, const uint32_t (&c)[4],
-                                                  int32_t o0, int32_t o1, int lane) {
+__device__ __forceinline__ void short_math_f16(const MainParams& P, int cat, const ShortLdH& L, const uint16_t (&xh)[4],
+                                               int lane) {
+    if (cat == 3) {                                      // singles (Alg. 5)
+        const float2 lo = u2f2(L.a0), hi = u2f2(L.a2);
+        const float v[4] = {lo.x, lo.y, hi.x, hi.y};
+#pragma unroll
+        for (int j = 0; j < 4; ++j) store_y<1>(P, L.o[j], v[j] * h2f(xh[j]));
+        return;
+    }
     const int g = lane >> 2, t = lane & 3;
     const int nseg = cat == 1 ? 1 : 2;
-    const uint16_t* x = static_cast<const uint16_t*>(P.x);
-    uint16_t xh[4];
-#pragma unroll
-    for (int e = 0; e < 4; ++e) xh[e] = gxh(x, c[e]);
     // element e: four-slot row group q = (e<2 ? 0 : 2) + (t>>1), slot 2(t&1) + (e&1); elements
     // 0,1 are this lane's slots of m16n8k8 block 0 (rows 0-15), elements 2,3 of block 1 (16-31)
     const int seg0 = seg_of(cat, 2 * (t & 1)), seg1 = seg_of(cat, 2 * (t & 1) + 1);
@@ -831,7 +993,7 @@ __device__ __forceinline__ void short_compute_f16(const MainParams& P, int cat, 
     float r0 = 0.f, r1 = 0.f;
     float slo[2], shi[2];
     if constexpr (VAR == VAR_CUDACORE) {
-        const float2 vl = u2f2(a0), vh = u2f2(a2);
+        const float2 vl = u2f2(L.a0), vh = u2f2(L.a2);
         const float p0 = vl.x * h2f(xh[0]), p1 = vl.y * h2f(xh[1]), p2 = vh.x * h2f(xh[2]), p3 = vh.y * h2f(xh[3]);
 #pragma unroll
         for (int s = 0; s < 2; ++s) {
@@ -850,7 +1012,7 @@ __device__ __forceinline__ void short_compute_f16(const MainParams& P, int cat, 
                 const int eb = (q >> 1) * 2;
                 const uint32_t b0 = mine ? pack2(m0 ? xh[eb] : 0, m1 ? xh[eb + 1] : 0) : 0u;
                 float cc0 = 0.f, cc1 = 0.f;
-                hmma(cc0, cc1, (q >> 1) ? a2 : a0, b0);
+                hmma(cc0, cc1, (q >> 1) ? L.a2 : L.a0, b0);
                 val = __shfl_sync(FULL, (g & 1) ? cc1 : cc0, 4 * gs + (gs >> 1));
             } else {
                 val = __shfl_sync(FULL, q < 2 ? slo[s] : shi[s], 4 * gs + 2 * (q & 1));
@@ -860,44 +1022,25 @@ __device__ __forceinline__ void short_compute_f16(const MainParams& P, int cat, 
             if ((lane >> 3) == blk - 4) r1 = val;
         }
     }
-    store_y<1>(P, o0, r0);
-    if (nseg == 2) store_y<1>(P, o1, r1);
+    store_y<1>(P, L.o[0], r0);
+    if (nseg == 2) store_y<1>(P, L.o[1], r1);
 }
 
-template <int VAR>
-__device__ __forceinline__ void short_tile_f16(const MainParams& P, int cat, int64_t tile, int64_t obase, int lane,
-                                               uint64_t pol) {
-    const int nseg = cat == 1 ? 1 : 2;
-    uint32_t a0, a2, c[4];
-    ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
-    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
-    const int32_t o0 = __ldg(P.short_out + obase + lane);
-    const int32_t o1 = nseg == 2 ? __ldg(P.short_out + obase + 32 + lane) : -1;
-    short_compute_f16<VAR>(P, cat, a0, a2, c, o0, o1, lane);
-}
-
-// singles (Alg. 5): lane handles 4 consecutive len-1 rows on CUDA cores
-template <int DT>
-__device__ __forceinline__ void singles_tile(const MainParams& P, int64_t tile, int64_t obase, int lane, uint64_t pol) {
-    uint32_t c[4], o[4];
-    ld4_b32(P.short_col + tile * 128 + lane * 4, pol, c);
-    ld4_b32(P.short_out + obase + lane * 4, pol, o);
-    if constexpr (DT != 1) {
-        using IO = ValIO<DT>;
-        double v[4];
-        IO::ld4(static_cast<const typename IO::T*>(P.short_val) + tile * 128 + lane * 4, pol, v);
-#pragma unroll
-        for (int j = 0; j < 4; ++j)
-            store_y<DT>(P, static_cast<int32_t>(o[j]), v[j] * IO::gx(static_cast<const typename IO::T*>(P.x), c[j]));
+// one tile, all three steps (split short kernel)
+template <int DT, int VAR>
+__device__ __forceinline__ void short_tile(const MainParams& P, const ShortRef& T, int lane, uint64_t pol) {
+    if constexpr (DT == 1) {
+        ShortLdH L;
+        uint16_t xh[4];
+        short_load_f16(P, T, lane, pol, L);
+        short_gather_f16(P, L, xh);
+        short_math_f16<VAR>(P, T.cat, L, xh, lane);
     } else {
-        uint32_t a0, a2;
-        ld2_b32(static_cast<const uint16_t*>(P.short_val) + tile * 128 + lane * 4, pol, a0, a2);
-        float2 lo = u2f2(a0);
-        float2 hi = u2f2(a2);
-        const float v[4] = {lo.x, lo.y, hi.x, hi.y};
-        const uint16_t* x = static_cast<const uint16_t*>(P.x);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) store_y<1>(P, static_cast<int32_t>(o[j]), v[j] * h2f(gxh(x, c[j])));
+        ShortLd<DT> L;
+        double xv[4];
+        short_load_f64<DT>(P, T, lane, pol, L);
+        short_gather_f64<DT>(P, L, xv);
+        short_math_f64<DT, VAR>(P, T.cat, L, xv, lane);
     }
 }
 
@@ -950,25 +1093,36 @@ __device__ __forceinline__ void finish_warp(const MainParams& P, int64_t fw, int
         if (e0 + j < P.n0) empty_row<DT>(P.y, __ldg(P.empty_rows + e0 + j), P.beta, P.extra);
 }
 
-// short tile t of panel D (tiles [1&3][len4][2&2][singles], Alg. 4-5)
+// short warp ws of panel D: tiles ws*TPW .. ws*TPW+TPW-1 (Alg. 4-5).  With TPW = 2 both tiles'
+// loads, then both tiles' gathers are in flight before either tile's arithmetic.
 template <int DT, int VAR>
-__device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc* D, int64_t t, int lane, uint64_t pol) {
-    const int64_t t13 = __ldg(&D->t13), t4 = __ldg(&D->t4), t22 = __ldg(&D->t22);
-    if (t >= t13 + t4 + t22 + __ldg(&D->ts) || !(P.class_mask & 4)) return;
-    const int64_t tile = __ldg(&D->tile0) + t;
-    const int64_t out0 = __ldg(&D->out0);
-    int cat;
-    int64_t obase;
-    if (t < t13) { cat = 0; obase = out0 + t * 64; }
-    else if (t < t13 + t4) { cat = 1; obase = out0 + 64 * t13 + (t - t13) * 32; }
-    else if (t < t13 + t4 + t22) { cat = 2; obase = out0 + 64 * t13 + 32 * t4 + (t - t13 - t4) * 64; }
-    else {
-        obase = out0 + 64 * t13 + 32 * t4 + 64 * t22 + (t - t13 - t4 - t22) * 128;
-        singles_tile<DT>(P, tile, obase, lane, pol);
-        return;
+__device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc* D, int64_t ws, int lane, uint64_t pol) {
+    const int64_t nt = __ldg(&D->t13) + __ldg(&D->t4) + __ldg(&D->t22) + __ldg(&D->ts);
+    constexpr int TPW = DASP_BY_DT(DT, DASP_SHORT_TPW);
+    const int64_t t0 = ws * TPW;
+    if (t0 >= nt || !(P.class_mask & 4)) return;
+    const ShortRef A = short_ref(D, t0);
+    if (TPW == 1 || t0 + 1 >= nt) { short_tile<DT, VAR>(P, A, lane, pol); return; }
+    const ShortRef B = short_ref(D, t0 + 1);
+    if constexpr (DT == 1) {
+        ShortLdH LA, LB;
+        uint16_t xa[4], xb[4];
+        short_load_f16(P, A, lane, pol, LA);
+        short_load_f16(P, B, lane, pol, LB);
+        short_gather_f16(P, LA, xa);
+        short_gather_f16(P, LB, xb);
+        short_math_f16<VAR>(P, A.cat, LA, xa, lane);
+        short_math_f16<VAR>(P, B.cat, LB, xb, lane);
+    } else {
+        ShortLd<DT> LA, LB;
+        double xa[4], xb[4];
+        short_load_f64<DT>(P, A, lane, pol, LA);
+        short_load_f64<DT>(P, B, lane, pol, LB);
+        short_gather_f64<DT>(P, LA, xa);
+        short_gather_f64<DT>(P, LB, xb);
+        short_math_f64<DT, VAR>(P, A.cat, LA, xa, lane);
+        short_math_f64<DT, VAR>(P, B.cat, LB, xb, lane);
     }
-    if constexpr (DT == 1) short_tile_f16<VAR>(P, cat, tile, obase, lane, pol);
-    else short_tile_f64<DT, VAR>(P, cat, tile, obase, lane, pol);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1108,9 +1262,7 @@ dasp_short_kernel(const MainParams P, const uint64_t* __restrict__ tile_meta, in
     const uint64_t meta = __ldg(tile_meta + t);
     const int cat = static_cast<int>(meta >> 62);
     const int64_t obase = static_cast<int64_t>(meta & ((1ull << 62) - 1));
-    if (cat == 3) { singles_tile<DT>(P, t, obase, lane, pol); return; }
-    if constexpr (DT == 1) short_tile_f16<VAR>(P, cat, t, obase, lane, pol);
-    else short_tile_f64<DT, VAR>(P, cat, t, obase, lane, pol);
+    short_tile<DT, VAR>(P, ShortRef{cat, t, obase}, lane, pol);
 }
 
 // long phase 2 (Alg. 2 l.17-25): one warp per long row, lane-strided sum of the group partials
@@ -1476,7 +1628,17 @@ __device__ __forceinline__ void short_stage_f16(const MainParams& P, const uint8
         store_y<1>(P, o.w, hi.y * h2f(gxh(x, c[3])));
         return;
     }
-    short_compute_f16<VAR>(P, cat, a.x, a.y, c, so[lane], cat == 1 ? -1 : so[32 + lane], lane);
+    ShortLdH L;
+    L.a0 = a.x;
+    L.a2 = a.y;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) L.c[e] = c[e];
+    L.o[0] = so[lane];
+    L.o[1] = cat == 1 ? -1 : so[32 + lane];
+    L.o[2] = L.o[3] = -1;
+    uint16_t xh[4];
+    short_gather_f16(P, L, xh);
+    short_math_f16<VAR>(P, cat, L, xh, lane);
 }
 
 template <int VAR>
@@ -1659,6 +1821,8 @@ __global__ void __launch_bounds__(256) dasp_long_meta_kernel(const int64_t* __re
     for (int64_t g = g0 + lane; g < g1; g += 32) group_row[g] = static_cast<int32_t>(r);
 }
 }  // namespace
+
+int short_tiles_per_warp(int dtype) { return DASP_BY_DT(dtype, DASP_SHORT_TPW); }
 
 cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,
                              cudaStream_t s) {

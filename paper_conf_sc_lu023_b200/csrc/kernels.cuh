@@ -92,6 +92,8 @@ struct FinishParams {
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
+// short tiles one main-kernel warp processes (build knob DASP_SHORT_TPW)
+int short_tiles_per_warp(int dtype);
 // co-scheduled mode metadata from group_ptr: long_cnt[r] = groups of row r, group_row[g] = row
 // (group_row must be pre-filled with -1 for the pad groups)
 cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,

@@ -413,3 +413,4 @@ def test_co_schedule_many_long_rows_one_launch_each():
         y_ref_dt, _ = oracle_ref(A, x, dt)
         for _ in range(20):
             assert np.array_equal(run(plan, x, dt), y_ref_dt), dt
+
