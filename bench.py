@@ -267,6 +267,12 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
+    elif args.fused:   # the fused scatter mode rendezvouses symmetric memory over a process group
+        import socket
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1, device_id=dev)
     variant = dasp.DASP_VARIANT_MMA if args.variant == "mma" else dasp.DASP_VARIANT_CUDACORE
 
     # ---- inputs: this rank's slab (whole matrix at N = 1), generated per row ----
@@ -491,16 +497,20 @@ def main():
             d_rp = torch.from_numpy(slab.row_ptr).to(dev)
             d_col = torch.from_numpy(np.ascontiguousarray(slab.col)).to(dev)
             d_val = torch.from_numpy(np.ascontiguousarray(slab.val)).to(vdt).to(dev)
-            torch.cuda.synchronize(dev)
-            t0 = time.perf_counter()
-            dplan = dasp.dasp_plan_create_device(d_rp, d_col, d_val, slab.rows, spec.n, args.dtype, device=local,
-                                                 panel_rows=args.panel_rows)
-            wall = (time.perf_counter() - t0) * 1e3
-            gpu_build = {"gpu_build_ms": dplan.info["build_ms"], "wall_ms": wall,
+            builds = []
+            for _ in range(2):   # the first call also pays CUDA lazy module loading of the builder kernels
+                torch.cuda.synchronize(dev)
+                t0 = time.perf_counter()
+                dplan = dasp.dasp_plan_create_device(d_rp, d_col, d_val, slab.rows, spec.n, args.dtype,
+                                                     device=local, panel_rows=args.panel_rows)
+                builds.append((dplan.info["build_ms"], (time.perf_counter() - t0) * 1e3))
+                dplan.destroy()
+            (cold_ms, cold_wall), (warm_ms, wall) = builds
+            gpu_build = {"gpu_build_ms": warm_ms, "wall_ms": wall, "first_call_ms": cold_ms,
+                         "first_call_note": "first call in the process includes CUDA lazy loading of the builder kernels",
                          "host_build_ms": info["build_ms"], "host_upload_ms": info["upload_ms"],
-                         "spmv_equivalents": dplan.info["build_ms"] / ms_step,
+                         "spmv_equivalents": warm_ms / ms_step,
                          "host_spmv_equivalents": (info["build_ms"] + info["upload_ms"]) / ms_step}
-            dplan.destroy()
             del d_rp, d_col, d_val
             torch.cuda.empty_cache()
         except Exception as exc:   # reported, not fatal: the bench line is about the SpMV
@@ -548,7 +558,7 @@ def main():
                      "medium_rb_per_warp": info["medium_rb_per_warp"]},
         }
         print(json.dumps(line))
-    if world > 1:
+    if dist.is_initialized():
         dist.destroy_process_group()
 
 
