@@ -28,7 +28,7 @@ $(PKG)/libdasp.so: $(OBJ)/builder.o $(OBJ)/kernels.o $(OBJ)/gpu_builder.o $(OBJ)
 	$(NVCC) $(ARCH) -shared -o $@ $^ -Xcompiler -fopenmp -lgomp
 
 oracle/liboracle.so: oracle/oracle.c
-	gcc -O2 -ffp-contract=off -fno-fast-math -fPIC -shared -o $@ $< -lm
+	gcc -O2 -ffp-contract=off -fno-fast-math -fopenmp -fPIC -shared -o $@ $< -lm
 
 synth/libsynth.so: synth/synth.c
 	gcc -O2 -fopenmp -fPIC -shared -o $@ $< -lm

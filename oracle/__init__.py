@@ -36,7 +36,8 @@ COUNTS = ["m", "n", "nnz", "n0", "n1", "n2", "n3", "n4", "row_medium", "row_long
 def build_lib() -> str:
     src = os.path.join(_HERE, "oracle.c")
     if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
-        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared", "-o", _SO, src, "-lm"])
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-fPIC", "-shared",
+                               "-o", _SO, src, "-lm"])
     return _SO
 
 
@@ -50,6 +51,8 @@ def _L():
         lib = ctypes.CDLL(_SO)
         vp, i64, d = ctypes.c_void_p, ctypes.c_int64, ctypes.c_double
         lib.oracle_spmv.argtypes = [i64, vp, vp, vp, vp, d, d, vp, vp, vp]
+        lib.oracle_spmv_mt.argtypes = [i64, vp, vp, vp, vp, d, d, vp, vp, vp, ctypes.c_int]
+        lib.oracle_spmv_mt.restype = ctypes.c_int
         lib.oracle_build.argtypes = [ctypes.c_int, i64, i64, vp, vp, vp, i64, i64, d]
         lib.oracle_build.restype = vp
         lib.oracle_free.argtypes = [vp]
@@ -79,6 +82,21 @@ def spmv(row_ptr, col, val, x, alpha=1.0, beta=0.0, y0=None):
         y0 = None
     _L().oracle_spmv(m, _p(row_ptr), _p(col), _p(val), _p(x), float(alpha), float(beta), _p(y0), _p(y), _p(s))
     return y, s
+
+
+def spmv_mt(row_ptr, col, val, x, alpha=1.0, beta=0.0, y0=None, threads=0):
+    """The same as spmv with the rows split over host threads (OpenMP); returns (y, s, threads)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    val = np.ascontiguousarray(np.asarray(val).astype(np.float64))
+    x = np.ascontiguousarray(np.asarray(x).astype(np.float64))
+    m = len(row_ptr) - 1
+    y = np.empty(max(m, 1))[:m]
+    s = np.empty(max(m, 1))[:m]
+    y0 = np.ascontiguousarray(np.asarray(y0).astype(np.float64)) if beta != 0.0 else None
+    used = _L().oracle_spmv_mt(m, _p(row_ptr), _p(col), _p(val), _p(x), float(alpha), float(beta), _p(y0), _p(y),
+                               _p(s), int(threads))
+    return y, s, used
 
 
 def spmv_csr(A, x, alpha=1.0, beta=0.0, y0=None):

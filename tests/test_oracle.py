@@ -240,3 +240,18 @@ def test_empty_and_degenerate():
     A0 = synth.CSR(0, 0, np.zeros(1, dtype=np.int64), np.zeros(0, np.int32), np.zeros(0))
     F0 = oracle.build(A0, "f64")
     assert all(v == 0 for k, v in F0.counts.items() if k not in ("panel_rows", "n_panels"))
+
+
+def test_oracle_multithreaded_copy_is_bitwise_identical():
+    """oracle_spmv_mt runs the same per-row loop with rows split over threads (bench.py's all-core
+    oracle timing): every row is computed by one thread in the same order, so y and s are
+    bit-identical to the single-thread oracle, with and without alpha/beta."""
+    for name, scale in (("c1b", 1.0), ("c3", 0.002)):
+        A = synth.generate(synth.config(name, scale=scale))
+        x = synth.vector(3, A.n)
+        y0 = synth.vector(4, A.m)
+        for alpha, beta in ((1.0, 0.0), (-0.5, 2.0)):
+            y1, s1 = oracle.spmv(A.row_ptr, A.col, A.val, x, alpha, beta, y0)
+            y2, s2, used = oracle.spmv_mt(A.row_ptr, A.col, A.val, x, alpha, beta, y0, threads=4)
+            assert used == 4
+            assert np.array_equal(y1, y2) and np.array_equal(s1, s2)
