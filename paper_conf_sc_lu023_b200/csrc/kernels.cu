@@ -3,7 +3,9 @@
 // Two launches per SpMV: the long-row phase-1 kernel (Alg. 2 l.1-16), then the
 // main kernel, whose warps are (warp-uniform dispatch on the global warp index) long-row
 // phase 2 + empty rows first (Alg. 2 l.17-25), then per row panel the medium row-blocks
-// (Alg. 3) and short tiles (Alg. 4-5).  Every block inner product is computed by one of two
+// (Alg. 3) and short tiles, two per warp (Alg. 4-5).  Opt-in (options.co_schedule): one launch,
+// the long units as blocks of the main kernel and phase 2 run by the warp that completes a
+// row's group counter (long_unit_complete).  Every block inner product is computed by one of two
 // variants that read the SAME packed arrays (north_star (3)):
 //   VAR_MMA      legacy warp MMA: DMMA m8n8k4 f64 (Listing 1) / HMMA m16n8k8
 //                f16->f32; the block dot products sit on the diagonal of C (Fig. 4)
