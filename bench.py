@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--variant", default="cudacore", choices=["mma", "cudacore"])
     ap.add_argument("--no-compare", action="store_true", help="skip timing the other compute variant")
     ap.add_argument("--no-graph", action="store_true", help="skip the CUDA-graph replay measurement (N=1 SpMV)")
+    ap.add_argument("--no-library", action="store_true", help="skip the cuSPARSE (torch CSR) context timing")
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--pipeline", action="store_true", help="use the TMA-staged persistent kernel")
@@ -417,6 +418,37 @@ def main():
         except Exception as exc:   # reported, not fatal
             graph = {"error": str(exc)}
 
+    # context only (the paper compares against cuSPARSE CSR SpMV): the same matrix and
+    # x through torch's CSR tensor @ vector, i.e. cuSPARSE SpMV on this GPU, same timing protocol
+    library = None
+    if not use_slab and not args.no_library and args.dtype in ("f64", "f32"):
+        try:
+            vdt = torch.float64 if args.dtype == "f64" else torch.float32
+            Acsr = torch.sparse_csr_tensor(torch.from_numpy(slab.row_ptr).to(dev),
+                                           torch.from_numpy(np.ascontiguousarray(slab.col)).to(dev),
+                                           torch.from_numpy(np.ascontiguousarray(slab.val)).to(vdt).to(dev),
+                                           size=(slab.rows, spec.n))
+            xl = xd.to(vdt)
+            with torch.cuda.stream(stream):
+                for _ in range(5):
+                    yl = torch.mv(Acsr, xl)
+                l0, l1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                nrep = min(args.steps, 200)
+                l0.record(stream)
+                for _ in range(nrep):
+                    yl = torch.mv(Acsr, xl)
+                l1.record(stream)
+            torch.cuda.synchronize(dev)
+            lms = l0.elapsed_time(l1) / nrep
+            err = float(torch.max(torch.abs(yl.to(torch.float64) - yd.to(torch.float64) / alpha)))
+            library = {"impl": "cuSPARSE CSR SpMV via torch.mv(sparse_csr)", "ms_per_step": lms,
+                       "GFLOPS": 2.0 * float(lens.sum()) / (lms * 1e-3) / 1e9, "steps": nrep,
+                       "max_abs_diff_vs_dasp": err}
+            del Acsr, xl, yl
+            torch.cuda.empty_cache()
+        except Exception as exc:   # reported, not fatal
+            library = {"error": str(exc)[:200]}
+
     nnz_total = int(lens.sum())
     flops_step = 2.0 * nnz_total
     gflops = flops_step / (ms_step * 1e-3) / 1e9
@@ -558,7 +590,8 @@ def main():
             "gpu_launches": launches_step * args.steps,
             "gpu_launches_per_step": launches_step,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-            "variant_compare": compare, "cuda_graph": graph, "preprocessing": gpu_build,
+            "variant_compare": compare, "cuda_graph": graph, "library_context": library,
+            "preprocessing": gpu_build,
             "plan": {"build_ms": info["build_ms"], "upload_ms": info["upload_ms"], "gen_s": gen_s, "plan_s": plan_s,
                      "rows": {"empty": info["n_empty"], "short": info["n_len1"] + info["n_len2"] + info["n_len3"]
                               + info["n_len4"], "medium": info["row_medium"], "long": info["row_long"]},
