@@ -424,10 +424,11 @@ def main():
     if not use_slab and not args.no_library and args.dtype in ("f64", "f32"):
         try:
             vdt = torch.float64 if args.dtype == "f64" else torch.float32
-            Acsr = torch.sparse_csr_tensor(torch.from_numpy(slab.row_ptr).to(dev),
-                                           torch.from_numpy(np.ascontiguousarray(slab.col)).to(dev),
+            idt = np.int32 if int(slab.row_ptr[-1]) < 2 ** 31 - 1 else np.int64   # one index dtype for both
+            Acsr = torch.sparse_csr_tensor(torch.from_numpy(slab.row_ptr.astype(idt)).to(dev),
+                                           torch.from_numpy(np.ascontiguousarray(slab.col).astype(idt)).to(dev),
                                            torch.from_numpy(np.ascontiguousarray(slab.val)).to(vdt).to(dev),
-                                           size=(slab.rows, spec.n))
+                                           size=(slab.rows, spec.n), check_invariants=False)
             xl = xd.to(vdt)
             with torch.cuda.stream(stream):
                 for _ in range(5):
