@@ -193,6 +193,23 @@ dasp_status_t dasp_spmv_scatter(dasp_plan_t plan, const void* x, void* const* y_
 dasp_status_t dasp_spmv_host(dasp_plan_t plan, const void* x_host, void* y_host, double alpha,
                              double beta, void* stream);
 
+/*
+ * dasp_spmv_host_stream — dasp_spmv_host over a stream of `nvec` independent right-hand sides:
+ * y_j = alpha*A*x_j + beta*y_j for j = 0..nvec-1 (Alg. 1; the iterated / many-vector use
+ * the paper amortises its preprocessing over).  x_host holds the vectors at a stride of
+ * ldx >= n elements, y_host at a stride of ldy >= m elements (element types as dasp_spmv).  The
+ * call pipelines them through two plan-owned device slots: the host->device copy of x_{j+1} and
+ * the device->host copy of y_{j-1} run on two plan-owned copy streams while SpMV j runs on
+ * `stream`, so per vector the cost approaches max(H2D, kernel, D2H) rather than their sum.  Every
+ * vector is copied in and its result copied out (no caching).  Results are identical to nvec
+ * dasp_spmv_host calls.  Synchronises `stream` before returning; the host buffers must stay valid
+ * until then and should be pinned (pageable memory serialises the copies).  Returns INVALID_ARG
+ * (null plan, nvec < 0, ldx < n with x needed, ldy < m, null buffers), UNSUPPORTED (host-only plan),
+ * OUT_OF_MEMORY or CUDA.
+ */
+dasp_status_t dasp_spmv_host_stream(dasp_plan_t plan, const void* x_host, int64_t ldx, void* y_host,
+                                    int64_t ldy, int64_t nvec, double alpha, double beta, void* stream);
+
 /* Frees every host and device buffer of the plan.  No call on the plan may be in flight
  * (the call synchronises the plan's device).  NULL is accepted. */
 dasp_status_t dasp_plan_destroy(dasp_plan_t plan);

@@ -32,6 +32,11 @@ struct dasp_plan_s {
     void* d_partial = nullptr;
     void* d_xh = nullptr;                 // dasp_spmv_host staging
     void* d_yh = nullptr;
+    // dasp_spmv_host_stream: double-buffered device x/y, two copy streams, per-slot events
+    void* d_xs[2] = {};
+    void* d_ys[2] = {};
+    cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+    cudaEvent_t ev_x[2] = {}, ev_done[2] = {}, ev_yout[2] = {};
     int64_t device_bytes = 0;
     double build_ms = 0, upload_ms = 0;
     int64_t blocks = 0;                   // grid of the medium/short kernel
@@ -122,6 +127,18 @@ void free_device(dasp_plan_s* p) {
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
+    for (int b = 0; b < 2; ++b) {
+        if (p->d_xs[b]) cudaFree(p->d_xs[b]);
+        if (p->d_ys[b]) cudaFree(p->d_ys[b]);
+        p->d_xs[b] = p->d_ys[b] = nullptr;
+        for (cudaEvent_t* e : {&p->ev_x[b], &p->ev_done[b], &p->ev_yout[b]}) {
+            if (*e) cudaEventDestroy(*e);
+            *e = nullptr;
+        }
+    }
+    if (p->s_h2d) cudaStreamDestroy(p->s_h2d);
+    if (p->s_d2h) cudaStreamDestroy(p->s_d2h);
+    p->s_h2d = p->s_d2h = nullptr;
     for (auto& r : p->recs) { (void)r; }
     for (auto e : p->pool) cudaEventDestroy(e);
     p->pool.clear();
@@ -672,6 +689,62 @@ dasp_status_t dasp_spmv_host(dasp_plan_t p, const void* x_host, void* y_host, do
     dasp_status_t st = dasp_spmv(p, p->d_xh, p->d_yh, alpha, beta, stream);
     if (st != DASP_OK) return st;
     if (cudaMemcpyAsync(y_host, p->d_yh, yb, cudaMemcpyDeviceToHost, s) != cudaSuccess) return DASP_ERR_CUDA;
+    return cudaStreamSynchronize(s) == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
+}
+
+dasp_status_t dasp_spmv_host_stream(dasp_plan_t p, const void* x_host, int64_t ldx, void* y_host, int64_t ldy,
+                                    int64_t nvec, double alpha, double beta, void* stream) {
+    if (!p || nvec < 0) return DASP_ERR_INVALID_ARG;
+    if (p->device < 0) return DASP_ERR_UNSUPPORTED;
+    const HostFormat& f = p->host;
+    if (f.m == 0 || nvec == 0) return DASP_OK;
+    const bool need_x = f.n > 0 && alpha != 0.0;
+    if (!y_host || (!x_host && need_x)) return DASP_ERR_INVALID_ARG;
+    if ((need_x && ldx < f.n) || ldy < f.m) return DASP_ERR_INVALID_ARG;
+    DeviceGuard guard(p->device);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const size_t xb = static_cast<size_t>(f.n) * sx(p->dtype), yb = static_cast<size_t>(f.m) * sy(p->dtype);
+    const size_t xs = static_cast<size_t>(ldx) * sx(p->dtype), ys = static_cast<size_t>(ldy) * sy(p->dtype);
+    for (int b = 0; b < 2; ++b) {
+        if (!p->d_xs[b] && xb && cudaMalloc(&p->d_xs[b], xb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
+        if (!p->d_ys[b] && cudaMalloc(&p->d_ys[b], yb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
+        for (cudaEvent_t* e : {&p->ev_x[b], &p->ev_done[b], &p->ev_yout[b]})
+            if (!*e && cudaEventCreateWithFlags(e, cudaEventDisableTiming) != cudaSuccess) return DASP_ERR_CUDA;
+    }
+    if (!p->s_h2d && cudaStreamCreateWithFlags(&p->s_h2d, cudaStreamNonBlocking) != cudaSuccess) return DASP_ERR_CUDA;
+    if (!p->s_d2h && cudaStreamCreateWithFlags(&p->s_d2h, cudaStreamNonBlocking) != cudaSuccess) return DASP_ERR_CUDA;
+    // order the copy streams after everything already enqueued on `stream`
+    if (cudaEventRecord(p->ev_yout[0], s) != cudaSuccess || cudaEventRecord(p->ev_yout[1], s) != cudaSuccess ||
+        cudaEventRecord(p->ev_done[0], s) != cudaSuccess || cudaEventRecord(p->ev_done[1], s) != cudaSuccess)
+        return DASP_ERR_CUDA;
+    const char* xh = static_cast<const char*>(x_host);
+    char* yh = static_cast<char*>(y_host);
+    bool ok = true;
+    for (int64_t j = 0; j < nvec && ok; ++j) {
+        const int b = static_cast<int>(j & 1);
+        // h2d: vector j into slot b once SpMV j-2 has read it (and, for beta != 0, y_j once y_{j-2} left)
+        ok = ok && cudaStreamWaitEvent(p->s_h2d, p->ev_done[b], 0) == cudaSuccess;
+        if (need_x) ok = ok && cudaMemcpyAsync(p->d_xs[b], xh + j * xs, xb, cudaMemcpyHostToDevice, p->s_h2d) == cudaSuccess;
+        if (beta != 0.0) {
+            ok = ok && cudaStreamWaitEvent(p->s_h2d, p->ev_yout[b], 0) == cudaSuccess;
+            ok = ok && cudaMemcpyAsync(p->d_ys[b], yh + j * ys, yb, cudaMemcpyHostToDevice, p->s_h2d) == cudaSuccess;
+        }
+        ok = ok && cudaEventRecord(p->ev_x[b], p->s_h2d) == cudaSuccess;
+        // compute: SpMV j on `stream` after its inputs landed and y slot b was drained
+        ok = ok && cudaStreamWaitEvent(s, p->ev_x[b], 0) == cudaSuccess;
+        ok = ok && cudaStreamWaitEvent(s, p->ev_yout[b], 0) == cudaSuccess;
+        if (!ok) break;
+        dasp_status_t st = dasp_spmv(p, p->d_xs[b], p->d_ys[b], alpha, beta, stream);
+        if (st != DASP_OK) return st;
+        ok = ok && cudaEventRecord(p->ev_done[b], s) == cudaSuccess;
+        // d2h: y_j back while x_{j+1} comes in and SpMV j+1 runs
+        ok = ok && cudaStreamWaitEvent(p->s_d2h, p->ev_done[b], 0) == cudaSuccess;
+        ok = ok && cudaMemcpyAsync(yh + j * ys, p->d_ys[b], yb, cudaMemcpyDeviceToHost, p->s_d2h) == cudaSuccess;
+        ok = ok && cudaEventRecord(p->ev_yout[b], p->s_d2h) == cudaSuccess;
+    }
+    if (!ok) return DASP_ERR_CUDA;
+    if (cudaStreamWaitEvent(s, p->ev_yout[0], 0) != cudaSuccess || cudaStreamWaitEvent(s, p->ev_yout[1], 0) != cudaSuccess)
+        return DASP_ERR_CUDA;
     return cudaStreamSynchronize(s) == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
 }
 

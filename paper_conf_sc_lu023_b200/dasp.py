@@ -27,6 +27,7 @@ STATUS = ["DASP_OK", "DASP_ERR_INVALID_ARG", "DASP_ERR_INVALID_CSR", "DASP_ERR_O
 
 # every symbol include/dasp.h declares (tests check the library exports all of them)
 EXPORTS = ["dasp_options_default", "dasp_plan_create", "dasp_plan_create_device", "dasp_spmv", "dasp_spmv_ex", "dasp_spmv_scatter", "dasp_spmv_host",
+           "dasp_spmv_host_stream",
            "dasp_plan_destroy", "dasp_status_string", "dasp_plan_get_info", "dasp_plan_copy_array",
            "dasp_partition_rows", "dasp_remap_columns", "dasp_gather_halo", "dasp_plan_set_timing", "dasp_plan_read_timing",
            "dasp_version"]
@@ -78,6 +79,7 @@ def _load():
         "dasp_spmv": ([vp, vp, vp, d, d, vp], ctypes.c_int),
         "dasp_spmv_ex": ([vp, vp, vp, d, d, vp, i32], ctypes.c_int),
         "dasp_spmv_host": ([vp, vp, vp, d, d, vp], ctypes.c_int),
+        "dasp_spmv_host_stream": ([vp, vp, i64, vp, i64, i64, d, d, vp], ctypes.c_int),
         "dasp_spmv_scatter": ([vp, vp, ctypes.POINTER(vp), i32, d, d, vp], ctypes.c_int),
         "dasp_plan_destroy": ([vp], ctypes.c_int),
         "dasp_status_string": ([ctypes.c_int], ctypes.c_char_p),
@@ -262,6 +264,15 @@ def dasp_spmv_host(plan: Plan, x: np.ndarray, y: np.ndarray, alpha: float = 1.0,
     """End-to-end call with host buffers (copies inside; synchronises)."""
     st = _lib.dasp_spmv_host(plan.handle, _ptr(x), _ptr(y), float(alpha), float(beta), _stream_ptr(stream))
     _check(st, "dasp_spmv_host")
+
+
+def dasp_spmv_host_stream(plan: Plan, x, ldx: int, y, ldy: int, nvec: int, alpha: float = 1.0, beta: float = 0.0,
+                          stream=None):
+    """nvec end-to-end SpMVs with host buffers (vectors at strides ldx / ldy elements), H2D / SpMV / D2H
+    pipelined over two device slots; synchronises."""
+    st = _lib.dasp_spmv_host_stream(plan.handle, _ptr(x), int(ldx), _ptr(y), int(ldy), int(nvec), float(alpha),
+                                    float(beta), _stream_ptr(stream))
+    _check(st, "dasp_spmv_host_stream")
 
 
 def dasp_plan_destroy(plan: Plan):

@@ -220,6 +220,38 @@ def test_spmv_host_end_to_end():
     assert oracle.tolerance_ok(y, y_ref, s).all()
 
 
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("beta", [0.0, -0.5])
+def test_spmv_host_stream_pipelined(dt, beta):
+    """dasp_spmv_host_stream: nvec vectors at padded strides through the two-slot H2D/SpMV/D2H
+    pipeline; every y_j matches the oracle and equals the one-call-per-vector result bit for bit."""
+    A = synth.generate(synth.config("c1b"))
+    nvec, ldx, ldy = 5, A.n + 3, A.m + 5
+    X = np.zeros((nvec, ldx), dtype=NP_VAL[dt])
+    for j in range(nvec):
+        X[j, :A.n] = synth.vector(20 + j, A.n).astype(NP_VAL[dt])
+    ynp = np.float64 if dt == "f64" else np.float32
+    Y0 = np.zeros((nvec, ldy), dtype=ynp)
+    for j in range(nvec):
+        Y0[j, :A.m] = synth.vector(40 + j, A.m).astype(ynp)
+    Xh = torch.from_numpy(X).pin_memory()
+    Yh = torch.from_numpy(Y0.copy()).pin_memory()
+    plan = make(A, dt)
+    dasp.dasp_spmv_host_stream(plan, Xh.data_ptr(), ldx, Yh.data_ptr(), ldy, nvec, 1.5, beta)
+    Y = Yh.numpy()
+    val64 = A.val.astype(NP_VAL[dt]).astype(np.float64)
+    for j in range(nvec):
+        y_ref, s = oracle.spmv(A.row_ptr, A.col, val64, X[j, :A.n].astype(np.float64), 1.5, beta,
+                               Y0[j, :A.m].astype(np.float64))
+        assert oracle.tolerance_ok(Y[j, :A.m].astype(np.float64), y_ref, s, dt).all(), j
+        assert np.array_equal(Y[j, A.m:], Y0[j, A.m:])          # stride padding untouched
+        y1 = Y0[j, :A.m].copy()
+        dasp.dasp_spmv_host(plan, np.ascontiguousarray(X[j, :A.n]), y1, 1.5, beta)
+        assert np.array_equal(y1, Y[j, :A.m]), j
+    with pytest.raises(dasp.DaspError):
+        dasp.dasp_spmv_host_stream(plan, Xh.data_ptr(), A.n - 1, Yh.data_ptr(), ldy, nvec, 1.0, 0.0)
+
+
 def test_bad_device_args():
     A = synth.generate(synth.config("c1a"))
     plan = make(A, "f64")
