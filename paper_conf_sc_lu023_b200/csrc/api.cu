@@ -223,10 +223,27 @@ namespace {
 // the medium/short kernel, the long-unit schedule, the pipelined kernel's item words, and their
 // device copies.  `panel_table` (host) is the DASP_ARR_PANELS content; `unit_first_col[u]` the
 // column of the first element of long unit u (for the column-bucket schedule).
+// narrow_slots[rb] = max(K nreg, longest row) = K nreg(rb) + irregular length of the row-block's
+// first (longest) row: the slots each of its rows spans (rows are sorted by length, so within a
+// panel this is non-increasing and the narrow row-blocks are a suffix).  rb_ptr [nrb+1] and
+// irr_first [2 nrb] = irr_ptr[8 rb], irr_ptr[8 rb + 1], host copies.
+std::vector<int32_t> narrow_slots(const HostFormat& f, const int64_t* rb_ptr, const int64_t* irr_first) {
+    std::vector<int32_t> ns(static_cast<size_t>(f.nrb));
+    const int64_t be = static_cast<int64_t>(f.geo.K) * 8;
+    for (int64_t rb = 0; rb < f.nrb; ++rb)
+        ns[rb] = static_cast<int32_t>((rb_ptr[rb + 1] - rb_ptr[rb]) / be * f.geo.K + (irr_first[2 * rb + 1] - irr_first[2 * rb]));
+    return ns;
+}
+
 dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_t* panel_table,
-                           const std::vector<int32_t>& unit_first_col) {
+                           const std::vector<int32_t>& unit_first_col, const std::vector<int32_t>& nslots) {
     HostFormat& f = p->host;
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
+    int64_t nrw = dasp::narrow_rb_per_warp(p->dtype);
+    {
+        const char* ne = std::getenv("DASP_NARROW");   // 0 = every row-block on the wide path (experiments)
+        if ((ne && std::atoi(ne) == 0) || static_cast<int64_t>(nslots.size()) != f.nrb) nrw = 0;
+    }
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<uint64_t> blk_word;
     std::vector<uint64_t> tile_meta;
@@ -245,7 +262,12 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
         dasp::PanelDesc& d = desc[q];
         d.blk0 = blk;
-        d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5]; d.nmw = (e[5] + p->rbw - 1) / p->rbw;
+        d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5];
+        d.rbn = d.nrb;
+        if (nrw > 0)
+            while (d.rbn > 0 && nslots[d.rb0 + d.rbn - 1] <= dasp::narrow_max_slots()) --d.rbn;
+        d.nmwd = (d.rbn + p->rbw - 1) / p->rbw;
+        d.nmw = d.nmwd + (nrw > 0 ? (d.nrb - d.rbn + nrw - 1) / nrw : 0);
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
         if (p->split_short) {   // tiles leave the main kernel; per-tile metadata for the short kernel
             for (int64_t t = 0; t < d.t13 + d.t4 + d.t22 + d.ts; ++t) {
@@ -475,9 +497,16 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         const int64_t ue = static_cast<int64_t>(f.geo.UG) * f.geo.G;
         for (size_t u = 0; u < first_col.size(); ++u) first_col[u] = lc[u * ue];
     }
+    std::vector<int64_t> irr_first(static_cast<size_t>(2 * f.nrb));
+    {
+        const int64_t* ip = static_cast<const int64_t*>(f.arr[DASP_ARR_IRR_PTR].ptr);
+        for (int64_t rb = 0; rb < f.nrb; ++rb) { irr_first[2 * rb] = ip[8 * rb]; irr_first[2 * rb + 1] = ip[8 * rb + 1]; }
+    }
+    const std::vector<int32_t> nslots =
+        f.nrb ? narrow_slots(f, static_cast<const int64_t*>(f.arr[DASP_ARR_RB_PTR].ptr), irr_first.data()) : std::vector<int32_t>();
     std::unique_ptr<DeviceGuard> guard;
     if (p->device >= 0) guard.reset(new DeviceGuard(p->device));
-    st = setup_launch(p, o, static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr), first_col);
+    st = setup_launch(p, o, static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr), first_col, nslots);
     if (st != DASP_OK) return fail(p, st);
     if (p->device >= 0) {
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
@@ -538,7 +567,17 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
         dasp::gather_unit_first_col(static_cast<const int32_t*>(p->d[DASP_ARR_LONG_COL]), f.geo.UG * f.geo.G,
                                     static_cast<int64_t>(first_col.size()), first_col.data(), s) != cudaSuccess)
         return fail(p, DASP_ERR_CUDA);
-    st = setup_launch(p, o, f.panel_table.data(), first_col);
+    std::vector<int32_t> nslots;
+    if (f.nrb > 0) {   // rb_ptr and irr_ptr[8 rb .. 8 rb + 1] back from the device
+        std::vector<int64_t> rbp(static_cast<size_t>(f.nrb + 1)), irr_first(static_cast<size_t>(2 * f.nrb));
+        if (cudaMemcpyAsync(rbp.data(), p->d[DASP_ARR_RB_PTR], rbp.size() * 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+            cudaMemcpy2DAsync(irr_first.data(), 16, p->d[DASP_ARR_IRR_PTR], 64, 16, static_cast<size_t>(f.nrb),
+                              cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+            cudaStreamSynchronize(s) != cudaSuccess)
+            return fail(p, DASP_ERR_CUDA);
+        nslots = narrow_slots(f, rbp.data(), irr_first.data());
+    }
+    st = setup_launch(p, o, f.panel_table.data(), first_col, nslots);
     if (st != DASP_OK) return fail(p, st);
     if ((st = init_cosched(p)) != DASP_OK) return fail(p, st);
     *plan_out = p;

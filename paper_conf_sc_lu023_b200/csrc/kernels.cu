@@ -1129,6 +1129,75 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 
 // ------------------------------------------------------------------------------------------
 // the fused main kernel
+// Narrow row-blocks: the suffix [rbn, nrb) of a panel's sorted row-blocks in which every row
+// fits in two 4-slot quads (max(4 nreg, longest row) <= 8: rows of 5-8 nonzeros, ~40 % of a
+// power-law matrix's medium rows).  The warp-per-row-block path spends three dependent memory
+// round trips (metadata, streams, gathers) on ~0.6 KB there; here one lane owns one row, so a
+// warp works on four row-blocks side by side (lane = 8 q + g: row-block q, row g) and each lane
+// issues its row's two quads in one round: a regular block's row g is 4 contiguous elements at
+// 32 b + 4 g (the block-after-block ragged layout, R18, nreg <= 2 < CW), an irregular quad is the
+// row's tail in irr_val.  CUDA-core arithmetic (FP64 FMA; FP32 storage widened exactly).
+#ifndef DASP_NARROW_RB
+#define DASP_NARROW_RB 8     // row-blocks per narrow warp: 4 side by side x 2 passes
+#endif
+template <int DT>
+__device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
+    using IO = ValIO<DT>;
+    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
+    const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
+    const int g = lane & 7;
+    for (int64_t rq = rbs + (lane >> 3); rq < rbe; rq += 4) {   // no warp collectives below
+        const int64_t i = rq * 8 + g;
+        const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
+        const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 5);
+        const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
+        const int32_t orow = __ldg(P.med_out + i);
+        typename IO::R v[2][4];
+        uint32_t c[2][4];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            if (q < nreg) {
+                IO::ld4r(rv + base + 32 * q + 4 * g, pol, v[q]);
+                ld4_b32(P.reg_col + base + 32 * q + 4 * g, pol, c[q]);
+            } else {
+                const int k0 = 4 * (q - nreg);
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    v[q][e] = 0; c[q][e] = 0xffffffffu;
+                    if (k0 + e < ilen) { v[q][e] = IO::ld1r(iv + ib + k0 + e, pol); c[q][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                }
+            }
+        }
+        double xv[2][4];
+#pragma unroll
+        for (int q = 0; q < 2; ++q)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) xv[q][e] = IO::gx(x, c[q][e]);
+        double acc = 0.0;
+#pragma unroll
+        for (int q = 0; q < 2; ++q)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc = fma(IO::cv(v[q][e]), xv[q][e], acc);
+        store_y<DT>(P, orow, acc);
+    }
+}
+
+// medium warp w of panel D: a wide warp (LOOP_NUM row-blocks, warp per row-block) or a narrow one
+template <int DT, int VAR>
+__device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc* D, int64_t w, int lane, uint64_t pol) {
+    const int64_t rbp0 = __ldg(&D->rb0), nmwd = __ldg(&D->nmwd);
+    if (w < nmwd) {
+        const int64_t rb0 = rbp0 + w * P.rbw;
+        medium_rbs<DT, VAR>(P, rb0, min(rb0 + P.rbw, rbp0 + __ldg(&D->rbn)), lane, pol);
+        return;
+    }
+    const int64_t rb0 = rbp0 + __ldg(&D->rbn) + (w - nmwd) * DASP_NARROW_RB;
+    const int64_t rb1 = min(rb0 + DASP_NARROW_RB, rbp0 + __ldg(&D->nrb));
+    if constexpr (VAR == VAR_CUDACORE && DT != 1) medium_narrow<DT>(P, rb0, rb1, lane, pol);
+    else medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);   // MMA variant: the paper's warp per row-block
+}
+
 // ------------------------------------------------------------------------------------------
 #ifndef DASP_MIN_BLOCKS
 #define DASP_MIN_BLOCKS 4   // caps registers at 64: >= 32 resident warps per SM, no spills
@@ -1189,14 +1258,14 @@ dasp_main_kernel(const MainParams P) {
     const int64_t nmw = __ldg(&D->nmw);
     if (w < nmw) {                                       // medium rows
         if (!(P.class_mask & 2)) return;
+#if DASP_MED_ASYNC
         const int64_t rbp0 = __ldg(&D->rb0);
         const int64_t rb0 = rbp0 + w * P.rbw;
         const int64_t rb1 = min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb));
-#if DASP_MED_ASYNC
         __shared__ __align__(16) uint8_t med_smem[WARPS_PER_BLOCK * 2 * MED_STAGE];
         medium_rbs_async<DT, VAR>(P, rb0, rb1, lane, pol, med_smem + (threadIdx.x >> 5) * 2 * MED_STAGE);
 #else
-        medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);
+        medium_warp<DT, VAR>(P, D, w, lane, pol);
 #endif
         return;
     }
@@ -1230,11 +1299,7 @@ dasp_main_dyn_kernel(const MainParams P, int64_t n_items) {
         const int64_t local = ci - __ldg(P.item_start + q);
         const int64_t nmw = __ldg(&D->nmw);
         if (local < nmw) {
-            if (P.class_mask & 2) {
-                const int64_t rbp0 = __ldg(&D->rb0);
-                const int64_t rb0 = rbp0 + local * P.rbw;
-                medium_rbs<DT, VAR>(P, rb0, min(rb0 + P.rbw, rbp0 + __ldg(&D->nrb)), lane, pol);
-            }
+            if (P.class_mask & 2) medium_warp<DT, VAR>(P, D, local, lane, pol);
         } else {
             short_item<DT, VAR>(P, D, local - nmw, lane, pol);
         }
@@ -1825,6 +1890,7 @@ __global__ void __launch_bounds__(256) dasp_long_meta_kernel(const int64_t* __re
 }  // namespace
 
 int short_tiles_per_warp(int dtype) { return DASP_BY_DT(dtype, DASP_SHORT_TPW); }
+int narrow_rb_per_warp(int dtype) { return (dtype == 1 || DASP_MED_ASYNC) ? 0 : DASP_NARROW_RB; }
 
 cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,
                              cudaStream_t s) {
