@@ -265,7 +265,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         d.unit0 = e[2]; d.nunits = e[3]; d.rb0 = e[4]; d.nrb = e[5];
         d.rbn = d.nrb;
         if (nrw > 0)
-            while (d.rbn > 0 && nslots[d.rb0 + d.rbn - 1] <= dasp::narrow_max_slots()) --d.rbn;
+            while (d.rbn > 0 && nslots[d.rb0 + d.rbn - 1] <= dasp::narrow_max_slots(f.geo.K)) --d.rbn;
         d.nmwd = (d.rbn + p->rbw - 1) / p->rbw;
         d.nmw = d.nmwd + (nrw > 0 ? (d.nrb - d.rbn + nrw - 1) / nrw : 0);
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];

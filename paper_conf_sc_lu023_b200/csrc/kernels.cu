@@ -1130,7 +1130,7 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 // ------------------------------------------------------------------------------------------
 // the fused main kernel
 // Narrow row-blocks: the suffix [rbn, nrb) of a panel's sorted row-blocks in which every row
-// fits in two 4-slot quads (max(4 nreg, longest row) <= 8: rows of 5-8 nonzeros, ~40 % of a
+// fits in two K-slot groups (max(K nreg, longest row) <= 2K; FP64/FP32 K = 4: rows of 5-8 nonzeros, ~40 % of a
 // power-law matrix's medium rows).  The warp-per-row-block path spends three dependent memory
 // round trips (metadata, streams, gathers) on ~0.6 KB there; here one lane owns one row, so a
 // warp works on four row-blocks side by side (lane = 8 q + g: row-block q, row g) and each lane
@@ -1183,6 +1183,55 @@ __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t rbs, 
     }
 }
 
+// FP16 (8 x 8 blocks, K = 8): narrow rows span <= 16 slots = two octets; a regular block's row g
+// is 8 contiguous halves at 64 b + 8 g (16-B value and 32-B column loads), FP32 accumulation.
+__device__ __forceinline__ void medium_narrow_f16(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
+    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
+    const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    const int g = lane & 7;
+    for (int64_t rq = rbs + (lane >> 3); rq < rbe; rq += 4) {
+        const int64_t i = rq * 8 + g;
+        const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
+        const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 6);
+        const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
+        const int32_t orow = __ldg(P.med_out + i);
+        uint32_t v[2][4], c[2][8];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            if (q < nreg) {
+                ld4_b32(rv + base + 64 * q + 8 * g, pol, v[q]);
+                ld8_b32(P.reg_col + base + 64 * q + 8 * g, pol, c[q]);
+            } else {
+                const int k0 = 8 * (q - nreg);
+#pragma unroll
+                for (int e = 0; e < 8; e += 2) {
+                    uint32_t lo = 0, hi = 0;
+                    c[q][e] = c[q][e + 1] = 0xffffffffu;
+                    if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); c[q][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                    if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); c[q][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
+                    v[q][e >> 1] = lo | (hi << 16);
+                }
+            }
+        }
+        uint16_t xh[2][8];
+#pragma unroll
+        for (int q = 0; q < 2; ++q)
+#pragma unroll
+            for (int e = 0; e < 8; ++e) xh[q][e] = gxh(x, c[q][e]);
+        float acc = 0.f;
+#pragma unroll
+        for (int q = 0; q < 2; ++q)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const float2 av = u2f2(v[q][j]);
+                acc = fmaf(av.x, h2f(xh[q][2 * j]), acc);
+                acc = fmaf(av.y, h2f(xh[q][2 * j + 1]), acc);
+            }
+        store_y<1>(P, orow, acc);
+    }
+}
+
 // medium warp w of panel D: a wide warp (LOOP_NUM row-blocks, warp per row-block) or a narrow one
 template <int DT, int VAR>
 __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc* D, int64_t w, int lane, uint64_t pol) {
@@ -1194,7 +1243,8 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
     }
     const int64_t rb0 = rbp0 + __ldg(&D->rbn) + (w - nmwd) * DASP_NARROW_RB;
     const int64_t rb1 = min(rb0 + DASP_NARROW_RB, rbp0 + __ldg(&D->nrb));
-    if constexpr (VAR == VAR_CUDACORE && DT != 1) medium_narrow<DT>(P, rb0, rb1, lane, pol);
+    if constexpr (VAR == VAR_CUDACORE && DT == 1) medium_narrow_f16(P, rb0, rb1, lane, pol);
+    else if constexpr (VAR == VAR_CUDACORE) medium_narrow<DT>(P, rb0, rb1, lane, pol);
     else medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);   // MMA variant: the paper's warp per row-block
 }
 
@@ -1890,7 +1940,10 @@ __global__ void __launch_bounds__(256) dasp_long_meta_kernel(const int64_t* __re
 }  // namespace
 
 int short_tiles_per_warp(int dtype) { return DASP_BY_DT(dtype, DASP_SHORT_TPW); }
-int narrow_rb_per_warp(int dtype) { return (dtype == 1 || DASP_MED_ASYNC) ? 0 : DASP_NARROW_RB; }
+#ifndef DASP_NARROW_F16
+#define DASP_NARROW_F16 1
+#endif
+int narrow_rb_per_warp(int dtype) { return (DASP_MED_ASYNC || (dtype == 1 && !DASP_NARROW_F16)) ? 0 : DASP_NARROW_RB; }
 
 cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,
                              cudaStream_t s) {

@@ -97,10 +97,10 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
 // short tiles one main-kernel warp processes (build knob DASP_SHORT_TPW)
 int short_tiles_per_warp(int dtype);
-// narrow medium row-blocks (rows of at most narrow_max_slots() slots: max(K*nreg, longest row)):
-// row-blocks one narrow warp processes, 0 = no narrow path for this dtype
+// narrow medium row-blocks (rows of at most narrow_max_slots(K) = 2K slots: max(K*nreg, longest
+// row)): row-blocks one narrow warp processes, 0 = no narrow path for this dtype
 int narrow_rb_per_warp(int dtype);
-constexpr int narrow_max_slots() { return 8; }
+constexpr int narrow_max_slots(int K) { return 2 * K; }
 // co-scheduled mode metadata from group_ptr: long_cnt[r] = groups of row r, group_row[g] = row
 // (group_row must be pre-filled with -1 for the pad groups)
 cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,
