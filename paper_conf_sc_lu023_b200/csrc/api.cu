@@ -244,6 +244,11 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         const char* ne = std::getenv("DASP_NARROW");   // 0 = every row-block on the wide path (experiments)
         if ((ne && std::atoi(ne) == 0) || static_cast<int64_t>(nslots.size()) != f.nrb) nrw = 0;
     }
+    bool mid = true;   // two-lanes-per-row narrow warps (DASP_NARROW_MID=0: off, experiments)
+    {
+        const char* me = std::getenv("DASP_NARROW_MID");
+        if (me && std::atoi(me) == 0) mid = false;
+    }
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<uint64_t> blk_word;
     std::vector<uint64_t> tile_meta;
@@ -266,8 +271,12 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         d.rbn = d.nrb;
         if (nrw > 0)
             while (d.rbn > 0 && nslots[d.rb0 + d.rbn - 1] <= dasp::narrow_max_slots(f.geo.K)) --d.rbn;
-        d.nmwd = (d.rbn + p->rbw - 1) / p->rbw;
-        d.nmw = d.nmwd + (nrw > 0 ? (d.nrb - d.rbn + nrw - 1) / nrw : 0);
+        d.rbm = d.rbn;
+        if (nrw > 0 && mid)
+            while (d.rbm > 0 && nslots[d.rb0 + d.rbm - 1] <= dasp::mid_max_slots(f.geo.K)) --d.rbm;
+        d.nmwd = (d.rbm + p->rbw - 1) / p->rbw;
+        d.nmwm = d.nmwd + (nrw > 0 ? (d.rbn - d.rbm + nrw - 1) / nrw : 0);
+        d.nmw = d.nmwm + (nrw > 0 ? (d.nrb - d.rbn + nrw - 1) / nrw : 0);
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
         if (p->split_short) {   // tiles leave the main kernel; per-tile metadata for the short kernel
             for (int64_t t = 0; t < d.t13 + d.t4 + d.t22 + d.ts; ++t) {

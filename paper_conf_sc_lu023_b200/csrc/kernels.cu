@@ -1140,112 +1140,144 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 #ifndef DASP_NARROW_RB
 #define DASP_NARROW_RB 8     // row-blocks per narrow warp: 4 side by side x 2 passes
 #endif
-template <int DT>
+template <int DT, int LPR>
 __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
     using IO = ValIO<DT>;
+    constexpr int SIDE = 4 / LPR;                        // row-blocks side by side
     const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
     const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
     const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
-    const int g = lane & 7;
-    for (int64_t rq = rbs + (lane >> 3); rq < rbe; rq += 4) {   // no warp collectives below
-        const int64_t i = rq * 8 + g;
-        const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
-        const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 5);
-        const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
-        const int32_t orow = __ldg(P.med_out + i);
-        typename IO::R v[2][4];
-        uint32_t c[2][4];
+    const int g = (lane / LPR) & 7, sub = lane % LPR;     // row g of row-block lane / (8 LPR); quads 2 sub, 2 sub + 1
+    const int64_t passes = (rbe - rbs + SIDE - 1) / SIDE;
+    for (int64_t ps = 0; ps < passes; ++ps) {            // warp-uniform trip count (LPR > 1 shuffles)
+        const int64_t rq = rbs + ps * SIDE + lane / (8 * LPR);
+        const bool act = rq < rbe;
+        double acc = 0.0;
+        int32_t orow = -1;
+        if (act) {
+            const int64_t i = rq * 8 + g;
+            const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
+            const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 5);
+            const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
+            orow = __ldg(P.med_out + i);
+            typename IO::R v[2][4];
+            uint32_t c[2][4];
 #pragma unroll
-        for (int q = 0; q < 2; ++q) {
-            if (q < nreg) {
-                IO::ld4r(rv + base + 32 * q + 4 * g, pol, v[q]);
-                ld4_b32(P.reg_col + base + 32 * q + 4 * g, pol, c[q]);
-            } else {
-                const int k0 = 4 * (q - nreg);
+            for (int h = 0; h < 2; ++h) {
+                const int q = 2 * sub + h;
+                if (q < nreg) {   // nreg = 4 (mid rows only): one full lane-interleaved chunk, row g at 16 g
+                    const int64_t off = base + (nreg >= 4 ? 16 * g + 8 * sub + 4 * h : 32 * q + 4 * g);
+                    IO::ld4r(rv + off, pol, v[h]);
+                    ld4_b32(P.reg_col + off, pol, c[h]);
+                } else {
+                    const int k0 = 4 * (q - nreg);
 #pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                    v[q][e] = 0; c[q][e] = 0xffffffffu;
-                    if (k0 + e < ilen) { v[q][e] = IO::ld1r(iv + ib + k0 + e, pol); c[q][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                    for (int e = 0; e < 4; ++e) {
+                        v[h][e] = 0; c[h][e] = 0xffffffffu;
+                        if (k0 + e < ilen) { v[h][e] = IO::ld1r(iv + ib + k0 + e, pol); c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                    }
                 }
             }
+            double xv[2][4];
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+                for (int e = 0; e < 4; ++e) xv[h][e] = IO::gx(x, c[h][e]);
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+                for (int e = 0; e < 4; ++e) acc = fma(IO::cv(v[h][e]), xv[h][e], acc);
         }
-        double xv[2][4];
-#pragma unroll
-        for (int q = 0; q < 2; ++q)
-#pragma unroll
-            for (int e = 0; e < 4; ++e) xv[q][e] = IO::gx(x, c[q][e]);
-        double acc = 0.0;
-#pragma unroll
-        for (int q = 0; q < 2; ++q)
-#pragma unroll
-            for (int e = 0; e < 4; ++e) acc = fma(IO::cv(v[q][e]), xv[q][e], acc);
-        store_y<DT>(P, orow, acc);
+        if constexpr (LPR == 2) acc += __shfl_xor_sync(FULL, acc, 1);
+        if (sub == 0) store_y<DT>(P, orow, acc);         // orow -1 (inactive / virtual row): no store
     }
 }
 
-// FP16 (8 x 8 blocks, K = 8): narrow rows span <= 16 slots = two octets; a regular block's row g
-// is 8 contiguous halves at 64 b + 8 g (16-B value and 32-B column loads), FP32 accumulation.
+// FP16 (8 x 8 blocks, K = 8): narrow rows span <= 16 LPR slots = two octets per lane; a regular
+// block's row g is 8 contiguous halves at 64 b + 8 g (16-B value and 32-B column loads), FP32
+// accumulation.
+template <int LPR>
 __device__ __forceinline__ void medium_narrow_f16(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
+    constexpr int SIDE = 4 / LPR;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
     const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
-    const int g = lane & 7;
-    for (int64_t rq = rbs + (lane >> 3); rq < rbe; rq += 4) {
-        const int64_t i = rq * 8 + g;
-        const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
-        const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 6);
-        const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
-        const int32_t orow = __ldg(P.med_out + i);
-        uint32_t v[2][4], c[2][8];
+    const int g = (lane / LPR) & 7, sub = lane % LPR;
+    const int64_t passes = (rbe - rbs + SIDE - 1) / SIDE;
+    for (int64_t ps = 0; ps < passes; ++ps) {
+        const int64_t rq = rbs + ps * SIDE + lane / (8 * LPR);
+        const bool act = rq < rbe;
+        float acc = 0.f;
+        int32_t orow = -1;
+        if (act) {
+            const int64_t i = rq * 8 + g;
+            const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
+            const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 6);
+            const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
+            orow = __ldg(P.med_out + i);
+            uint32_t v[2][4], c[2][8];
 #pragma unroll
-        for (int q = 0; q < 2; ++q) {
-            if (q < nreg) {
-                ld4_b32(rv + base + 64 * q + 8 * g, pol, v[q]);
-                ld8_b32(P.reg_col + base + 64 * q + 8 * g, pol, c[q]);
-            } else {
-                const int k0 = 8 * (q - nreg);
+            for (int h = 0; h < 2; ++h) {
+                const int q = 2 * sub + h;
+                if (q < nreg) {   // nreg = 4 (mid rows only): one full lane-interleaved chunk, row g at 32 g
+                    const int64_t off = base + (nreg >= 4 ? 32 * g + 16 * sub + 8 * h : 64 * q + 8 * g);
+                    ld4_b32(rv + off, pol, v[h]);
+                    ld8_b32(P.reg_col + off, pol, c[h]);
+                } else {
+                    const int k0 = 8 * (q - nreg);
 #pragma unroll
-                for (int e = 0; e < 8; e += 2) {
-                    uint32_t lo = 0, hi = 0;
-                    c[q][e] = c[q][e + 1] = 0xffffffffu;
-                    if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); c[q][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
-                    if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); c[q][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
-                    v[q][e >> 1] = lo | (hi << 16);
+                    for (int e = 0; e < 8; e += 2) {
+                        uint32_t lo = 0, hi = 0;
+                        c[h][e] = c[h][e + 1] = 0xffffffffu;
+                        if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                        if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); c[h][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
+                        v[h][e >> 1] = lo | (hi << 16);
+                    }
                 }
             }
+            uint16_t xh[2][8];
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+                for (int e = 0; e < 8; ++e) xh[h][e] = gxh(x, c[h][e]);
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const float2 av = u2f2(v[h][j]);
+                    acc = fmaf(av.x, h2f(xh[h][2 * j]), acc);
+                    acc = fmaf(av.y, h2f(xh[h][2 * j + 1]), acc);
+                }
         }
-        uint16_t xh[2][8];
-#pragma unroll
-        for (int q = 0; q < 2; ++q)
-#pragma unroll
-            for (int e = 0; e < 8; ++e) xh[q][e] = gxh(x, c[q][e]);
-        float acc = 0.f;
-#pragma unroll
-        for (int q = 0; q < 2; ++q)
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const float2 av = u2f2(v[q][j]);
-                acc = fmaf(av.x, h2f(xh[q][2 * j]), acc);
-                acc = fmaf(av.y, h2f(xh[q][2 * j + 1]), acc);
-            }
-        store_y<1>(P, orow, acc);
+        if constexpr (LPR == 2) acc += __shfl_xor_sync(FULL, acc, 1);
+        if (sub == 0) store_y<1>(P, orow, acc);
     }
 }
 
-// medium warp w of panel D: a wide warp (LOOP_NUM row-blocks, warp per row-block) or a narrow one
+// medium warp w of panel D: a wide warp (LOOP_NUM row-blocks, warp per row-block), a mid narrow
+// warp (two lanes per row: rows spanning <= 4K slots) or a narrow one (a lane per row: <= 2K)
 template <int DT, int VAR>
 __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc* D, int64_t w, int lane, uint64_t pol) {
     const int64_t rbp0 = __ldg(&D->rb0), nmwd = __ldg(&D->nmwd);
     if (w < nmwd) {
         const int64_t rb0 = rbp0 + w * P.rbw;
-        medium_rbs<DT, VAR>(P, rb0, min(rb0 + P.rbw, rbp0 + __ldg(&D->rbn)), lane, pol);
+        medium_rbs<DT, VAR>(P, rb0, min(rb0 + P.rbw, rbp0 + __ldg(&D->rbm)), lane, pol);
         return;
     }
-    const int64_t rb0 = rbp0 + __ldg(&D->rbn) + (w - nmwd) * DASP_NARROW_RB;
-    const int64_t rb1 = min(rb0 + DASP_NARROW_RB, rbp0 + __ldg(&D->nrb));
-    if constexpr (VAR == VAR_CUDACORE && DT == 1) medium_narrow_f16(P, rb0, rb1, lane, pol);
-    else if constexpr (VAR == VAR_CUDACORE) medium_narrow<DT>(P, rb0, rb1, lane, pol);
-    else medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);   // MMA variant: the paper's warp per row-block
+    const int64_t nmwm = __ldg(&D->nmwm);
+    const bool mid = w < nmwm;
+    const int64_t rb0 = mid ? rbp0 + __ldg(&D->rbm) + (w - nmwd) * DASP_NARROW_RB
+                            : rbp0 + __ldg(&D->rbn) + (w - nmwm) * DASP_NARROW_RB;
+    const int64_t rb1 = min(rb0 + DASP_NARROW_RB, rbp0 + (mid ? __ldg(&D->rbn) : __ldg(&D->nrb)));
+    if constexpr (VAR == VAR_CUDACORE && DT == 1) {
+        if (mid) medium_narrow_f16<2>(P, rb0, rb1, lane, pol);
+        else medium_narrow_f16<1>(P, rb0, rb1, lane, pol);
+    } else if constexpr (VAR == VAR_CUDACORE) {
+        if (mid) medium_narrow<DT, 2>(P, rb0, rb1, lane, pol);
+        else medium_narrow<DT, 1>(P, rb0, rb1, lane, pol);
+    } else {
+        medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);   // MMA variant: the paper's warp per row-block
+    }
 }
 
 // ------------------------------------------------------------------------------------------

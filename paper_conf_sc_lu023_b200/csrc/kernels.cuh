@@ -19,10 +19,11 @@ struct ExtraDst {
 constexpr int WARPS_PER_BLOCK = MAIN_THREADS / 32;
 
 // One row panel (R28) as the medium/short kernel sees it.  Its main warps are, in
-// order: nmw medium warps -- nmwd of them over the row-blocks [0, rbn) with rbw row-blocks each
-// (Alg. 3, LOOP_NUM P:L271), then nmw - nmwd narrow warps over the row-blocks [rbn, nrb) whose
-// rows all fit in 2K slots, narrow_rb_per_warp() each (one lane per row) -- then one warp per
-// short tile (1&3 | len4 | 2&2 | singles).  Its long units (unit0, nunits) run either in their own kernel
+// order: nmw medium warps -- nmwd of them over the row-blocks [0, rbm) with rbw row-blocks each
+// (Alg. 3, LOOP_NUM P:L271), nmwm - nmwd mid narrow warps over [rbm, rbn) whose rows all fit in
+// 4K slots (two lanes per row), nmw - nmwm narrow warps over [rbn, nrb) whose rows fit in 2K
+// slots (one lane per row), narrow_rb_per_warp() row-blocks each -- then one warp per short tile
+// (1&3 | len4 | 2&2 | singles).  Its long units (unit0, nunits) run either in their own kernel
 // (dasp_long_kernel) or, co-scheduled, as long blocks of the main kernel interleaved with the
 // panel's main blocks (MainParams::blk_word).
 struct PanelDesc {
@@ -30,7 +31,7 @@ struct PanelDesc {
     int64_t unit0, nunits;
     int64_t rb0, nrb, nmw;
     int64_t tile0, t13, t4, t22, ts, out0;
-    int64_t rbn, nmwd;
+    int64_t rbm, rbn, nmwd, nmwm;
 };
 
 // Everything the fused main kernel reads.
@@ -101,6 +102,7 @@ int short_tiles_per_warp(int dtype);
 // row)): row-blocks one narrow warp processes, 0 = no narrow path for this dtype
 int narrow_rb_per_warp(int dtype);
 constexpr int narrow_max_slots(int K) { return 2 * K; }
+constexpr int mid_max_slots(int K) { return 4 * K; }
 // co-scheduled mode metadata from group_ptr: long_cnt[r] = groups of row r, group_row[g] = row
 // (group_row must be pre-filled with -1 for the pad groups)
 cudaError_t launch_long_meta(const int64_t* group_ptr, int64_t row_long, int32_t* long_cnt, int32_t* group_row,

@@ -220,6 +220,38 @@ def test_spmv_host_end_to_end():
     assert oracle.tolerance_ok(y, y_ref, s).all()
 
 
+NARROW_LENS = {
+    "len5-8": list(range(5, 9)),          # FP64/FP32 narrow (one lane per row); FP16 narrow
+    "len9-16": list(range(9, 17)),        # FP64/FP32 mid (two lanes per row), nreg up to 4 (full chunk)
+    "len13-16": list(range(13, 17)),      # every row-block nreg = 4 in FP64/FP32
+    "len17-32": list(range(17, 33)),      # FP16 mid, nreg up to 4; FP64/FP32 wide
+    "len29-32": list(range(29, 33)),      # FP16 nreg = 4 (full chunk)
+    "mixed": list(range(5, 40)) + [0, 1, 2, 3, 4, 300],
+}
+
+
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("name", list(NARROW_LENS))
+@pytest.mark.parametrize("narrow", ["1", "0"])
+def test_narrow_medium_paths(dt, name, narrow, monkeypatch):
+    """Narrow / mid medium row-blocks (a lane or two lanes per row) vs the oracle, and the same
+    plan built with DASP_NARROW=0 (every row-block on the warp-per-row-block path)."""
+    monkeypatch.setenv("DASP_NARROW", narrow)
+    rng = np.random.default_rng(len(name))
+    lens = list(rng.choice(NARROW_LENS[name], size=3001))          # ragged: 375 row-blocks + 1 row
+    A = synth.from_lengths(lens, n=5000, seed=11)
+    x = synth.vector(3, A.n)
+    y_ref, s = oracle_ref(A, x, dt)
+    for variant in VARIANTS:
+        plan = make(A, dt)
+        y = run(plan, x, dt, variant=variant)
+        assert oracle.tolerance_ok(y, y_ref, s, dt).all(), (VNAME[variant], int((~oracle.tolerance_ok(y, y_ref, s, dt)).sum()))
+        y0 = synth.vector(4, A.m)
+        y = run(plan, x, dt, 2.0, -0.5, y0, variant=variant)
+        y_ref2, s2 = oracle_ref(A, x, dt, 2.0, -0.5, y0)
+        assert oracle.tolerance_ok(y, y_ref2, s2, dt).all()
+
+
 @pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("beta", [0.0, -0.5])
 def test_spmv_host_stream_pipelined(dt, beta):
