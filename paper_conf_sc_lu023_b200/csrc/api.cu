@@ -417,6 +417,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
             if (lim > 0 && win > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim) == cudaSuccess) {
                 p->apw_bytes = win;
                 p->apw_hit = std::min(1.0f, static_cast<float>(lim) / static_cast<float>(win));
+                if (const char* h = std::getenv("DASP_X_APW_HIT")) p->apw_hit = static_cast<float>(std::atof(h));
             }
         }
         cudaGetLastError();
@@ -670,7 +671,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
         if (c >= 1 && c <= 3) mp.class_mask = 1 << (c - 1);
     }
     if (!p->pipe && !p->cosched && p->n_units > 0 && (mp.class_mask & 1)) {
-        e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s); });
+        e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s, x, p->apw_bytes, p->apw_hit); });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }
     if (!p->pipe && p->split_short && p->n_tiles > 0 && (mp.class_mask & 4)) {

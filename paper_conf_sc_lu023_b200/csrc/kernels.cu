@@ -1140,117 +1140,156 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 #ifndef DASP_NARROW_RB
 #define DASP_NARROW_RB 8     // row-blocks per narrow warp: 4 side by side x 2 passes
 #endif
-template <int DT, int LPR>
-__device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
-    using IO = ValIO<DT>;
-    constexpr int SIDE = 4 / LPR;                        // row-blocks side by side
-    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
-    const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
-    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
-    const int g = (lane / LPR) & 7, sub = lane % LPR;     // row g of row-block lane / (8 LPR); quads 2 sub, 2 sub + 1
-    const int64_t passes = (rbe - rbs + SIDE - 1) / SIDE;
-    for (int64_t ps = 0; ps < passes; ++ps) {            // warp-uniform trip count (LPR > 1 shuffles)
-        const int64_t rq = rbs + ps * SIDE + lane / (8 * LPR);
-        const bool act = rq < rbe;
-        double acc = 0.0;
-        int32_t orow = -1;
-        if (act) {
-            const int64_t i = rq * 8 + g;
-            const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
-            const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 5);
-            const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
-            orow = __ldg(P.med_out + i);
-            typename IO::R v[2][4];
-            uint32_t c[2][4];
+// 1: the next pass's stream loads are issued before this pass's gathers.  Measured
+// (profiles/r01d/narrow_pipe.jsonl): FP16 C3 main kernel -3 %, stencils -1 %; FP64 +6 % (spills at
+// 64 registers), FP32 neutral -- so FP16 only.
+#ifndef DASP_NARROW_PIPE_F64
+#define DASP_NARROW_PIPE_F64 0
+#endif
+#ifndef DASP_NARROW_PIPE_F16
+#define DASP_NARROW_PIPE_F16 1
+#endif
+#ifndef DASP_NARROW_PIPE_F32
+#define DASP_NARROW_PIPE_F32 0
+#endif
+template <int DT> struct NarLd {                   // one pass of one lane: two K-slot groups
+    typename ValIO<DT>::R v[2][4];
+    uint32_t c[2][4];
+    int32_t orow;
+};
+template <> struct NarLd<1> {                      // FP16: two octets
+    uint32_t v[2][4];
+    uint32_t c[2][8];
+    int32_t orow;
+};
+// stream loads of row g of row-block rq (rq < rbe) for this lane's groups 2 sub, 2 sub + 1
+template <int DT>
+__device__ __forceinline__ void narrow_load(const MainParams& P, int64_t rq, bool act, int g, int sub, uint64_t pol,
+                                            NarLd<DT>& L) {
+    L.orow = -1;
+    if (!act) {
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int q = 2 * sub + h;
-                if (q < nreg) {   // nreg = 4 (mid rows only): one full lane-interleaved chunk, row g at 16 g
-                    const int64_t off = base + (nreg >= 4 ? 16 * g + 8 * sub + 4 * h : 32 * q + 4 * g);
-                    IO::ld4r(rv + off, pol, v[h]);
-                    ld4_b32(P.reg_col + off, pol, c[h]);
-                } else {
-                    const int k0 = 4 * (q - nreg);
+        for (int h = 0; h < 2; ++h) {
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) {
-                        v[h][e] = 0; c[h][e] = 0xffffffffu;
-                        if (k0 + e < ilen) { v[h][e] = IO::ld1r(iv + ib + k0 + e, pol); c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
-                    }
+            for (int e = 0; e < (DT == 1 ? 4 : 4); ++e) L.v[h][e] = 0;
+#pragma unroll
+            for (int e = 0; e < (DT == 1 ? 8 : 4); ++e) L.c[h][e] = 0xffffffffu;
+        }
+        return;
+    }
+    const int64_t i = rq * 8 + g;
+    const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
+    const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
+    L.orow = __ldg(P.med_out + i);
+    if constexpr (DT == 1) {
+        const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
+        const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
+        const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 6);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int q = 2 * sub + h;
+            if (q < nreg) {   // nreg = 4 (mid rows only): one full lane-interleaved chunk, row g at 32 g
+                const int64_t off = base + (nreg >= 4 ? 32 * g + 16 * sub + 8 * h : 64 * q + 8 * g);
+                ld4_b32(rv + off, pol, L.v[h]);
+                ld8_b32(P.reg_col + off, pol, L.c[h]);
+            } else {
+                const int k0 = 8 * (q - nreg);
+#pragma unroll
+                for (int e = 0; e < 8; e += 2) {
+                    uint32_t lo = 0, hi = 0;
+                    L.c[h][e] = L.c[h][e + 1] = 0xffffffffu;
+                    if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); L.c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                    if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); L.c[h][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
+                    L.v[h][e >> 1] = lo | (hi << 16);
                 }
             }
-            double xv[2][4];
-#pragma unroll
-            for (int h = 0; h < 2; ++h)
-#pragma unroll
-                for (int e = 0; e < 4; ++e) xv[h][e] = IO::gx(x, c[h][e]);
-#pragma unroll
-            for (int h = 0; h < 2; ++h)
-#pragma unroll
-                for (int e = 0; e < 4; ++e) acc = fma(IO::cv(v[h][e]), xv[h][e], acc);
         }
-        if constexpr (LPR == 2) acc += __shfl_xor_sync(FULL, acc, 1);
-        if (sub == 0) store_y<DT>(P, orow, acc);         // orow -1 (inactive / virtual row): no store
+    } else {
+        using IO = ValIO<DT>;
+        const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
+        const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+        const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 5);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int q = 2 * sub + h;
+            if (q < nreg) {   // nreg = 4 (mid rows only): one full lane-interleaved chunk, row g at 16 g
+                const int64_t off = base + (nreg >= 4 ? 16 * g + 8 * sub + 4 * h : 32 * q + 4 * g);
+                IO::ld4r(rv + off, pol, L.v[h]);
+                ld4_b32(P.reg_col + off, pol, L.c[h]);
+            } else {
+                const int k0 = 4 * (q - nreg);
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    L.v[h][e] = 0; L.c[h][e] = 0xffffffffu;
+                    if (k0 + e < ilen) { L.v[h][e] = IO::ld1r(iv + ib + k0 + e, pol); L.c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                }
+            }
+        }
     }
 }
-
-// FP16 (8 x 8 blocks, K = 8): narrow rows span <= 16 LPR slots = two octets per lane; a regular
-// block's row g is 8 contiguous halves at 64 b + 8 g (16-B value and 32-B column loads), FP32
-// accumulation.
-template <int LPR>
-__device__ __forceinline__ void medium_narrow_f16(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
-    constexpr int SIDE = 4 / LPR;
-    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
-    const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
-    const uint16_t* x = static_cast<const uint16_t*>(P.x);
-    const int g = (lane / LPR) & 7, sub = lane % LPR;
-    const int64_t passes = (rbe - rbs + SIDE - 1) / SIDE;
-    for (int64_t ps = 0; ps < passes; ++ps) {
-        const int64_t rq = rbs + ps * SIDE + lane / (8 * LPR);
-        const bool act = rq < rbe;
+// gathers, the row's dot product (fixed order), the LPR-lane sum and the y store
+template <int DT, int LPR>
+__device__ __forceinline__ void narrow_finish(const MainParams& P, const NarLd<DT>& L, int sub) {
+    if constexpr (DT == 1) {
+        const uint16_t* x = static_cast<const uint16_t*>(P.x);
+        uint16_t xh[2][8];
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+            for (int e = 0; e < 8; ++e) xh[h][e] = gxh(x, L.c[h][e]);
         float acc = 0.f;
-        int32_t orow = -1;
-        if (act) {
-            const int64_t i = rq * 8 + g;
-            const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
-            const int nreg = static_cast<int>((__ldg(P.rb_ptr + rq + 1) - base) >> 6);
-            const int ilen = static_cast<int>(__ldg(P.irr_ptr + i + 1) - ib);
-            orow = __ldg(P.med_out + i);
-            uint32_t v[2][4], c[2][8];
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int q = 2 * sub + h;
-                if (q < nreg) {   // nreg = 4 (mid rows only): one full lane-interleaved chunk, row g at 32 g
-                    const int64_t off = base + (nreg >= 4 ? 32 * g + 16 * sub + 8 * h : 64 * q + 8 * g);
-                    ld4_b32(rv + off, pol, v[h]);
-                    ld8_b32(P.reg_col + off, pol, c[h]);
-                } else {
-                    const int k0 = 8 * (q - nreg);
+        for (int h = 0; h < 2; ++h)
 #pragma unroll
-                    for (int e = 0; e < 8; e += 2) {
-                        uint32_t lo = 0, hi = 0;
-                        c[h][e] = c[h][e + 1] = 0xffffffffu;
-                        if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
-                        if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); c[h][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
-                        v[h][e >> 1] = lo | (hi << 16);
-                    }
-                }
+            for (int j = 0; j < 4; ++j) {
+                const float2 av = u2f2(L.v[h][j]);
+                acc = fmaf(av.x, h2f(xh[h][2 * j]), acc);
+                acc = fmaf(av.y, h2f(xh[h][2 * j + 1]), acc);
             }
-            uint16_t xh[2][8];
-#pragma unroll
-            for (int h = 0; h < 2; ++h)
-#pragma unroll
-                for (int e = 0; e < 8; ++e) xh[h][e] = gxh(x, c[h][e]);
-#pragma unroll
-            for (int h = 0; h < 2; ++h)
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    const float2 av = u2f2(v[h][j]);
-                    acc = fmaf(av.x, h2f(xh[h][2 * j]), acc);
-                    acc = fmaf(av.y, h2f(xh[h][2 * j + 1]), acc);
-                }
-        }
         if constexpr (LPR == 2) acc += __shfl_xor_sync(FULL, acc, 1);
-        if (sub == 0) store_y<1>(P, orow, acc);
+        if (sub == 0) store_y<1>(P, L.orow, acc);        // orow -1 (inactive / virtual row): no store
+    } else {
+        using IO = ValIO<DT>;
+        const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
+        double xv[2][4];
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) xv[h][e] = IO::gx(x, L.c[h][e]);
+        double acc = 0.0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc = fma(IO::cv(L.v[h][e]), xv[h][e], acc);
+        if constexpr (LPR == 2) acc += __shfl_xor_sync(FULL, acc, 1);
+        if (sub == 0) store_y<DT>(P, L.orow, acc);
+    }
+}
+// LPR lanes per row (1: rows spanning <= 2K slots, 4 row-blocks side by side; 2: <= 4K, 2 side
+// by side), passes over [rbs, rbe) with a warp-uniform trip count (the LPR = 2 shuffle)
+template <int DT, int LPR>
+__device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
+    constexpr int SIDE = 4 / LPR;
+    const int g = (lane / LPR) & 7, sub = lane % LPR;
+    const int64_t r0 = rbs + lane / (8 * LPR);
+    const int64_t passes = (rbe - rbs + SIDE - 1) / SIDE;
+    if constexpr (DASP_BY_DT(DT, DASP_NARROW_PIPE) != 0) {
+        NarLd<DT> A;
+        narrow_load<DT>(P, r0, r0 < rbe, g, sub, pol, A);
+        for (int64_t ps = 0; ps < passes; ++ps) {
+            NarLd<DT> B;
+            const int64_t rn = r0 + (ps + 1) * SIDE;
+            narrow_load<DT>(P, rn, rn < rbe, g, sub, pol, B);
+            narrow_finish<DT, LPR>(P, A, sub);
+            A = B;
+        }
+    } else {
+        for (int64_t ps = 0; ps < passes; ++ps) {
+            NarLd<DT> A;
+            const int64_t rq = r0 + ps * SIDE;
+            narrow_load<DT>(P, rq, rq < rbe, g, sub, pol, A);
+            narrow_finish<DT, LPR>(P, A, sub);
+        }
     }
 }
 
@@ -1269,10 +1308,7 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
     const int64_t rb0 = mid ? rbp0 + __ldg(&D->rbm) + (w - nmwd) * DASP_NARROW_RB
                             : rbp0 + __ldg(&D->rbn) + (w - nmwm) * DASP_NARROW_RB;
     const int64_t rb1 = min(rb0 + DASP_NARROW_RB, rbp0 + (mid ? __ldg(&D->rbn) : __ldg(&D->nrb)));
-    if constexpr (VAR == VAR_CUDACORE && DT == 1) {
-        if (mid) medium_narrow_f16<2>(P, rb0, rb1, lane, pol);
-        else medium_narrow_f16<1>(P, rb0, rb1, lane, pol);
-    } else if constexpr (VAR == VAR_CUDACORE) {
+    if constexpr (VAR == VAR_CUDACORE) {
         if (mid) medium_narrow<DT, 2>(P, rb0, rb1, lane, pol);
         else medium_narrow<DT, 1>(P, rb0, rb1, lane, pol);
     } else {
@@ -1937,9 +1973,9 @@ __global__ void __launch_bounds__(256) dasp_gather_kernel(const W* __restrict__ 
 
 }  // namespace
 
-template <typename Kern>
+template <typename Kern, typename... Args>
 static cudaError_t launch_ex(Kern kernel, unsigned blocks, cudaStream_t s, const void* apw_base, size_t apw_bytes,
-                             float apw_hit, const MainParams& p) {
+                             float apw_hit, Args... args) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(blocks);
     cfg.blockDim = dim3(MAIN_THREADS);
@@ -1955,7 +1991,7 @@ static cudaError_t launch_ex(Kern kernel, unsigned blocks, cudaStream_t s, const
         cfg.attrs = attr;
         cfg.numAttrs = 1;
     }
-    return cudaLaunchKernelEx(&cfg, kernel, p);
+    return cudaLaunchKernelEx(&cfg, kernel, args...);
 }
 
 namespace {
@@ -2061,7 +2097,8 @@ cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint6
     return cudaGetLastError();
 }
 
-cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s) {
+cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s,
+                        const void* apw_base, size_t apw_bytes, float apw_hit) {
     if (n_units <= 0) return cudaSuccess;
     const int64_t blocks = (n_units * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
@@ -2070,6 +2107,7 @@ cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_u
     auto k = dtype == 0 ? (mma ? dasp_long_kernel<0, VAR_MMA> : dasp_long_kernel<0, VAR_CUDACORE>)
            : dtype == 1 ? (mma ? dasp_long_kernel<1, VAR_MMA> : dasp_long_kernel<1, VAR_CUDACORE>)
                         : (mma ? dasp_long_kernel<2, VAR_MMA> : dasp_long_kernel<2, VAR_CUDACORE>);
+    if (apw_bytes) return launch_ex(k, grid.x, s, apw_base, apw_bytes, apw_hit, p, n_units);
     k<<<grid, block, 0, s>>>(p, n_units);
     return cudaGetLastError();
 }

@@ -95,7 +95,8 @@ struct FinishParams {
 // apw_bytes > 0: launch with an L2 access-policy window (persisting) over [apw_base, +apw_bytes)
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s,
                         const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
-cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
+cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s,
+                        const void* apw_base = nullptr, size_t apw_bytes = 0, float apw_hit = 1.0f);
 // short tiles one main-kernel warp processes (build knob DASP_SHORT_TPW)
 int short_tiles_per_warp(int dtype);
 // narrow medium row-blocks (rows of at most narrow_max_slots(K) = 2K slots: max(K*nreg, longest
