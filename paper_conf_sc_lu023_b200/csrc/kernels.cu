@@ -110,6 +110,14 @@ __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
     return static_cast<int32_t>(c) >= 0 ? __ldg(reinterpret_cast<const unsigned short*>(x) + static_cast<int32_t>(c))
                                         : static_cast<uint16_t>(0);
 }
+// L2 bulk prefetch of a contiguous range (one instruction, no registers, no shared memory):
+// addr 16-B aligned, bytes a multiple of 16 (callers pass whole 32-element regular regions)
+__device__ __forceinline__ void bulk_prefetch_l2(const void* addr, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
+}
+#ifndef DASP_BULK_PF
+#define DASP_BULK_PF 0     // 1: wide medium warps L2-prefetch the next row-block's regular region (measured slower on C2 / C5, profiles/r01d/bulk_prefetch_negative.jsonl)
+#endif
 // Value streams of the m8n8k4-geometry paths: FP64 (DT 0) and FP32 storage (DT 2, computed in
 // FP64: every float converts exactly, so the DMMA / FMA arithmetic is the FP64 path's).
 template <int DT> struct ValIO;
@@ -861,8 +869,17 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
         for (int64_t rb = rb0; rb < rb1; ++rb) {
             // (prefetching the next row-block's metadata here was measured: it costs registers
             // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta_prefetch_rbw.jsonl)
-            if constexpr (DT == 1) medium_rb_f16<VAR>(P, rb_meta(P, rb, lane), lane, pol);
-            else medium_rb_f64<DT, VAR>(P, rb_meta(P, rb, lane), lane, pol);
+            const RbMeta M = rb_meta(P, rb, lane);
+            if (DASP_BULK_PF && lane == 0 && rb + 1 < rb1 && M.nelem > 0) {
+                // row-block rb+1's regular region starts where rb's ends and is no longer (rows
+                // sorted by length): prefetch [base + nelem, base + 2 nelem) of values and columns
+                const int64_t nb = M.base + M.nelem;
+                bulk_prefetch_l2(static_cast<const char*>(P.reg_val) + nb * static_cast<int64_t>(sizeof(typename Tr<DT>::V)),
+                                 static_cast<uint32_t>(M.nelem * sizeof(typename Tr<DT>::V)));
+                bulk_prefetch_l2(P.reg_col + nb, static_cast<uint32_t>(M.nelem * 4));
+            }
+            if constexpr (DT == 1) medium_rb_f16<VAR>(P, M, lane, pol);
+            else medium_rb_f64<DT, VAR>(P, M, lane, pol);
         }
     }
 }
