@@ -928,10 +928,23 @@ template <int DT> struct ShortLd {          // FP64 / FP32 (m8n8k4 geometry)
     uint32_t c[4];
     int32_t o[4];
 };
+#ifndef DASP_SINGLES_T
+#define DASP_SINGLES_T 1   // singles: lane L takes singles L, L+32, L+64, L+96 (each store instruction
+#endif                     // covers 32 consecutive singles) instead of 4L..4L+3
 template <int DT>
 __device__ __forceinline__ void short_load_f64(const MainParams& P, const ShortRef& T, int lane, uint64_t pol, ShortLd<DT>& L) {
     using IO = ValIO<DT>;
-    IO::ld4r(static_cast<const typename IO::T*>(P.short_val) + T.tile * 128 + lane * 4, pol, L.v);
+    const typename IO::T* sv = static_cast<const typename IO::T*>(P.short_val) + T.tile * 128;
+    if (DASP_SINGLES_T && T.cat == 3) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            L.v[j] = IO::ld1r(sv + 32 * j + lane, pol);
+            L.c[j] = ld1_b32(P.short_col + T.tile * 128 + 32 * j + lane, pol);
+            L.o[j] = static_cast<int32_t>(ld1_b32(P.short_out + T.obase + 32 * j + lane, pol));
+        }
+        return;
+    }
+    IO::ld4r(sv + lane * 4, pol, L.v);
     ld4_b32(P.short_col + T.tile * 128 + lane * 4, pol, L.c);
     short_load_out(P, T, lane, pol, L.o);
 }
@@ -984,6 +997,19 @@ struct ShortLdH {                                    // FP16 (two m16n8k8 blocks
     int32_t o[4];
 };
 __device__ __forceinline__ void short_load_f16(const MainParams& P, const ShortRef& T, int lane, uint64_t pol, ShortLdH& L) {
+    const unsigned short* sv = static_cast<const unsigned short*>(P.short_val) + T.tile * 128;
+    if (DASP_SINGLES_T && T.cat == 3) {   // singles L + 32 j: (a0 lo, a0 hi, a2 lo, a2 hi) = j 0..3
+        uint32_t h[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            h[j] = __ldg(sv + 32 * j + lane);
+            L.c[j] = ld1_b32(P.short_col + T.tile * 128 + 32 * j + lane, pol);
+            L.o[j] = static_cast<int32_t>(ld1_b32(P.short_out + T.obase + 32 * j + lane, pol));
+        }
+        L.a0 = h[0] | (h[1] << 16);
+        L.a2 = h[2] | (h[3] << 16);
+        return;
+    }
     ld2_b32(static_cast<const uint16_t*>(P.short_val) + T.tile * 128 + lane * 4, pol, L.a0, L.a2);
     ld4_b32(P.short_col + T.tile * 128 + lane * 4, pol, L.c);
     short_load_out(P, T, lane, pol, L.o);
