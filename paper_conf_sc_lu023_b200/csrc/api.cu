@@ -25,6 +25,7 @@ struct TimingRec {
 
 struct dasp_plan_s {
     int dtype = 0, device = -1, variant = DASP_VARIANT_CUDACORE, rbw = 1;
+    int wide_il = 0;                      // interleaved wide medium warps (setup_launch)
     bool keep_host = false;
     HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
     void* d[DASP_ARR_COUNT] = {};
@@ -239,6 +240,11 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
                            const std::vector<int32_t>& unit_first_col, const std::vector<int32_t>& nslots) {
     HostFormat& f = p->host;
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
+    // a block's wide medium warps interleave their row-blocks when the medium rows are ragged
+    // (LOOP_NUM 4 or less): C5 +1 % (FP64) .. +7 % (FP16), C3 neutral; uniform stencil rows
+    // (LOOP_NUM 8) keep contiguous ranges (C2+ -2 % .. -5 % interleaved; profiles/r01d/wide_interleave.jsonl)
+    p->wide_il = p->rbw <= 4 ? 1 : 0;
+    if (const char* wi = std::getenv("DASP_WIDE_IL")) p->wide_il = std::atoi(wi) != 0;
     int64_t nrw = dasp::narrow_rb_per_warp(p->dtype);
     {
         const char* ne = std::getenv("DASP_NARROW");   // 0 = every row-block on the wide path (experiments)
@@ -658,6 +664,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.blk_word = static_cast<const uint64_t*>(p->d_blk_word);
     mp.unit_order = static_cast<const int32_t*>(p->d_unit_order);
     mp.rbw = p->rbw;
+    mp.wide_il = p->wide_il;
     mp.class_mask = 7;
     mp.extra = extra;
     mp.item_start = static_cast<const int64_t*>(p->d_item_start);

@@ -115,6 +115,9 @@ __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
 __device__ __forceinline__ void bulk_prefetch_l2(const void* addr, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
 }
+#ifndef DASP_META_PF
+#define DASP_META_PF 0     // CUDA-core wide medium warps: next row-block's metadata one row-block ahead
+#endif
 #ifndef DASP_BULK_PF
 #define DASP_BULK_PF 0     // 1: wide medium warps L2-prefetch the next row-block's regular region (measured slower on C2 / C5, profiles/r01d/bulk_prefetch_negative.jsonl)
 #endif
@@ -814,11 +817,12 @@ __device__ __forceinline__ void medium_rbs_async(const MainParams& P, int64_t rb
 template <int DT> __host__ __device__ constexpr int med_pair() { return DT == 0 ? DASP_PAIR_F64 : (DT == 1 ? DASP_PAIR_F16 : DASP_PAIR_F32); }
 
 template <int DT, int VAR>
-__device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int64_t rb1, int lane, uint64_t pol) {
+__device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int64_t rb1, int lane, uint64_t pol,
+                                           int64_t st = 1) {   // row-blocks rb0, rb0 + st, ... < rb1
     if constexpr (med_pair<DT>() == 2) {
-        for (int64_t rb = rb0; rb < rb1; rb += 2) {
+        for (int64_t rb = rb0; rb < rb1; rb += 2 * st) {
             const RbMeta MA = rb_meta(P, rb, lane);
-            const RbMeta MB = rb + 1 < rb1 ? rb_meta(P, rb + 1, lane) : RbMeta{0, 0, 0, 0, -1};
+            const RbMeta MB = rb + st < rb1 ? rb_meta(P, rb + st, lane) : RbMeta{0, 0, 0, 0, -1};
             if constexpr (DT == 1) {
                 MedLdH LA, LB;
                 medium_load_f16(P, MA, lane, pol, LA);
@@ -841,7 +845,7 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
         int64_t rb = rb0;
         while (rb < rb1) {
             const RbMeta MA = rb_meta(P, rb, lane);     // both metadata rounds issued together
-            const RbMeta MB = rb + 1 < rb1 ? rb_meta(P, rb + 1, lane) : RbMeta{0, 0, FULL_ELEMS, 0, -1};
+            const RbMeta MB = rb + st < rb1 ? rb_meta(P, rb + st, lane) : RbMeta{0, 0, FULL_ELEMS, 0, -1};
             {
                 if (MA.nelem < FULL_ELEMS && MB.nelem < FULL_ELEMS) {
                     if constexpr (DT == 1) {
@@ -857,20 +861,33 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
                         medium_finish_f64<DT, VAR, false>(P, MA, LA, lane, pol);
                         medium_finish_f64<DT, VAR, false>(P, MB, LB, lane, pol);
                     }
-                    rb += 2;
+                    rb += 2 * st;
                     continue;
                 }
             }
             if constexpr (DT == 1) medium_rb_f16<VAR>(P, MA, lane, pol);
             else medium_rb_f64<DT, VAR>(P, MA, lane, pol);
-            ++rb;
+            rb += st;
         }
     } else {
-        for (int64_t rb = rb0; rb < rb1; ++rb) {
+        if constexpr (DASP_META_PF != 0 && VAR == VAR_CUDACORE) {
+            // CUDA-core variant: row-block rb+1's metadata loads are issued before rb is processed
+            // (the MMA instantiation spills with it; profiles/r01/meta_prefetch_rbw.jsonl)
+            if (rb0 >= rb1) return;
+            RbMeta M = rb_meta(P, rb0, lane);
+            for (int64_t rb = rb0; rb < rb1; rb += st) {
+                const RbMeta N = rb + st < rb1 ? rb_meta(P, rb + st, lane) : RbMeta{0, 0, 0, 0, -1};
+                if constexpr (DT == 1) medium_rb_f16<VAR>(P, M, lane, pol);
+                else medium_rb_f64<DT, VAR>(P, M, lane, pol);
+                M = N;
+            }
+            return;
+        }
+        for (int64_t rb = rb0; rb < rb1; rb += st) {
             // (prefetching the next row-block's metadata here was measured: it costs registers
             // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta_prefetch_rbw.jsonl)
             const RbMeta M = rb_meta(P, rb, lane);
-            if (DASP_BULK_PF && lane == 0 && rb + 1 < rb1 && M.nelem > 0) {
+            if (DASP_BULK_PF && lane == 0 && rb + st < rb1 && M.nelem > 0) {
                 // row-block rb+1's regular region starts where rb's ends and is no longer (rows
                 // sorted by length): prefetch [base + nelem, base + 2 nelem) of values and columns
                 const int64_t nb = M.base + M.nelem;
@@ -1342,8 +1359,14 @@ template <int DT, int VAR>
 __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc* D, int64_t w, int lane, uint64_t pol) {
     const int64_t rbp0 = __ldg(&D->rb0), nmwd = __ldg(&D->nmwd);
     if (w < nmwd) {
-        const int64_t rb0 = rbp0 + w * P.rbw;
-        medium_rbs<DT, VAR>(P, rb0, min(rb0 + P.rbw, rbp0 + __ldg(&D->rbm)), lane, pol);
+        const int64_t rbe = rbp0 + __ldg(&D->rbm);
+        // (MainParams::wide_il) the 8 warps of a block take their group's 8 rbw row-blocks
+        // interleaved (warp j: j, j+8, ...; a short last group strides by its warp count), so at
+        // any time a block streams one contiguous region instead of 8 regions rbw row-blocks apart
+        const int64_t gw = w & ~int64_t(WARPS_PER_BLOCK - 1);
+        const int64_t stg = P.wide_il ? min(static_cast<int64_t>(WARPS_PER_BLOCK), nmwd - gw) : 1;
+        const int64_t rbs = P.wide_il ? rbp0 + gw * P.rbw + (w - gw) : rbp0 + w * P.rbw;
+        medium_rbs<DT, VAR>(P, rbs, min(rbs - (w - gw) * (P.wide_il != 0) + stg * P.rbw, rbe), lane, pol, stg);
         return;
     }
     const int64_t nmwm = __ldg(&D->nmwm);
