@@ -26,6 +26,7 @@ struct TimingRec {
 struct dasp_plan_s {
     int dtype = 0, device = -1, variant = DASP_VARIANT_CUDACORE, rbw = 1;
     int wide_il = 0;                      // interleaved wide medium warps (setup_launch)
+    int narrow_il = 0;                    // interleaved narrow / mid medium warps (measured neutral / slower: off)
     bool keep_host = false;
     HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
     void* d[DASP_ARR_COUNT] = {};
@@ -77,6 +78,7 @@ int sa(int dtype) { return dtype == DASP_R_16F ? 4 : 8; }   // long-group partia
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 constexpr int kColBuckets = 16;
+constexpr int kLongOrderDefault = 1;   // long units bucketed one by one (setup_launch; 2 measured slower, profiles/r01d/interleave_long_order.jsonl)
 constexpr bool kSplitShortDefault = false;
 constexpr bool kDynSchedDefault = false;
 constexpr bool kCoschedDefault = false;  // long units inside the main kernel: measured slower
@@ -245,6 +247,8 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     // (LOOP_NUM 8) keep contiguous ranges (C2+ -2 % .. -5 % interleaved; profiles/r01d/wide_interleave.jsonl)
     p->wide_il = p->rbw <= 4 ? 1 : 0;
     if (const char* wi = std::getenv("DASP_WIDE_IL")) p->wide_il = std::atoi(wi) != 0;
+    p->narrow_il = 0;
+    if (const char* ni = std::getenv("DASP_NARROW_IL")) p->narrow_il = std::atoi(ni) != 0;
     int64_t nrw = dasp::narrow_rb_per_warp(p->dtype);
     {
         const char* ne = std::getenv("DASP_NARROW");   // 0 = every row-block on the wide path (experiments)
@@ -321,21 +325,28 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     // group order by the finish kernel: the result is bitwise independent of this order.
     std::vector<int32_t> unit_order(static_cast<size_t>(p->n_units));
     {
+        // DASP_LONG_ORDER: 0 = memory order, 1 (default) = bucketed per unit, 2 = bucketed per run
+        // of WARPS_PER_BLOCK consecutive units, so the warps of one block still stream one
+        // contiguous region (bucketed by the run's first unit)
         const char* lo_env = std::getenv("DASP_LONG_ORDER");
-        const bool bucketed = !(lo_env && std::atoi(lo_env) == 0) && f.n > 0;
+        const int mode = f.n > 0 ? (lo_env ? std::atoi(lo_env) : kLongOrderDefault) : 0;
+        const int64_t run = mode == 2 ? dasp::WARPS_PER_BLOCK : 1;
         for (const auto& d : desc) {
-            std::vector<int32_t> cnt(kColBuckets + 1, 0);
+            std::vector<int64_t> cnt(kColBuckets + 1, 0);
             auto bucket = [&](int64_t u) {
                 const int32_t c = unit_first_col[u];
                 return c < 0 ? kColBuckets - 1 : static_cast<int>(static_cast<int64_t>(c) * kColBuckets / f.n);
             };
-            if (!bucketed) {
+            if (mode == 0) {
                 for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + w] = static_cast<int32_t>(d.unit0 + w);
                 continue;
             }
-            for (int64_t w = 0; w < d.nunits; ++w) cnt[bucket(d.unit0 + w) + 1]++;
+            for (int64_t w = 0; w < d.nunits; w += run) cnt[bucket(d.unit0 + w) + 1] += std::min(run, d.nunits - w);
             for (int b = 0; b < kColBuckets; ++b) cnt[b + 1] += cnt[b];
-            for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + cnt[bucket(d.unit0 + w)]++] = static_cast<int32_t>(d.unit0 + w);
+            for (int64_t w = 0; w < d.nunits; w += run) {
+                const int b = bucket(d.unit0 + w);
+                for (int64_t k = w; k < std::min(w + run, d.nunits); ++k) unit_order[d.unit0 + cnt[b]++] = static_cast<int32_t>(d.unit0 + k);
+            }
         }
     }
     // item words of the pipelined kernel, panel by panel: long units (schedule order), medium
@@ -665,6 +676,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.unit_order = static_cast<const int32_t*>(p->d_unit_order);
     mp.rbw = p->rbw;
     mp.wide_il = p->wide_il;
+    mp.narrow_il = p->narrow_il;
     mp.class_mask = 7;
     mp.extra = extra;
     mp.item_start = static_cast<const int64_t*>(p->d_item_start);

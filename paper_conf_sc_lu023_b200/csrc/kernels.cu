@@ -1327,26 +1327,32 @@ __device__ __forceinline__ void narrow_finish(const MainParams& P, const NarLd<D
 }
 // LPR lanes per row (1: rows spanning <= 2K slots, 4 row-blocks side by side; 2: <= 4K, 2 side
 // by side), passes over [rbs, rbe) with a warp-uniform trip count (the LPR = 2 shuffle)
+// A narrow warp is warp jl of a group of nwg warps that share the DASP_NARROW_RB nwg row-blocks
+// from gb: pass ps of warp jl covers the SIDE row-blocks gb + SIDE (jl + ps nwg) .. (nwg = 1: the
+// warp's own contiguous DASP_NARROW_RB row-blocks; nwg = 8: a block's warps interleaved, so the
+// block streams one contiguous region at a time).  Row-blocks >= rbe are skipped.
 template <int DT, int LPR>
-__device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t rbs, int64_t rbe, int lane, uint64_t pol) {
+__device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t gb, int64_t jl, int64_t nwg, int64_t rbe,
+                                              int lane, uint64_t pol) {
     constexpr int SIDE = 4 / LPR;
     const int g = (lane / LPR) & 7, sub = lane % LPR;
-    const int64_t r0 = rbs + lane / (8 * LPR);
-    const int64_t passes = (rbe - rbs + SIDE - 1) / SIDE;
+    const int64_t r0 = gb + SIDE * jl + lane / (8 * LPR);
+    const int64_t step = SIDE * nwg;
+    constexpr int64_t passes = DASP_NARROW_RB / SIDE;
     if constexpr (DASP_BY_DT(DT, DASP_NARROW_PIPE) != 0) {
         NarLd<DT> A;
         narrow_load<DT>(P, r0, r0 < rbe, g, sub, pol, A);
         for (int64_t ps = 0; ps < passes; ++ps) {
             NarLd<DT> B;
-            const int64_t rn = r0 + (ps + 1) * SIDE;
-            narrow_load<DT>(P, rn, rn < rbe, g, sub, pol, B);
+            const int64_t rn = r0 + (ps + 1) * step;
+            narrow_load<DT>(P, rn, ps + 1 < passes && rn < rbe, g, sub, pol, B);
             narrow_finish<DT, LPR>(P, A, sub);
             A = B;
         }
     } else {
         for (int64_t ps = 0; ps < passes; ++ps) {
             NarLd<DT> A;
-            const int64_t rq = r0 + ps * SIDE;
+            const int64_t rq = r0 + ps * step;
             narrow_load<DT>(P, rq, rq < rbe, g, sub, pol, A);
             narrow_finish<DT, LPR>(P, A, sub);
         }
@@ -1371,13 +1377,18 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
     }
     const int64_t nmwm = __ldg(&D->nmwm);
     const bool mid = w < nmwm;
-    const int64_t rb0 = mid ? rbp0 + __ldg(&D->rbm) + (w - nmwd) * DASP_NARROW_RB
-                            : rbp0 + __ldg(&D->rbn) + (w - nmwm) * DASP_NARROW_RB;
-    const int64_t rb1 = min(rb0 + DASP_NARROW_RB, rbp0 + (mid ? __ldg(&D->rbn) : __ldg(&D->nrb)));
+    const int64_t j = mid ? w - nmwd : w - nmwm;                        // warp within its class
+    const int64_t rbc = rbp0 + (mid ? __ldg(&D->rbm) : __ldg(&D->rbn));  // the class's first row-block
+    const int64_t rbe = rbp0 + (mid ? __ldg(&D->rbn) : __ldg(&D->nrb));
     if constexpr (VAR == VAR_CUDACORE) {
-        if (mid) medium_narrow<DT, 2>(P, rb0, rb1, lane, pol);
-        else medium_narrow<DT, 1>(P, rb0, rb1, lane, pol);
+        const int64_t nwc = mid ? nmwm - nmwd : __ldg(&D->nmw) - nmwm;
+        const int64_t gw = P.narrow_il ? (j & ~int64_t(WARPS_PER_BLOCK - 1)) : j;
+        const int64_t nwg = P.narrow_il ? min(static_cast<int64_t>(WARPS_PER_BLOCK), nwc - gw) : 1;
+        const int64_t gb = rbc + gw * DASP_NARROW_RB;
+        if (mid) medium_narrow<DT, 2>(P, gb, j - gw, nwg, rbe, lane, pol);
+        else medium_narrow<DT, 1>(P, gb, j - gw, nwg, rbe, lane, pol);
     } else {
+        const int64_t rb0 = rbc + j * DASP_NARROW_RB, rb1 = min(rb0 + DASP_NARROW_RB, rbe);
         medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);   // MMA variant: the paper's warp per row-block
     }
 }

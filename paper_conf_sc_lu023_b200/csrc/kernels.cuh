@@ -60,6 +60,7 @@ struct MainParams {
     double alpha, beta;
     int32_t rbw;
     int32_t wide_il;          // 1: a block's wide medium warps interleave their row-blocks (kernels.cu medium_warp)
+    int32_t narrow_il;        // 1: a block's narrow / mid warps interleave their passes (medium_narrow)
     int32_t class_mask;       // bit 0 long, bit 1 medium, bit 2 short (profiling; 7 = all)
     ExtraDst extra;
     // dynamic schedule of the main kernel (launch_main_dyn): panel q's work items are
