@@ -28,6 +28,7 @@ struct dasp_plan_s {
     int dtype = 0, device = -1, variant = DASP_VARIANT_CUDACORE, rbw = 1;
     int wide_il = 0;                      // interleaved wide medium warps (setup_launch)
     int narrow_il = 0;                    // interleaved narrow / mid medium warps (measured neutral / slower: off)
+    int nrw = 0;                          // row-blocks per narrow / mid warp (0: no narrow path)
     bool keep_host = false;
     HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
     void* d[DASP_ARR_COUNT] = {};
@@ -255,6 +256,9 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         const char* ne = std::getenv("DASP_NARROW");   // 0 = every row-block on the wide path (experiments)
         if ((ne && std::atoi(ne) == 0) || static_cast<int64_t>(nslots.size()) != f.nrb) nrw = 0;
     }
+    // small matrices (LOOP_NUM 1) keep more warps in flight: one pass of 4 row-blocks
+    if (nrw > 4 && p->rbw <= 1) nrw = 4;
+    p->nrw = static_cast<int>(nrw);
     bool mid = true;   // two-lanes-per-row narrow warps (DASP_NARROW_MID=0: off, experiments)
     {
         const char* me = std::getenv("DASP_NARROW_MID");
@@ -678,6 +682,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.rbw = p->rbw;
     mp.wide_il = p->wide_il;
     mp.narrow_il = p->narrow_il;
+    mp.nrw = p->nrw;
     mp.class_mask = 7;
     mp.extra = extra;
     mp.item_start = static_cast<const int64_t*>(p->d_item_start);

@@ -49,10 +49,10 @@
 #define DASP_SHORT_TPW_F64 2
 #endif
 #ifndef DASP_SHORT_TPW_F16
-#define DASP_SHORT_TPW_F16 2
+#define DASP_SHORT_TPW_F16 4
 #endif
 #ifndef DASP_SHORT_TPW_F32
-#define DASP_SHORT_TPW_F32 2
+#define DASP_SHORT_TPW_F32 3
 #endif
 #define DASP_BY_DT(DT, K) ((DT) == 0 ? K##_F64 : ((DT) == 1 ? K##_F16 : K##_F32))
 
@@ -1163,6 +1163,31 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
     constexpr int TPW = DASP_BY_DT(DT, DASP_SHORT_TPW);
     const int64_t t0 = ws * TPW;
     if (t0 >= nt || !(P.class_mask & 4)) return;
+    if constexpr (TPW > 2) {   // generic: every tile's loads, then every tile's gathers, then the math
+        ShortRef R[TPW];
+#pragma unroll
+        for (int k = 0; k < TPW; ++k) R[k] = short_ref(D, min(t0 + k, nt - 1));
+        if constexpr (DT == 1) {
+            ShortLdH L[TPW];
+            uint16_t xh[TPW][4];
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_load_f16(P, R[k], lane, pol, L[k]);
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_gather_f16(P, L[k], xh[k]);
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_math_f16<VAR>(P, R[k].cat, L[k], xh[k], lane);
+        } else {
+            ShortLd<DT> L[TPW];
+            double xv[TPW][4];
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_load_f64<DT>(P, R[k], lane, pol, L[k]);
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_gather_f64<DT>(P, L[k], xv[k]);
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_math_f64<DT, VAR>(P, R[k].cat, L[k], xv[k], lane);
+        }
+        return;
+    }
     const ShortRef A = short_ref(D, t0);
     if (TPW == 1 || t0 + 1 >= nt) { short_tile<DT, VAR>(P, A, lane, pol); return; }
     const ShortRef B = short_ref(D, t0 + 1);
@@ -1198,7 +1223,7 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 // 32 b + 4 g (the block-after-block ragged layout, R18, nreg <= 2 < CW), an irregular quad is the
 // row's tail in irr_val.  CUDA-core arithmetic (FP64 FMA; FP32 storage widened exactly).
 #ifndef DASP_NARROW_RB
-#define DASP_NARROW_RB 8     // row-blocks per narrow warp: 4 side by side x 2 passes
+#define DASP_NARROW_RB 8     // row-blocks per narrow warp (at most; MainParams::nrw): 4 side by side x 2 passes
 #endif
 // 1: the next pass's stream loads are issued before this pass's gathers.  Measured
 // (profiles/r01d/narrow_pipe.jsonl): FP16 C3 main kernel -3 %, stencils -1 %; FP64 +6 % (spills at
@@ -1327,9 +1352,9 @@ __device__ __forceinline__ void narrow_finish(const MainParams& P, const NarLd<D
 }
 // LPR lanes per row (1: rows spanning <= 2K slots, 4 row-blocks side by side; 2: <= 4K, 2 side
 // by side), passes over [rbs, rbe) with a warp-uniform trip count (the LPR = 2 shuffle)
-// A narrow warp is warp jl of a group of nwg warps that share the DASP_NARROW_RB nwg row-blocks
+// A narrow warp is warp jl of a group of nwg warps that share the nrw nwg row-blocks (nrw = P.nrw)
 // from gb: pass ps of warp jl covers the SIDE row-blocks gb + SIDE (jl + ps nwg) .. (nwg = 1: the
-// warp's own contiguous DASP_NARROW_RB row-blocks; nwg = 8: a block's warps interleaved, so the
+// warp's own contiguous nrw row-blocks; nwg = 8: a block's warps interleaved, so the
 // block streams one contiguous region at a time).  Row-blocks >= rbe are skipped.
 template <int DT, int LPR>
 __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t gb, int64_t jl, int64_t nwg, int64_t rbe,
@@ -1338,7 +1363,7 @@ __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t gb, i
     const int g = (lane / LPR) & 7, sub = lane % LPR;
     const int64_t r0 = gb + SIDE * jl + lane / (8 * LPR);
     const int64_t step = SIDE * nwg;
-    constexpr int64_t passes = DASP_NARROW_RB / SIDE;
+    const int64_t passes = P.nrw / SIDE;
     if constexpr (DASP_BY_DT(DT, DASP_NARROW_PIPE) != 0) {
         NarLd<DT> A;
         narrow_load<DT>(P, r0, r0 < rbe, g, sub, pol, A);
@@ -1384,11 +1409,11 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
         const int64_t nwc = mid ? nmwm - nmwd : __ldg(&D->nmw) - nmwm;
         const int64_t gw = P.narrow_il ? (j & ~int64_t(WARPS_PER_BLOCK - 1)) : j;
         const int64_t nwg = P.narrow_il ? min(static_cast<int64_t>(WARPS_PER_BLOCK), nwc - gw) : 1;
-        const int64_t gb = rbc + gw * DASP_NARROW_RB;
+        const int64_t gb = rbc + gw * P.nrw;
         if (mid) medium_narrow<DT, 2>(P, gb, j - gw, nwg, rbe, lane, pol);
         else medium_narrow<DT, 1>(P, gb, j - gw, nwg, rbe, lane, pol);
     } else {
-        const int64_t rb0 = rbc + j * DASP_NARROW_RB, rb1 = min(rb0 + DASP_NARROW_RB, rbe);
+        const int64_t rb0 = rbc + j * P.nrw, rb1 = min(rb0 + P.nrw, rbe);
         medium_rbs<DT, VAR>(P, rb0, rb1, lane, pol);   // MMA variant: the paper's warp per row-block
     }
 }

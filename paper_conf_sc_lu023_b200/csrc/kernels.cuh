@@ -61,6 +61,7 @@ struct MainParams {
     int32_t rbw;
     int32_t wide_il;          // 1: a block's wide medium warps interleave their row-blocks (kernels.cu medium_warp)
     int32_t narrow_il;        // 1: a block's narrow / mid warps interleave their passes (medium_narrow)
+    int32_t nrw;              // row-blocks per narrow / mid warp (4 or 8: a multiple of 4)
     int32_t class_mask;       // bit 0 long, bit 1 medium, bit 2 short (profiling; 7 = all)
     ExtraDst extra;
     // dynamic schedule of the main kernel (launch_main_dyn): panel q's work items are
@@ -102,7 +103,7 @@ cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_u
 // short tiles one main-kernel warp processes (build knob DASP_SHORT_TPW)
 int short_tiles_per_warp(int dtype);
 // narrow medium row-blocks (rows of at most narrow_max_slots(K) = 2K slots: max(K*nreg, longest
-// row)): row-blocks one narrow warp processes, 0 = no narrow path for this dtype
+// row)): the most row-blocks one narrow warp processes, 0 = no narrow path for this dtype
 int narrow_rb_per_warp(int dtype);
 constexpr int narrow_max_slots(int K) { return 2 * K; }
 constexpr int mid_max_slots(int K) { return 4 * K; }
