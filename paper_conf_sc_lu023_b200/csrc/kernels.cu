@@ -328,30 +328,38 @@ __device__ __forceinline__ void long_unit_f64(const MainParams& P, int64_t u, in
 }
 
 // FP16: lane l reads 8-B value chunks l + 32j (j = 0..3): halves 4(l+32j)..+3, all in group j
-template <int VAR>
-__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol) {
+// one FP16 long unit in three steps (loads | gathers | block dots + transpose-reduce + partials),
+// so a warp can hold two units' memory round trips in flight (DASP_LONG_UPW_F16)
+struct LongLdH {
+    uint32_t vv[8], c[16];
+};
+__device__ __forceinline__ void long_load_f16(const MainParams& P, int64_t u, int lane, uint64_t pol, LongLdH& L) {
     const uint16_t* lv = static_cast<const uint16_t*>(P.long_val) + u * 512;
     const int32_t* lc = P.long_col + u * 512;
-    const uint16_t* x = static_cast<const uint16_t*>(P.x);
-    uint32_t vv[8], c[16];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-        ld2_b32(lv + 4 * (lane + 32 * j), pol, vv[2 * j], vv[2 * j + 1]);
-        ld4_b32(lc + 4 * (lane + 32 * j), pol, *reinterpret_cast<uint32_t(*)[4]>(&c[4 * j]));
+        ld2_b32(lv + 4 * (lane + 32 * j), pol, L.vv[2 * j], L.vv[2 * j + 1]);
+        ld4_b32(lc + 4 * (lane + 32 * j), pol, *reinterpret_cast<uint32_t(*)[4]>(&L.c[4 * j]));
     }
-    uint16_t xh[16];
+}
+__device__ __forceinline__ void long_gather_f16(const MainParams& P, const LongLdH& L, uint16_t (&xh)[16]) {
+    const uint16_t* x = static_cast<const uint16_t*>(P.x);
 #pragma unroll
-    for (int e = 0; e < 16; ++e) xh[e] = gxh(x, c[e]);
+    for (int e = 0; e < 16; ++e) xh[e] = gxh(x, L.c[e]);
+}
+template <int VAR>
+__device__ __forceinline__ void long_finish_f16(const MainParams& P, int64_t u, const LongLdH& L, const uint16_t (&xh)[16],
+                                                int lane) {
     float gsum[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
         if constexpr (VAR == VAR_MMA) {
             float c0 = 0.f, c1 = 0.f;
-            hmma(c0, c1, vv[2 * j], pack2(xh[4 * j], xh[4 * j + 1]));
-            hmma(c0, c1, vv[2 * j + 1], pack2(xh[4 * j + 2], xh[4 * j + 3]));
+            hmma(c0, c1, L.vv[2 * j], pack2(xh[4 * j], xh[4 * j + 1]));
+            hmma(c0, c1, L.vv[2 * j + 1], pack2(xh[4 * j + 2], xh[4 * j + 3]));
             gsum[j] = is_diag_holder(lane) ? (((lane >> 2) & 1) ? c1 : c0) : 0.f;
         } else {
-            const float2 a = u2f2(vv[2 * j]), b = u2f2(vv[2 * j + 1]);
+            const float2 a = u2f2(L.vv[2 * j]), b = u2f2(L.vv[2 * j + 1]);
             float sacc = a.x * h2f(xh[4 * j]);
             sacc = fmaf(a.y, h2f(xh[4 * j + 1]), sacc);
             sacc = fmaf(b.x, h2f(xh[4 * j + 2]), sacc);
@@ -370,7 +378,16 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
         kk += __shfl_xor_sync(FULL, kk, 2);
         kk += __shfl_xor_sync(FULL, kk, 1);
         if ((lane & 7) == 0) static_cast<float*>(P.partial)[u * 4 + 2 * (lane >> 4) + ((lane >> 3) & 1)] = kk;
-    }    if (P.long_cnt) long_unit_complete<1>(P, u, lane);
+    }
+    if (P.long_cnt) long_unit_complete<1>(P, u, lane);
+}
+template <int VAR>
+__device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, int lane, uint64_t pol) {
+    LongLdH L;
+    uint16_t xh[16];
+    long_load_f16(P, u, lane, pol, L);
+    long_gather_f16(P, L, xh);
+    long_finish_f16<VAR>(P, u, L, xh, lane);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1433,19 +1450,41 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
 // per SM) than the medium path, which needs 64 (profiles/r01/long_kernel_occupancy.jsonl).  Units run in
 // the column-bucketed schedule `unit_order`.
 #ifndef DASP_LONG_MIN_BLOCKS
-#define DASP_LONG_MIN_BLOCKS 6
+#define DASP_LONG_MIN_BLOCKS 8   // 32 registers, 64 warps/SM (C3 long -2 %, C5 -3 % vs 40 registers; profiles/r01d/long_occupancy*.jsonl)
 #endif
 #ifndef DASP_LONG_MIN_BLOCKS_F16
-#define DASP_LONG_MIN_BLOCKS_F16 6
+#define DASP_LONG_MIN_BLOCKS_F16 8   // 32 registers, 64 warps/SM (FP16 / FP32 long: -1..-7 %, profiles/r01d/long_occupancy.jsonl)
+#endif
+#ifndef DASP_LONG_MIN_BLOCKS_F32
+#define DASP_LONG_MIN_BLOCKS_F32 8
+#endif
+#ifndef DASP_LONG_UPW_F16
+#define DASP_LONG_UPW_F16 1   // FP16 long units per warp (2: both units' loads, then both gathers)
 #endif
 template <int DT, int VAR>
-__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_LONG_MIN_BLOCKS : DASP_LONG_MIN_BLOCKS_F16)
+__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_LONG_MIN_BLOCKS
+                                                         : (DT == 1 ? DASP_LONG_MIN_BLOCKS_F16 : DASP_LONG_MIN_BLOCKS_F32))
 dasp_long_kernel(const MainParams P, int64_t n_units) {
-    const int64_t w = (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5;
+    constexpr int UPW = DT == 1 ? DASP_LONG_UPW_F16 : 1;
+    const int64_t w = ((static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5) * UPW;
     if (w >= n_units) return;
     const int lane = threadIdx.x & 31;
     const uint64_t pol = stream_policy();
     const int64_t u = __ldg(P.unit_order + w);
+    if constexpr (DT == 1 && UPW == 2) {
+        if (w + 1 < n_units) {
+            const int64_t u2 = __ldg(P.unit_order + w + 1);
+            LongLdH A, B;
+            uint16_t xa[16], xb[16];
+            long_load_f16(P, u, lane, pol, A);
+            long_load_f16(P, u2, lane, pol, B);
+            long_gather_f16(P, A, xa);
+            long_gather_f16(P, B, xb);
+            long_finish_f16<VAR>(P, u, A, xa, lane);
+            long_finish_f16<VAR>(P, u2, B, xb, lane);
+            return;
+        }
+    }
     if constexpr (DT == 1) long_unit_f16<VAR>(P, u, lane, pol);
     else long_unit_f64<DT, VAR>(P, u, lane, pol);
 }
@@ -2202,7 +2241,8 @@ cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint6
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s,
                         const void* apw_base, size_t apw_bytes, float apw_hit) {
     if (n_units <= 0) return cudaSuccess;
-    const int64_t blocks = (n_units * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
+    const int64_t upw = dtype == 1 ? DASP_LONG_UPW_F16 : 1;
+    const int64_t blocks = ((n_units + upw - 1) / upw * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
     const bool mma = variant == VAR_MMA;
