@@ -258,6 +258,8 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     }
     // small matrices (LOOP_NUM 1) keep more warps in flight: one pass of 4 row-blocks
     if (nrw > 4 && p->rbw <= 1) nrw = 4;
+    if (const char* ev = std::getenv("DASP_NRW"))   // experiments: row-blocks per narrow warp (multiple of 4)
+        if (nrw > 0 && std::atoi(ev) >= 4) nrw = std::atoi(ev) / 4 * 4;
     p->nrw = static_cast<int>(nrw);
     bool mid = true;   // two-lanes-per-row narrow warps (DASP_NARROW_MID=0: off, experiments)
     {
