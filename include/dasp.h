@@ -115,6 +115,10 @@ typedef struct {
     double threshold;                                  /* resolved tau                       */
     double build_ms, upload_ms;                        /* host build; host->device upload   */
     int32_t co_scheduled;                              /* 1 if long units run co-scheduled   */
+    int64_t rowblocks_mid, rowblocks_narrow;           /* medium row-blocks on the two-lanes-
+                                                          per-row / one-lane-per-row warps
+                                                          (launch schedule)    */
+    int32_t narrow_rb_per_warp;                        /* row-blocks per narrow / mid warp   */
 } dasp_plan_info_t;
 
 /*

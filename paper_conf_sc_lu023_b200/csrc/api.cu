@@ -29,6 +29,7 @@ struct dasp_plan_s {
     int wide_il = 0;                      // interleaved wide medium warps (setup_launch)
     int narrow_il = 0;                    // interleaved narrow / mid medium warps (measured neutral / slower: off)
     int nrw = 0;                          // row-blocks per narrow / mid warp (0: no narrow path)
+    int64_t rb_mid = 0, rb_narrow = 0;    // row-blocks on mid / narrow warps (all panels)
     bool keep_host = false;
     HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
     void* d[DASP_ARR_COUNT] = {};
@@ -261,6 +262,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     if (const char* ev = std::getenv("DASP_NRW"))   // experiments: row-blocks per narrow warp (multiple of 4)
         if (nrw > 0 && std::atoi(ev) >= 4) nrw = std::atoi(ev) / 4 * 4;
     p->nrw = static_cast<int>(nrw);
+    p->rb_mid = p->rb_narrow = 0;
     bool mid = true;   // two-lanes-per-row narrow warps (DASP_NARROW_MID=0: off, experiments)
     {
         const char* me = std::getenv("DASP_NARROW_MID");
@@ -294,6 +296,8 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         d.nmwd = (d.rbm + p->rbw - 1) / p->rbw;
         d.nmwm = d.nmwd + (nrw > 0 ? (d.rbn - d.rbm + nrw - 1) / nrw : 0);
         d.nmw = d.nmwm + (nrw > 0 ? (d.nrb - d.rbn + nrw - 1) / nrw : 0);
+        p->rb_mid += d.rbn - d.rbm;
+        p->rb_narrow += d.nrb - d.rbn;
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
         if (p->split_short) {   // tiles leave the main kernel; per-tile metadata for the short kernel
             for (int64_t t = 0; t < d.t13 + d.t4 + d.t22 + d.ts; ++t) {
@@ -860,6 +864,9 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->n_panels = f.n_panels;
     o->pipeline = p->pipe ? 1 : 0;
     o->co_scheduled = p->cosched ? 1 : 0;
+    o->rowblocks_mid = p->rb_mid;
+    o->rowblocks_narrow = p->rb_narrow;
+    o->narrow_rb_per_warp = p->nrw;
     o->max_len = f.max_len;
     o->threshold = f.tau;
     o->build_ms = p->build_ms;

@@ -58,7 +58,8 @@ class PlanInfo(ctypes.Structure):
                [("medium_rb_per_warp", ctypes.c_int32), ("launches_per_spmv", ctypes.c_int32),
                 ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64), ("pipeline", ctypes.c_int32),
                 ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
-                ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double), ("co_scheduled", ctypes.c_int32)]
+                ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double), ("co_scheduled", ctypes.c_int32),
+                ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32)]
 
     def as_dict(self):
         return {name: getattr(self, name) for name, _ in self._fields_}

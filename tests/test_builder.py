@@ -177,3 +177,33 @@ def test_knob_closed_forms_on_stencil():
     assert info["nnz_reg_new"] == 0 and info["nnz_irreg"] == A.nnz
     with pytest.raises(dasp.DaspError):
         host_plan(A, "f64", max_len=3)
+
+
+@pytest.mark.parametrize("dt", ["f64", "f16", "f32"])
+@pytest.mark.parametrize("panel", [-1, 1000])
+def test_narrow_mid_split(dt, panel):
+    """The launch schedule's narrow / mid row-block counts: per panel, the trailing
+    row-blocks whose rows span at most 2K (narrow) / 4K (mid) slots, slots = K*nreg + irregular length
+    of the row-block's first row -- recomputed here from the oracle builder's rb_ptr / irr_ptr."""
+    rng = np.random.default_rng(3)
+    lens = list(rng.choice([0, 1, 3, 5, 6, 7, 8, 9, 12, 16, 20, 27, 31, 40, 100, 300], size=4000))
+    A = synth.from_lengths(lens, n=5000)
+    plan = host_plan(A, dt, panel_rows=panel)
+    info = plan.info
+    ref = oracle.build(A, dt, panel_rows=info["panel_rows"])
+    K = 8 if dt == "f16" else 4
+    rb_ptr, irr_ptr, pan = ref.view("rb_ptr"), ref.view("irr_ptr"), ref.view("panels").reshape(-1, 12)
+    narrow = mid = 0
+    for p in pan:
+        rb0, nrb = int(p[4]), int(p[5])
+        slots = [(rb_ptr[rb + 1] - rb_ptr[rb]) // (8 * K) * K + (irr_ptr[8 * rb + 1] - irr_ptr[8 * rb])
+                 for rb in range(rb0, rb0 + nrb)]
+        n_narrow = n_mid = 0
+        while n_narrow < nrb and slots[nrb - 1 - n_narrow] <= 2 * K:
+            n_narrow += 1
+        while n_narrow + n_mid < nrb and slots[nrb - 1 - n_narrow - n_mid] <= 4 * K:
+            n_mid += 1
+        narrow += n_narrow
+        mid += n_mid
+    assert (info["rowblocks_narrow"], info["rowblocks_mid"]) == (narrow, mid)
+    assert info["narrow_rb_per_warp"] in (4, 8)
