@@ -6,7 +6,10 @@
 
 namespace dasp {
 
-constexpr int MAIN_THREADS = 256;
+#ifndef DASP_MAIN_THREADS
+#define DASP_MAIN_THREADS 256
+#endif
+constexpr int MAIN_THREADS = DASP_MAIN_THREADS;   // threads per block of the main / long / short kernels
 constexpr int MAX_EXTRA_DST = 7;   // dasp_spmv_scatter: up to 8 destinations (this GPU + 7 peers)
 
 // Extra destinations of y (dasp_spmv_scatter): every value stored into y is also stored at the
