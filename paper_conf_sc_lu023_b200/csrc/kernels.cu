@@ -102,8 +102,21 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
     return v;
 }
 // x gather through the read-only path; column -1 (pad, R12) reads 0 without touching memory
+#ifndef DASP_GX_MODE
+#define DASP_GX_MODE 0   // x gathers: 0 ld.global.nc (LDG.CONSTANT), 1 + L1::evict_last, 2 ld.global.ca
+#endif
+// (DASP_GX_MODE 1 / 2 measured within noise on C2 / C2+ / C3 / C5, profiles/r01d/x_gather_cache_op.jsonl)
 __device__ __forceinline__ double gx(const double* x, uint32_t c) {
-    return static_cast<int32_t>(c) >= 0 ? __ldg(x + static_cast<int32_t>(c)) : 0.0;
+    if constexpr (DASP_GX_MODE == 0) {
+        return static_cast<int32_t>(c) >= 0 ? __ldg(x + static_cast<int32_t>(c)) : 0.0;
+    } else {
+        if (static_cast<int32_t>(c) < 0) return 0.0;
+        const double* a = x + static_cast<int32_t>(c);
+        double v;
+        if constexpr (DASP_GX_MODE == 1) asm("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(a));
+        else asm volatile("ld.global.ca.f64 %0, [%1];" : "=d"(v) : "l"(a));
+        return v;
+    }
 }
 __device__ __forceinline__ double gx_f64(const double* x, uint32_t c) { return gx(x, c); }
 __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
