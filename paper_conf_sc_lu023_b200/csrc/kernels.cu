@@ -128,6 +128,9 @@ __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
 __device__ __forceinline__ void bulk_prefetch_l2(const void* addr, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
 }
+#ifndef DASP_META_L2PF
+#define DASP_META_L2PF 0   // 1: wide warps L2-prefetch their metadata lines at warp start (C2 -2.5 %, C2+ +1..3 %, C5 -1 %: off)
+#endif
 #ifndef DASP_META_PF
 #define DASP_META_PF 0     // CUDA-core wide medium warps: next row-block's metadata one row-block ahead
 #endif
@@ -1427,7 +1430,20 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
         const int64_t gw = w & ~int64_t(WARPS_PER_BLOCK - 1);
         const int64_t stg = P.wide_il ? min(static_cast<int64_t>(WARPS_PER_BLOCK), nmwd - gw) : 1;
         const int64_t rbs = P.wide_il ? rbp0 + gw * P.rbw + (w - gw) : rbp0 + w * P.rbw;
-        medium_rbs<DT, VAR>(P, rbs, min(rbs - (w - gw) * (P.wide_il != 0) + stg * P.rbw, rbe), lane, pol, stg);
+        const int64_t rbend = min(rbs - (w - gw) * (P.wide_il != 0) + stg * P.rbw, rbe);
+        if constexpr (DASP_META_L2PF != 0) {
+            // the warp's row-block metadata (irr_ptr, med_out, rb_ptr lines of its whole range) into
+            // L2 with one prefetch per lane, so each row-block's metadata round trip is an L2 hit
+            const int64_t r0 = rbs - (w - gw) * (P.wide_il != 0);
+            const char* ip = reinterpret_cast<const char*>(P.irr_ptr + 8 * r0);
+            const char* mo = reinterpret_cast<const char*>(P.med_out + 8 * r0);
+            const int li = static_cast<int>((8 * (rbend - r0) * 8 + 8 + 127) >> 7);
+            const int lm = static_cast<int>((8 * (rbend - r0) * 4 + 127) >> 7);
+            const char* a = lane < li ? ip + 128 * lane
+                          : lane < li + lm ? mo + 128 * (lane - li) : reinterpret_cast<const char*>(P.rb_ptr + r0);
+            if (lane <= li + lm) asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+        }
+        medium_rbs<DT, VAR>(P, rbs, rbend, lane, pol, stg);
         return;
     }
     const int64_t nmwm = __ldg(&D->nmwm);
