@@ -2143,9 +2143,31 @@ __global__ void __launch_bounds__(256) dasp_gather_kernel(const W* __restrict__ 
 
 }  // namespace
 
+// DASP_CARVEOUT >= 0: preferred shared-memory carveout (percent) set once per kernel before its
+// first launch (experiment knob; -1 leaves the driver's choice)
+#ifndef DASP_CARVEOUT
+#define DASP_CARVEOUT -1
+#endif
+static void set_carveout(const void* k) {
+#if DASP_CARVEOUT >= 0
+    static const void* done[32] = {};
+    for (int i = 0; i < 32; ++i) {
+        if (done[i] == k) return;
+        if (!done[i]) {
+            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, DASP_CARVEOUT);
+            done[i] = k;
+            return;
+        }
+    }
+#else
+    (void)k;
+#endif
+}
+
 template <typename Kern, typename... Args>
 static cudaError_t launch_ex(Kern kernel, unsigned blocks, cudaStream_t s, const void* apw_base, size_t apw_bytes,
                              float apw_hit, Args... args) {
+    set_carveout(reinterpret_cast<const void*>(kernel));
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(blocks);
     cfg.blockDim = dim3(MAIN_THREADS);
@@ -2279,6 +2301,7 @@ cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_u
            : dtype == 1 ? (mma ? dasp_long_kernel<1, VAR_MMA> : dasp_long_kernel<1, VAR_CUDACORE>)
                         : (mma ? dasp_long_kernel<2, VAR_MMA> : dasp_long_kernel<2, VAR_CUDACORE>);
     if (apw_bytes) return launch_ex(k, grid.x, s, apw_base, apw_bytes, apw_hit, p, n_units);
+    set_carveout(reinterpret_cast<const void*>(k));
     k<<<grid, block, 0, s>>>(p, n_units);
     return cudaGetLastError();
 }
