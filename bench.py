@@ -547,6 +547,7 @@ def main():
                "h2d_bytes_per_step": int(x1.numel() * x1.element_size()),
                "d2h_bytes_per_step": int(slab.rows * yh.element_size()), "api": "dasp_spmv_host_stream",
                "steps": args.e2e_steps, "distinct_x": nv,
+               "h2d": "SM loads from pinned host (UVA)" if os.environ.get("DASP_H2D_SM", "0") not in ("", "0") else "copy engine",
                "single_call": {"api": "dasp_spmv_host", "value": flops_step / dt1 / 1e9, "ms_per_step": dt1 * 1e3}}
 
     # ---- preprocessing cost (Fig. 13): host builder vs the device builder (f2) ----

@@ -207,7 +207,11 @@ dasp_status_t dasp_spmv_host(dasp_plan_t plan, const void* x_host, void* y_host,
  * `stream`, so per vector the cost approaches max(H2D, kernel, D2H) rather than their sum.  Every
  * vector is copied in and its result copied out (no caching).  Results are identical to nvec
  * dasp_spmv_host calls.  Synchronises `stream` before returning; the host buffers must stay valid
- * until then and should be pinned (pageable memory serialises the copies).  Returns INVALID_ARG
+ * until then and should be pinned (pageable memory serialises the copies).  Copies use
+ * cudaMemcpyAsync; DASP_H2D_SM=1 in the environment makes page-locked host vectors of >= 1 MiB at
+ * 16-B aligned addresses be read by SM loads over UVA instead (an experiment knob: faster alone,
+ * slower inside the pipelined step).  dasp_spmv_host does the same.
+ * Returns INVALID_ARG
  * (null plan, nvec < 0, ldx < n with x needed, ldy < m, null buffers), UNSUPPORTED (host-only plan),
  * OUT_OF_MEMORY or CUDA.
  */

@@ -753,6 +753,28 @@ dasp_status_t dasp_spmv(dasp_plan_t p, const void* x, void* y, double alpha, dou
     return dasp_spmv_ex(p, x, y, alpha, beta, stream, DASP_VARIANT_DEFAULT);
 }
 
+// Host -> device copy of a caller's buffer: cudaMemcpyAsync (copy engine).  DASP_H2D_SM=1 in the
+// environment (read per call) instead reads page-locked host memory (device-accessible under UVA) of
+// >= 1 MiB at a 16-B aligned address with SM loads (dasp::launch_h2d_sm).  Alone that copy runs at
+// 49.5 GB/s against 42 GB/s (scripts/probe/h2d_probe.py), but inside the e2e step it shares the SMs
+// with the SpMV and the step got slower (C2 FP64 e2e 220 vs 283 GFLOPS, profiles/r01e/h2d_ab.jsonl):
+// off by default.
+static cudaError_t copy_h2d(void* dst, const void* src, size_t bytes, cudaStream_t s) {
+    const char* env = std::getenv("DASP_H2D_SM");
+    const int sm_mode = env ? std::atoi(env) : 0;
+    if (sm_mode && bytes >= (1u << 20) && (reinterpret_cast<uintptr_t>(src) & 15) == 0) {
+        cudaPointerAttributes a{};
+        if (cudaPointerGetAttributes(&a, src) == cudaSuccess && a.type == cudaMemoryTypeHost && a.devicePointer) {
+            int dev = 0, sms = 0;
+            if (cudaGetDevice(&dev) == cudaSuccess &&
+                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && sms > 0)
+                return dasp::launch_h2d_sm(dst, a.devicePointer, bytes, sms, s);
+        }
+        cudaGetLastError();   // a failed attribute query is not an error of this call
+    }
+    return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s);
+}
+
 dasp_status_t dasp_spmv_host(dasp_plan_t p, const void* x_host, void* y_host, double alpha, double beta, void* stream) {
     if (!p) return DASP_ERR_INVALID_ARG;
     if (p->device < 0) return DASP_ERR_UNSUPPORTED;
@@ -764,8 +786,8 @@ dasp_status_t dasp_spmv_host(dasp_plan_t p, const void* x_host, void* y_host, do
     const size_t xb = static_cast<size_t>(f.n) * sx(p->dtype), yb = static_cast<size_t>(f.m) * sy(p->dtype);
     if (!p->d_xh && xb && cudaMalloc(&p->d_xh, xb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
     if (!p->d_yh && cudaMalloc(&p->d_yh, yb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
-    if (xb && alpha != 0.0 && cudaMemcpyAsync(p->d_xh, x_host, xb, cudaMemcpyHostToDevice, s) != cudaSuccess) return DASP_ERR_CUDA;
-    if (beta != 0.0 && cudaMemcpyAsync(p->d_yh, y_host, yb, cudaMemcpyHostToDevice, s) != cudaSuccess) return DASP_ERR_CUDA;
+    if (xb && alpha != 0.0 && copy_h2d(p->d_xh, x_host, xb, s) != cudaSuccess) return DASP_ERR_CUDA;
+    if (beta != 0.0 && copy_h2d(p->d_yh, y_host, yb, s) != cudaSuccess) return DASP_ERR_CUDA;
     dasp_status_t st = dasp_spmv(p, p->d_xh, p->d_yh, alpha, beta, stream);
     if (st != DASP_OK) return st;
     if (cudaMemcpyAsync(y_host, p->d_yh, yb, cudaMemcpyDeviceToHost, s) != cudaSuccess) return DASP_ERR_CUDA;
@@ -804,10 +826,10 @@ dasp_status_t dasp_spmv_host_stream(dasp_plan_t p, const void* x_host, int64_t l
         const int b = static_cast<int>(j & 1);
         // h2d: vector j into slot b once SpMV j-2 has read it (and, for beta != 0, y_j once y_{j-2} left)
         ok = ok && cudaStreamWaitEvent(p->s_h2d, p->ev_done[b], 0) == cudaSuccess;
-        if (need_x) ok = ok && cudaMemcpyAsync(p->d_xs[b], xh + j * xs, xb, cudaMemcpyHostToDevice, p->s_h2d) == cudaSuccess;
+        if (need_x) ok = ok && copy_h2d(p->d_xs[b], xh + j * xs, xb, p->s_h2d) == cudaSuccess;
         if (beta != 0.0) {
             ok = ok && cudaStreamWaitEvent(p->s_h2d, p->ev_yout[b], 0) == cudaSuccess;
-            ok = ok && cudaMemcpyAsync(p->d_ys[b], yh + j * ys, yb, cudaMemcpyHostToDevice, p->s_h2d) == cudaSuccess;
+            ok = ok && copy_h2d(p->d_ys[b], yh + j * ys, yb, p->s_h2d) == cudaSuccess;
         }
         ok = ok && cudaEventRecord(p->ev_x[b], p->s_h2d) == cudaSuccess;
         // compute: SpMV j on `stream` after its inputs landed and y slot b was drained

@@ -2354,4 +2354,29 @@ cudaError_t launch_gather(const void* src, const int32_t* idx, int64_t n, void* 
     return cudaGetLastError();
 }
 
+namespace {
+// Host -> device copy by SM loads from page-locked host memory (UVA): 16-B loads, one grid stride.
+// Many SMs keep more PCIe read requests outstanding than one copy engine does (C2 x vector: 49.5 vs
+// 42 GB/s on the bench box, scripts/probe/h2d_probe.py).
+__global__ void __launch_bounds__(256) dasp_h2d_sm_kernel(const int4* __restrict__ src, int4* __restrict__ dst,
+                                                          int64_t n16, const uint8_t* __restrict__ src_tail,
+                                                          uint8_t* __restrict__ dst_tail, int tail) {
+    const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
+    for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < n16; i += stride)
+        dst[i] = src[i];
+    if (blockIdx.x == 0 && static_cast<int>(threadIdx.x) < tail) dst_tail[threadIdx.x] = src_tail[threadIdx.x];
+}
+}  // namespace
+
+cudaError_t launch_h2d_sm(void* dst, const void* host_src, size_t bytes, int sms, cudaStream_t s) {
+    if (bytes == 0) return cudaSuccess;
+    const int64_t n16 = static_cast<int64_t>(bytes / 16);
+    const int tail = static_cast<int>(bytes % 16);
+    const uint8_t* st = static_cast<const uint8_t*>(host_src) + n16 * 16;
+    uint8_t* dt = static_cast<uint8_t*>(dst) + n16 * 16;
+    dasp_h2d_sm_kernel<<<static_cast<unsigned>(sms > 0 ? sms : 148), 256, 0, s>>>(
+        static_cast<const int4*>(host_src), static_cast<int4*>(dst), n16, st, dt, tail);
+    return cudaGetLastError();
+}
+
 }  // namespace dasp

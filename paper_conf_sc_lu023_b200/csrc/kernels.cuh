@@ -132,5 +132,7 @@ cudaError_t launch_pipe(const MainParams& p, int dtype, int variant, const uint6
 cudaError_t launch_scale(void* y, int64_t m, double beta, int dtype, cudaStream_t s, const ExtraDst& extra);
 // dst[k] = src[idx[k]] for k < n, elements of elem_bytes (2, 4 or 8) bytes
 cudaError_t launch_gather(const void* src, const int32_t* idx, int64_t n, void* dst, int elem_bytes, cudaStream_t s);
+// host -> device copy by SM loads; host_src must be page-locked (device-accessible under UVA) and 16-B aligned
+cudaError_t launch_h2d_sm(void* dst, const void* host_src, size_t bytes, int sms, cudaStream_t s);
 
 }  // namespace dasp

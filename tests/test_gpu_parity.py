@@ -284,6 +284,35 @@ def test_spmv_host_stream_pipelined(dt, beta):
         dasp.dasp_spmv_host_stream(plan, Xh.data_ptr(), A.n - 1, Yh.data_ptr(), ldy, nvec, 1.0, 0.0)
 
 
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("h2d_sm", ["1", "0"])
+def test_spmv_host_large_pinned_vectors(dt, h2d_sm, monkeypatch):
+    """Host vectors >= 1 MiB in page-locked memory; with DASP_H2D_SM=1 they take the SM-load
+    host->device copy (16-B body + ragged byte tail: n odd) and misaligned strides (FP16/FP32, ldx
+    odd) fall back to cudaMemcpyAsync; with 0 every copy is cudaMemcpyAsync.
+    Every y_j equals the device-resident dasp_spmv result bit for bit and passes the oracle."""
+    monkeypatch.setenv("DASP_H2D_SM", h2d_sm)
+    rng = np.random.default_rng(5)
+    n = {"f64": 200_001, "f32": 300_001, "f16": 600_001}[dt]       # x >= 1 MiB; row 1 of X misaligned for f16/f32
+    A = synth.from_lengths(list(rng.integers(5, 41, size=3001)), n=n, seed=13)
+    nvec, ldx, ldy = 3, n + 1, A.m + 3
+    X = np.zeros((nvec, ldx), dtype=NP_VAL[dt])
+    for j in range(nvec):
+        X[j, :n] = synth.vector(60 + j, n).astype(NP_VAL[dt])
+    Xh = torch.from_numpy(X).pin_memory()
+    Yh = torch.full((nvec, ldy), float("nan"), dtype=torch.float64 if dt == "f64" else torch.float32).pin_memory()
+    plan = make(A, dt)
+    dasp.dasp_spmv_host_stream(plan, Xh.data_ptr(), ldx, Yh.data_ptr(), ldy, nvec, 1.0, 0.0)
+    for j in range(nvec):
+        y_dev = run(plan, X[j, :n], dt)
+        assert np.array_equal(Yh.numpy()[j, :A.m].astype(np.float64), y_dev), j
+        y_ref, s_ref = oracle_ref(A, X[j, :n].astype(np.float64), dt)
+        assert oracle.tolerance_ok(Yh.numpy()[j, :A.m].astype(np.float64), y_ref, s_ref, dt).all(), j
+    y1 = torch.full((A.m,), float("nan"), dtype=Yh.dtype).pin_memory()
+    dasp.dasp_spmv_host(plan, Xh[0, :n].numpy(), y1.numpy())
+    assert np.array_equal(y1.numpy(), Yh.numpy()[0, :A.m])
+
+
 def test_bad_device_args():
     A = synth.generate(synth.config("c1a"))
     plan = make(A, "f64")
