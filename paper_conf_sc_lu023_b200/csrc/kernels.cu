@@ -104,6 +104,9 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
 // x gather through the read-only path; column -1 (pad, R12) reads 0 without touching memory
 #ifndef DASP_GX_MODE
 #define DASP_GX_MODE 0   // x gathers: 0 ld.global.nc (LDG.CONSTANT), 1 + L1::evict_last, 2 ld.global.ca
+#ifndef DASP_PDL
+#define DASP_PDL 0       // programmatic dependent launch between consecutive main / long kernels
+#endif
 #endif
 // (DASP_GX_MODE 1 / 2 measured within noise on C2 / C2+ / C3 / C5, profiles/r01d/x_gather_cache_op.jsonl)
 __device__ __forceinline__ double gx(const double* x, uint32_t c) {
@@ -1494,6 +1497,10 @@ template <int DT, int VAR>
 __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_LONG_MIN_BLOCKS
                                                          : (DT == 1 ? DASP_LONG_MIN_BLOCKS_F16 : DASP_LONG_MIN_BLOCKS_F32))
 dasp_long_kernel(const MainParams P, int64_t n_units) {
+#if DASP_PDL
+    asm volatile("griddepcontrol.wait;" ::: "memory");      // the previous grid's writes are visible
+    asm volatile("griddepcontrol.launch_dependents;" :::);  // the next SpMV may be dispatched behind us
+#endif
     constexpr int UPW = DT == 1 ? DASP_LONG_UPW_F16 : 1;
     const int64_t w = ((static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5) * UPW;
     if (w >= n_units) return;
@@ -1522,6 +1529,10 @@ dasp_long_kernel(const MainParams P, int64_t n_units) {
 template <int DT, int VAR>
 __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32))
 dasp_main_kernel(const MainParams P) {
+#if DASP_PDL
+    asm volatile("griddepcontrol.wait;" ::: "memory");      // the previous grid's writes are visible
+    asm volatile("griddepcontrol.launch_dependents;" :::);  // the next SpMV may be dispatched behind us
+#endif
     const int lane = threadIdx.x & 31;
     const int64_t fin_blocks = (P.fin_warps + WARPS_PER_BLOCK - 1) / WARPS_PER_BLOCK;
     if (blockIdx.x < fin_blocks) {                       // long-row phase 2 + empty rows
@@ -2172,16 +2183,25 @@ static cudaError_t launch_ex(Kern kernel, unsigned blocks, cudaStream_t s, const
     cfg.gridDim = dim3(blocks);
     cfg.blockDim = dim3(MAIN_THREADS);
     cfg.stream = s;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
+    unsigned na = 0;
     if (apw_bytes) {
-        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-        attr[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(apw_base);
-        attr[0].val.accessPolicyWindow.num_bytes = apw_bytes;
-        attr[0].val.accessPolicyWindow.hitRatio = apw_hit;
-        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        attr[na].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[na].val.accessPolicyWindow.base_ptr = const_cast<void*>(apw_base);
+        attr[na].val.accessPolicyWindow.num_bytes = apw_bytes;
+        attr[na].val.accessPolicyWindow.hitRatio = apw_hit;
+        attr[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        ++na;
+    }
+#if DASP_PDL
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+#endif
+    if (na) {
         cfg.attrs = attr;
-        cfg.numAttrs = 1;
+        cfg.numAttrs = na;
     }
     return cudaLaunchKernelEx(&cfg, kernel, args...);
 }
@@ -2300,7 +2320,7 @@ cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_u
     auto k = dtype == 0 ? (mma ? dasp_long_kernel<0, VAR_MMA> : dasp_long_kernel<0, VAR_CUDACORE>)
            : dtype == 1 ? (mma ? dasp_long_kernel<1, VAR_MMA> : dasp_long_kernel<1, VAR_CUDACORE>)
                         : (mma ? dasp_long_kernel<2, VAR_MMA> : dasp_long_kernel<2, VAR_CUDACORE>);
-    if (apw_bytes) return launch_ex(k, grid.x, s, apw_base, apw_bytes, apw_hit, p, n_units);
+    if (apw_bytes || DASP_PDL) return launch_ex(k, grid.x, s, apw_base, apw_bytes, apw_hit, p, n_units);
     set_carveout(reinterpret_cast<const void*>(k));
     k<<<grid, block, 0, s>>>(p, n_units);
     return cudaGetLastError();
