@@ -104,6 +104,9 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
 // x gather through the read-only path; column -1 (pad, R12) reads 0 without touching memory
 #ifndef DASP_GX_MODE
 #define DASP_GX_MODE 0   // x gathers: 0 ld.global.nc (LDG.CONSTANT), 1 + L1::evict_last, 2 ld.global.ca
+#ifndef DASP_Y_ST
+#define DASP_Y_ST 0      // y stores: 0 plain, 1 st.global.cs (streaming), 2 st.global.cg
+#endif
 #ifndef DASP_PDL
 #define DASP_PDL 0       // programmatic dependent launch between consecutive main / long kernels
 #endif
@@ -238,7 +241,13 @@ __device__ __forceinline__ void store_y(const MainParams& P, int32_t row, typena
     A ra = static_cast<A>(P.alpha) * acc;                // in the accumulator type, one final rounding
     if (P.beta != 0.0) ra += static_cast<A>(P.beta) * static_cast<A>(y[row]);   // (FP32 variant, R29)
     const Y r = static_cast<Y>(ra);
+#if DASP_Y_ST == 1
+    __stcs(y + row, r);                                  // streaming store (evict-first in L1/L2)
+#elif DASP_Y_ST == 2
+    __stcg(y + row, r);                                  // cache at L2 only
+#else
     y[row] = r;
+#endif
     for (int d = 0; d < P.extra.n; ++d) static_cast<Y*>(P.extra.ptr[d])[row] = r;   // peers (scatter)
 }
 
