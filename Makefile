@@ -38,10 +38,17 @@ clean:
 
 .PHONY: all clean
 
-# experiment builds: one libdasp_<VAR=value[+VAR=value]>.so per EXPVARS entry (comma-separated -D settings)
-EXPVARS ?= DASP_NSTAGE=3 DASP_NSTAGE=4
-exp: $(OBJ)/builder.o $(OBJ)/api.o $(OBJ)/gpu_builder.o
+# experiment builds: one build/libdasp_<VAR=value[+VAR=value]>.so per EXPVARS entry (comma-separated
+# -D settings applied to every translation unit); select one with DASP_LIB=<path> (dasp.py)
+EXPVARS ?= DASP_NARROW_IL=1
+exp:
 	for v in $(EXPVARS); do \
-	  $(NVCC) $(NVFLAGS) -D$$(echo $$v | sed 's/,/ -D/g') -c $(SRC)/kernels.cu -o $(OBJ)/kernels_$$(echo $$v | tr , +).o 2> $(OBJ)/kernels_$$(echo $$v | tr , +).ptxas.txt && \
-	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$(echo $$v | tr , +).so $(OBJ)/builder.o $(OBJ)/kernels_$$(echo $$v | tr , +).o $(OBJ)/gpu_builder.o $(OBJ)/api.o -Xcompiler -fopenmp -lgomp; \
+	  t=$$(echo $$v | tr , +); d="-D$$(echo $$v | sed 's/,/ -D/g')"; mkdir -p $(OBJ)/exp_$$t; \
+	  g++ $(CXXFLAGS) $$d -c $(SRC)/builder.cpp -o $(OBJ)/exp_$$t/builder.o && \
+	  $(NVCC) $(NVFLAGS) $$d -c $(SRC)/kernels.cu -o $(OBJ)/exp_$$t/kernels.o 2> $(OBJ)/exp_$$t/kernels.ptxas.txt && \
+	  $(NVCC) $(NVFLAGS) $$d -c $(SRC)/gpu_builder.cu -o $(OBJ)/exp_$$t/gpu_builder.o 2> /dev/null && \
+	  $(NVCC) $(NVFLAGS) $$d -c $(SRC)/api.cu -o $(OBJ)/exp_$$t/api.o && \
+	  $(NVCC) $(ARCH) -shared -o $(OBJ)/libdasp_$$t.so $(OBJ)/exp_$$t/*.o -Xcompiler -fopenmp -lgomp || exit 1; \
 	done
+
+.PHONY: exp

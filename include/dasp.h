@@ -72,24 +72,15 @@ typedef struct {
                                    rows is classified, sorted and pieced on its own so x and y
                                    windows stay L2-resident; 0 = automatic, -1 = one panel
                                    (the paper's global format)                        */
-    int32_t pipeline;           /* 1: persistent kernel whose producer lane stages every item's
-                                   packed arrays in shared memory with cp.async.bulk (TMA) and
-                                   mbarriers; 0 (default): one warp per item, loads straight to
-                                   registers (faster on B200 in our measurements) */
     int32_t max_len;            /* MAX_LEN, "an adjustable parameter": long iff len >
                                    max_len; 0 = 256; must be >= 4                             */
     double threshold;           /* tau, "a customized parameter": an 8 x MMA_K block is
                                    regular iff it holds more than 8*MMA_K*tau nonzeros;
                                    0 = 0.75; must be <= 1                                     */
-    int32_t co_schedule;        /* 1: the long-row units run as blocks of the medium/short
-                                   kernel, interleaved with each panel's medium/short blocks,
-                                   and the warp that completes a long row runs its phase 2
-                                   (Alg. 2 l.17-25) -- one launch per SpMV; 0: long units in
-                                   their own launch before it; -1 (default): automatic (0)    */
 } dasp_options_t;
 
 /* Fills `opts` with the defaults: device 0, CUDA-core variant, validate, no keep_host, auto
- * LOOP_NUM, automatic panel size, direct (non-pipelined) kernel. */
+ * LOOP_NUM, automatic panel size, MAX_LEN 256, tau 0.75. */
 void dasp_options_default(dasp_options_t* opts);
 
 /* Plan statistics (Fig. 12's class shares; build cost). */
@@ -110,11 +101,9 @@ typedef struct {
     int32_t medium_rb_per_warp;
     int32_t launches_per_spmv;                         /* kernels one dasp_spmv enqueues    */
     int64_t panel_rows, n_panels;                      /* resolved panel size and count     */
-    int32_t pipeline;                                  /* 1 if the TMA-staged kernel is used */
     int64_t max_len;                                   /* resolved MAX_LEN                   */
     double threshold;                                  /* resolved tau                       */
     double build_ms, upload_ms;                        /* host build; host->device upload   */
-    int32_t co_scheduled;                              /* 1 if long units run co-scheduled   */
     int64_t rowblocks_mid, rowblocks_narrow;           /* medium row-blocks on the two-lanes-
                                                           per-row / one-lane-per-row warps
                                                           (launch schedule)    */
@@ -148,7 +137,8 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
  * double or binary16 [nnz]); classification, sorts, scans and scatters run as kernels on `stream`
  * (cudaStream_t as void*), the packed arrays are written in place in device memory and are
  * byte-identical to dasp_plan_create's.  Synchronises `stream`.  opts->device must be >= 0;
- * keep_host is ignored.  Errors as dasp_plan_create.
+ * keep_host is ignored.  nnz must equal d_row_ptr[m] (checked before any kernel reads col/val:
+ * INVALID_CSR otherwise).  Errors as dasp_plan_create.
  */
 dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz,
                                       const int64_t* d_row_ptr, const int32_t* d_col_idx, const void* d_val,
@@ -208,10 +198,7 @@ dasp_status_t dasp_spmv_host(dasp_plan_t plan, const void* x_host, void* y_host,
  * vector is copied in and its result copied out (no caching).  Results are identical to nvec
  * dasp_spmv_host calls.  Synchronises `stream` before returning; the host buffers must stay valid
  * until then and should be pinned (pageable memory serialises the copies).  Copies use
- * cudaMemcpyAsync; DASP_H2D_SM=1 in the environment makes page-locked host vectors of >= 1 MiB at
- * 16-B aligned addresses be read by SM loads over UVA instead (an experiment knob: faster alone,
- * slower inside the pipelined step).  dasp_spmv_host does the same.
- * Returns INVALID_ARG
+ * cudaMemcpyAsync on the copy engines.  Returns INVALID_ARG
  * (null plan, nvec < 0, ldx < n with x needed, ldy < m, null buffers), UNSUPPORTED (host-only plan),
  * OUT_OF_MEMORY or CUDA.
  */
@@ -275,14 +262,11 @@ dasp_status_t dasp_gather_halo(const void* src, const int32_t* idx, int64_t n, v
 
 /* Kernel ids of the per-kernel timing below. */
 typedef enum {
-    DASP_K_MAIN = 0,      /* medium + short/single kernel, panel by panel (Alg. 3-5); with
-                             options.pipeline the persistent kernel that also does the long units */
-    DASP_K_FINISH = 1,    /* long phase 2 (Alg. 2 l.17-25) + empty rows: only with options.pipeline; otherwise
-                             they are the first warps of DASP_K_MAIN */
+    DASP_K_MAIN = 0,      /* dasp_main_kernel: long phase 2 (Alg. 2 l.17-25) + empty rows as its
+                             first warps, then medium + short/single warps panel by panel (Alg. 3-5) */
+    DASP_K_LONG = 1,      /* dasp_long_kernel: long phase 1 (Alg. 2 l.1-16) */
     DASP_K_SCALE = 2,     /* alpha == 0 quick path */
-    DASP_K_LONG = 3,      /* long phase 1 (Alg. 2 l.1-16) */
-    DASP_K_SHORT = 4,     /* short tiles when they run in their own kernel (DASP_SPLIT_SHORT) */
-    DASP_K_COUNT = 5
+    DASP_K_COUNT = 3
 } dasp_kernel_t;
 
 /*

@@ -46,24 +46,9 @@ struct dasp_plan_s {
     double build_ms = 0, upload_ms = 0;
     int64_t blocks = 0;                   // grid of the medium/short kernel
     int64_t n_units = 0;                  // long units (long kernel)
-    bool split_short = false;             // short tiles in their own kernel (else in the main kernel)
-    int64_t n_tiles = 0;
-    void* d_tile_meta = nullptr;          // uint64 cat << 62 | output base, per tile (split mode)
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
-    void* d_blk_word = nullptr;           // uint64 role of every main-kernel block (kernels.cuh)
-    bool cosched = false;                 // long units co-scheduled inside the main kernel
-    void* d_long_cnt = nullptr;           // int32 per long row: groups not yet summed (co-scheduled)
-    void* d_group_row = nullptr;          // int32 per group: its long row, -1 for pad groups
+    void* d_blk_word = nullptr;           // uint64 panel of every main-kernel block (kernels.cuh)
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
-    void* d_items = nullptr;              // uint64 item words of the pipelined kernel
-    int64_t n_items = 0, pipe_blocks = 0;
-    bool pipe = false;                    // persistent TMA-staged kernel (else the one-warp-per-item kernel)
-    bool dyn = false;                     // persistent main kernel with the dynamic (atomic) schedule
-    void* d_item_start = nullptr;         // int64 [n_panels + 1] first work item of every panel
-    void* d_sched = nullptr;              // 2 x u64 counters of the dynamic schedule (self-resetting)
-    int64_t dyn_items = 0, dyn_blocks = 0;
-    size_t apw_bytes = 0;                 // L2 persisting access-policy window over x (0 = off)
-    float apw_hit = 1.0f;
     // timing
     int32_t timing_cap = 0, timing_calls = 0;
     std::vector<TimingRec> recs;
@@ -80,12 +65,23 @@ int sa(int dtype) { return dtype == DASP_R_16F ? 4 : 8; }   // long-group partia
 // automatic panel: ~1M rows keeps a panel's x window and y (8 B each per row) well inside the
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
-constexpr int kColBuckets = 16;
-constexpr int kLongOrderDefault = 1;   // long units bucketed one by one (setup_launch; 2 measured slower, profiles/r01d/interleave_long_order.jsonl)
-constexpr bool kSplitShortDefault = false;
-constexpr bool kDynSchedDefault = false;
-constexpr bool kCoschedDefault = false;  // long units inside the main kernel: measured slower
-constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // TMA windows may read up to 16 B past an array's end
+#ifndef DASP_COL_BUCKETS
+#define DASP_COL_BUCKETS 16
+#endif
+#ifndef DASP_LONG_ORDER
+#define DASP_LONG_ORDER 1   // long-unit schedule: 0 memory order, 1 column buckets per panel, 2 global buckets
+#endif
+constexpr int kColBuckets = DASP_COL_BUCKETS;
+constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read up to 16 B past an array's end
+// build knobs (experiments only; the product reads no environment): DASP_CLASS_MASK restricts the
+// main kernel to medium (2) or short (4) warps for per-class timings -- the other rows are then
+// NOT computed; DASP_NARROW_IL interleaves narrow warps (measured neutral / slower)
+#ifndef DASP_CLASS_MASK
+#define DASP_CLASS_MASK 7
+#endif
+#ifndef DASP_NARROW_IL
+#define DASP_NARROW_IL 0
+#endif
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
 // small matrices keep the paper's 1 / 2; for large ones, uniform medium rows (coefficient of
@@ -120,16 +116,8 @@ void free_device(dasp_plan_s* p) {
     if (p->d_partial) cudaFree(p->d_partial);
     if (p->d_panels) cudaFree(p->d_panels);
     if (p->d_blk_word) cudaFree(p->d_blk_word);
-    if (p->d_long_cnt) cudaFree(p->d_long_cnt);
-    if (p->d_group_row) cudaFree(p->d_group_row);
-    p->d_long_cnt = p->d_group_row = nullptr;
     if (p->d_unit_order) cudaFree(p->d_unit_order);
-    if (p->d_items) cudaFree(p->d_items);
-    if (p->d_tile_meta) cudaFree(p->d_tile_meta);
-    if (p->d_item_start) cudaFree(p->d_item_start);
-    if (p->d_sched) cudaFree(p->d_sched);
-    p->d_panels = p->d_blk_word = p->d_unit_order = p->d_items = p->d_tile_meta = nullptr;
-    p->d_item_start = p->d_sched = nullptr;
+    p->d_panels = p->d_blk_word = p->d_unit_order = nullptr;
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -179,7 +167,6 @@ int64_t alg_bytes(const dasp_plan_s* p, bool beta) {
     const int64_t nout = 64 * f.t13 + 32 * f.t4 + 64 * f.t22 + 128 * f.ts;
     int64_t b = 0;
     b += f.n_groups_padded * f.geo.G * (s_v + 4) + 2 * f.n_groups_padded * s_a + 8 * (f.row_long + 1) + 4 * f.row_long;
-    if (p->cosched) b += 4 * f.n_groups_padded;   // group_row (co-scheduled phase 2)
     b += (f.nnz_reg_new + f.nnz_irreg) * (s_v + 4) + 8 * (f.nrb + 1) + 8 * (nmp + 1) + 4 * nmp;
     b += f.nnz_short_new * (s_v + 4) + 4 * nout;
     b += 4 * f.n0;
@@ -202,10 +189,8 @@ void dasp_options_default(dasp_options_t* o) {
     o->medium_rb_per_warp = 0;
     o->num_threads = 0;
     o->panel_rows = 0;
-    o->pipeline = 0;
     o->max_len = 256;
     o->threshold = 0.75;
-    o->co_schedule = -1;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -226,8 +211,7 @@ const char* dasp_status_string(dasp_status_t s) {
 namespace {
 
 // Launch metadata shared by host- and device-built plans: LOOP_NUM, the per-panel descriptors of
-// the medium/short kernel, the long-unit schedule, the pipelined kernel's item words, and their
-// device copies.  `panel_table` (host) is the DASP_ARR_PANELS content; `unit_first_col[u]` the
+// the medium/short kernel, the long-unit schedule, and their device copies.  `panel_table` (host) is the DASP_ARR_PANELS content; `unit_first_col[u]` the
 // column of the first element of long unit u (for the column-bucket schedule).
 // narrow_slots[rb] = max(K nreg, longest row) = K nreg(rb) + irregular length of the row-block's
 // first (longest) row: the slots each of its rows spans (rows are sorted by length, so within a
@@ -249,39 +233,15 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     // (LOOP_NUM 4 or less): C5 +1 % (FP64) .. +7 % (FP16), C3 neutral; uniform stencil rows
     // (LOOP_NUM 8) keep contiguous ranges (C2+ -2 % .. -5 % interleaved; profiles/r01d/wide_interleave.jsonl)
     p->wide_il = p->rbw <= 4 ? 1 : 0;
-    if (const char* wi = std::getenv("DASP_WIDE_IL")) p->wide_il = std::atoi(wi) != 0;
-    p->narrow_il = 0;
-    if (const char* ni = std::getenv("DASP_NARROW_IL")) p->narrow_il = std::atoi(ni) != 0;
-    int64_t nrw = dasp::narrow_rb_per_warp(p->dtype);
-    {
-        const char* ne = std::getenv("DASP_NARROW");   // 0 = every row-block on the wide path (experiments)
-        if ((ne && std::atoi(ne) == 0) || static_cast<int64_t>(nslots.size()) != f.nrb) nrw = 0;
-    }
+    p->narrow_il = DASP_NARROW_IL;
+    int64_t nrw = static_cast<int64_t>(nslots.size()) == f.nrb ? dasp::narrow_rb_per_warp(p->dtype) : 0;
     // small matrices (LOOP_NUM 1) keep more warps in flight: one pass of 4 row-blocks
     if (nrw > 4 && p->rbw <= 1) nrw = 4;
-    if (const char* ev = std::getenv("DASP_NRW"))   // experiments: row-blocks per narrow warp (multiple of 4)
-        if (nrw > 0 && std::atoi(ev) >= 4) nrw = std::atoi(ev) / 4 * 4;
     p->nrw = static_cast<int>(nrw);
     p->rb_mid = p->rb_narrow = 0;
-    bool mid = true;   // two-lanes-per-row narrow warps (DASP_NARROW_MID=0: off, experiments)
-    {
-        const char* me = std::getenv("DASP_NARROW_MID");
-        if (me && std::atoi(me) == 0) mid = false;
-    }
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<uint64_t> blk_word;
-    std::vector<uint64_t> tile_meta;
-    {
-        const char* ss = std::getenv("DASP_SPLIT_SHORT");
-        p->split_short = ss ? std::atoi(ss) != 0 : kSplitShortDefault;
-        const char* cs = std::getenv("DASP_COSCHED");
-        const char* pe = std::getenv("DASP_PIPE");
-        const bool pipe_wanted = pe ? std::atoi(pe) != 0 : o.pipeline != 0;
-        p->cosched = (cs ? std::atoi(cs) != 0 : (o.co_schedule < 0 ? kCoschedDefault : o.co_schedule != 0)) &&
-                     f.n_groups_padded > 0 && !pipe_wanted;
-    }
     int64_t blk = 0;
-    std::vector<int64_t> item_start(1, 0);
     for (int64_t q = 0; q < f.n_panels; ++q) {
         const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
         dasp::PanelDesc& d = desc[q];
@@ -291,7 +251,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         if (nrw > 0)
             while (d.rbn > 0 && nslots[d.rb0 + d.rbn - 1] <= dasp::narrow_max_slots(f.geo.K)) --d.rbn;
         d.rbm = d.rbn;
-        if (nrw > 0 && mid)
+        if (nrw > 0)
             while (d.rbm > 0 && nslots[d.rb0 + d.rbm - 1] <= dasp::mid_max_slots(f.geo.K)) --d.rbm;
         d.nmwd = (d.rbm + p->rbw - 1) / p->rbw;
         d.nmwm = d.nmwd + (nrw > 0 ? (d.rbn - d.rbm + nrw - 1) / nrw : 0);
@@ -299,36 +259,14 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         p->rb_mid += d.rbn - d.rbm;
         p->rb_narrow += d.nrb - d.rbn;
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
-        if (p->split_short) {   // tiles leave the main kernel; per-tile metadata for the short kernel
-            for (int64_t t = 0; t < d.t13 + d.t4 + d.t22 + d.ts; ++t) {
-                uint64_t cat;
-                int64_t ob;
-                if (t < d.t13) { cat = 0; ob = d.out0 + t * 64; }
-                else if (t < d.t13 + d.t4) { cat = 1; ob = d.out0 + 64 * d.t13 + (t - d.t13) * 32; }
-                else if (t < d.t13 + d.t4 + d.t22) { cat = 2; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + (t - d.t13 - d.t4) * 64; }
-                else { cat = 3; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + 64 * d.t22 + (t - d.t13 - d.t4 - d.t22) * 128; }
-                tile_meta.push_back((cat << 62) | static_cast<uint64_t>(ob));
-            }
-            d.t13 = d.t4 = d.t22 = d.ts = 0;
-        }
         const int64_t tpw = dasp::short_tiles_per_warp(p->dtype);
         const int64_t warps = d.nmw + (d.t13 + d.t4 + d.t22 + d.ts + tpw - 1) / tpw;   // long units: own kernel
-        item_start.push_back(item_start.back() + warps);
         const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
-        // co-scheduled: the panel's long blocks are spread evenly among its main blocks, so the
-        // SMs always hold a mix of HBM-streaming long units and latency-bound medium/short warps
-        const int64_t nl = p->cosched ? (d.nunits + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK : 0;
-        int64_t il = 0, im = 0;
-        for (int64_t i = 0; i < nl + nb; ++i) {
-            const bool is_long = (i + 1) * nl / (nl + nb) > i * nl / (nl + nb);
-            const uint64_t idx = static_cast<uint64_t>(is_long ? il++ : im++);
-            blk_word.push_back((is_long ? (1ull << 63) : 0ull) | (static_cast<uint64_t>(q) << 32) | idx);
-        }
-        blk += nb + nl;
+        for (int64_t i = 0; i < nb; ++i) blk_word.push_back((static_cast<uint64_t>(q) << 32) | static_cast<uint64_t>(i));
+        blk += nb;
     }
     p->blocks = blk;
     p->n_units = f.n_groups_padded / f.geo.UG;
-    p->n_tiles = static_cast<int64_t>(tile_meta.size());
     // long-unit execution order (a launch schedule, not part of the format): inside each panel
     // the units run bucketed by the column of their first element, so that the warps in flight
     // gather from ~1/kColBuckets of x at a time instead of all of it (long rows' columns are
@@ -336,13 +274,12 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     // group order by the finish kernel: the result is bitwise independent of this order.
     std::vector<int32_t> unit_order(static_cast<size_t>(p->n_units));
     {
-        // DASP_LONG_ORDER: 0 = memory order, 1 (default) = bucketed per unit, 2 = bucketed per run
-        // of WARPS_PER_BLOCK consecutive units, so the warps of one block still stream one
-        // contiguous region (bucketed by the run's first unit)
-        const char* lo_env = std::getenv("DASP_LONG_ORDER");
-        const int mode = f.n > 0 ? (lo_env ? std::atoi(lo_env) : kLongOrderDefault) : 0;
-        const int64_t run = mode == 2 ? dasp::WARPS_PER_BLOCK : 1;
-        for (const auto& d : desc) {
+        // memory order when there is no column space to bucket (n = 0)
+        const int mode = f.n > 0 ? DASP_LONG_ORDER : 0;
+        std::vector<dasp::PanelDesc> all(1);   // global order: one pseudo-panel over every unit
+        all[0].unit0 = 0;
+        all[0].nunits = p->n_units;
+        for (const auto& d : (mode == 2 ? all : desc)) {
             std::vector<int64_t> cnt(kColBuckets + 1, 0);
             auto bucket = [&](int64_t u) {
                 const int32_t c = unit_first_col[u];
@@ -352,40 +289,11 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
                 for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + w] = static_cast<int32_t>(d.unit0 + w);
                 continue;
             }
-            for (int64_t w = 0; w < d.nunits; w += run) cnt[bucket(d.unit0 + w) + 1] += std::min(run, d.nunits - w);
+            for (int64_t w = 0; w < d.nunits; ++w) ++cnt[bucket(d.unit0 + w) + 1];
             for (int b = 0; b < kColBuckets; ++b) cnt[b + 1] += cnt[b];
-            for (int64_t w = 0; w < d.nunits; w += run) {
-                const int b = bucket(d.unit0 + w);
-                for (int64_t k = w; k < std::min(w + run, d.nunits); ++k) unit_order[d.unit0 + cnt[b]++] = static_cast<int32_t>(d.unit0 + k);
-            }
+            for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + cnt[bucket(d.unit0 + w)]++] = static_cast<int32_t>(d.unit0 + w);
         }
     }
-    // item words of the pipelined kernel, panel by panel: long units (schedule order), medium
-    // row-blocks, short tiles (kind<<62 | payload; kernels.cu produce())
-    std::vector<uint64_t> items;
-    bool items_ok = true;
-    const char* pe = std::getenv("DASP_PIPE");   // overrides the option (experiments)
-    const bool want_pipe = pe ? std::atoi(pe) != 0 : o.pipeline != 0;
-    if (want_pipe) {
-        for (const auto& d : desc) {
-            for (int64_t w = 0; w < d.nunits; ++w) items.push_back((1ull << 62) | static_cast<uint64_t>(unit_order[d.unit0 + w]));
-            for (int64_t r = 0; r < d.nrb; ++r) items.push_back((2ull << 62) | static_cast<uint64_t>(d.rb0 + r));
-            const int64_t nt = d.t13 + d.t4 + d.t22 + d.ts;
-            for (int64_t t = 0; t < nt; ++t) {
-                int64_t cat, ob;
-                if (t < d.t13) { cat = 0; ob = d.out0 + t * 64; }
-                else if (t < d.t13 + d.t4) { cat = 1; ob = d.out0 + 64 * d.t13 + (t - d.t13) * 32; }
-                else if (t < d.t13 + d.t4 + d.t22) { cat = 2; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + (t - d.t13 - d.t4) * 64; }
-                else { cat = 3; ob = d.out0 + 64 * d.t13 + 32 * d.t4 + 64 * d.t22 + (t - d.t13 - d.t4 - d.t22) * 128; }
-                const int64_t tile = d.tile0 + t;
-                if (tile >= (int64_t(1) << 27) || ob >= (int64_t(1) << 33)) items_ok = false;
-                items.push_back((3ull << 62) | (static_cast<uint64_t>(cat) << 60) | (static_cast<uint64_t>(tile) << 33) |
-                                static_cast<uint64_t>(ob));
-            }
-        }
-    }
-    p->n_items = static_cast<int64_t>(items.size());
-    p->pipe = want_pipe && items_ok && p->dtype != DASP_R_32F;   // the staged kernel covers FP64 / FP16
     if (p->device < 0) return DASP_OK;
 
     auto upload = [&](void** dst, const void* src, size_t bytes) -> dasp_status_t {
@@ -401,72 +309,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
     if ((st = upload(&p->d_blk_word, blk_word.data(), blk_word.size() * 8)) != DASP_OK) return st;
     if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
-    if (p->split_short && (st = upload(&p->d_tile_meta, tile_meta.data(), tile_meta.size() * 8)) != DASP_OK) return st;
-    if (p->pipe) {
-        int bps = 0, nsm = 0;
-        if ((st = upload(&p->d_items, items.data(), items.size() * 8)) != DASP_OK) return st;
-        if (dasp::pipe_occupancy(p->dtype, DASP_VARIANT_CUDACORE, &bps) != cudaSuccess ||   // sets both kernels'
-            dasp::pipe_occupancy(p->dtype, DASP_VARIANT_MMA, &bps) != cudaSuccess ||        // smem attribute
-            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess)
-            return DASP_ERR_CUDA;
-        // persistent grid: every SM full, never more warps than items
-        const int64_t wpb = dasp::pipe_warps_per_block();
-        p->pipe_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (p->n_items + wpb - 1) / wpb);
-    }
-    // dynamic schedule of the main kernel (DASP_SCHED=1 / options)
-    {
-        const char* se = std::getenv("DASP_SCHED");
-        p->dyn = (se ? std::atoi(se) == 1 : kDynSchedDefault) && !p->cosched;
-        p->dyn_items = item_start.back();
-        const int64_t all_items = p->dyn_items + dasp::finish_warps(f.row_long, f.n0);
-        if (p->dyn && !p->pipe && all_items > 0) {
-            int bps = 0, nsm = 0;
-            if (dasp::main_dyn_occupancy(p->dtype, p->variant, &bps) != cudaSuccess ||
-                cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device) != cudaSuccess)
-                return DASP_ERR_CUDA;
-            const int64_t wpb = dasp::WARPS_PER_BLOCK;
-            p->dyn_blocks = std::min<int64_t>(static_cast<int64_t>(std::max(bps, 1)) * nsm, (all_items + wpb - 1) / wpb);
-            if ((st = upload(&p->d_item_start, item_start.data(), item_start.size() * 8)) != DASP_OK) return st;
-            const uint64_t zero[2] = {0, 0};
-            if ((st = upload(&p->d_sched, zero, sizeof(zero))) != DASP_OK) return st;
-        } else {
-            p->dyn = false;
-        }
-    }
-    // optional persisting L2 access-policy window over x (DASP_X_APW=1; measured slower on C3,
-    // profiles/r01, so off by default)
-    const char* apw = std::getenv("DASP_X_APW");
-    if (apw && std::atoi(apw) > 0) {
-        cudaDeviceProp prop;
-        if (cudaGetDeviceProperties(&prop, p->device) == cudaSuccess && prop.persistingL2CacheMaxSize > 0) {
-            const size_t xb = static_cast<size_t>(f.n) * sx(p->dtype);
-            size_t lim = std::min<size_t>(static_cast<size_t>(prop.persistingL2CacheMaxSize), xb);
-            size_t win = std::min<size_t>(static_cast<size_t>(prop.accessPolicyMaxWindowSize), xb);
-            if (lim > 0 && win > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim) == cudaSuccess) {
-                p->apw_bytes = win;
-                p->apw_hit = std::min(1.0f, static_cast<float>(lim) / static_cast<float>(win));
-                if (const char* h = std::getenv("DASP_X_APW_HIT")) p->apw_hit = static_cast<float>(std::atof(h));
-            }
-        }
-        cudaGetLastError();
-    }
     return DASP_OK;
-}
-
-// co-scheduled mode: per-row group counters and per-group rows, from the device group_ptr
-dasp_status_t init_cosched(dasp_plan_s* p) {
-    const HostFormat& f = p->host;
-    if (!p->cosched || p->device < 0) return DASP_OK;
-    const size_t cb = static_cast<size_t>(std::max<int64_t>(f.row_long, 1)) * 4;
-    const size_t gb = static_cast<size_t>(std::max<int64_t>(f.n_groups_padded, 1)) * 4;
-    if (cudaMalloc(&p->d_long_cnt, cb) != cudaSuccess || cudaMalloc(&p->d_group_row, gb) != cudaSuccess)
-        return DASP_ERR_OUT_OF_MEMORY;
-    p->device_bytes += static_cast<int64_t>(cb + gb);
-    if (cudaMemset(p->d_group_row, 0xff, gb) != cudaSuccess) return DASP_ERR_CUDA;
-    if (dasp::launch_long_meta(static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]), f.row_long,
-                               static_cast<int32_t*>(p->d_long_cnt), static_cast<int32_t*>(p->d_group_row), nullptr) != cudaSuccess)
-        return DASP_ERR_CUDA;
-    return cudaDeviceSynchronize() == cudaSuccess ? DASP_OK : DASP_ERR_CUDA;
 }
 
 dasp_status_t check_create_args(dasp_plan_t* plan_out, int64_t m, int64_t n, int64_t nnz, const void* row_ptr,
@@ -484,10 +327,8 @@ dasp_status_t check_create_args(dasp_plan_t* plan_out, int64_t m, int64_t n, int
 }
 
 int64_t resolve_panel_rows(const dasp_options_t& o) {
-    // panel size (R28): -1 one panel (the paper's global format); 0 automatic; env override
-    int64_t panel_rows = o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
-    if (const char* pr = std::getenv("DASP_PANEL_ROWS")) panel_rows = std::atoll(pr);
-    return panel_rows;
+    // panel size (R28): -1 one panel (the paper's global format); 0 automatic
+    return o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
 }
 
 dasp_status_t fail(dasp_plan_s* p, dasp_status_t st) {
@@ -563,7 +404,6 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         auto u1 = std::chrono::steady_clock::now();
         p->upload_ms = std::chrono::duration<double, std::milli>(u1 - u0).count();
         if (!p->keep_host) f.release();
-        if ((st = init_cosched(p)) != DASP_OK) return fail(p, st);
     }
     *plan_out = p;
     return DASP_OK;
@@ -585,7 +425,7 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
     DeviceGuard guard(p->device);
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     auto t0 = std::chrono::steady_clock::now();
-    int bst = dasp::build_format_device(p->host, p->d, dtype, m, n, d_row_ptr, d_col_idx, d_val, o.validate != 0,
+    int bst = dasp::build_format_device(p->host, p->d, dtype, m, n, nnz, d_row_ptr, d_col_idx, d_val, o.validate != 0,
                                         resolve_panel_rows(o), o.max_len, o.threshold, s);
     auto t1 = std::chrono::steady_clock::now();
     p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
@@ -594,7 +434,6 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
         return static_cast<dasp_status_t>(bst);
     }
     HostFormat& f = p->host;
-    if (f.nnz != nnz) return fail(p, DASP_ERR_INVALID_CSR);
     for (int a = 0; a < DASP_ARR_COUNT; ++a) {
         p->bytes[a] = f.arr[a].bytes;
         p->device_bytes += p->bytes[a];
@@ -617,7 +456,6 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
     }
     st = setup_launch(p, o, f.panel_table.data(), first_col, nslots);
     if (st != DASP_OK) return fail(p, st);
-    if ((st = init_cosched(p)) != DASP_OK) return fail(p, st);
     *plan_out = p;
     return DASP_OK;
 }
@@ -689,63 +527,24 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.wide_il = p->wide_il;
     mp.narrow_il = p->narrow_il;
     mp.nrw = p->nrw;
-    mp.class_mask = 7;
     mp.extra = extra;
-    mp.item_start = static_cast<const int64_t*>(p->d_item_start);
-    mp.sched = static_cast<unsigned long long*>(p->d_sched);
-    mp.group_row = static_cast<const int32_t*>(p->d_group_row);
-    mp.long_cnt = p->cosched ? static_cast<int32_t*>(p->d_long_cnt) : nullptr;   // null: no phase 2 in the units
-    // DASP_PROFILE_CLASS (profiling only; the other classes' rows are then NOT computed):
-    // 1 = long units, 2 = medium warps, 3 = short tiles
-    if (const char* pc = std::getenv("DASP_PROFILE_CLASS")) {
-        const int c = std::atoi(pc);
-        if (c >= 1 && c <= 3) mp.class_mask = 1 << (c - 1);
-    }
-    if (!p->pipe && !p->cosched && p->n_units > 0 && (mp.class_mask & 1)) {
-        e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s, x, p->apw_bytes, p->apw_hit); });
-        if (e != cudaSuccess) return DASP_ERR_CUDA;
-    }
-    if (!p->pipe && p->split_short && p->n_tiles > 0 && (mp.class_mask & 4)) {
-        e = timed(p, DASP_K_SHORT, s, on, [&] {
-            return dasp::launch_short(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_tile_meta), p->n_tiles, s);
-        });
+    mp.class_mask = DASP_CLASS_MASK;
+    if (p->n_units > 0) {
+        e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s); });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }
     const int64_t n0 = (beta == 1.0 && extra.n == 0) ? 0 : f.n0;   // scatter mode must still copy them
     // long-row phase 2 and the empty rows run as the first warps of the main kernel (the long
-    // kernel before it has written every partial); only the pipelined kernel keeps a finish launch
+    // kernel before it has written every partial)
     mp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
     mp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
     mp.empty_rows = static_cast<const int32_t*>(p->d[DASP_ARR_EMPTY_ROWS]);
-    // co-scheduled: phase 2 runs in the long units' completion (kernels.cu long_unit_complete),
-    // so the fin warps only write the empty rows
-    mp.row_long = p->cosched ? 0 : f.row_long;
+    mp.row_long = f.row_long;
     mp.n0 = n0;
-    mp.fin_warps = (!p->pipe && (mp.class_mask & 1)) ? dasp::finish_warps(mp.row_long, n0) : 0;
+    mp.fin_warps = dasp::finish_warps(mp.row_long, n0);
     const int64_t fin_blocks = (mp.fin_warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
-    e = timed(p, DASP_K_MAIN, s, on, [&] {
-        if (p->pipe)
-            return dasp::launch_pipe(mp, p->dtype, variant, static_cast<const uint64_t*>(p->d_items), p->n_items,
-                                     p->pipe_blocks, s);
-        if (p->dyn) return dasp::launch_main_dyn(mp, p->dtype, variant, p->dyn_blocks, mp.fin_warps + p->dyn_items, s);
-        return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s, x, p->apw_bytes, p->apw_hit);
-    });
+    e = timed(p, DASP_K_MAIN, s, on, [&] { return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s); });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
-    if (p->pipe && f.row_long + n0 > 0) {
-        dasp::FinishParams fp;
-        fp.partial = p->d_partial;
-        fp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
-        fp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
-        fp.empty_rows = static_cast<const int32_t*>(p->d[DASP_ARR_EMPTY_ROWS]);
-        fp.y = y;
-        fp.alpha = alpha;
-        fp.beta = beta;
-        fp.row_long = f.row_long;
-        fp.n0 = n0;
-        fp.extra = extra;
-        e = timed(p, DASP_K_FINISH, s, on, [&] { return dasp::launch_finish(fp, p->dtype, s); });
-        if (e != cudaSuccess) return DASP_ERR_CUDA;
-    }
     return DASP_OK;
 }
 
@@ -753,25 +552,9 @@ dasp_status_t dasp_spmv(dasp_plan_t p, const void* x, void* y, double alpha, dou
     return dasp_spmv_ex(p, x, y, alpha, beta, stream, DASP_VARIANT_DEFAULT);
 }
 
-// Host -> device copy of a caller's buffer: cudaMemcpyAsync (copy engine).  DASP_H2D_SM=1 in the
-// environment (read per call) instead reads page-locked host memory (device-accessible under UVA) of
-// >= 1 MiB at a 16-B aligned address with SM loads (dasp::launch_h2d_sm).  Alone that copy runs at
-// 49.5 GB/s against 42 GB/s (scripts/probe/h2d_probe.py), but inside the e2e step it shares the SMs
-// with the SpMV and the step got slower (C2 FP64 e2e 220 vs 283 GFLOPS, profiles/r01e/h2d_ab.jsonl):
-// off by default.
+// Host -> device copy of a caller's buffer (copy engine; SM loads over UVA measured slower inside the
+// pipelined e2e step)
 static cudaError_t copy_h2d(void* dst, const void* src, size_t bytes, cudaStream_t s) {
-    const char* env = std::getenv("DASP_H2D_SM");
-    const int sm_mode = env ? std::atoi(env) : 0;
-    if (sm_mode && bytes >= (1u << 20) && (reinterpret_cast<uintptr_t>(src) & 15) == 0) {
-        cudaPointerAttributes a{};
-        if (cudaPointerGetAttributes(&a, src) == cudaSuccess && a.type == cudaMemoryTypeHost && a.devicePointer) {
-            int dev = 0, sms = 0;
-            if (cudaGetDevice(&dev) == cudaSuccess &&
-                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && sms > 0)
-                return dasp::launch_h2d_sm(dst, a.devicePointer, bytes, sms, s);
-        }
-        cudaGetLastError();   // a failed attribute query is not an error of this call
-    }
     return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s);
 }
 
@@ -879,13 +662,9 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta0 = alg_bytes(p, false);
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
-    o->launches_per_spmv = p->pipe ? (p->n_items > 0 ? 1 : 0) + (f.row_long + f.n0 > 0 ? 1 : 0)
-                                   : (p->n_units > 0 && !p->cosched ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0) +
-                                         (p->n_tiles > 0 ? 1 : 0);
+    o->launches_per_spmv = (p->n_units > 0 ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
-    o->pipeline = p->pipe ? 1 : 0;
-    o->co_scheduled = p->cosched ? 1 : 0;
     o->rowblocks_mid = p->rb_mid;
     o->rowblocks_narrow = p->rb_narrow;
     o->narrow_rb_per_warp = p->nrw;

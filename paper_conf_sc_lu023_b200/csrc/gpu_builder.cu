@@ -326,9 +326,12 @@ int bits_for(uint64_t maxkey) {
     return b;
 }
 
-// DASP_GB_TRACE=1 prints the time of every builder phase (stderr)
+// build knob DASP_GB_TRACE=1 prints the time of every builder phase (stderr)
+#ifndef DASP_GB_TRACE
+#define DASP_GB_TRACE 0
+#endif
 struct Trace {
-    bool on = std::getenv("DASP_GB_TRACE") != nullptr;
+    bool on = DASP_GB_TRACE != 0;
     cudaStream_t s;
     std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
     void operator()(const char* what) {
@@ -554,9 +557,9 @@ cudaError_t gather_unit_first_col(const int32_t* d_long_col, int64_t unit_elems,
     return d2h(host_out, tmp.p, n_units * 4, s);
 }
 
-int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, int64_t n, const int64_t* d_row_ptr,
-                        const int32_t* d_col, const void* d_val, bool validate, int64_t panel_rows, int64_t max_len,
-                        double tau, cudaStream_t s) {
+int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, int64_t n, int64_t nnz,
+                        const int64_t* d_row_ptr, const int32_t* d_col, const void* d_val, bool validate,
+                        int64_t panel_rows, int64_t max_len, double tau, cudaStream_t s) {
     f = HostFormat{};
     f.geo = geometry(dtype);
     f.dtype = dtype;
@@ -567,6 +570,8 @@ int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, in
     if (f.max_len < 4 || f.tau > 1.0) return DASP_ERR_INVALID_ARG;
     f.panel_rows = (panel_rows <= 0 || panel_rows >= m) ? std::max<int64_t>(m, 1) : panel_rows;
     if (d2h(&f.nnz, d_row_ptr + m, 8, s) != cudaSuccess) return DASP_ERR_CUDA;
+    // every kernel below reads col / val up to row_ptr[m]: it must be the caller's array length
+    if (f.nnz != nnz) return DASP_ERR_INVALID_CSR;
     if (validate) {
         int64_t r0 = 0;
         if (d2h(&r0, d_row_ptr, 8, s) != cudaSuccess) return DASP_ERR_CUDA;

@@ -6,15 +6,16 @@
 
 namespace dasp {
 
-constexpr int64_t kDeviceArrayPad = 64;   // every device array gets this tail (16-B TMA windows)
+constexpr int64_t kDeviceArrayPad = 64;   // every device array gets this tail (vector loads past the end)
 
 // Builds the format from a device CSR (d_row_ptr[m+1], d_col[nnz], d_val[nnz] on the current
 // device) straight into device arrays d_arrays[DASP_ARR_COUNT] (cudaMalloc'ed here, byte sizes in
-// f.arr[a].bytes, host pointers null) and fills f's counts and f.panel_table.  Returns a
-// dasp_status_t; on error nothing stays allocated.
-int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, int64_t n, const int64_t* d_row_ptr,
-                        const int32_t* d_col, const void* d_val, bool validate, int64_t panel_rows, int64_t max_len,
-                        double tau, cudaStream_t s);
+// f.arr[a].bytes, host pointers null) and fills f's counts and f.panel_table.  nnz is the length of
+// d_col / d_val: DASP_ERR_INVALID_CSR unless d_row_ptr[m] == nnz (checked before any kernel reads
+// them).  Returns a dasp_status_t; on error nothing stays allocated.
+int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, int64_t n, int64_t nnz,
+                        const int64_t* d_row_ptr, const int32_t* d_col, const void* d_val, bool validate,
+                        int64_t panel_rows, int64_t max_len, double tau, cudaStream_t s);
 
 // host_out[u] = long_col[u * unit_elems] for u < n_units (device gather + one copy)
 cudaError_t gather_unit_first_col(const int32_t* d_long_col, int64_t unit_elems, int64_t n_units, int32_t* host_out,

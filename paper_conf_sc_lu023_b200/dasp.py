@@ -17,8 +17,8 @@ LIB_PATH = os.environ.get("DASP_LIB", os.path.join(_HERE, "libdasp.so"))   # ove
 
 DASP_R_64F, DASP_R_16F, DASP_R_32F = 0, 1, 2
 DASP_VARIANT_DEFAULT, DASP_VARIANT_MMA, DASP_VARIANT_CUDACORE = 0, 1, 2
-DASP_K_MAIN, DASP_K_FINISH, DASP_K_SCALE, DASP_K_LONG, DASP_K_SHORT, DASP_K_COUNT = 0, 1, 2, 3, 4, 5
-KERNEL_NAMES = ["dasp_main_kernel", "dasp_finish_kernel", "dasp_scale_kernel", "dasp_long_kernel", "dasp_short_kernel"]
+DASP_K_MAIN, DASP_K_LONG, DASP_K_SCALE, DASP_K_COUNT = 0, 1, 2, 3
+KERNEL_NAMES = ["dasp_main_kernel", "dasp_long_kernel", "dasp_scale_kernel"]
 
 ARRAYS = ["long_val", "long_col", "group_ptr", "long_out", "rb_ptr", "reg_val", "reg_col", "irr_ptr",
           "irr_val", "irr_col", "med_out", "short_val", "short_col", "short_out", "empty_rows", "panels"]
@@ -43,8 +43,8 @@ class DaspError(RuntimeError):
 class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("variant", ctypes.c_int32), ("validate", ctypes.c_int32),
                 ("keep_host", ctypes.c_int32), ("medium_rb_per_warp", ctypes.c_int32),
-                ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64), ("pipeline", ctypes.c_int32),
-                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double), ("co_schedule", ctypes.c_int32)]
+                ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64),
+                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -56,9 +56,9 @@ class PlanInfo(ctypes.Structure):
                    "nnz_long_new", "nnz_reg_new", "nnz_irreg", "nnz_short_new", "nnz_long", "nnz_medium",
                    "nnz_short", "device_bytes", "alg_bytes_beta0", "alg_bytes_beta1")] + \
                [("medium_rb_per_warp", ctypes.c_int32), ("launches_per_spmv", ctypes.c_int32),
-                ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64), ("pipeline", ctypes.c_int32),
+                ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64),
                 ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
-                ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double), ("co_scheduled", ctypes.c_int32),
+                ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double),
                 ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32)]
 
     def as_dict(self):
@@ -161,14 +161,12 @@ class Plan:
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                      variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, keep_host: bool = False,
                      medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0,
-                     pipeline: bool = False, max_len: int = 256, threshold: float = 0.75,
-                     co_schedule: int = -1) -> Plan:
+                     max_len: int = 256, threshold: float = 0.75) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
     (dtype "f16"; passed as binary16 bits) or float32[nnz] (dtype "f32").  panel_rows: 0 automatic,
-    -1 one global panel.  co_schedule: 1 long-row units inside the medium/short kernel (one
-    launch), 0 in their own launch, -1 automatic."""
+    -1 one global panel."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     if dtype == "f64":
@@ -185,14 +183,15 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     if len(row_ptr) != m + 1:
         raise ValueError("row_ptr must have m+1 entries")
     nnz = int(row_ptr[-1]) if m >= 0 else 0
+    # the C call trusts nnz: both arrays must hold it (a short array would be read past its end)
+    if len(col_idx) != len(val) or len(col_idx) < nnz:
+        raise ValueError(f"col_idx ({len(col_idx)}) and val ({len(val)}) must both hold row_ptr[m] = {nnz} entries")
     opts = Options()
     _lib.dasp_options_default(ctypes.byref(opts))
     opts.device, opts.variant, opts.validate = device, variant, int(validate)
     opts.keep_host, opts.medium_rb_per_warp, opts.num_threads = int(keep_host), medium_rb_per_warp, num_threads
     opts.panel_rows = panel_rows
-    opts.pipeline = int(pipeline)
     opts.max_len, opts.threshold = int(max_len), float(threshold)
-    opts.co_schedule = int(co_schedule)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))
@@ -202,8 +201,8 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
 
 def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                             variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, medium_rb_per_warp: int = 0,
-                            panel_rows: int = 0, pipeline: bool = False, max_len: int = 256, threshold: float = 0.75,
-                            stream=None, co_schedule: int = -1) -> Plan:
+                            panel_rows: int = 0, max_len: int = 256, threshold: float = 0.75,
+                            stream=None) -> Plan:
     """Build the plan on the GPU from a device CSR (torch CUDA tensors: int64 row_ptr, int32
     col_idx, float64 / float16 val) -- SURVEY.md §8(f) f2."""
     import torch
@@ -213,12 +212,13 @@ def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = 
             raise ValueError("dasp_plan_create_device needs contiguous CUDA tensors (int64, int32, value dtype)")
     if row_ptr.numel() != m + 1:
         raise ValueError("row_ptr must have m+1 entries")
+    if val.numel() != col_idx.numel():
+        raise ValueError("col_idx and val must have the same length")
     opts = Options()
     _lib.dasp_options_default(ctypes.byref(opts))
     opts.device, opts.variant, opts.validate = device, variant, int(validate)
-    opts.medium_rb_per_warp, opts.panel_rows, opts.pipeline = medium_rb_per_warp, panel_rows, int(pipeline)
+    opts.medium_rb_per_warp, opts.panel_rows = medium_rb_per_warp, panel_rows
     opts.max_len, opts.threshold = int(max_len), float(threshold)
-    opts.co_schedule = int(co_schedule)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create_device(ctypes.byref(h), m, n, int(col_idx.numel()), _ptr(row_ptr), _ptr(col_idx),
                                       _ptr(val), {"f64": DASP_R_64F, "f16": DASP_R_16F, "f32": DASP_R_32F}[dtype],
@@ -226,6 +226,48 @@ def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = 
                                       _stream_ptr(stream))
     _check(st, "dasp_plan_create_device")
     return Plan(h, dtype, m, n)
+
+
+def _xy_dtypes(dtype):
+    """(x, y) torch dtypes of a plan dtype."""
+    import torch
+    return {"f64": (torch.float64, torch.float64), "f16": (torch.float16, torch.float32),
+            "f32": (torch.float32, torch.float32)}[dtype]
+
+
+def _xy_np(dtype):
+    """(x, y) numpy dtypes of a plan dtype."""
+    return {"f64": (np.float64, np.float64), "f16": (np.float16, np.float32), "f32": (np.float32, np.float32)}[dtype]
+
+
+def _check_host(a, need, want, name):
+    """A host buffer passed by pointer to the C call: a numpy array or a CPU torch tensor of the
+    plan's element type, contiguous, with at least `need` elements (the library reads / writes
+    exactly that many).  Raw integer pointers are the caller's responsibility."""
+    if isinstance(a, int):
+        return
+    if isinstance(a, np.ndarray):
+        ok = a.dtype == np.dtype(want) and a.flags.c_contiguous and a.size >= need
+        got = f"{a.dtype}[{a.size}]"
+    else:
+        import torch
+        tw = {np.float64: torch.float64, np.float32: torch.float32, np.float16: torch.float16}[want]
+        ok = (isinstance(a, torch.Tensor) and not a.is_cuda and a.dtype == tw and a.is_contiguous()
+              and a.numel() >= need)
+        got = f"{getattr(a, 'dtype', type(a))}[{a.numel() if isinstance(a, torch.Tensor) else '?'}]"
+    if not ok:
+        raise ValueError(f"{name}: need a contiguous host {np.dtype(want).name} buffer of >= {need} elements, got {got}")
+
+
+def _default_stream(plan, stream):
+    """stream=None means torch's current stream on the plan's device (not the legacy NULL stream,
+    which torch's pool streams do not synchronise with)."""
+    if stream is not None:
+        return stream
+    import torch
+    if not hasattr(plan, "_dev"):
+        plan._dev = plan.info["device"]
+    return torch.cuda.current_stream(plan._dev)
 
 
 def _check_vec(t, length, want_dtype, name, plan_device):
@@ -240,15 +282,15 @@ def _check_vec(t, length, want_dtype, name, plan_device):
 
 def dasp_spmv(plan: Plan, x, y, alpha: float = 1.0, beta: float = 0.0, stream=None,
               variant: int = DASP_VARIANT_DEFAULT, check: bool = True):
-    """y = alpha*A*x + beta*y on the plan's device (x, y torch CUDA tensors; enqueue only)."""
+    """y = alpha*A*x + beta*y on the plan's device (x, y torch CUDA tensors; enqueue only on
+    `stream`, default torch's current stream)."""
     if check:
-        import torch
         dev = plan.info["device"] if not hasattr(plan, "_dev") else plan._dev
         plan._dev = dev
-        xd, yd = {"f64": (torch.float64, torch.float64), "f16": (torch.float16, torch.float32),
-                  "f32": (torch.float32, torch.float32)}[plan.dtype]
+        xd, yd = _xy_dtypes(plan.dtype)
         _check_vec(x, plan.n, xd, "x", dev)
         _check_vec(y, plan.m, yd, "y", dev)
+    stream = _default_stream(plan, stream)
     st = _lib.dasp_spmv_ex(plan.handle, _ptr(x), _ptr(y), float(alpha), float(beta), _stream_ptr(stream), variant)
     _check(st, "dasp_spmv")
 
@@ -256,6 +298,7 @@ def dasp_spmv(plan: Plan, x, y, alpha: float = 1.0, beta: float = 0.0, stream=No
 def dasp_spmv_scatter(plan: Plan, x, dsts, alpha: float = 1.0, beta: float = 0.0, stream=None):
     """y = alpha*A*x + beta*y written to every pointer of `dsts` (dsts[0] is this GPU's y; the rest
     are raw device pointers or tensors, e.g. peer x buffers mapped over NVLink)."""
+    stream = _default_stream(plan, stream)
     ptrs = (ctypes.c_void_p * len(dsts))(*[_ptr(d) for d in dsts])
     st = _lib.dasp_spmv_scatter(plan.handle, _ptr(x), ptrs, len(dsts), float(alpha), float(beta), _stream_ptr(stream))
     _check(st, "dasp_spmv_scatter")
@@ -263,6 +306,11 @@ def dasp_spmv_scatter(plan: Plan, x, dsts, alpha: float = 1.0, beta: float = 0.0
 
 def dasp_spmv_host(plan: Plan, x: np.ndarray, y: np.ndarray, alpha: float = 1.0, beta: float = 0.0, stream=None):
     """End-to-end call with host buffers (copies inside; synchronises)."""
+    xt, yt = _xy_np(plan.dtype)
+    if alpha != 0.0 and plan.n > 0:
+        _check_host(x, plan.n, xt, "x")
+    _check_host(y, plan.m, yt, "y")
+    stream = _default_stream(plan, stream)
     st = _lib.dasp_spmv_host(plan.handle, _ptr(x), _ptr(y), float(alpha), float(beta), _stream_ptr(stream))
     _check(st, "dasp_spmv_host")
 
@@ -271,6 +319,14 @@ def dasp_spmv_host_stream(plan: Plan, x, ldx: int, y, ldy: int, nvec: int, alpha
                           stream=None):
     """nvec end-to-end SpMVs with host buffers (vectors at strides ldx / ldy elements), H2D / SpMV / D2H
     pipelined over two device slots; synchronises."""
+    if nvec < 0 or ldx < 0 or ldy < 0:
+        raise ValueError("nvec, ldx and ldy must be >= 0")
+    xt, yt = _xy_np(plan.dtype)
+    if nvec > 0:
+        if alpha != 0.0 and plan.n > 0:
+            _check_host(x, (nvec - 1) * ldx + plan.n, xt, "x")
+        _check_host(y, (nvec - 1) * ldy + plan.m, yt, "y")
+    stream = _default_stream(plan, stream)
     st = _lib.dasp_spmv_host_stream(plan.handle, _ptr(x), int(ldx), _ptr(y), int(ldy), int(nvec), float(alpha),
                                     float(beta), _stream_ptr(stream))
     _check(st, "dasp_spmv_host_stream")

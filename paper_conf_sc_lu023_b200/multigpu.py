@@ -39,6 +39,19 @@ import numpy as np
 
 from . import dasp
 
+# iterated SpMV feeds y back as the next x, so x and y must share one element type: FP64 (the
+# north-star mode) or FP32 (R29).  FP16 plans take binary16 x but write FP32 y (R15), which would
+# need a cast inside the loop; they are not part of the multi-GPU mode.
+_ITER_DTYPES = {"f64": ("float64", 8), "f32": ("float32", 4)}
+
+
+def _iter_dtype(dtype):
+    if dtype not in _ITER_DTYPES:
+        raise ValueError(f"row-slab iteration needs x and y of one type (f64 or f32), not {dtype!r}")
+    import torch
+    name, size = _ITER_DTYPES[dtype]
+    return getattr(torch, name), size
+
 
 def slab_bounds(row_lengths: np.ndarray, nparts: int) -> np.ndarray:
     """nnz-balanced contiguous row slabs from the global row lengths (via the C-ABI)."""
@@ -110,7 +123,8 @@ class SlabSpMV:
         self.device = torch.device(device)
         self.dtype = dtype
         self.fused = fused
-        tdt = torch.float64
+        tdt, self.elem_bytes = _iter_dtype(dtype)
+        self._checked = False
         n_pad = world * slab.S
         self.n_pad = n_pad
         if fused:
@@ -132,7 +146,8 @@ class SlabSpMV:
 
             def _local(x, y, alpha):
                 dasp.dasp_spmv(self.plan, x, y, alpha, 0.0, torch.cuda.current_stream(self.device),
-                               variant=variant, check=False)
+                               variant=variant, check=not self._checked)   # full checks on the first call
+                self._checked = True
             self.local_spmv = _local
         else:
             self.plan = None
@@ -142,7 +157,7 @@ class SlabSpMV:
         """Load the global x (length n) into the padded layout of the current buffer."""
         import torch
         st, S = self.slab.starts, self.slab.S
-        buf = np.zeros(self.world * S)
+        buf = np.zeros(self.world * S, dtype=_ITER_DTYPES[self.dtype][0])
         for q in range(self.world):
             buf[q * S: q * S + st[q + 1] - st[q]] = x_global[st[q]:st[q + 1]]
         self.x[self.cur].copy_(torch.from_numpy(buf))
@@ -176,7 +191,7 @@ class SlabSpMV:
         """One iteration with the all-gather fused into the SpMV epilogue (see module doc)."""
         import torch
         nb = 1 - self.cur
-        dsts = scatter_destinations(self.peer_base, self.rank, self.world, nb, self.n_pad, self.slab.S, 8)
+        dsts = scatter_destinations(self.peer_base, self.rank, self.world, nb, self.n_pad, self.slab.S, self.elem_bytes)
         dasp.dasp_spmv_scatter(self.plan, self.x[self.cur], dsts, alpha, 0.0, torch.cuda.current_stream(self.device))
         self.hdl.barrier(channel=0)          # every rank's stores have landed before x is read
         self.cur = nb
@@ -265,13 +280,14 @@ class HaloSlabSpMV:
             raise ValueError("HaloSlabSpMV needs a slab with global columns (build_slab(remap=False))")
         self.slab, self.world, self.rank, self.group = slab, world, rank, group
         self.device = torch.device(device)
+        self.dtype = dtype
+        tdt, self.elem_bytes = _iter_dtype(dtype)
         self.split = split_halo(slab.row_ptr, slab.col, slab.val, slab.starts, rank)
         if world > 1:
             send_idx, self.send_counts = exchange_lists(self.split, slab.starts, rank, world, group,
                                                         self.device if self.device.type == "cuda" else "cpu")
         else:
             send_idx, self.send_counts = np.zeros(0, np.int32), np.zeros(1, np.int64)
-        tdt = torch.float64
         self.x = [torch.zeros(slab.rows, dtype=tdt, device=self.device) for _ in range(2)]
         self.cur = 0
         self.send_idx = torch.from_numpy(send_idx).to(self.device)
@@ -309,12 +325,13 @@ class HaloSlabSpMV:
     @property
     def halo_bytes(self) -> int:
         """x bytes this rank receives per step (an all-gather would receive (n - rows)*8)."""
-        return self.n_halo * 8
+        return self.n_halo * self.elem_bytes
 
     def set_x(self, x_global: np.ndarray):
         import torch
         r0 = self.slab.row0
-        self.x[self.cur].copy_(torch.from_numpy(np.ascontiguousarray(x_global[r0:r0 + self.slab.rows], dtype=np.float64)))
+        self.x[self.cur].copy_(torch.from_numpy(np.ascontiguousarray(x_global[r0:r0 + self.slab.rows],
+                                                                     dtype=_ITER_DTYPES[self.dtype][0])))
 
     def my_x(self):
         return self.x[self.cur]
@@ -351,7 +368,7 @@ class HaloSlabSpMV:
         if self.world == 1:
             return self.x[self.cur].cpu().numpy().copy()
         S = int(max(np.diff(st)))
-        buf = torch.zeros(S, dtype=torch.float64, device=self.device)
+        buf = torch.zeros(S, dtype=self.x[0].dtype, device=self.device)
         buf[:self.slab.rows] = self.x[self.cur]
         parts = [torch.empty_like(buf) for _ in range(self.world)]
         dist.all_gather(parts, buf, group=self.group)

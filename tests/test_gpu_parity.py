@@ -232,24 +232,30 @@ NARROW_LENS = {
 
 @pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("name", list(NARROW_LENS))
-@pytest.mark.parametrize("narrow", ["1", "0"])
-def test_narrow_medium_paths(dt, name, narrow, monkeypatch):
-    """Narrow / mid medium row-blocks (a lane or two lanes per row) vs the oracle, and the same
-    plan built with DASP_NARROW=0 (every row-block on the warp-per-row-block path)."""
-    monkeypatch.setenv("DASP_NARROW", narrow)
+def test_narrow_medium_paths(dt, name):
+    """Narrow / mid medium row-blocks (the CUDA-core variant gives a lane or two lanes to a row)
+    vs the oracle, and vs the MMA variant, which runs the same row-blocks on the paper's
+    warp-per-row-block path (Alg. 3): real values within tolerance, integers bit-exact."""
     rng = np.random.default_rng(len(name))
     lens = list(rng.choice(NARROW_LENS[name], size=3001))          # ragged: 375 row-blocks + 1 row
     A = synth.from_lengths(lens, n=5000, seed=11)
     x = synth.vector(3, A.n)
     y_ref, s = oracle_ref(A, x, dt)
+    plan = make(A, dt)
+    assert plan.info["rowblocks_narrow"] + plan.info["rowblocks_mid"] > 0 or name == "len17-32" or dt == "f16"
     for variant in VARIANTS:
-        plan = make(A, dt)
         y = run(plan, x, dt, variant=variant)
         assert oracle.tolerance_ok(y, y_ref, s, dt).all(), (VNAME[variant], int((~oracle.tolerance_ok(y, y_ref, s, dt)).sum()))
         y0 = synth.vector(4, A.m)
         y = run(plan, x, dt, 2.0, -0.5, y0, variant=variant)
         y_ref2, s2 = oracle_ref(A, x, dt, 2.0, -0.5, y0)
         assert oracle.tolerance_ok(y, y_ref2, s2, dt).all()
+    Ai = synth.from_lengths(lens, n=5000, seed=11, val_mode=synth.VAL_INT)
+    xi = synth.vector(5, Ai.n, synth.VAL_INT)
+    plan = make(Ai, dt)
+    yi_ref, _ = oracle_ref(Ai, xi, dt)
+    for variant in VARIANTS:
+        assert np.array_equal(run(plan, xi, dt, variant=variant), yi_ref), VNAME[variant]
 
 
 @pytest.mark.parametrize("dt", DTYPES)
@@ -285,13 +291,9 @@ def test_spmv_host_stream_pipelined(dt, beta):
 
 
 @pytest.mark.parametrize("dt", DTYPES)
-@pytest.mark.parametrize("h2d_sm", ["1", "0"])
-def test_spmv_host_large_pinned_vectors(dt, h2d_sm, monkeypatch):
-    """Host vectors >= 1 MiB in page-locked memory; with DASP_H2D_SM=1 they take the SM-load
-    host->device copy (16-B body + ragged byte tail: n odd) and misaligned strides (FP16/FP32, ldx
-    odd) fall back to cudaMemcpyAsync; with 0 every copy is cudaMemcpyAsync.
+def test_spmv_host_large_pinned_vectors(dt):
+    """Host vectors >= 1 MiB in page-locked memory at odd strides (misaligned rows for FP16/FP32).
     Every y_j equals the device-resident dasp_spmv result bit for bit and passes the oracle."""
-    monkeypatch.setenv("DASP_H2D_SM", h2d_sm)
     rng = np.random.default_rng(5)
     n = {"f64": 200_001, "f32": 300_001, "f16": 600_001}[dt]       # x >= 1 MiB; row 1 of X misaligned for f16/f32
     A = synth.from_lengths(list(rng.integers(5, 41, size=3001)), n=n, seed=13)
@@ -323,83 +325,15 @@ def test_bad_device_args():
         dasp.dasp_spmv(plan, x, x, check=False)   # aliasing x == y
 
 
-# full-size configs, in the launch configuration bench.py times: sampled rows vs the oracle
-def _sampled_parity(A, dt, nsample=20000, seed=0):
-    x = synth.vector(13, A.n)
-    plan = make(A, dt)
-    y = run(plan, x, dt)
-    rng = np.random.default_rng(seed)
-    lens = np.diff(A.row_ptr)
-    rows = np.unique(np.concatenate([rng.integers(0, A.m, nsample), np.flatnonzero(lens > 256)[:2000],
-                                     [0, A.m - 1]]))
-    starts, ends = A.row_ptr[rows], A.row_ptr[rows + 1]
-    sub_rp = np.concatenate([[0], np.cumsum(ends - starts)]).astype(np.int64)
-    idx = np.concatenate([np.arange(s, e) for s, e in zip(starts, ends)]) if len(rows) else np.zeros(0, np.int64)
-    sub = synth.CSR(len(rows), A.n, sub_rp, A.col[idx], A.val[idx])
-    y_ref, s = oracle_ref(sub, x, dt)
-    ok = oracle.tolerance_ok(y[rows], y_ref, s, dt)
-    assert ok.all(), f"{(~ok).sum()} sampled rows off"
-    return plan
-
-
-@pytest.mark.parametrize("dt", DTYPES)
-def test_full_size_stencil_sampled(dt):
-    A = synth.generate(synth.config("c2"))
-    _sampled_parity(A, dt)
-
-
-@pytest.mark.parametrize("dt", DTYPES)
-def test_full_size_powerlaw_sampled(dt):
-    A = synth.generate(synth.config("c3"))
-    _sampled_parity(A, dt)
-
-
-def test_long_unit_order_is_result_neutral(monkeypatch):
-    """The column-bucketed long-unit schedule changes only execution order: bitwise same y."""
-    A = synth.generate(synth.config("c3", scale=0.02))
-    x = synth.vector(31, A.n)
-    ys = []
-    for order in ["0", "1"]:
-        monkeypatch.setenv("DASP_LONG_ORDER", order)
-        for v in VARIANTS:
-            ys.append(run(make(A, "f64", panel_rows=50000), x, "f64", variant=v))
-    assert np.array_equal(ys[0], ys[2]) and np.array_equal(ys[1], ys[3])
-    y_ref, s = oracle_ref(A, x, "f64")
-    assert oracle.tolerance_ok(ys[0], y_ref, s).all()
-
-
-# the TMA-staged persistent kernel (dasp_options_t.pipeline): same bits as the direct kernel on
-# integer inputs, every class, both dtypes and variants, several panel sizes
-@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
-@pytest.mark.parametrize("dt", ["f64", "f16"])
-@pytest.mark.parametrize("name,gen", CASES, ids=[c[0] for c in CASES])
-def test_pipeline_kernel_parity(name, gen, dt, variant):
-    A = gen(synth.VAL_INT)
-    x = synth.vector(41, A.n, synth.VAL_INT)
-    y0 = synth.vector(42, A.m, synth.VAL_INT)
-    for panel in [-1, 700]:
-        plan = make(A, dt, pipeline=True, panel_rows=panel)
-        assert plan.info["pipeline"] == 1
-        y = run(plan, x, dt, 2.0, -1.0, y0, variant=variant)
-        y_ref, _ = oracle_ref(A, x, dt, 2.0, -1.0, y0)
-        assert np.array_equal(y, y_ref)
-    A = gen(synth.VAL_UNIFORM)
-    x = synth.vector(43, A.n)
-    plan = make(A, dt, pipeline=True)
-    y = run(plan, x, dt, variant=variant)
-    y_ref, s = oracle_ref(A, x, dt)
-    assert oracle.tolerance_ok(y, y_ref, s, dt).all()
-
-
 # dasp_spmv_scatter: the fused SpMV + all-gather epilogue writes the same values to every
 # destination (here several local buffers stand in for the peers' x buffers)
+@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
 @pytest.mark.parametrize("dt", DTYPES)
-@pytest.mark.parametrize("pipeline", [False, True])
-def test_scatter_epilogue_writes_every_destination(dt, pipeline):
+def test_scatter_epilogue_writes_every_destination(dt, variant):
     A = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
     x = synth.vector(51, A.n, synth.VAL_INT)
     y0 = synth.vector(52, A.m, synth.VAL_INT)
-    plan = make(A, dt, pipeline=pipeline)
+    plan = make(A, dt, variant=variant)
     xd = torch.from_numpy(x.astype(NP_VAL[dt])).cuda()
     ydt = torch.float64 if dt == "f64" else torch.float32
     for alpha, beta in [(1.0, 0.0), (2.0, -1.0), (1.0, 1.0), (0.0, 3.0)]:
@@ -427,19 +361,6 @@ def test_parity_knobs(dt, max_len, tau):
         assert np.array_equal(run(plan, x, dt, variant=v), y_ref)
 
 
-# short tiles in their own launch (DASP_SPLIT_SHORT=1): same bits as the fused main kernel
-@pytest.mark.parametrize("dt", DTYPES)
-def test_split_short_kernel_parity(dt, monkeypatch):
-    monkeypatch.setenv("DASP_SPLIT_SHORT", "1")
-    for name, gen in CASES:
-        A = gen(synth.VAL_INT)
-        x = synth.vector(101, A.n, synth.VAL_INT)
-        y_ref, _ = oracle_ref(A, x, dt)
-        for v in VARIANTS:
-            plan = make(A, dt, panel_rows=900)
-            assert np.array_equal(run(plan, x, dt, variant=v), y_ref), name
-
-
 @pytest.mark.parametrize("dt", ["f64", "f16", "f32"])
 def test_cuda_graph_capture_replay(dt):
     """dasp_spmv enqueues only kernels on the given stream (no host sync, no allocation), so a loop
@@ -464,46 +385,75 @@ def test_cuda_graph_capture_replay(dt):
     assert np.array_equal(yd.cpu().numpy().astype(np.float64), eager.astype(np.float64))
 
 
-# co-scheduled long rows (dasp_options_t.co_schedule): the long units run inside the
-# main kernel and the warp that completes a row's group counter runs its phase 2.  Both modes on
-# every long-row case; repeated launches check that the counters reset themselves (a stale
-# counter would skip or double a row's phase 2), and the two latest launches must be bitwise equal
-# (the phase-2 order is fixed whichever warp runs it).
+# P:L91 (CSR): a column index per nonzero, no order implied, so the boundary accepts unsorted
+# columns and duplicate (row, col) entries (summed like any other entry; include/dasp.h), and
+# rectangular shapes.  Integer values: every summation order gives the same bits.
+def _shuffle_rows(A, rng):
+    """The same matrix with each row's entries in a random order."""
+    rows = np.repeat(np.arange(A.m), np.diff(A.row_ptr))
+    perm = np.lexsort((rng.random(A.nnz), rows))
+    return synth.CSR(A.m, A.n, A.row_ptr, A.col[perm], A.val[perm])
+
+
+def _with_duplicates(A, rng, frac=0.3):
+    """Every chosen entry repeated 1-3 extra times right after itself (same column, own value):
+    rows grow, so rows move between the short / medium / long classes."""
+    rep = np.ones(A.nnz, dtype=np.int64)
+    pick = rng.random(A.nnz) < frac
+    rep[pick] += rng.integers(1, 4, int(pick.sum()))
+    rows = np.repeat(np.arange(A.m), np.diff(A.row_ptr))
+    lens = np.bincount(rows, weights=rep, minlength=A.m).astype(np.int64)
+    rp = np.zeros(A.m + 1, dtype=np.int64)
+    np.cumsum(lens, out=rp[1:])
+    col = np.repeat(A.col, rep)
+    val = np.repeat(A.val, rep)
+    val = np.where(rng.random(len(val)) < 0.5, val, -val + 1.0)   # duplicates carry other values
+    return synth.CSR(A.m, A.n, rp, col.astype(np.int32), val)
+
+
+def _rectangular(m, n, rng, lens_choice):
+    lens = rng.choice(lens_choice, size=m)
+    lens = np.minimum(lens, n)
+    rp = np.zeros(m + 1, dtype=np.int64)
+    np.cumsum(lens, out=rp[1:])
+    col = np.concatenate([rng.choice(n, L, replace=False) for L in lens]).astype(np.int32) if rp[-1] else np.zeros(0, np.int32)
+    val = rng.integers(-3, 4, int(rp[-1])).astype(np.float64)
+    return synth.CSR(m, n, rp, col, val)
+
+
+def _irregular_cases():
+    rng = np.random.default_rng(77)
+    base = synth.generate(synth.config("c1b", val_mode=synth.VAL_INT))
+    yield "c1b_unsorted", _shuffle_rows(base, rng)
+    yield "c1b_duplicates", _with_duplicates(base, rng)
+    yield "c3s_unsorted_dup", _shuffle_rows(_with_duplicates(
+        synth.generate(synth.config("c3", scale=0.004, val_mode=synth.VAL_INT)), rng), rng)
+    lens = [0, 1, 2, 3, 4, 5, 9, 17, 33, 256, 257, 700]
+    yield "tall_6000x700", _rectangular(6000, 700, rng, lens)
+    yield "wide_900x20000", _rectangular(900, 20000, rng, lens + [3000])
+    yield "one_column", _rectangular(3000, 1, rng, [0, 1])
+    yield "dup_single_column", _with_duplicates(_rectangular(2000, 1, rng, [1]), rng, frac=1.0)
+
+
+IRREGULAR = list(_irregular_cases())
+
+
 @pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
 @pytest.mark.parametrize("dt", DTYPES)
-@pytest.mark.parametrize("cs", [0, 1])
-def test_co_schedule_parity_repeated(cs, dt, variant):
-    for name, gen in CASES:
-        for vm, seed in ((synth.VAL_UNIFORM, 41), (synth.VAL_INT, 42)):
-            A = gen(vm)
-            x = synth.vector(seed, A.n, vm)
-            plan = make(A, dt, co_schedule=cs, panel_rows=700)
-            assert plan.info["co_scheduled"] == (1 if cs and plan.info["row_long"] > 0 else 0), name
-            y_ref, s = oracle_ref(A, x, dt)
-            ys = [run(plan, x, dt, variant=variant) for _ in range(3)]
-            for y in ys:
-                if vm == synth.VAL_INT:
-                    assert np.array_equal(y, y_ref), name
-                else:
-                    assert oracle.tolerance_ok(y, y_ref, s, dt).all(), name
-            assert np.array_equal(ys[1], ys[2]), name
-            y0 = synth.vector(seed + 1, A.m, vm)
-            y = run(plan, x, dt, -0.5, 2.0, y0, variant=variant)
-            y_ref, s = oracle_ref(A, x, dt, -0.5, 2.0, y0)
-            assert oracle.tolerance_ok(y, y_ref, s, dt).all(), name
-
-
-def test_co_schedule_many_long_rows_one_launch_each():
-    """Rows of 257..20000 nonzeros (5..313 groups), so units straddle row ends and several rows
-    complete inside one unit; 20 launches, every one compared with the oracle."""
-    lens = list(np.random.default_rng(5).integers(257, 20000, size=300)) + [257] * 40 + [300, 5, 3, 0] * 10
-    A = synth.from_lengths(lens, n=60000, val_mode=synth.VAL_INT)
-    x = synth.vector(51, A.n, synth.VAL_INT)
-    y_ref, _ = oracle_ref(A, x, "f64")
-    for dt in DTYPES:
-        plan = make(A, dt, co_schedule=1)
-        assert plan.info["co_scheduled"] == 1
-        y_ref_dt, _ = oracle_ref(A, x, dt)
-        for _ in range(20):
-            assert np.array_equal(run(plan, x, dt), y_ref_dt), dt
-
+@pytest.mark.parametrize("name,A", IRREGULAR, ids=[c[0] for c in IRREGULAR])
+def test_unsorted_duplicate_rectangular_bit_exact(name, A, dt, variant):
+    x = synth.vector(81, A.n, synth.VAL_INT)
+    y0 = synth.vector(82, A.m, synth.VAL_INT)
+    for panel in (0, 333):
+        plan = make(A, dt, panel_rows=panel)
+        y_ref, _ = oracle_ref(A, x, dt)
+        assert np.array_equal(run(plan, x, dt, variant=variant), y_ref), name
+        y_ref, _ = oracle_ref(A, x, dt, -2.0, 1.0, y0)
+        assert np.array_equal(run(plan, x, dt, -2.0, 1.0, y0, variant=variant), y_ref), name
+    # the device builder takes the same input and gives the same bytes
+    if A.nnz:
+        dplan = dasp.dasp_plan_create_device(torch.from_numpy(A.row_ptr).cuda(), torch.from_numpy(A.col).cuda(),
+                                             torch.from_numpy(A.val.astype(NP_VAL[dt])).cuda(), A.m, A.n, dt)
+        hplan = make(A, dt)
+        for arr in dasp.ARRAYS:
+            assert np.array_equal(dasp.dasp_plan_copy_array(dplan, arr), dasp.dasp_plan_copy_array(hplan, arr)), arr
