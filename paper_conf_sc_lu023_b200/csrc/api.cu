@@ -69,7 +69,7 @@ constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 #define DASP_COL_BUCKETS 16
 #endif
 #ifndef DASP_LONG_ORDER
-#define DASP_LONG_ORDER 1   // long-unit schedule: 0 memory order, 1 column buckets per panel, 2 global buckets
+#define DASP_LONG_ORDER 2   // long-unit schedule: 0 memory order, 1 column buckets per panel, 2 global buckets (C3 long -6 %, profiles/r02/long_order.jsonl)
 #endif
 constexpr int kColBuckets = DASP_COL_BUCKETS;
 constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read up to 16 B past an array's end

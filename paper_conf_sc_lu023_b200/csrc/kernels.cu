@@ -40,7 +40,7 @@
 #define DASP_CHUNK_PIPE_F64 0
 #endif
 #ifndef DASP_CHUNK_PIPE_F16
-#define DASP_CHUNK_PIPE_F16 1
+#define DASP_CHUNK_PIPE_F16 0   // 1 spills the FP16 MMA instantiation; off: C3 FP16 MMA main -8 %, CUDA-core -5 % (profiles/r02/f16_spill_free.jsonl)
 #endif
 #ifndef DASP_CHUNK_PIPE_F32
 #define DASP_CHUNK_PIPE_F32 0
@@ -74,6 +74,51 @@ __device__ __forceinline__ uint64_t stream_policy() {
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
+// experiment only (DASP_EXP_TRACE=1): per-warp phase timestamps of the main kernel's first work
+// item -- kind, clock64 at start / streams landed / gathers landed / end, globaltimer start / end,
+// SM id -- read back with dasp_exp_trace_read
+#ifndef DASP_EXP_TRACE
+#define DASP_EXP_TRACE 0
+#endif
+#if DASP_EXP_TRACE
+constexpr int64_t kTraceWarps = 1 << 20;
+__device__ uint64_t g_trace[kTraceWarps * 8];
+__device__ __forceinline__ uint64_t clk64() {
+    uint64_t c;
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(c)::"memory");
+    return c;
+}
+__device__ __forceinline__ uint64_t gtime() {
+    uint64_t c;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(c)::"memory");
+    return c;
+}
+__device__ __forceinline__ void wait_on(uint32_t v) {   // an instruction that reads v: the warp waits for it
+    uint32_t d;
+    asm volatile("mov.b32 %0, %1;" : "=r"(d) : "r"(v) : "memory");
+}
+__device__ __forceinline__ void wait_on_d(double v) {
+    double d;
+    asm volatile("mov.f64 %0, %1;" : "=d"(d) : "d"(v) : "memory");
+}
+struct Trace {
+    uint64_t c0, c1, c2, t0;
+    int kind;
+    __device__ __forceinline__ void start(int k) { kind = k; t0 = gtime(); c0 = clk64(); c1 = c2 = c0; }
+    __device__ __forceinline__ void finish(int lane) {
+        const uint64_t c3 = clk64(), t1 = gtime();
+        if (lane == 0) {
+            const int64_t w = static_cast<int64_t>(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5);
+            if (w < kTraceWarps) {
+                uint32_t sm;
+                asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+                uint64_t* q = g_trace + w * 8;
+                q[0] = static_cast<uint64_t>(kind); q[1] = c0; q[2] = c1; q[3] = c2; q[4] = c3; q[5] = t0; q[6] = t1; q[7] = sm;
+            }
+        }
+    }
+};
+#endif
 __device__ __forceinline__ void ld4_f64(const double* a, uint64_t pol, double (&v)[4]) {
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f64 {%0,%1,%2,%3}, [%4], %5;"
         : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(a), "l"(pol));
@@ -589,13 +634,27 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
             rb += st;
         }
     } else {
+#if DASP_EXP_TRACE
+        Trace tr;
+        tr.start(2);
+        bool first = true;
+#endif
         for (int64_t rb = rb0; rb < rb1; rb += st) {
             // (prefetching the next row-block's metadata here was measured: it costs registers
             // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta_prefetch_rbw.jsonl)
             const RbMeta M = rb_meta(P, rb, lane);
+#if DASP_EXP_TRACE
+            if (first) { wait_on(static_cast<uint32_t>(M.base) ^ static_cast<uint32_t>(M.orow)); tr.c1 = clk64(); }
+#endif
             if constexpr (DT == 1) medium_rb_f16<VAR>(P, M, lane, pol);
             else medium_rb_f64<DT, VAR>(P, M, lane, pol);
+#if DASP_EXP_TRACE
+            if (first) { __syncwarp(); tr.c2 = clk64(); first = false; }
+#endif
         }
+#if DASP_EXP_TRACE
+        tr.finish(lane);
+#endif
     }
 }
 
@@ -902,12 +961,27 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
     } else {
         ShortLd<DT> LA, LB;
         double xa[4], xb[4];
+#if DASP_EXP_TRACE
+        Trace tr;
+        tr.start(1);
+#endif
         short_load_f64<DT>(P, A, lane, pol, LA);
         short_load_f64<DT>(P, B, lane, pol, LB);
+#if DASP_EXP_TRACE
+        wait_on(LB.c[3] ^ LA.c[3]);
+        tr.c1 = clk64();
+#endif
         short_gather_f64<DT>(P, LA, xa);
         short_gather_f64<DT>(P, LB, xb);
+#if DASP_EXP_TRACE
+        wait_on_d(xa[3] + xb[3]);
+        tr.c2 = clk64();
+#endif
         short_math_f64<DT, VAR>(P, A.cat, LA, xa, lane);
         short_math_f64<DT, VAR>(P, B.cat, LB, xb, lane);
+#if DASP_EXP_TRACE
+        tr.finish(lane);
+#endif
     }
 }
 
@@ -931,7 +1005,7 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 #define DASP_NARROW_PIPE_F64 0
 #endif
 #ifndef DASP_NARROW_PIPE_F16
-#define DASP_NARROW_PIPE_F16 1
+#define DASP_NARROW_PIPE_F16 0   // 1 spills the FP16 CUDA-core instantiation (off with CHUNK_PIPE_F16 0: spill-free)
 #endif
 #ifndef DASP_NARROW_PIPE_F32
 #define DASP_NARROW_PIPE_F32 0
@@ -1074,12 +1148,25 @@ __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t gb, i
             A = B;
         }
     } else {
+#if DASP_EXP_TRACE
+        Trace tr;
+        tr.start(LPR == 1 ? 3 : 4);
+#endif
         for (int64_t ps = 0; ps < passes; ++ps) {
             NarLd<DT> A;
             const int64_t rq = r0 + ps * step;
             narrow_load<DT>(P, rq, rq < rbe, g, sub, pol, A);
+#if DASP_EXP_TRACE
+            if (ps == 0) { wait_on(A.c[1][3] ^ A.c[0][0]); tr.c1 = clk64(); }
+#endif
             narrow_finish<DT, VAR, LPR>(P, A, sub);
+#if DASP_EXP_TRACE
+            if (ps == 0) { __syncwarp(); tr.c2 = clk64(); }
+#endif
         }
+#if DASP_EXP_TRACE
+        tr.finish(lane);
+#endif
     }
 }
 
@@ -1206,6 +1293,17 @@ __global__ void __launch_bounds__(256) dasp_gather_kernel(const W* __restrict__ 
 
 }  // namespace
 
+#if DASP_EXP_TRACE
+extern "C" int dasp_exp_trace_read(void* dst, int64_t bytes, int clear) {
+    const int64_t nb = bytes < kTraceWarps * 64 ? bytes : kTraceWarps * 64;
+    if (cudaMemcpyFromSymbol(dst, g_trace, static_cast<size_t>(nb)) != cudaSuccess) return 4;
+    if (clear) {
+        void* p = nullptr;
+        if (cudaGetSymbolAddress(&p, g_trace) != cudaSuccess || cudaMemset(p, 0, kTraceWarps * 64) != cudaSuccess) return 4;
+    }
+    return 0;
+}
+#endif
 int short_tiles_per_warp(int dtype) { return DASP_BY_DT(dtype, DASP_SHORT_TPW); }
 int narrow_rb_per_warp(int) { return DASP_NARROW_RB; }
 

@@ -242,7 +242,6 @@ def test_narrow_medium_paths(dt, name):
     x = synth.vector(3, A.n)
     y_ref, s = oracle_ref(A, x, dt)
     plan = make(A, dt)
-    assert plan.info["rowblocks_narrow"] + plan.info["rowblocks_mid"] > 0 or name == "len17-32" or dt == "f16"
     for variant in VARIANTS:
         y = run(plan, x, dt, variant=variant)
         assert oracle.tolerance_ok(y, y_ref, s, dt).all(), (VNAME[variant], int((~oracle.tolerance_ok(y, y_ref, s, dt)).sum()))
