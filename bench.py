@@ -204,11 +204,22 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def load_traffic(workload, dtype, variant, kernel):
-    """ncu DRAM bytes (read + write) per launch recorded by scripts/ncu_summary.py."""
+def load_traffic(workload, dtype, variant, kernel, what=""):
+    """ncu DRAM bytes (read + write) per launch recorded by scripts/ncu_summary.py (what="": bytes;
+    "l2_read_requests": L1 -> L2 read requests per launch)."""
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-            return json.load(f).get(f"{workload}/{dtype}/{variant}/{kernel}")
+            return json.load(f).get(f"{workload}/{dtype}/{variant}/{kernel}" + (f"/{what}" if what else ""))
+    except Exception:
+        return None
+
+
+def load_l2_ceiling():
+    """Measured ceiling of scattered 8-B gathers served by L2 (one 32-B sector request each):
+    profiles/l2_gather_ceiling.json, written from scripts/probe/l2peak.py on this pool's B200s."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "l2_gather_ceiling.json")) as f:
+            return float(json.load(f)["Grequests_per_s"])
     except Exception:
         return None
 
@@ -244,10 +255,17 @@ def roofline(info, dtype, kern, ms_step, workload, variant, peak, peak_src, tria
         avg = ms / nl
         alg = bm.get(k)
         tr = load_traffic(workload, dtype, variant, k)
+        req = load_traffic(workload, dtype, variant, k, "l2_read_requests")
+        ceil = load_l2_ceiling()
         kernels[k] = {"avg_ms": avg, "launches": nl, "share_of_step": avg / ms_step, "alg_bytes": alg,
                       "alg_gbs": alg / (avg * 1e-3) / 1e9 if alg else None,
                       "frac": alg / (avg * 1e-3) / 1e9 / peak if alg else None,
-                      "traffic": tr, "traffic_over_alg": tr / alg if (tr and alg) else None}
+                      "traffic": tr, "traffic_over_alg": tr / alg if (tr and alg) else None,
+                      # second roofline axis: L1 -> L2 read requests (ncu, per launch) over this launch's
+                      # time, against the measured scattered-gather ceiling
+                      "l2_requests": ({"per_launch": req, "achieved_G_per_s": req / (avg * 1e-3) / 1e9,
+                                       "ceiling_G_per_s": ceil, "frac": req / (avg * 1e-3) / 1e9 / ceil}
+                                      if (req and ceil) else None)}
     dom = max(per, key=lambda k: per[k][0]) if per else "dasp_main_kernel"
     d = kernels.get(dom, {})
     ach = d.get("alg_gbs")

@@ -86,6 +86,9 @@ constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read 
 #ifndef DASP_NARROW_IL
 #define DASP_NARROW_IL 0
 #endif
+#ifndef DASP_HEAVY_FIRST
+#define DASP_HEAVY_FIRST 0   // leading blocks of every panel dispatched at the start of the main grid
+#endif
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
 // small matrices keep the paper's 1 / 2; for large ones, uniform medium rows (coefficient of
@@ -277,6 +280,19 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         blk += nb;
     }
     p->blocks = blk;
+    // heavy blocks first: a panel's first blocks hold its longest medium row-blocks (rows are
+    // length-sorted), whose warps walk many chunks one round trip after the other and finish long
+    // after the panel's other blocks.  Dispatching those blocks of every panel at the start of the
+    // grid overlaps them with everything else instead of leaving them as the tail of the launch.
+    if (DASP_HEAVY_FIRST > 0 && f.n_panels > 1) {
+        std::vector<uint64_t> order;
+        order.reserve(blk_word.size());
+        for (uint64_t w : blk_word)
+            if ((w & 0xffffffffu) < static_cast<uint64_t>(DASP_HEAVY_FIRST)) order.push_back(w);
+        for (uint64_t w : blk_word)
+            if ((w & 0xffffffffu) >= static_cast<uint64_t>(DASP_HEAVY_FIRST)) order.push_back(w);
+        blk_word.swap(order);
+    }
     p->n_units = f.n_groups_padded / f.geo.UG;
     // medium chunk units: every full chunk (CW regular blocks) of the wide row-blocks [rb0, rb0 +
     // rbm) of each panel, in memory order, runs in the long-row launch (kernels.cu mchunk_pair_*);

@@ -35,6 +35,12 @@ WANT = [
     ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", "FMA pipe inst %"),
     ("sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active", "FP64 pipe inst %"),
     ("smsp__inst_executed.sum", "warp instructions"),
+    ("lts__t_sectors_srcunit_tex_op_read.sum", "L2 read sectors from L1 (streams + x gathers)"),
+    ("lts__t_sectors_srcunit_tex_op_read_lookup_miss.sum", "L2 read sector misses"),
+    ("lts__t_requests_srcunit_tex_op_read.sum", "L2 read requests from L1"),
+    ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "L2 (LTS) throughput % of peak"),
+    ("lts__t_sectors.sum.pct_of_peak_sustained_elapsed", "L2 sectors % of peak"),
+    ("l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "L1 throughput % of peak"),
 ]
 
 
@@ -62,8 +68,7 @@ def main():
         key, rep = arg.split("=", 1)
         for k, d in enumerate(raw(rep)):
             kname = d.get("Kernel Name", ("", ""))[1]
-            kern = next((n for n in ("dasp_main_kernel", "dasp_long_kernel", "dasp_finish_kernel", "dasp_pipe_kernel")
-                         if n in kname), None)
+            kern = next((n for n in ("dasp_main_kernel", "dasp_long_kernel") if n in kname), None)
             if kern is None:
                 continue
             lines.append(f"## {key} — {kern}  ({os.path.basename(rep)})")
@@ -80,8 +85,15 @@ def main():
             rd = to_bytes(*d["dram__bytes_read.sum"])
             wr = to_bytes(*d["dram__bytes_write.sum"])
             traffic[f"{key}/{kern}"] = rd + wr
-            if kern == "dasp_main_kernel":
-                traffic[key] = rd + wr
+            sec = d.get("lts__t_sectors_srcunit_tex_op_read.sum")
+            dur = d.get("gpu__time_duration.sum")
+            if sec and dur:
+                ns = float(dur[1].replace(",", "")) * {"ns": 1, "us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6}.get(dur[0], 1)
+                traffic[f"{key}/{kern}/l2_read_sectors"] = float(sec[1].replace(",", ""))
+                traffic[f"{key}/{kern}/l2_read_Gsectors_per_s"] = float(sec[1].replace(",", "")) / ns
+            req = d.get("lts__t_requests_srcunit_tex_op_read.sum")
+            if req:
+                traffic[f"{key}/{kern}/l2_read_requests"] = float(req[1].replace(",", ""))
             lines.append("")
     with open(out_md, "w") as f:
         f.write("\n".join(lines) + "\n")

@@ -48,6 +48,8 @@ def main():
                 assert np.array_equal(dasp.dasp_plan_copy_array(dplan, arr), dasp.dasp_plan_copy_array(plan, arr)), arr
             dplan.destroy()
             plan.destroy()
+    torch.cuda.synchronize()
+    torch.cuda.empty_cache()   # torch's caching allocator keeps its blocks otherwise (reported as leaks)
     print("sanitize workload ok")
 
 
