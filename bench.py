@@ -62,9 +62,6 @@ def parse(argv=None):
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--panel-rows", type=int, default=0, help="rows per panel (0 auto, -1 one global panel)")
-    ap.add_argument("--medium-units", type=int, default=-1, choices=[-1, 0, 1],
-                    help="1: full chunks of wide medium row-blocks as chunk units in the long launch; 0: one warp "
-                    "per row-block (Alg. 3 as printed); -1: library default")
     ap.add_argument("--iterate", action="store_true", help="N=1: run the row-slab iteration (x <- alpha*A*x)")
     ap.add_argument("--halo", action="store_true", help="slab mode: sparse halo exchange (all_to_all of the referenced "
                     "remote x only) overlapped with the local sub-matrix SpMV (SURVEY.md 8(f) f1)")
@@ -178,18 +175,13 @@ def byte_model(info, dtype, beta_nonzero=False):
     ngp, nrb, rl = info["n_groups_padded"], info["rowblocks"], info["row_long"]
     nout_short = 64 * info["tiles_13"] + 32 * info["tiles_4"] + 64 * info["tiles_22"] + 128 * info["tiles_single"]
     long_ = ngp * G * (sv + 4) + ngp * sa
-    # medium chunk units (full chunks of the wide row-blocks) stream in the long launch
-    nch = info.get("medium_chunk_units", 0)
-    chunk_slots = nch * (256 if dtype == "f16" else 128)
-    long_ += chunk_slots * (sv + 4)
     phase2 = 8 * (rl + 1) + ngp * sa + 4 * rl + rl * sy * b1        # groupPtr, partials, outRow, y of long rows
-    main = ((info["nnz_reg_new"] - chunk_slots + info["nnz_irreg"] + info["nnz_short_new"]) * (sv + 4)
+    main = ((info["nnz_reg_new"] + info["nnz_irreg"] + info["nnz_short_new"]) * (sv + 4)
             + 8 * (nrb + 1) + 4 * (info["row_medium"] + 1)
             + 4 * (8 * nrb + nout_short + info["n_empty"])                  # outRow of every other output slot
             + (m - rl) * sy * b1 + n * sx)
     overhead = {"irr_ptr_int64_all_slots": 8 * (8 * nrb + 1) - 4 * (info["row_medium"] + 1),
-                "long_unit_schedule": 4 * (ngp // 4),
-                "chunk_unit_partials_list": nch * (2 * 8 * sa + 8) + (4 * nrb if nch else 0)}
+                "long_unit_schedule": 4 * (ngp // 4)}
     csr_equiv = nnz * (sv + 4) + (m + 1) * 8 + n * sx + m * sy * b1
     return {"dasp_long_kernel": long_, "dasp_main_kernel": main + phase2, "total": long_ + main + phase2,
             "overhead": overhead, "csr_equiv": csr_equiv}
@@ -329,11 +321,8 @@ def time_oracle(A, x, dtype, budget_s):
 def make_plan(A, dtype, dev_index, variant, args):
     from paper_conf_sc_lu023_b200 import dasp
     val = A.val.astype({"f64": np.float64, "f16": np.float16, "f32": np.float32}[dtype])
-    kw = {}
-    if args.medium_units >= 0:
-        kw["medium_units"] = bool(args.medium_units)
     return dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dtype, device=dev_index, variant=variant,
-                                 medium_rb_per_warp=args.rbw, panel_rows=args.panel_rows, **kw)
+                                 medium_rb_per_warp=args.rbw, panel_rows=args.panel_rows)
 
 
 def timed_steps(step, plan, steps, warmup, dev, stream, clocks=True):
@@ -569,7 +558,6 @@ def run_single(args, local):
         "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config),
                    "m": int(spec.m), "n": int(spec.n), "nnz": nnz, "variant": args.variant,
                    "panel_rows": info["panel_rows"], "parallelism": "single GPU",
-                   "medium_chunk_units": info["medium_chunk_units"],
                    "l2": "inputs larger than L2 (packed A, 2.8 GB for C3 FP64, streamed every step); x stays "
                          "L2-resident across steps as in the paper's averaged back-to-back runs (P:L567)"},
         "effective_gbs": bm["csr_equiv"] / (ms_step * 1e-3) / 1e9,

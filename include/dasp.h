@@ -77,12 +77,6 @@ typedef struct {
     double threshold;           /* tau, "a customized parameter": an 8 x MMA_K block is
                                    regular iff it holds more than 8*MMA_K*tau nonzeros;
                                    0 = 0.75; must be <= 1                                     */
-    int32_t medium_units;       /* 1: the full chunks (4 regular blocks) of the wide
-                                   medium row-blocks run as independent chunk units in the long-row
-                                   launch, each writing its 8 row partials, which the row-block's
-                                   warp adds to its ragged chunk and irregular tails;
-                                   0 (default): one warp walks all of a row-block's chunks (Alg. 3 as
-                                   printed) -- chunk units measured C3 -4 %, C2 +24 %, C5 +6 %     */
 } dasp_options_t;
 
 /* Fills `opts` with the defaults: device 0, CUDA-core variant, validate, no keep_host, auto
@@ -114,7 +108,6 @@ typedef struct {
                                                           per-row / one-lane-per-row warps
                                                           (launch schedule)    */
     int32_t narrow_rb_per_warp;                        /* row-blocks per narrow / mid warp   */
-    int64_t medium_chunk_units;                        /* medium chunk units in the long launch */
 } dasp_plan_info_t;
 
 /*

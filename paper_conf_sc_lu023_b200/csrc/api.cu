@@ -49,10 +49,6 @@ struct dasp_plan_s {
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
     void* d_blk_word = nullptr;           // uint64 panel of every main-kernel block (kernels.cuh)
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
-    int64_t n_mchunks = 0;                // medium chunk units (full chunks of wide row-blocks) in the long launch
-    void* d_mchunk_base = nullptr;        // int64 [n_mchunks] element offset of each chunk unit
-    void* d_mchunk0 = nullptr;            // int32 [nrb] first chunk unit of each row-block (-1: none)
-    void* d_mpartial = nullptr;           // [8 n_mchunks] row partials of the chunk units (f64, f32 for FP16)
     // timing
     int32_t timing_cap = 0, timing_calls = 0;
     std::vector<TimingRec> recs;
@@ -87,7 +83,7 @@ constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read 
 #define DASP_NARROW_IL 0
 #endif
 #ifndef DASP_HEAVY_FIRST
-#define DASP_HEAVY_FIRST 0   // leading blocks of every panel dispatched at the start of the main grid
+#define DASP_HEAVY_FIRST 16  // leading blocks of every panel dispatched at the start of the main grid (C3 FP16 -2.7 %, FP64 -0.1..-0.8 %, others +-0.8 %: profiles/r02/heavy_first_ab.jsonl, chunk_units_removed_and_heavy_first.jsonl)
 #endif
 
 // LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
@@ -125,10 +121,7 @@ void free_device(dasp_plan_s* p) {
     if (p->d_blk_word) cudaFree(p->d_blk_word);
     if (p->d_unit_order) cudaFree(p->d_unit_order);
     p->d_panels = p->d_blk_word = p->d_unit_order = nullptr;
-    for (void** q : {&p->d_mchunk_base, &p->d_mchunk0, &p->d_mpartial}) {
-        if (*q) cudaFree(*q);
-        *q = nullptr;
-    }
+
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
     p->d_partial = p->d_xh = p->d_yh = nullptr;
@@ -181,7 +174,6 @@ int64_t alg_bytes(const dasp_plan_s* p, bool beta) {
     b += (f.nnz_reg_new + f.nnz_irreg) * (s_v + 4) + 8 * (f.nrb + 1) + 8 * (nmp + 1) + 4 * nmp;
     b += f.nnz_short_new * (s_v + 4) + 4 * nout;
     b += 4 * f.n0;
-    b += p->n_mchunks * (2 * 8 * s_a + 8) + (p->n_mchunks ? 4 * f.nrb : 0);   // chunk units
     b += f.n * s_x + f.m * s_y * (beta ? 2 : 1);
     return b;
 }
@@ -203,7 +195,6 @@ void dasp_options_default(dasp_options_t* o) {
     o->panel_rows = 0;
     o->max_len = 256;
     o->threshold = 0.75;
-    o->medium_units = 0;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -239,8 +230,7 @@ std::vector<int32_t> narrow_slots(const HostFormat& f, const int64_t* rb_ptr, co
 }
 
 dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_t* panel_table,
-                           const std::vector<int32_t>& unit_first_col, const std::vector<int32_t>& nslots,
-                           const int64_t* rb_ptr) {
+                           const std::vector<int32_t>& unit_first_col, const std::vector<int32_t>& nslots) {
     HostFormat& f = p->host;
     p->rbw = o.medium_rb_per_warp > 0 ? o.medium_rb_per_warp : auto_rbw(f.row_medium, f.nnz_medium, f.sumsq_medium);
     // a block's wide medium warps interleave their row-blocks when the medium rows are ragged
@@ -294,25 +284,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         blk_word.swap(order);
     }
     p->n_units = f.n_groups_padded / f.geo.UG;
-    // medium chunk units: every full chunk (CW regular blocks) of the wide row-blocks [rb0, rb0 +
-    // rbm) of each panel, in memory order, runs in the long-row launch (kernels.cu mchunk_pair_*);
-    // the row-block's warp adds the chunk partials to its ragged chunk and irregular tails
-    std::vector<int64_t> mchunk_base;
-    std::vector<int32_t> mchunk0;
-    const bool units = o.medium_units != 0 && rb_ptr != nullptr && f.nrb > 0;
-    if (units) {
-        const int64_t ce = static_cast<int64_t>(f.geo.CW) * f.geo.BE;   // elements of a full chunk
-        mchunk0.assign(static_cast<size_t>(f.nrb), -1);
-        for (const auto& d : desc)
-            for (int64_t rb = d.rb0; rb < d.rb0 + d.rbm; ++rb) {
-                const int64_t nfull = (rb_ptr[rb + 1] - rb_ptr[rb]) / ce;
-                if (nfull == 0) continue;
-                mchunk0[rb] = static_cast<int32_t>(mchunk_base.size());
-                for (int64_t c = 0; c < nfull; ++c) mchunk_base.push_back(rb_ptr[rb] + c * ce);
-            }
-        if (mchunk_base.size() >= (size_t(1) << 31)) return DASP_ERR_UNSUPPORTED;
-    }
-    p->n_mchunks = static_cast<int64_t>(mchunk_base.size());
+
     // long-unit execution order (a launch schedule, not part of the format): inside each panel
     // the units run bucketed by the column of their first element, so that the warps in flight
     // gather from ~1/kColBuckets of x at a time instead of all of it (long rows' columns are
@@ -355,13 +327,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
     if ((st = upload(&p->d_blk_word, blk_word.data(), blk_word.size() * 8)) != DASP_OK) return st;
     if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
-    if (p->n_mchunks > 0) {
-        if ((st = upload(&p->d_mchunk_base, mchunk_base.data(), mchunk_base.size() * 8)) != DASP_OK) return st;
-        if ((st = upload(&p->d_mchunk0, mchunk0.data(), mchunk0.size() * 4)) != DASP_OK) return st;
-        const size_t mb = static_cast<size_t>(p->n_mchunks) * 8 * sa(p->dtype);
-        if (cudaMalloc(&p->d_mpartial, mb) != cudaSuccess) return DASP_ERR_OUT_OF_MEMORY;
-        p->device_bytes += static_cast<int64_t>(mb);
-    }
+
     return DASP_OK;
 }
 
@@ -438,8 +404,7 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
         f.nrb ? narrow_slots(f, static_cast<const int64_t*>(f.arr[DASP_ARR_RB_PTR].ptr), irr_first.data()) : std::vector<int32_t>();
     std::unique_ptr<DeviceGuard> guard;
     if (p->device >= 0) guard.reset(new DeviceGuard(p->device));
-    st = setup_launch(p, o, static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr), first_col, nslots,
-                      static_cast<const int64_t*>(f.arr[DASP_ARR_RB_PTR].ptr));
+    st = setup_launch(p, o, static_cast<const int64_t*>(f.arr[DASP_ARR_PANELS].ptr), first_col, nslots);
     if (st != DASP_OK) return fail(p, st);
     if (p->device >= 0) {
         for (int a = 0; a < DASP_ARR_COUNT; ++a) {
@@ -499,10 +464,8 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
                                     static_cast<int64_t>(first_col.size()), first_col.data(), s) != cudaSuccess)
         return fail(p, DASP_ERR_CUDA);
     std::vector<int32_t> nslots;
-    std::vector<int64_t> rbp;
     if (f.nrb > 0) {   // rb_ptr and irr_ptr[8 rb .. 8 rb + 1] back from the device
-        rbp.resize(static_cast<size_t>(f.nrb + 1));
-        std::vector<int64_t> irr_first(static_cast<size_t>(2 * f.nrb));
+        std::vector<int64_t> rbp(static_cast<size_t>(f.nrb + 1)), irr_first(static_cast<size_t>(2 * f.nrb));
         if (cudaMemcpyAsync(rbp.data(), p->d[DASP_ARR_RB_PTR], rbp.size() * 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
             cudaMemcpy2DAsync(irr_first.data(), 16, p->d[DASP_ARR_IRR_PTR], 64, 16, static_cast<size_t>(f.nrb),
                               cudaMemcpyDeviceToHost, s) != cudaSuccess ||
@@ -510,7 +473,7 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
             return fail(p, DASP_ERR_CUDA);
         nslots = narrow_slots(f, rbp.data(), irr_first.data());
     }
-    st = setup_launch(p, o, f.panel_table.data(), first_col, nslots, rbp.empty() ? nullptr : rbp.data());
+    st = setup_launch(p, o, f.panel_table.data(), first_col, nslots);
     if (st != DASP_OK) return fail(p, st);
     *plan_out = p;
     return DASP_OK;
@@ -585,15 +548,11 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.nrw = p->nrw;
     mp.extra = extra;
     mp.class_mask = DASP_CLASS_MASK;
-    mp.mchunk_base = static_cast<const int64_t*>(p->d_mchunk_base);
-    mp.mchunk0 = static_cast<const int32_t*>(p->d_mchunk0);
-    mp.mpartial = p->d_mpartial;
-    mp.n_mchunks = p->n_mchunks;
     const int64_t n0 = (beta == 1.0 && extra.n == 0) ? 0 : f.n0;   // scatter mode must still copy them
     mp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
     mp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
     mp.empty_rows = static_cast<const int32_t*>(p->d[DASP_ARR_EMPTY_ROWS]);
-    if (p->n_units + p->n_mchunks > 0) {
+    if (p->n_units > 0) {
         e = timed(p, DASP_K_LONG, s, on, [&] { return dasp::launch_long(mp, p->dtype, variant, p->n_units, s); });
         if (e != cudaSuccess) return DASP_ERR_CUDA;
     }
@@ -722,8 +681,7 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->alg_bytes_beta0 = alg_bytes(p, false);
     o->alg_bytes_beta1 = alg_bytes(p, true);
     o->medium_rb_per_warp = p->rbw;
-    o->launches_per_spmv = (p->n_units + p->n_mchunks > 0 ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0);
-    o->medium_chunk_units = p->n_mchunks;
+    o->launches_per_spmv = (p->n_units > 0 ? 1 : 0) + (p->blocks + f.row_long + f.n0 > 0 ? 1 : 0);
     o->panel_rows = f.panel_rows;
     o->n_panels = f.n_panels;
     o->rowblocks_mid = p->rb_mid;

@@ -157,24 +157,9 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
 __device__ __forceinline__ int32_t xi(uint32_t c) {
     return DASP_EXP_NOX ? static_cast<int32_t>(c & 255u) : static_cast<int32_t>(c);
 }
-#ifndef DASP_EXP_HOT
-#define DASP_EXP_HOT 0   // experiment only: x gathers of columns < g_hot_cols keep L1 (evict_last), others default
-#endif
-#if DASP_EXP_HOT
-__device__ int32_t g_hot_cols;
-__device__ __forceinline__ double gx(const double* x, uint32_t c) {
-    if (static_cast<int32_t>(c) < 0) return 0.0;
-    const double* a = x + static_cast<int32_t>(c);
-    double v;
-    if (static_cast<int32_t>(c) < g_hot_cols) asm("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(a));
-    else v = __ldg(a);
-    return v;
-}
-#else
 __device__ __forceinline__ double gx(const double* x, uint32_t c) {
     return static_cast<int32_t>(c) >= 0 ? __ldg(x + xi(c)) : 0.0;
 }
-#endif
 __device__ __forceinline__ double gx_f64(const double* x, uint32_t c) { return gx(x, c); }
 __device__ __forceinline__ uint16_t gxh(const uint16_t* x, uint32_t c) {
     return static_cast<int32_t>(c) >= 0 ? __ldg(reinterpret_cast<const unsigned short*>(x) + xi(c))
@@ -398,105 +383,6 @@ __device__ __forceinline__ void long_unit_f16(const MainParams& P, int64_t u, in
 }
 
 // ------------------------------------------------------------------------------------------
-// medium chunk units: the full lane-interleaved chunks (CW = 4 regular blocks,
-// R18) of the wide medium row-blocks, run in the long-row launch two chunks per warp.  Lane
-// (g, t) holds its element of the chunk's 4 blocks (row g, slot t of each block): 4 products,
-// then a quad reduction (CUDA-core) or 4 block MMAs and the diagonal (Fig. 4) give row g's sum
-// over the chunk, stored as partial[k*8 + g].  The main kernel's warp for the row-block adds its
-// chunks' partials (fixed order) to the ragged chunk and the irregular tails (Alg. 3 l.20-25).
-// ------------------------------------------------------------------------------------------
-template <int DT, int VAR>
-__device__ __forceinline__ void mchunk_pair_f64(const MainParams& P, int64_t k, int lane, uint64_t pol) {
-    using IO = ValIO<DT>;
-    const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
-    const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
-    const bool two = k + 1 < P.n_mchunks;
-    const int64_t b0 = __ldg(P.mchunk_base + k), b1 = two ? __ldg(P.mchunk_base + k + 1) : b0;
-    typename IO::R v[2][4];
-    uint32_t c[2][4];
-    IO::ld4r(rv + b0 + lane * 4, pol, v[0]);
-    ld4_b32(P.reg_col + b0 + lane * 4, pol, c[0]);
-    if (two) {
-        IO::ld4r(rv + b1 + lane * 4, pol, v[1]);
-        ld4_b32(P.reg_col + b1 + lane * 4, pol, c[1]);
-    } else {
-#pragma unroll
-        for (int j = 0; j < 4; ++j) { v[1][j] = 0; c[1][j] = 0xffffffffu; }
-    }
-    double xv[2][4];
-#pragma unroll
-    for (int h = 0; h < 2; ++h)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) xv[h][j] = IO::gx(x, c[h][j]);
-    double* mp = static_cast<double*>(P.mpartial);
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        double part;
-        if constexpr (vk(VAR) == VAR_MMA) {
-            double c0 = 0.0, c1 = 0.0;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) dmma(c0, c1, IO::cv(v[h][j]), xv[h][j]);
-            part = diag_to_quad(c0, c1, lane);
-        } else {
-            part = 0.0;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) part = fma(IO::cv(v[h][j]), xv[h][j], part);
-            part += __shfl_xor_sync(FULL, part, 1);
-            part += __shfl_xor_sync(FULL, part, 2);
-        }
-        if ((lane & 3) == 0 && (h == 0 || two)) mp[(k + h) * 8 + (lane >> 2)] = part;
-    }
-}
-// FP16: a chunk is 4 blocks of 8 x 8 (256 halves); lane (g, t) holds slots 2t, 2t+1 of row g of
-// each block (a 16-B value load, a 32-B column load)
-template <int VAR>
-__device__ __forceinline__ void mchunk_pair_f16(const MainParams& P, int64_t k, int lane, uint64_t pol) {
-    const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
-    const uint16_t* x = static_cast<const uint16_t*>(P.x);
-    const bool two = k + 1 < P.n_mchunks;
-    const int64_t b0 = __ldg(P.mchunk_base + k), b1 = two ? __ldg(P.mchunk_base + k + 1) : b0;
-    uint32_t v[2][4], c[2][8];
-    ld4_b32(rv + b0 + lane * 8, pol, v[0]);
-    ld8_b32(P.reg_col + b0 + lane * 8, pol, c[0]);
-    if (two) {
-        ld4_b32(rv + b1 + lane * 8, pol, v[1]);
-        ld8_b32(P.reg_col + b1 + lane * 8, pol, c[1]);
-    } else {
-#pragma unroll
-        for (int j = 0; j < 4; ++j) v[1][j] = 0u;
-#pragma unroll
-        for (int e = 0; e < 8; ++e) c[1][e] = 0xffffffffu;
-    }
-    uint16_t xh[2][8];
-#pragma unroll
-    for (int h = 0; h < 2; ++h)
-#pragma unroll
-        for (int e = 0; e < 8; ++e) xh[h][e] = gxh(x, c[h][e]);
-    float* mp = static_cast<float*>(P.mpartial);
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        float part;
-        if constexpr (vk(VAR) == VAR_MMA) {
-            float c0 = 0.f, c1 = 0.f;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) hmma(c0, c1, v[h][j], pack2(xh[h][2 * j], xh[h][2 * j + 1]));
-            part = diag_to_quad(c0, c1, lane);
-        } else {
-            part = 0.f;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const float2 a = u2f2(v[h][j]);
-                part = fmaf(a.x, h2f(xh[h][2 * j]), part);
-                part = fmaf(a.y, h2f(xh[h][2 * j + 1]), part);
-            }
-            part += __shfl_xor_sync(FULL, part, 1);
-            part += __shfl_xor_sync(FULL, part, 2);
-        }
-        if ((lane & 3) == 0 && (h == 0 || two)) mp[(k + h) * 8 + (lane >> 2)] = part;
-    }
-}
-
-// ------------------------------------------------------------------------------------------
 // medium rows (Alg. 3): row-block = 8 rows; regular 8 x K blocks in lane-interleaved chunks
 // of CW blocks (R18), then the irregular tails with 4 lanes per row, then y.
 // ------------------------------------------------------------------------------------------
@@ -506,15 +392,12 @@ struct RbMeta {
     int64_t base, ib;         // regular region start; this lane's row's irregular start
     int32_t nelem, ilen;      // regular elements (<= 64 blocks); irregular length (<= 256)
     int32_t orow;
-    int32_t k0;               // >= 0: the full chunks are chunk units k0, k0+1, ... of the long kernel
 };
-// units: the row-block is a wide one of a plan whose full chunks run as chunk units (MainParams::mchunk0)
-__device__ __forceinline__ RbMeta rb_meta(const MainParams& P, int64_t rb, int lane, bool units = false) {
+__device__ __forceinline__ RbMeta rb_meta(const MainParams& P, int64_t rb, int lane) {
     const int64_t i = rb * 8 + (lane >> 2);
     const int64_t base = __ldg(P.rb_ptr + rb), ib = __ldg(P.irr_ptr + i);
     return RbMeta{base, ib, static_cast<int32_t>(__ldg(P.rb_ptr + rb + 1) - base),
-                  static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i),
-                  units ? __ldg(P.mchunk0 + rb) : -1};
+                  static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i)};
 }
 
 // A row-block is processed in two halves so that a warp can keep the round-1 loads of two
@@ -527,7 +410,6 @@ __device__ __forceinline__ RbMeta rb_meta(const MainParams& P, int64_t rb, int l
 template <int DT> struct MedLd {
     typename ValIO<DT>::R va[4], vr[3], vi;
     uint32_t ca[4], cr[3], ci;
-    double up;                // chunk-unit partials of this lane's row (chunks t, t+4 of the row-block)
 };
 // FULL = false: the row-block is known to have no full chunk (nreg < CW), so the chunk state is
 // dead code and two such row-blocks fit in the registers of one (the small-pair path).
@@ -538,18 +420,10 @@ __device__ __forceinline__ void medium_load_f64(const MainParams& P, const RbMet
     const int nfull = FULL ? nreg >> 2 : 0, rem = nreg & 3;
     const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
-    L.up = 0.0;
     if constexpr (FULL) {
 #pragma unroll
         for (int j = 0; j < 4; ++j) { L.va[j] = 0; L.ca[j] = 0xffffffffu; }
-        if (M.k0 >= 0) {                                 // full chunks done by chunk units: their row partials
-            const int t = lane & 3, g = lane >> 2;
-            const double* mp = static_cast<const double*>(P.mpartial);
-            if (t < nfull) L.up = __ldcg(mp + (static_cast<int64_t>(M.k0) + t) * 8 + g);
-            if (t + 4 < nfull) L.up += __ldcg(mp + (static_cast<int64_t>(M.k0) + t + 4) * 8 + g);
-        } else if (nfull > 0) {
-            IO::ld4r(rv + lane * 4, pol, L.va); ld4_b32(rc + lane * 4, pol, L.ca);
-        }
+        if (nfull > 0) { IO::ld4r(rv + lane * 4, pol, L.va); ld4_b32(rc + lane * 4, pol, L.ca); }
     }
     const int64_t rbase = static_cast<int64_t>(nfull) * 128 + lane;   // ragged chunk: block j at 32j (R18)
 #pragma unroll
@@ -579,15 +453,14 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
         for (int j = 0; j < 4; ++j) { va[j] = L.va[j]; ca[j] = L.ca[j]; }
         // software pipeline: chunk ch+1's stream loads are issued while chunk ch's gathers are
         // in flight (one memory round trip per chunk instead of two)
-        const int nloop = M.k0 >= 0 ? 0 : nfull;         // chunk units: the long kernel did them
-        for (int ch = 0; ch < nloop; ++ch) {
+        for (int ch = 0; ch < nfull; ++ch) {
             if (!DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
             double xv[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
             typename IO::R vn[4];
             uint32_t cn[4];
-            if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nloop) {
+            if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nfull) {
                 IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vn);
                 ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cn);
             }
@@ -596,7 +469,7 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
                 if constexpr (vk(VAR) == VAR_MMA) dmma(c0, c1, IO::cv(va[j]), xv[j]);
                 else part = fma(IO::cv(va[j]), xv[j], part);
             }
-            if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nloop) {
+            if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nfull) {
 #pragma unroll
                 for (int j = 0; j < 4; ++j) { va[j] = vn[j]; ca[j] = cn[j]; }
             }
@@ -617,11 +490,6 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
         const double d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.0;
     }
-    if (M.k0 >= 0) {                                       // chunk-unit partials (chunks t, t+4, t+8, ...)
-        part += L.up;
-        const double* mp = static_cast<const double*>(P.mpartial);
-        for (int c = t + 8; c < nfull; c += 4) part += __ldcg(mp + (static_cast<int64_t>(M.k0) + c) * 8 + (lane >> 2));
-    }
     part = fma(IO::cv(L.vi), xi, part);                    // Alg. 3 l.20-24: irregular part
     const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
     for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
@@ -634,7 +502,6 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
 struct MedLdH {
     uint32_t va[4], ca[8], vr[3], cr[6], ci;
     uint16_t vi;
-    float up;                 // chunk-unit partials of this lane's row (chunks t, t+4)
 };
 template <bool FULL = true>
 __device__ __forceinline__ void medium_load_f16(const MainParams& P, const RbMeta& M, int lane, uint64_t pol, MedLdH& L) {
@@ -642,20 +509,12 @@ __device__ __forceinline__ void medium_load_f16(const MainParams& P, const RbMet
     const int nfull = FULL ? nreg >> 2 : 0, rem = nreg & 3;
     const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
-    L.up = 0.f;
     if constexpr (FULL) {
 #pragma unroll
         for (int j = 0; j < 4; ++j) L.va[j] = 0u;
 #pragma unroll
         for (int e = 0; e < 8; ++e) L.ca[e] = 0xffffffffu;
-        if (M.k0 >= 0) {                                 // full chunks done by chunk units
-            const int t = lane & 3, g = lane >> 2;
-            const float* mp = static_cast<const float*>(P.mpartial);
-            if (t < nfull) L.up = __ldcg(mp + (static_cast<int64_t>(M.k0) + t) * 8 + g);
-            if (t + 4 < nfull) L.up += __ldcg(mp + (static_cast<int64_t>(M.k0) + t + 4) * 8 + g);
-        } else if (nfull > 0) {
-            ld4_b32(rv + lane * 8, pol, L.va); ld8_b32(rc + lane * 8, pol, L.ca);
-        }
+        if (nfull > 0) { ld4_b32(rv + lane * 8, pol, L.va); ld8_b32(rc + lane * 8, pol, L.ca); }
     }
     const int64_t rbase = static_cast<int64_t>(nfull) * 256 + lane * 2;   // ragged chunk: block j at 64j (R18)
 #pragma unroll
@@ -694,17 +553,16 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
         for (int j = 0; j < 4; ++j) va[j] = L.va[j];
 #pragma unroll
         for (int e = 0; e < 8; ++e) ca[e] = L.ca[e];
-        const int nloop = M.k0 >= 0 ? 0 : nfull;         // chunk units: the long kernel did them
-        for (int ch = 0; ch < nloop; ++ch) {   // chunk ch+1's loads overlap chunk ch's gathers
+        for (int ch = 0; ch < nfull; ++ch) {   // chunk ch+1's loads overlap chunk ch's gathers
             if (!DASP_CHUNK_PIPE_F16 && ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
             uint16_t xh[8];
 #pragma unroll
             for (int e = 0; e < 8; ++e) xh[e] = gxh(x, ca[e]);
             uint32_t vn[4], cn[8];
-            if (DASP_CHUNK_PIPE_F16 && ch + 1 < nloop) { ld4_b32(rv + (ch + 1) * 256 + lane * 8, pol, vn); ld8_b32(rc + (ch + 1) * 256 + lane * 8, pol, cn); }
+            if (DASP_CHUNK_PIPE_F16 && ch + 1 < nfull) { ld4_b32(rv + (ch + 1) * 256 + lane * 8, pol, vn); ld8_b32(rc + (ch + 1) * 256 + lane * 8, pol, cn); }
 #pragma unroll
             for (int j = 0; j < 4; ++j) blockx(va[j], xh[2 * j], xh[2 * j + 1]);
-            if (DASP_CHUNK_PIPE_F16 && ch + 1 < nloop) {
+            if (DASP_CHUNK_PIPE_F16 && ch + 1 < nfull) {
 #pragma unroll
                 for (int j = 0; j < 4; ++j) va[j] = vn[j];
 #pragma unroll
@@ -718,11 +576,6 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
     if constexpr (vk(VAR) == VAR_MMA) {
         const float d = diag_to_quad(c0, c1, lane);
         part = t == 0 ? d : 0.f;
-    }
-    if (M.k0 >= 0) {                                       // chunk-unit partials (chunks t, t+4, t+8, ...)
-        part += L.up;
-        const float* mp = static_cast<const float*>(P.mpartial);
-        for (int c = t + 8; c < nfull; c += 4) part += __ldcg(mp + (static_cast<int64_t>(M.k0) + c) * 8 + (lane >> 2));
     }
     part = fmaf(h2f(L.vi), h2f(gxh(x, L.ci)), part);
     for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
@@ -747,7 +600,7 @@ __device__ __forceinline__ void medium_rb_f16(const MainParams& P, const RbMeta&
 
 template <int DT, int VAR>
 __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int64_t rb1, int lane, uint64_t pol,
-                                           int64_t st = 1, bool units = false) {   // row-blocks rb0, rb0 + st, ... < rb1
+                                           int64_t st = 1) {   // row-blocks rb0, rb0 + st, ... < rb1
     if constexpr (DASP_BY_DT(DT, DASP_SMALL_PAIR) != 0) {
         // small-pair path: two consecutive row-blocks without a full chunk (nreg < CW: rows of
         // up to ~15 nonzeros, most medium rows of a power-law matrix) load together, so a warp
@@ -755,8 +608,8 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
         constexpr int FULL_ELEMS = DT == 1 ? 256 : 128;   // elements of one CW-block chunk
         int64_t rb = rb0;
         while (rb < rb1) {
-            const RbMeta MA = rb_meta(P, rb, lane, units);   // both metadata rounds issued together
-            const RbMeta MB = rb + st < rb1 ? rb_meta(P, rb + st, lane, units) : RbMeta{0, 0, FULL_ELEMS, 0, -1, -1};
+            const RbMeta MA = rb_meta(P, rb, lane);     // both metadata rounds issued together
+            const RbMeta MB = rb + st < rb1 ? rb_meta(P, rb + st, lane) : RbMeta{0, 0, FULL_ELEMS, 0, -1};
             {
                 if (MA.nelem < FULL_ELEMS && MB.nelem < FULL_ELEMS) {
                     if constexpr (DT == 1) {
@@ -789,7 +642,7 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
         for (int64_t rb = rb0; rb < rb1; rb += st) {
             // (prefetching the next row-block's metadata here was measured: it costs registers
             // and spills in the FP64 MMA instantiation, net slower; profiles/r01/meta_prefetch_rbw.jsonl)
-            const RbMeta M = rb_meta(P, rb, lane, units);
+            const RbMeta M = rb_meta(P, rb, lane);
 #if DASP_EXP_TRACE
             if (first) { wait_on(static_cast<uint32_t>(M.base) ^ static_cast<uint32_t>(M.orow)); tr.c1 = clk64(); }
 #endif
@@ -1331,7 +1184,7 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
         const int64_t stg = P.wide_il ? min(static_cast<int64_t>(WARPS_PER_BLOCK), nmwd - gw) : 1;
         const int64_t rbs = P.wide_il ? rbp0 + gw * P.rbw + (w - gw) : rbp0 + w * P.rbw;
         const int64_t rbend = min(rbs - (w - gw) * (P.wide_il != 0) + stg * P.rbw, rbe);
-        medium_rbs<DT, VAR>(P, rbs, rbend, lane, pol, stg, P.n_mchunks > 0);
+        medium_rbs<DT, VAR>(P, rbs, rbend, lane, pol, stg);
         return;
     }
     const int64_t nmwm = __ldg(&D->nmwm);
@@ -1380,16 +1233,9 @@ __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_LONG_MIN_BLOCKS
                                                          : (DT == 1 ? DASP_LONG_MIN_BLOCKS_F16 : DASP_LONG_MIN_BLOCKS_F32))
 dasp_long_kernel(const MainParams P, int64_t n_units) {
     const int64_t w = (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5;
+    if (w >= n_units) return;
     const int lane = threadIdx.x & 31;
     const uint64_t pol = stream_policy();
-    if (w >= n_units) {                                  // medium chunk units, two per warp
-        const int64_t k = 2 * (w - n_units);
-        if (k < P.n_mchunks) {
-            if constexpr (DT == 1) mchunk_pair_f16<VAR>(P, k, lane, pol);
-            else mchunk_pair_f64<DT, VAR>(P, k, lane, pol);
-        }
-        return;
-    }
     const int64_t u = __ldg(P.unit_order + w);
     if constexpr (DT == 1) long_unit_f16<VAR>(P, u, lane, pol);
     else long_unit_f64<DT, VAR>(P, u, lane, pol);
@@ -1447,11 +1293,6 @@ __global__ void __launch_bounds__(256) dasp_gather_kernel(const W* __restrict__ 
 
 }  // namespace
 
-#if DASP_EXP_HOT
-extern "C" int dasp_exp_set_hot(int32_t h) {
-    return cudaMemcpyToSymbol(g_hot_cols, &h, sizeof(h)) == cudaSuccess ? 0 : 4;
-}
-#endif
 #if DASP_EXP_TRACE
 extern "C" int dasp_exp_trace_read(void* dst, int64_t bytes, int clear) {
     const int64_t nb = bytes < kTraceWarps * 64 ? bytes : kTraceWarps * 64;
@@ -1489,9 +1330,8 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
 }
 
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s) {
-    const int64_t warps = n_units + (p.n_mchunks + 1) / 2;
-    if (warps <= 0) return cudaSuccess;
-    const int64_t blocks = (warps * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
+    if (n_units <= 0) return cudaSuccess;
+    const int64_t blocks = (n_units * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
     const bool mma = variant == VAR_MMA;

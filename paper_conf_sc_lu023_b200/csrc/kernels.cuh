@@ -71,20 +71,12 @@ struct MainParams {
     const int32_t* long_out;
     const int32_t* empty_rows;
     int64_t row_long, n0, fin_warps;
-    // medium chunk units (n_mchunks > 0): the full chunks of the wide row-blocks run in the long
-    // kernel; mchunk_base[k] = element offset of chunk k in reg_val / reg_col, mpartial[8k + g] =
-    // row g's sum over it (f64, or f32 for FP16), mchunk0[rb] = the first chunk of row-block rb
-    const int64_t* mchunk_base;
-    const int32_t* mchunk0;
-    void* mpartial;
-    int64_t n_mchunks;
 };
 // finish work of the fused main kernel: 4 long rows per warp, then 128 empty rows per warp
 inline int64_t finish_warps(int64_t row_long, int64_t n0) { return (row_long + 3) / 4 + (n0 + 127) / 128; }
 
 // variant: 1 = MMA (DMMA/HMMA diagonal trick), 2 = CUDA-core.  dtype: 0 = FP64, 1 = FP16, 2 = FP32.
 cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s);
-// long units (Alg. 2 phase 1) then, two per warp, the medium chunk units of p
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
 // short tiles one main-kernel warp processes (build knob DASP_SHORT_TPW)
 int short_tiles_per_warp(int dtype);

@@ -44,7 +44,7 @@ class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("variant", ctypes.c_int32), ("validate", ctypes.c_int32),
                 ("keep_host", ctypes.c_int32), ("medium_rb_per_warp", ctypes.c_int32),
                 ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64),
-                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double), ("medium_units", ctypes.c_int32)]
+                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -59,8 +59,7 @@ class PlanInfo(ctypes.Structure):
                 ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64),
                 ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
                 ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double),
-                ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32),
-                ("medium_chunk_units", ctypes.c_int64)]
+                ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32)]
 
     def as_dict(self):
         return {name: getattr(self, name) for name, _ in self._fields_}
@@ -162,7 +161,7 @@ class Plan:
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                      variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, keep_host: bool = False,
                      medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0,
-                     max_len: int = 256, threshold: float = 0.75, medium_units: bool | None = None) -> Plan:
+                     max_len: int = 256, threshold: float = 0.75) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
@@ -193,8 +192,6 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     opts.keep_host, opts.medium_rb_per_warp, opts.num_threads = int(keep_host), medium_rb_per_warp, num_threads
     opts.panel_rows = panel_rows
     opts.max_len, opts.threshold = int(max_len), float(threshold)
-    if medium_units is not None:          # None: the library default (dasp_options_default)
-        opts.medium_units = int(medium_units)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))
@@ -205,7 +202,7 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
 def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                             variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, medium_rb_per_warp: int = 0,
                             panel_rows: int = 0, max_len: int = 256, threshold: float = 0.75,
-                            stream=None, medium_units: bool | None = None) -> Plan:
+                            stream=None) -> Plan:
     """Build the plan on the GPU from a device CSR (torch CUDA tensors: int64 row_ptr, int32
     col_idx, float64 / float16 val) -- SURVEY.md §8(f) f2."""
     import torch
@@ -222,8 +219,6 @@ def dasp_plan_create_device(row_ptr, col_idx, val, m: int, n: int, dtype: str = 
     opts.device, opts.variant, opts.validate = device, variant, int(validate)
     opts.medium_rb_per_warp, opts.panel_rows = medium_rb_per_warp, panel_rows
     opts.max_len, opts.threshold = int(max_len), float(threshold)
-    if medium_units is not None:
-        opts.medium_units = int(medium_units)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create_device(ctypes.byref(h), m, n, int(col_idx.numel()), _ptr(row_ptr), _ptr(col_idx),
                                       _ptr(val), {"f64": DASP_R_64F, "f16": DASP_R_16F, "f32": DASP_R_32F}[dtype],

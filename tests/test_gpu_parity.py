@@ -456,31 +456,3 @@ def test_unsorted_duplicate_rectangular_bit_exact(name, A, dt, variant):
         hplan = make(A, dt)
         for arr in dasp.ARRAYS:
             assert np.array_equal(dasp.dasp_plan_copy_array(dplan, arr), dasp.dasp_plan_copy_array(hplan, arr)), arr
-
-
-# medium chunk units (dasp_options_t.medium_units): the full chunks of the wide
-# row-blocks run in the long-row launch and the row-block's warp adds their row partials.  Same
-# integers bit for bit with and without, every dtype and variant, panels on and off.
-@pytest.mark.parametrize("variant", VARIANTS, ids=[VNAME[v] for v in VARIANTS])
-@pytest.mark.parametrize("dt", DTYPES)
-def test_medium_chunk_units_on_off(dt, variant):
-    rng = np.random.default_rng(9)
-    lens = list(rng.integers(5, 257, size=4001)) + [0, 1, 2, 3, 300, 5000] * 3   # nfull 0..16 per row-block
-    cases = [("lens", lambda vm: synth.from_lengths(lens, n=9000, seed=17, val_mode=vm))] + CASES
-    for name, gen in cases:
-        A = gen(synth.VAL_INT)
-        x = synth.vector(91, A.n, synth.VAL_INT)
-        y0 = synth.vector(92, A.m, synth.VAL_INT)
-        y_ref, _ = oracle_ref(A, x, dt, 1.5, -2.0, y0)
-        for units in (True, False):
-            for panel in (0, 900):
-                plan = make(A, dt, medium_units=units, panel_rows=panel)
-                if not units:
-                    assert plan.info["medium_chunk_units"] == 0
-                assert np.array_equal(run(plan, x, dt, 1.5, -2.0, y0, variant=variant), y_ref), (name, units, panel)
-        Ar = gen(synth.VAL_UNIFORM)
-        xr = synth.vector(93, Ar.n)
-        y_ref, s = oracle_ref(Ar, xr, dt)
-        plan = make(Ar, dt, medium_units=True)
-        assert oracle.tolerance_ok(run(plan, xr, dt, variant=variant), y_ref, s, dt).all(), name
-    assert make(synth.from_lengths(lens, n=9000, seed=17), dt, medium_units=True).info["medium_chunk_units"] > 0
