@@ -264,9 +264,11 @@ def _default_stream(plan, stream):
     which torch's pool streams do not synchronise with)."""
     if stream is not None:
         return stream
-    import torch
     if not hasattr(plan, "_dev"):
         plan._dev = plan.info["device"]
+    if plan._dev < 0:                     # host-only plan: the library reports UNSUPPORTED
+        return None
+    import torch
     return torch.cuda.current_stream(plan._dev)
 
 

@@ -207,3 +207,24 @@ def test_narrow_mid_split(dt, panel):
         mid += n_mid
     assert (info["rowblocks_narrow"], info["rowblocks_mid"]) == (narrow, mid)
     assert info["narrow_rb_per_warp"] in (4, 8)
+
+
+def test_binding_rejects_short_and_mistyped_host_buffers():
+    """The ctypes binding checks what the C call trusts: col / val must hold row_ptr[m] entries, and
+    host x / y buffers must have the plan's element types and enough elements."""
+    A = synth.generate(synth.config("c1a"))
+    with pytest.raises(ValueError):
+        dasp.dasp_plan_create(A.row_ptr, A.col[:-5], A.val[:-5], A.m, A.n, "f64", device=-1)
+    with pytest.raises(ValueError):
+        dasp.dasp_plan_create(A.row_ptr, A.col, A.val[:-1], A.m, A.n, "f64", device=-1)
+    p = dasp.dasp_plan_create(A.row_ptr, A.col, A.val, A.m, A.n, "f64", device=-1)
+    x = np.zeros(A.n)
+    y = np.zeros(A.m)
+    for bad_x, bad_y in [(x[:-1], y), (x, y[:-1]), (x.astype(np.float32), y), (x, y.astype(np.float32)),
+                         (np.zeros((2, A.n))[:, 0], y)]:
+        with pytest.raises(ValueError):
+            dasp.dasp_spmv_host(p, bad_x, bad_y)
+    with pytest.raises(ValueError):
+        dasp.dasp_spmv_host_stream(p, np.zeros(2 * A.n - 1), A.n, np.zeros(2 * A.m), A.m, 2)
+    with pytest.raises(ValueError):
+        dasp.dasp_spmv_host_stream(p, np.zeros(2 * A.n), A.n, np.zeros(2 * A.m - 1), A.m, 2)

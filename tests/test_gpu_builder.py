@@ -101,3 +101,19 @@ def test_device_builder_full_size_matches_host():
     for arr in dasp.ARRAYS:
         assert np.array_equal(dasp.dasp_plan_copy_array(dplan, arr), dasp.dasp_plan_copy_array(hplan, arr)), arr
     # (the build time itself is reported by bench.py "preprocessing", not asserted here)
+
+
+def test_device_builder_rejects_short_arrays_before_reading_them():
+    """row_ptr[m] larger than the col / val arrays handed over (nnz = their length): INVALID_CSR is
+    returned before any kernel reads past them, and the context stays usable."""
+    A = synth.generate(synth.config("c1a"))
+    rp = torch.from_numpy(A.row_ptr).cuda()
+    short = A.nnz - 1000
+    col = torch.from_numpy(A.col[:short].copy()).cuda()
+    val = torch.from_numpy(A.val[:short].copy()).cuda()
+    with pytest.raises(dasp.DaspError) as e:
+        dasp.dasp_plan_create_device(rp, col, val, A.m, A.n, "f64")
+    assert e.value.status == 2
+    torch.cuda.synchronize()                      # no sticky fault
+    plan = device_plan(A, "f64")
+    assert plan.info["nnz"] == A.nnz
