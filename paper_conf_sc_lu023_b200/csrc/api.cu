@@ -86,17 +86,21 @@ constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read 
 #define DASP_HEAVY_FIRST 16  // leading blocks of every panel dispatched at the start of the main grid (C3 FP16 -2.7 %, FP64 -0.1..-0.8 %, others +-0.8 %: profiles/r02/heavy_first_ab.jsonl, chunk_units_removed_and_heavy_first.jsonl)
 #endif
 
-// LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl):
-// small matrices keep the paper's 1 / 2; for large ones, uniform medium rows (coefficient of
-// variation of the length < 0.5, e.g. stencils) run best with 8 row-blocks per warp, ragged
-// ones (power-law) with 4 -- more would leave warps with very unequal work.
+// LOOP_NUM (row-blocks per warp, R11) re-tuned on B200 (profiles/r01/rbw_sweep.jsonl,
+// profiles/r02/loop_num_recheck.jsonl): small matrices keep the paper's 1 / 2; for large ones, uniform
+// medium rows (coefficient of variation of the length < 0.5, e.g. stencils) run best with 8 row-blocks
+// per warp, ragged ones with 4, heavy-tailed ones (cv >= 1, power law) with 2 -- more would leave
+// warps with very unequal work.
 int auto_rbw(int64_t row_medium, int64_t nnz_medium, int64_t sumsq_medium) {
     if (row_medium < 59990) return 1;
     if (row_medium < 400000) return 2;
     const double mean = static_cast<double>(nnz_medium) / static_cast<double>(row_medium);
     const double var = static_cast<double>(sumsq_medium) / static_cast<double>(row_medium) - mean * mean;
     const double cv = var > 0 ? std::sqrt(var) / mean : 0.0;
-    return cv < 0.5 ? 8 : 4;
+    // heavy-tailed lengths (power law, cv >= 1) leave a few warps with far more chunks than the rest:
+    // 2 row-blocks per warp (C3 main -4.3 %, FP16 -1.4 %; C5, cv 0.55, keeps 4: +2 % at 2;
+    // profiles/r02/loop_num_recheck.jsonl)
+    return cv < 0.5 ? 8 : (cv < 1.0 ? 4 : 2);
 }
 
 struct DeviceGuard {
