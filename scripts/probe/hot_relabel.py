@@ -46,7 +46,9 @@ def time_plan(A, x, dtype, steps=200):
 
 def main():
     cfg = sys.argv[1] if len(sys.argv) > 1 else "c3"
-    A = synth.generate(synth.config(cfg))
+    scale = float(sys.argv[2]) if len(sys.argv) > 2 else 1.0
+    hs = [int(h) for h in sys.argv[3].split(",")] if len(sys.argv) > 3 else [250_000, 1_000_000, 2_000_000, 4_000_000]
+    A = synth.generate(synth.config(cfg, scale=scale))
     x = synth.vector(101, A.n)
     base, y0 = time_plan(A, x, "f64")
     print(json.dumps({"case": "original", **base}), flush=True)
@@ -54,7 +56,7 @@ def main():
     order = np.argsort(-cnt, kind="stable")
     lens = np.diff(A.row_ptr)
     rows = torch.repeat_interleave(torch.arange(A.m, device="cuda"), torch.from_numpy(lens).cuda())
-    for H in (250_000, 1_000_000, 2_000_000, 4_000_000):
+    for H in hs:
         hot = np.sort(order[:H])
         is_hot = np.zeros(A.n, dtype=bool)
         is_hot[hot] = True
