@@ -108,6 +108,9 @@ typedef struct {
                                                           per-row / one-lane-per-row warps
                                                           (launch schedule)    */
     int32_t narrow_rb_per_warp;                        /* row-blocks per narrow / mid warp   */
+    int32_t main_blocks_per_sm;                        /* 4, or 5 for FP16 plans without a wide-
+                                                          medium majority      */
+    int32_t short_tiles_per_warp;                      /* short tiles per short warp         */
 } dasp_plan_info_t;
 
 /*

@@ -29,6 +29,8 @@ struct dasp_plan_s {
     int wide_il = 0;                      // interleaved wide medium warps (setup_launch)
     int narrow_il = 0;                    // interleaved narrow / mid medium warps (measured neutral / slower: off)
     int nrw = 0;                          // row-blocks per narrow / mid warp (0: no narrow path)
+    bool occ5 = false;                    // FP16: CUDA-core main kernel at 5 blocks / SM (setup_launch)
+    int tpw = 0;                          // short tiles per short warp of the layout
     int64_t rb_mid = 0, rb_narrow = 0;    // row-blocks on mid / narrow warps (all panels)
     bool keep_host = false;
     HostFormat host;                      // counts always valid; arrays freed after upload unless keep_host
@@ -250,6 +252,20 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
     std::vector<uint64_t> blk_word;
     int64_t blk = 0;
+    // FP16 with the CUDA-core default: the main kernel runs its 5-block / 48-register instantiation
+    // unless wide medium row-blocks (the register-hungry path, which spills there) are the majority
+    // of the plan's row-blocks: C2 FP16 -13 %, C2+ -15 %, C6 -5 %, C3 +-0; C5 (wide rows) +4 % and
+    // keeps 4 blocks (profiles/r02/f16_occupancy5.jsonl)
+    int64_t wide_rbs = 0;
+    for (int64_t q = 0; q < f.n_panels; ++q) {
+        const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
+        int64_t rbm = e[5];
+        if (nrw > 0)
+            while (rbm > 0 && nslots[e[4] + rbm - 1] <= dasp::mid_max_slots(f.geo.K)) --rbm;
+        wide_rbs += rbm;
+    }
+    p->occ5 = p->dtype == DASP_R_16F && p->variant == DASP_VARIANT_CUDACORE && 4 * wide_rbs <= f.nrb;
+    p->tpw = dasp::short_tiles_per_warp(p->dtype, p->occ5);
     for (int64_t q = 0; q < f.n_panels; ++q) {
         const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
         dasp::PanelDesc& d = desc[q];
@@ -267,7 +283,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         p->rb_mid += d.rbn - d.rbm;
         p->rb_narrow += d.nrb - d.rbn;
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
-        const int64_t tpw = dasp::short_tiles_per_warp(p->dtype);
+        const int64_t tpw = p->tpw;
         const int64_t warps = d.nmw + (d.t13 + d.t4 + d.t22 + d.ts + tpw - 1) / tpw;   // long units: own kernel
         const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
         for (int64_t i = 0; i < nb; ++i) blk_word.push_back((static_cast<uint64_t>(q) << 32) | static_cast<uint64_t>(i));
@@ -552,6 +568,7 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.nrw = p->nrw;
     mp.extra = extra;
     mp.class_mask = DASP_CLASS_MASK;
+    mp.tpw = p->tpw;
     const int64_t n0 = (beta == 1.0 && extra.n == 0) ? 0 : f.n0;   // scatter mode must still copy them
     mp.group_ptr = static_cast<const int64_t*>(p->d[DASP_ARR_GROUP_PTR]);
     mp.long_out = static_cast<const int32_t*>(p->d[DASP_ARR_LONG_OUT]);
@@ -566,7 +583,9 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.n0 = n0;
     mp.fin_warps = dasp::finish_warps(mp.row_long, n0);
     const int64_t fin_blocks = (mp.fin_warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
-    e = timed(p, DASP_K_MAIN, s, on, [&] { return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s); });
+    e = timed(p, DASP_K_MAIN, s, on, [&] {
+        return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s, p->occ5);
+    });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
     return DASP_OK;
 }
@@ -691,6 +710,8 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->rowblocks_mid = p->rb_mid;
     o->rowblocks_narrow = p->rb_narrow;
     o->narrow_rb_per_warp = p->nrw;
+    o->main_blocks_per_sm = p->occ5 ? 5 : 4;
+    o->short_tiles_per_warp = p->tpw;
     o->max_len = f.max_len;
     o->threshold = f.tau;
     o->build_ms = p->build_ms;

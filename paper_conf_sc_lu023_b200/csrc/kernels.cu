@@ -54,6 +54,9 @@
 #ifndef DASP_SHORT_TPW_F32
 #define DASP_SHORT_TPW_F32 3
 #endif
+#ifndef DASP_SHORT_TPW_OCC5
+#define DASP_SHORT_TPW_OCC5 2   // the FP16 5-block instantiation (VAR_OCC5): 2 tiles fit its 48 registers
+#endif
 #define DASP_BY_DT(DT, K) ((DT) == 0 ? K##_F64 : ((DT) == 1 ? K##_F16 : K##_F32))
 
 namespace dasp {
@@ -61,10 +64,12 @@ namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
 // variant template argument: bits 0-1 the block-dot path, bit 2 the scatter epilogue
-// (dasp_spmv_scatter), instantiated separately so the plain kernels carry no extra stores
-enum { VAR_MMA = 1, VAR_CUDACORE = 2, VAR_SCATTER = 4 };
+// (dasp_spmv_scatter), bit 3 the FP16 CUDA-core instantiation at 5 blocks / 48 registers per
+// thread (VAR_OCC5, plans without a wide-medium majority: main_occ5), each instantiated separately
+enum { VAR_MMA = 1, VAR_CUDACORE = 2, VAR_SCATTER = 4, VAR_OCC5 = 8 };
 __host__ __device__ constexpr int vk(int v) { return v & 3; }
 __host__ __device__ constexpr bool vs(int v) { return (v & VAR_SCATTER) != 0; }
+__host__ __device__ constexpr bool vo(int v) { return (v & VAR_OCC5) != 0; }
 
 // ------------------------------------------------------------------------------------------
 // memory helpers
@@ -918,36 +923,40 @@ __device__ __forceinline__ void finish_warp(const MainParams& P, int64_t fw, int
 template <int DT, int VAR>
 __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc* D, int64_t ws, int lane, uint64_t pol) {
     const int64_t nt = __ldg(&D->t13) + __ldg(&D->t4) + __ldg(&D->t22) + __ldg(&D->ts);
-    constexpr int TPW = DASP_BY_DT(DT, DASP_SHORT_TPW);
-    const int64_t t0 = ws * TPW;
+    // compile-time tiles per warp (register arrays); the plan's layout may use fewer (P.tpw: an
+    // FP16 plan laid out for the 5-block instantiation, run with another variant)
+    constexpr int TPW = vo(VAR) ? DASP_SHORT_TPW_OCC5 : DASP_BY_DT(DT, DASP_SHORT_TPW);
+    const int tpw = P.tpw;
+    const int64_t t0 = ws * tpw;
     if (t0 >= nt || !(P.class_mask & 4)) return;
     if constexpr (TPW > 2) {   // generic: every tile's loads, then every tile's gathers, then the math
         ShortRef R[TPW];
+        const int64_t te = min(t0 + tpw, nt);           // this warp's tiles [t0, te)
 #pragma unroll
         for (int k = 0; k < TPW; ++k) R[k] = short_ref(D, min(t0 + k, nt - 1));
         if constexpr (DT == 1) {
             ShortLdH L[TPW];
             uint16_t xh[TPW][4];
 #pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_load_f16(P, R[k], lane, pol, L[k]);
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_load_f16(P, R[k], lane, pol, L[k]);
 #pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_gather_f16(P, L[k], xh[k]);
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_gather_f16(P, L[k], xh[k]);
 #pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_math_f16<VAR>(P, R[k].cat, L[k], xh[k], lane);
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_math_f16<VAR>(P, R[k].cat, L[k], xh[k], lane);
         } else {
             ShortLd<DT> L[TPW];
             double xv[TPW][4];
 #pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_load_f64<DT>(P, R[k], lane, pol, L[k]);
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_load_f64<DT>(P, R[k], lane, pol, L[k]);
 #pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_gather_f64<DT>(P, L[k], xv[k]);
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_gather_f64<DT>(P, L[k], xv[k]);
 #pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < nt) short_math_f64<DT, VAR>(P, R[k].cat, L[k], xv[k], lane);
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_math_f64<DT, VAR>(P, R[k].cat, L[k], xv[k], lane);
         }
         return;
     }
     const ShortRef A = short_ref(D, t0);
-    if (TPW == 1 || t0 + 1 >= nt) { short_tile<DT, VAR>(P, A, lane, pol); return; }
+    if (TPW == 1 || tpw < 2 || t0 + 1 >= nt) { short_tile<DT, VAR>(P, A, lane, pol); return; }
     const ShortRef B = short_ref(D, t0 + 1);
     if constexpr (DT == 1) {
         ShortLdH LA, LB;
@@ -1212,6 +1221,7 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
 #ifndef DASP_MIN_BLOCKS_F16
 #define DASP_MIN_BLOCKS_F16 4
 #endif
+
 #ifndef DASP_MIN_BLOCKS_F32
 #define DASP_MIN_BLOCKS_F32 4
 #endif
@@ -1243,7 +1253,8 @@ dasp_long_kernel(const MainParams P, int64_t n_units) {
 
 // medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
 template <int DT, int VAR>
-__global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32))
+__global__ void __launch_bounds__(MAIN_THREADS, vo(VAR) ? 5
+                                                         : (DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32)))
 dasp_main_kernel(const MainParams P) {
     const int lane = threadIdx.x & 31;
     const int64_t fin_blocks = (P.fin_warps + WARPS_PER_BLOCK - 1) / WARPS_PER_BLOCK;
@@ -1304,11 +1315,18 @@ extern "C" int dasp_exp_trace_read(void* dst, int64_t bytes, int clear) {
     return 0;
 }
 #endif
-int short_tiles_per_warp(int dtype) { return DASP_BY_DT(dtype, DASP_SHORT_TPW); }
+int short_tiles_per_warp(int dtype, bool occ5) { return occ5 ? DASP_SHORT_TPW_OCC5 : DASP_BY_DT(dtype, DASP_SHORT_TPW); }
 int narrow_rb_per_warp(int) { return DASP_NARROW_RB; }
 
 template <int DT>
-static cudaError_t launch_main_dt(const MainParams& p, int variant, bool scatter, unsigned nb, cudaStream_t s) {
+static cudaError_t launch_main_dt(const MainParams& p, int variant, bool scatter, bool occ5, unsigned nb, cudaStream_t s) {
+    if constexpr (DT == 1) {
+        if (occ5 && variant != VAR_MMA) {
+            if (scatter) dasp_main_kernel<1, VAR_CUDACORE | VAR_SCATTER | VAR_OCC5><<<nb, MAIN_THREADS, 0, s>>>(p);
+            else dasp_main_kernel<1, VAR_CUDACORE | VAR_OCC5><<<nb, MAIN_THREADS, 0, s>>>(p);
+            return cudaGetLastError();
+        }
+    }
     if (variant == VAR_MMA) {
         if (scatter) dasp_main_kernel<DT, VAR_MMA | VAR_SCATTER><<<nb, MAIN_THREADS, 0, s>>>(p);
         else dasp_main_kernel<DT, VAR_MMA><<<nb, MAIN_THREADS, 0, s>>>(p);
@@ -1319,14 +1337,14 @@ static cudaError_t launch_main_dt(const MainParams& p, int variant, bool scatter
     return cudaGetLastError();
 }
 
-cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s) {
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s, bool occ5) {
     if (blocks <= 0) return cudaSuccess;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     const unsigned nb = static_cast<unsigned>(blocks);
     const bool scatter = p.extra.n > 0;
-    if (dtype == 0) return launch_main_dt<0>(p, variant, scatter, nb, s);
-    if (dtype == 1) return launch_main_dt<1>(p, variant, scatter, nb, s);
-    return launch_main_dt<2>(p, variant, scatter, nb, s);
+    if (dtype == 0) return launch_main_dt<0>(p, variant, scatter, false, nb, s);
+    if (dtype == 1) return launch_main_dt<1>(p, variant, scatter, occ5, nb, s);
+    return launch_main_dt<2>(p, variant, scatter, false, nb, s);
 }
 
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s) {

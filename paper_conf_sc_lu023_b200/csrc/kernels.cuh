@@ -64,6 +64,7 @@ struct MainParams {
     int32_t narrow_il;        // 1: a block's narrow / mid warps interleave their passes (medium_narrow)
     int32_t nrw;              // row-blocks per narrow / mid warp (4 or 8: a multiple of 4)
     int32_t class_mask;       // bit 1 medium, bit 2 short (7 = all; build knob DASP_CLASS_MASK for class timings)
+    int32_t tpw;              // short tiles per short warp in the plan's layout (short_tiles_per_warp)
     ExtraDst extra;           // scatter destinations (extra.n > 0 selects the scatter instantiation)
     // long-row phase 2 + empty rows fused into the main kernel (its first fin_warps warps; the
     // long kernel has completed, so every group partial is final)
@@ -76,10 +77,12 @@ struct MainParams {
 inline int64_t finish_warps(int64_t row_long, int64_t n0) { return (row_long + 3) / 4 + (n0 + 127) / 128; }
 
 // variant: 1 = MMA (DMMA/HMMA diagonal trick), 2 = CUDA-core.  dtype: 0 = FP64, 1 = FP16, 2 = FP32.
-cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s);
+// occ5: FP16 CUDA-core plans without a wide-medium majority run the 5-block / 48-register
+// instantiation (its short warps take DASP_SHORT_TPW_OCC5 tiles: short_tiles_per_warp(dtype, true))
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s, bool occ5 = false);
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
-// short tiles one main-kernel warp processes (build knob DASP_SHORT_TPW)
-int short_tiles_per_warp(int dtype);
+// short tiles one main-kernel warp processes (build knobs DASP_SHORT_TPW_*)
+int short_tiles_per_warp(int dtype, bool occ5 = false);
 // narrow medium row-blocks (rows of at most narrow_max_slots(K) = 2K slots: max(K*nreg, longest
 // row)): the most row-blocks one narrow warp processes
 int narrow_rb_per_warp(int dtype);

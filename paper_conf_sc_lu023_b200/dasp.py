@@ -59,7 +59,8 @@ class PlanInfo(ctypes.Structure):
                 ("panel_rows", ctypes.c_int64), ("n_panels", ctypes.c_int64),
                 ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
                 ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double),
-                ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32)]
+                ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32),
+                ("main_blocks_per_sm", ctypes.c_int32), ("short_tiles_per_warp", ctypes.c_int32)]
 
     def as_dict(self):
         return {name: getattr(self, name) for name, _ in self._fields_}

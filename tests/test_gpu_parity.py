@@ -456,3 +456,22 @@ def test_unsorted_duplicate_rectangular_bit_exact(name, A, dt, variant):
         hplan = make(A, dt)
         for arr in dasp.ARRAYS:
             assert np.array_equal(dasp.dasp_plan_copy_array(dplan, arr), dasp.dasp_plan_copy_array(hplan, arr)), arr
+
+
+# FP16 plans without a wide-medium majority run the 5-block main-kernel instantiation with 2 short
+# tiles per warp; every variant must honour the plan's layout (the MMA kernel is compiled for 4)
+@pytest.mark.parametrize("name,expect5", [("c2s", True), ("c6s", True), ("c5s", False), ("c1a", True)])
+def test_fp16_occupancy5_layout(name, expect5):
+    gen = dict(CASES)[name]
+    A = gen(synth.VAL_INT)
+    x = synth.vector(97, A.n, synth.VAL_INT)
+    plan = make(A, "f16")
+    assert plan.info["main_blocks_per_sm"] == (5 if expect5 else 4)
+    assert plan.info["short_tiles_per_warp"] == (2 if expect5 else 4)
+    y_ref, _ = oracle_ref(A, x, "f16")
+    for v in VARIANTS:
+        assert np.array_equal(run(plan, x, "f16", variant=v), y_ref), (name, VNAME[v])
+    mplan = make(A, "f16", variant=dasp.DASP_VARIANT_MMA)           # MMA default: never the 5-block layout
+    assert mplan.info["main_blocks_per_sm"] == 4
+    for v in VARIANTS:
+        assert np.array_equal(run(mplan, x, "f16", variant=v), y_ref), (name, VNAME[v])
