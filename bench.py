@@ -801,7 +801,10 @@ def run_reference(args, rank, world):
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "GFLOPS", "n_gpus": world,
             "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": dt * 1e3, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
-            "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config), "nnz": nnz},
+            "config": {"workload": workload, "matrix": CONFIG_DOC.get(args.config, args.config),
+                       "m": int(spec.m), "n": int(spec.n), "nnz": nnz, "variant": "oracle (double-double CSR loop)",
+                       "panel_rows": None, "parallelism": f"host CPU, rows over {used} OpenMP threads",
+                       "l2": "n/a (CPU); a strided row sample of the workload per step"},
             "cpu_baseline": {"value": v, "unit": "GFLOPS", "cores": used, "kind": "oracle",
                              "sample": f"every {stride}th row ({rows_n} rows, {int(rp[-1])} nnz) per step, "
                                        f"double-double CSR loop over {used} OpenMP threads"},

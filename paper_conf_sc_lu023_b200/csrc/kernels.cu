@@ -1229,9 +1229,6 @@ __device__ __forceinline__ void medium_warp(const MainParams& P, const PanelDesc
 // and is gather-latency bound, so it runs at higher occupancy (40 registers, 48 warps
 // per SM) than the medium path, which needs 64 (profiles/r01/long_kernel_occupancy.jsonl).  Units run in
 // the column-bucketed schedule `unit_order`.
-#ifndef DASP_LONG_UPW2
-#define DASP_LONG_UPW2 0   // experiment: two long units per warp (schedule entries fetched together)
-#endif
 #ifndef DASP_LONG_MIN_BLOCKS
 #define DASP_LONG_MIN_BLOCKS 8   // 32 registers, 64 warps/SM (C3 long -2 %, C5 -3 % vs 40 registers; profiles/r01d/long_occupancy*.jsonl)
 #endif
@@ -1245,25 +1242,13 @@ template <int DT, int VAR>
 __global__ void __launch_bounds__(MAIN_THREADS, DT == 0 ? DASP_LONG_MIN_BLOCKS
                                                          : (DT == 1 ? DASP_LONG_MIN_BLOCKS_F16 : DASP_LONG_MIN_BLOCKS_F32))
 dasp_long_kernel(const MainParams P, int64_t n_units) {
-    const int64_t w = ((static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5) * (DASP_LONG_UPW2 ? 2 : 1);
+    const int64_t w = (static_cast<int64_t>(blockIdx.x) * MAIN_THREADS + threadIdx.x) >> 5;
     if (w >= n_units) return;
     const int lane = threadIdx.x & 31;
     const uint64_t pol = stream_policy();
-#if DASP_LONG_UPW2
-    // experiment: two units per warp, both schedule entries loaded in one round trip
-    const int64_t u0 = __ldg(P.unit_order + w);
-    const int64_t u1 = w + 1 < n_units ? __ldg(P.unit_order + w + 1) : -1;
-    if constexpr (DT == 1) long_unit_f16<VAR>(P, u0, lane, pol);
-    else long_unit_f64<DT, VAR>(P, u0, lane, pol);
-    if (u1 >= 0) {
-        if constexpr (DT == 1) long_unit_f16<VAR>(P, u1, lane, pol);
-        else long_unit_f64<DT, VAR>(P, u1, lane, pol);
-    }
-#else
     const int64_t u = __ldg(P.unit_order + w);
     if constexpr (DT == 1) long_unit_f16<VAR>(P, u, lane, pol);
     else long_unit_f64<DT, VAR>(P, u, lane, pol);
-#endif
 }
 
 // medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
@@ -1364,8 +1349,7 @@ cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blo
 
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s) {
     if (n_units <= 0) return cudaSuccess;
-    const int64_t warps = DASP_LONG_UPW2 ? (n_units + 1) / 2 : n_units;
-    const int64_t blocks = (warps * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
+    const int64_t blocks = (n_units * 32 + MAIN_THREADS - 1) / MAIN_THREADS;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     dim3 grid(static_cast<unsigned>(blocks)), block(MAIN_THREADS);
     const bool mma = variant == VAR_MMA;
