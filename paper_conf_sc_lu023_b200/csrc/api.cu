@@ -365,9 +365,34 @@ dasp_status_t check_create_args(dasp_plan_t* plan_out, int64_t m, int64_t n, int
     return DASP_OK;
 }
 
-int64_t resolve_panel_rows(const dasp_options_t& o) {
-    // panel size (R28): -1 one panel (the paper's global format); 0 automatic
-    return o.panel_rows == 0 ? kAutoPanelRows : (o.panel_rows < 0 ? 0 : o.panel_rows);
+// Automatic panel size (R28).  Default 2^20 rows.  Ragged medium lengths (coefficient of variation >=
+// 0.5) take 8192-row panels -- a row-block's 8 length-sorted rows, and a block's row-blocks, then come
+// from within 8192 original rows, so their local x windows overlap in L1 and the gathers issue fewer
+// L2 requests -- except heavy-tailed lengths (cv >= 1) in FP64 / FP32, whose main kernel is latency-
+// bound and pays the small panels' fragmentation instead (profiles/r02/panel_size_small*.jsonl:
+// 8192 rows C5 FP64 -4.8 %, FP32 -8.6 %, FP16 -5.9 %, C3 FP16 -5.3 %; C3 FP64 +2 %, stencils +0.5..+2.5 %).
+constexpr int64_t kSmallPanelRows = 8192;
+int64_t auto_panel_rows(int dtype, int64_t cnt, int64_t sum, int64_t sumsq) {
+    if (cnt < 2) return kAutoPanelRows;
+    const double mean = static_cast<double>(sum) / static_cast<double>(cnt);
+    const double var = static_cast<double>(sumsq) / static_cast<double>(cnt) - mean * mean;
+    const double cv = var > 0 ? std::sqrt(var) / mean : 0.0;
+    if (cv >= 0.5 && (dtype == DASP_R_16F || cv < 1.0)) return kSmallPanelRows;
+    return kAutoPanelRows;
+}
+int64_t resolve_panel_rows(const dasp_options_t& o, int dtype, int64_t cnt, int64_t sum, int64_t sumsq) {
+    // -1 one panel (the paper's global format); 0 automatic; > 0 as given
+    return o.panel_rows == 0 ? auto_panel_rows(dtype, cnt, sum, sumsq) : (o.panel_rows < 0 ? 0 : o.panel_rows);
+}
+// medium-class length statistics of a host row_ptr (automatic panel size)
+void host_medium_stats(const int64_t* rp, int64_t m, int64_t max_len, int64_t* cnt, int64_t* sum, int64_t* sumsq) {
+    int64_t c = 0, s1 = 0, s2 = 0;
+#pragma omp parallel for schedule(static) reduction(+ : c, s1, s2)
+    for (int64_t i = 0; i < m; ++i) {
+        const int64_t L = rp[i + 1] - rp[i];
+        if (L >= dasp::MIN_MEDIUM_LEN && L <= max_len) { ++c; s1 += L; s2 += L * L; }
+    }
+    *cnt = c; *sum = s1; *sumsq = s2;
 }
 
 dasp_status_t fail(dasp_plan_s* p, dasp_status_t st) {
@@ -399,8 +424,10 @@ dasp_status_t dasp_plan_create(dasp_plan_t* plan_out, int64_t m, int64_t n, int6
     p->keep_host = o.keep_host != 0 || o.device < 0;
 
     auto t0 = std::chrono::steady_clock::now();
+    int64_t mc = 0, ms = 0, mq = 0;
+    if (o.panel_rows == 0) host_medium_stats(row_ptr, m, o.max_len > 0 ? o.max_len : dasp::MAX_LEN, &mc, &ms, &mq);
     int bst = dasp::build_format(p->host, dtype, m, n, row_ptr, col_idx, val, o.num_threads, o.validate != 0,
-                                 resolve_panel_rows(o), o.max_len, o.threshold);
+                                 resolve_panel_rows(o, dtype, mc, ms, mq), o.max_len, o.threshold);
     auto t1 = std::chrono::steady_clock::now();
     p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
     if (bst != DASP_OK) {
@@ -464,8 +491,14 @@ dasp_status_t dasp_plan_create_device(dasp_plan_t* plan_out, int64_t m, int64_t 
     DeviceGuard guard(p->device);
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     auto t0 = std::chrono::steady_clock::now();
+    int64_t mc = 0, ms = 0, mq = 0;
+    if (o.panel_rows == 0 &&
+        dasp::medium_length_stats(d_row_ptr, m, o.max_len > 0 ? o.max_len : dasp::MAX_LEN, &mc, &ms, &mq, s) != cudaSuccess) {
+        delete p;
+        return DASP_ERR_CUDA;
+    }
     int bst = dasp::build_format_device(p->host, p->d, dtype, m, n, nnz, d_row_ptr, d_col_idx, d_val, o.validate != 0,
-                                        resolve_panel_rows(o), o.max_len, o.threshold, s);
+                                        resolve_panel_rows(o, dtype, mc, ms, mq), o.max_len, o.threshold, s);
     auto t1 = std::chrono::steady_clock::now();
     p->build_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
     if (bst != DASP_OK) {

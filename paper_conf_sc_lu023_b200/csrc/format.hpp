@@ -28,6 +28,7 @@ inline Geometry geometry(int dtype) {
 }
 
 constexpr int MAX_LEN = 256;     // P:L152 (default; plan option max_len)
+constexpr int MIN_MEDIUM_LEN = 5; // short iff len <= 4
 constexpr int MMA_M = 8;
 constexpr int32_t PAD_COL = -1;  // R12: sentinel column of pads (x read as 0)
 constexpr int SHORT_TILE = 128;  // elements per short tile (32 four-slot rows)

@@ -547,6 +547,40 @@ __global__ void k_first_col(const int32_t* lc, int64_t ue, int64_t nu, int32_t* 
 
 }  // namespace
 
+namespace {
+// medium-class length statistics (count, sum, sum of squares) of rows with lo <= len <= hi
+__global__ void k_medium_stats(const int64_t* __restrict__ rp, int64_t m, int64_t lo, int64_t hi,
+                               unsigned long long* __restrict__ out) {
+    unsigned long long c = 0, s1 = 0, s2 = 0;
+    for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < m;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t L = rp[i + 1] - rp[i];
+        if (L >= lo && L <= hi) { ++c; s1 += L; s2 += static_cast<unsigned long long>(L * L); }
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+        c += __shfl_xor_sync(0xffffffffu, c, o);
+        s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+    }
+    if ((threadIdx.x & 31) == 0) { atomicAdd(out, c); atomicAdd(out + 1, s1); atomicAdd(out + 2, s2); }
+}
+}  // namespace
+
+cudaError_t medium_length_stats(const int64_t* d_row_ptr, int64_t m, int64_t max_len, int64_t* count, int64_t* sum,
+                                int64_t* sumsq, cudaStream_t s) {
+    *count = *sum = *sumsq = 0;
+    if (m <= 0) return cudaSuccess;
+    Buf acc;
+    cudaError_t e = acc.alloc(3 * 8);
+    if (e != cudaSuccess || (e = cudaMemsetAsync(acc.p, 0, 24, s)) != cudaSuccess) return e;
+    k_medium_stats<<<148 * 4, 256, 0, s>>>(d_row_ptr, m, MIN_MEDIUM_LEN, max_len, acc.as<unsigned long long>());
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    int64_t h[3];
+    if ((e = d2h(h, acc.p, 24, s)) != cudaSuccess) return e;
+    *count = h[0]; *sum = h[1]; *sumsq = h[2];
+    return cudaSuccess;
+}
+
 cudaError_t gather_unit_first_col(const int32_t* d_long_col, int64_t unit_elems, int64_t n_units, int32_t* host_out,
                                   cudaStream_t s) {
     Buf tmp;

@@ -17,6 +17,11 @@ int build_format_device(HostFormat& f, void** d_arrays, int dtype, int64_t m, in
                         const int64_t* d_row_ptr, const int32_t* d_col, const void* d_val, bool validate,
                         int64_t panel_rows, int64_t max_len, double tau, cudaStream_t s);
 
+// count / sum / sum of squares of the row lengths in [MIN_MEDIUM_LEN, max_len] (the medium class) of a
+// device row_ptr (the automatic panel size, api.cu)
+cudaError_t medium_length_stats(const int64_t* d_row_ptr, int64_t m, int64_t max_len, int64_t* count, int64_t* sum,
+                                int64_t* sumsq, cudaStream_t s);
+
 // host_out[u] = long_col[u * unit_elems] for u < n_units (device gather + one copy)
 cudaError_t gather_unit_first_col(const int32_t* d_long_col, int64_t unit_elems, int64_t n_units, int32_t* host_out,
                                   cudaStream_t s);
