@@ -49,7 +49,8 @@ struct dasp_plan_s {
     int64_t blocks = 0;                   // grid of the medium/short kernel
     int64_t n_units = 0;                  // long units (long kernel)
     void* d_panels = nullptr;             // dasp::PanelDesc[n_panels]
-    void* d_blk_word = nullptr;           // uint64 panel of every main-kernel block (kernels.cuh)
+    void* d_warp_word = nullptr;          // uint64 panel / warp of every main-kernel warp (kernels.cuh)
+    int64_t n_mwarps = 0;
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
     // timing
     int32_t timing_cap = 0, timing_calls = 0;
@@ -83,6 +84,9 @@ constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read 
 #endif
 #ifndef DASP_NARROW_IL
 #define DASP_NARROW_IL 0
+#endif
+#ifndef DASP_PACK_WARPS
+#define DASP_PACK_WARPS 1   // 1: panels' warps packed back to back in the main grid; 0: each panel padded to whole blocks
 #endif
 #ifndef DASP_HEAVY_FIRST
 #define DASP_HEAVY_FIRST 16  // leading blocks of every panel dispatched at the start of the main grid (C3 FP16 -2.7 %, FP64 -0.1..-0.8 %, others +-0.8 %: profiles/r02/heavy_first_ab.jsonl, chunk_units_removed_and_heavy_first.jsonl)
@@ -124,9 +128,9 @@ void free_device(dasp_plan_s* p) {
     }
     if (p->d_partial) cudaFree(p->d_partial);
     if (p->d_panels) cudaFree(p->d_panels);
-    if (p->d_blk_word) cudaFree(p->d_blk_word);
+    if (p->d_warp_word) cudaFree(p->d_warp_word);
     if (p->d_unit_order) cudaFree(p->d_unit_order);
-    p->d_panels = p->d_blk_word = p->d_unit_order = nullptr;
+    p->d_panels = p->d_warp_word = p->d_unit_order = nullptr;
 
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
@@ -250,7 +254,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     p->nrw = static_cast<int>(nrw);
     p->rb_mid = p->rb_narrow = 0;
     std::vector<dasp::PanelDesc> desc(static_cast<size_t>(f.n_panels));
-    std::vector<uint64_t> blk_word;
+    std::vector<int64_t> panel_warps(static_cast<size_t>(f.n_panels));
     int64_t blk = 0;
     // FP16 with the CUDA-core default: the main kernel runs its 5-block / 48-register instantiation
     // unless wide medium row-blocks (the register-hungry path, which spills there) are the majority
@@ -285,24 +289,27 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         d.tile0 = e[6]; d.t13 = e[7]; d.t4 = e[8]; d.t22 = e[9]; d.ts = e[10]; d.out0 = e[11];
         const int64_t tpw = p->tpw;
         const int64_t warps = d.nmw + (d.t13 + d.t4 + d.t22 + d.ts + tpw - 1) / tpw;   // long units: own kernel
-        const int64_t nb = (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
-        for (int64_t i = 0; i < nb; ++i) blk_word.push_back((static_cast<uint64_t>(q) << 32) | static_cast<uint64_t>(i));
-        blk += nb;
+        panel_warps[q] = warps;
+        blk += (warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
     }
-    p->blocks = blk;
-    // heavy blocks first: a panel's first blocks hold its longest medium row-blocks (rows are
-    // length-sorted), whose warps walk many chunks one round trip after the other and finish long
-    // after the panel's other blocks.  Dispatching those blocks of every panel at the start of the
-    // grid overlaps them with everything else instead of leaving them as the tail of the launch.
-    if (DASP_HEAVY_FIRST > 0 && f.n_panels > 1) {
-        std::vector<uint64_t> order;
-        order.reserve(blk_word.size());
-        for (uint64_t w : blk_word)
-            if ((w & 0xffffffffu) < static_cast<uint64_t>(DASP_HEAVY_FIRST)) order.push_back(w);
-        for (uint64_t w : blk_word)
-            if ((w & 0xffffffffu) >= static_cast<uint64_t>(DASP_HEAVY_FIRST)) order.push_back(w);
-        blk_word.swap(order);
+    // warp table of the main kernel.  Heavy warps first: a panel's first warps hold its longest
+    // medium row-blocks (rows are length-sorted), which walk many chunks one round trip after the
+    // other and finish long after the panel's other warps; dispatching them for every panel at the
+    // start of the grid overlaps them with everything else instead of leaving them as the tail of
+    // the launch.  Panels are packed back to back (DASP_PACK_WARPS) or each padded to whole blocks.
+    std::vector<uint64_t> warp_word;
+    {
+        const int64_t heavy = (f.n_panels > 1 ? DASP_HEAVY_FIRST : 0) * dasp::WARPS_PER_BLOCK;
+        auto emit = [&](int64_t q, int64_t w0, int64_t w1) {
+            for (int64_t w = w0; w < w1; ++w) warp_word.push_back((static_cast<uint64_t>(q) << 32) | static_cast<uint64_t>(w));
+            if (!DASP_PACK_WARPS)
+                while (warp_word.size() % dasp::WARPS_PER_BLOCK) warp_word.push_back(~0ull);
+        };
+        for (int64_t q = 0; q < f.n_panels; ++q) emit(q, 0, std::min(heavy, panel_warps[q]));
+        for (int64_t q = 0; q < f.n_panels; ++q) emit(q, std::min(heavy, panel_warps[q]), panel_warps[q]);
     }
+    p->n_mwarps = static_cast<int64_t>(warp_word.size());
+    p->blocks = (p->n_mwarps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
     p->n_units = f.n_groups_padded / f.geo.UG;
 
     // long-unit execution order (a launch schedule, not part of the format): inside each panel
@@ -345,7 +352,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     p->device_bytes += pb;
     dasp_status_t st;
     if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
-    if ((st = upload(&p->d_blk_word, blk_word.data(), blk_word.size() * 8)) != DASP_OK) return st;
+    if ((st = upload(&p->d_warp_word, warp_word.data(), warp_word.size() * 8)) != DASP_OK) return st;
     if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
 
     return DASP_OK;
@@ -593,7 +600,8 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.alpha = alpha;
     mp.beta = beta;
     mp.panels = static_cast<const dasp::PanelDesc*>(p->d_panels);
-    mp.blk_word = static_cast<const uint64_t*>(p->d_blk_word);
+    mp.warp_word = static_cast<const uint64_t*>(p->d_warp_word);
+    mp.n_mwarps = p->n_mwarps;
     mp.unit_order = static_cast<const int32_t*>(p->d_unit_order);
     mp.rbw = p->rbw;
     mp.wide_il = p->wide_il;

@@ -1263,11 +1263,14 @@ dasp_main_kernel(const MainParams P) {
         if (fw < P.fin_warps) finish_warp<DT, VAR>(P, fw, lane);
         return;
     }
-    // role of this warp inside its panel; the descriptor fields are loaded only on the branch
-    // that needs them so they do not stay live (register pressure = occupancy)
-    const uint64_t bw = __ldg(P.blk_word + (static_cast<int64_t>(blockIdx.x) - fin_blocks));
-    const PanelDesc* D = P.panels + static_cast<int32_t>((bw >> 32) & 0x7fffffffu);
-    int64_t w = static_cast<int64_t>(bw & 0xffffffffu) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+    // role of this warp inside its panel (MainParams::warp_word); the descriptor fields are loaded
+    // only on the branch that needs them so they do not stay live (register pressure = occupancy)
+    const int64_t gw = (static_cast<int64_t>(blockIdx.x) - fin_blocks) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+    if (gw >= P.n_mwarps) return;
+    const uint64_t ww = __ldg(P.warp_word + gw);
+    if (ww == ~0ull) return;                             // padding slot (per-panel block alignment)
+    const PanelDesc* D = P.panels + static_cast<int32_t>(ww >> 32);
+    const int64_t w = static_cast<int64_t>(ww & 0xffffffffu);
     const uint64_t pol = stream_policy();
     const int64_t nmw = __ldg(&D->nmw);
     if (w < nmw) {                                       // medium rows

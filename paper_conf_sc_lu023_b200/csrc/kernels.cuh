@@ -52,9 +52,10 @@ struct MainParams {
     const int32_t* short_col;
     const int32_t* short_out;
     const PanelDesc* panels;
-    // panel of every main-kernel block after the fin blocks: bits 32..62 = panel, bits 0..31 =
-    // block index among the panel's blocks
-    const uint64_t* blk_word;
+    // every main-kernel warp after the fin warps: panel << 32 | warp index within the panel
+    // (~0 = an idle padding slot); n_mwarps entries
+    const uint64_t* warp_word;
+    int64_t n_mwarps;
     const int32_t* unit_order;// long units in execution order (column-bucketed per panel)
     const void* x;
     void* y;
