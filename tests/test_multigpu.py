@@ -193,3 +193,19 @@ def test_halo_iteration_matches_oracle(tmp_path, cfg, world):
     for _ in range(iters):
         x, _ = oracle.spmv_csr(A, x, alpha=1.0 / inf_norm)
     assert np.allclose(got, x, rtol=0, atol=1e-13 * max(1.0, np.abs(x).max()))
+
+
+def test_slab_iteration_dtypes():
+    """The iteration feeds y back as x: x and y buffers take the plan's one element type (f64 / f32);
+    FP16 plans (binary16 x, f32 y) are rejected instead of reading float64 storage as halves."""
+    spec = synth.config("c1b")
+    lens = synth.row_lengths(spec)
+    slab = build_slab(lambda r0, nr: synth.generate(spec, r0, nr), lens, 0, 1)
+    for dt, tdt in (("f64", torch.float64), ("f32", torch.float32)):
+        it = SlabSpMV(slab, 1, 0, "cpu", dtype=dt, local_spmv=lambda x, y, a: y.copy_(x[:len(y)] * a))
+        assert it.x[0].dtype == tdt and it.elem_bytes == tdt.itemsize
+        it.set_x(synth.vector(3, spec.n))
+        it.step(0.5)
+        assert it.x_global().dtype == (np.float64 if dt == "f64" else np.float32)
+    with pytest.raises(ValueError):
+        SlabSpMV(slab, 1, 0, "cpu", dtype="f16", local_spmv=lambda x, y, a: None)
