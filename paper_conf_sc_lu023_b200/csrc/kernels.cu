@@ -926,7 +926,7 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
     // compile-time tiles per warp (register arrays); the plan's layout may use fewer (P.tpw: an
     // FP16 plan laid out for the 5-block instantiation, run with another variant)
     constexpr int TPW = vo(VAR) ? DASP_SHORT_TPW_OCC5 : DASP_BY_DT(DT, DASP_SHORT_TPW);
-    const int tpw = P.tpw;
+    const int tpw = (DT == 1 && !vo(VAR)) ? P.tpw : TPW;   // only FP16 layouts vary (main_occ5)
     const int64_t t0 = ws * tpw;
     if (t0 >= nt || !(P.class_mask & 4)) return;
     if constexpr (TPW > 2) {   // generic: every tile's loads, then every tile's gathers, then the math
