@@ -128,3 +128,27 @@ def test_halo_iteration_world1(pg):
     for _ in range(3):
         x, _ = oracle.spmv_csr(A, x, alpha=alpha)
     assert np.allclose(it.x_global(), x, rtol=0, atol=1e-12)
+
+
+def test_slab_iteration_world1_f32(pg):
+    """The row-slab iteration on an FP32 plan (x and y both float32, R29): three steps against the oracle
+    applied to the GPU's own previous iterate, each within the FP32 tolerance."""
+    from paper_conf_sc_lu023_b200.multigpu import SlabSpMV, build_slab
+    spec = synth.config("c5", scale=4e-4)
+    lens = synth.row_lengths(spec)
+    slab = build_slab(lambda r0, nr: synth.generate(spec, r0, nr), lens, 0, 1)
+    slab.val = slab.val.astype(np.float32)
+    it = SlabSpMV(slab, 1, 0, "cuda:0", dtype="f32")
+    assert it.x[0].dtype == torch.float32
+    x = synth.vector(62, spec.n).astype(np.float32)
+    it.set_x(x)
+    alpha = 1.0 / slab.inf_norm
+    A = synth.generate(spec)
+    val = A.val.astype(np.float32).astype(np.float64)
+    for _ in range(3):
+        it.step(alpha)
+        torch.cuda.synchronize()
+        got = it.x_global().astype(np.float64)
+        ref, s = oracle.spmv(A.row_ptr, A.col, val, x.astype(np.float64), alpha=alpha)
+        assert oracle.tolerance_ok(got, ref, s, "f32").all()
+        x = got.astype(np.float32)
