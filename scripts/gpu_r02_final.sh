@@ -2,7 +2,7 @@
 # round 2 final evidence at HEAD: smoke, GPU suite, default bench line, reference arm, config sweep,
 # C5 at full size (N = 1: SpMV and the row-slab iteration), ncu launch list of the default command and
 # --set full captures (summarised + traffic JSON), sanitizers.  Everything under gpurun_out/r02_final.
-O=gpurun_out/r02_final2
+O=gpurun_out/r02_final3
 mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw,power.limit --format=csv > $O/smi.txt
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?"
