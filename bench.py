@@ -62,6 +62,9 @@ def parse(argv=None):
     ap.add_argument("--impl", default="dasp", choices=["dasp", "reference"])
     ap.add_argument("--rbw", type=int, default=0, help="medium row-blocks per warp (LOOP_NUM); 0 = auto")
     ap.add_argument("--panel-rows", type=int, default=0, help="rows per panel (0 auto, -1 one global panel)")
+    ap.add_argument("--max-len", type=int, default=0, help="MAX_LEN (P:L152): long iff len > max_len; 0 = auto")
+    ap.add_argument("--tau", type=float, default=0.75, help="regular-block threshold tau (P:L158)")
+    ap.add_argument("--x-stage", type=int, default=0, help="x-window staging: 0 auto, 1 off, 2 on")
     ap.add_argument("--iterate", action="store_true", help="N=1: run the row-slab iteration (x <- alpha*A*x)")
     ap.add_argument("--halo", action="store_true", help="slab mode: sparse halo exchange (all_to_all of the referenced "
                     "remote x only) overlapped with the local sub-matrix SpMV (SURVEY.md 8(f) f1)")
@@ -322,7 +325,8 @@ def make_plan(A, dtype, dev_index, variant, args):
     from paper_conf_sc_lu023_b200 import dasp
     val = A.val.astype({"f64": np.float64, "f16": np.float16, "f32": np.float32}[dtype])
     return dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dtype, device=dev_index, variant=variant,
-                                 medium_rb_per_warp=args.rbw, panel_rows=args.panel_rows)
+                                 medium_rb_per_warp=args.rbw, panel_rows=args.panel_rows,
+                                 max_len=args.max_len, threshold=args.tau, x_stage=args.x_stage)
 
 
 def timed_steps(step, plan, steps, warmup, dev, stream, clocks=True):

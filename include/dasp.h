@@ -77,10 +77,17 @@ typedef struct {
     double threshold;           /* tau, "a customized parameter": an 8 x MMA_K block is
                                    regular iff it holds more than 8*MMA_K*tau nonzeros;
                                    0 = 0.75; must be <= 1                                     */
+    int32_t x_stage;            /* shared-memory staging of x windows for the wide medium
+                                   row-blocks ("shared-memory or TMA staging where reuse exists",
+                                   north_star (3)): 0 = automatic (the build's
+                                   DASP_X_STAGE_AUTO rule; default build: off, staging measured
+                                   slower than the L1-served gathers), 1 = off, 2 = on for every
+                                   block whose warps gather from a few dense column windows
+                                   (e.g. stencils).  Host-built CUDA-core plans only.            */
 } dasp_options_t;
 
 /* Fills `opts` with the defaults: device 0, CUDA-core variant, validate, no keep_host, auto
- * LOOP_NUM, automatic panel size, MAX_LEN 256, tau 0.75. */
+ * LOOP_NUM, automatic panel size, MAX_LEN 256, tau 0.75, automatic x staging. */
 void dasp_options_default(dasp_options_t* opts);
 
 /* Plan statistics (Fig. 12's class shares; build cost). */
@@ -111,6 +118,8 @@ typedef struct {
     int32_t main_blocks_per_sm;                        /* 4, or 5 for FP16 plans without a wide-
                                                           medium majority      */
     int32_t short_tiles_per_warp;                      /* short tiles per short warp         */
+    int64_t x_stage_blocks;                            /* main blocks that stage x windows   */
+    int32_t x_stage_smem;                              /* their dynamic shared memory (bytes) */
 } dasp_plan_info_t;
 
 /*

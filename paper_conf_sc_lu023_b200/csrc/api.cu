@@ -7,10 +7,12 @@
 #include <chrono>
 #include <cmath>
 #include <cstdio>
+#include <cstdint>
 #include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <new>
+#include <utility>
 #include <vector>
 
 #include "format.hpp"
@@ -52,6 +54,11 @@ struct dasp_plan_s {
     void* d_warp_word = nullptr;          // uint64 panel / warp of every main-kernel warp (kernels.cuh)
     int64_t n_mwarps = 0;
     void* d_unit_order = nullptr;         // int32 long-unit execution order (column buckets)
+    void* d_stage = nullptr;              // dasp::StageEnt per main block (x-window staging), or null
+    void* d_stage_map = nullptr;          // the staged blocks' tile maps
+    int stage_smem = 0;                   // dynamic shared memory of the staged instantiation
+    int stage_map_bytes = 0;              // tile-map bytes in front of the staged tiles
+    int64_t stage_blocks = 0;             // staged main blocks
     // timing
     int32_t timing_cap = 0, timing_calls = 0;
     std::vector<TimingRec> recs;
@@ -130,7 +137,9 @@ void free_device(dasp_plan_s* p) {
     if (p->d_panels) cudaFree(p->d_panels);
     if (p->d_warp_word) cudaFree(p->d_warp_word);
     if (p->d_unit_order) cudaFree(p->d_unit_order);
-    p->d_panels = p->d_warp_word = p->d_unit_order = nullptr;
+    if (p->d_stage) cudaFree(p->d_stage);
+    if (p->d_stage_map) cudaFree(p->d_stage_map);
+    p->d_panels = p->d_warp_word = p->d_unit_order = p->d_stage = p->d_stage_map = nullptr;
 
     if (p->d_xh) cudaFree(p->d_xh);
     if (p->d_yh) cudaFree(p->d_yh);
@@ -205,6 +214,7 @@ void dasp_options_default(dasp_options_t* o) {
     o->panel_rows = 0;
     o->max_len = 256;
     o->threshold = 0.75;
+    o->x_stage = 0;
 }
 
 const char* dasp_status_string(dasp_status_t s) {
@@ -237,6 +247,105 @@ std::vector<int32_t> narrow_slots(const HostFormat& f, const int64_t* rb_ptr, co
     for (int64_t rb = 0; rb < f.nrb; ++rb)
         ns[rb] = static_cast<int32_t>((rb_ptr[rb + 1] - rb_ptr[rb]) / be * f.geo.K + (irr_first[2 * rb + 1] - irr_first[2 * rb]));
     return ns;
+}
+
+// x-window staging table (kernels.cuh StageEnt; north_star (3) "shared-memory or TMA staging where
+// reuse exists"), from the host arrays of a host-built plan.  A main block is staged when all its
+// warps are wide medium warps, the columns they gather span at most STAGE_MAX_SPAN tiles of STAGE_T
+// columns, the referenced tiles (after merging the smallest gaps down to STAGE_RUNS runs) fill at
+// most STAGE_MAX_SLOTS slots, and each staged column is gathered at least kStageReuse times on
+// average (a 27-point stencil block: ~5.5; a power-law block: far below 1).  Tiles not wholly
+// inside x are never staged.  Returns the staged block count; st[b].ntile = 0 for the others.
+constexpr double kStageReuse = 2.0;
+// automatic mode (x_stage = 0) stages a plan when a quarter of its main blocks qualify; 0: the
+// automatic mode never stages (measured slower than the L1-served gathers)
+#ifndef DASP_X_STAGE_AUTO
+#define DASP_X_STAGE_AUTO 0
+#endif
+int64_t build_stage_table(const HostFormat& f, const std::vector<uint64_t>& warp_word,
+                          const std::vector<dasp::PanelDesc>& desc, int rbw, int wide_il,
+                          std::vector<dasp::StageEnt>& st, int* max_span, int* max_slots) {
+    using dasp::STAGE_T;
+    const int64_t nb = static_cast<int64_t>(warp_word.size() + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
+    st.assign(static_cast<size_t>(nb), dasp::StageEnt{});
+    const int64_t* rbp = static_cast<const int64_t*>(f.arr[DASP_ARR_RB_PTR].ptr);
+    const int64_t* ip = static_cast<const int64_t*>(f.arr[DASP_ARR_IRR_PTR].ptr);
+    const int32_t* rc = static_cast<const int32_t*>(f.arr[DASP_ARR_REG_COL].ptr);
+    const int32_t* ic = static_cast<const int32_t*>(f.arr[DASP_ARR_IRR_COL].ptr);
+    if (!rbp || !ip || (!rc && f.nnz_reg_new) || (!ic && f.nnz_irreg)) return 0;
+    const int64_t full_tiles = f.n / STAGE_T;   // tiles wholly inside x
+    int64_t staged = 0;
+    int mspan = 0, mslots = 0;
+#pragma omp parallel for schedule(dynamic, 16) reduction(+ : staged) reduction(max : mspan, mslots)
+    for (int64_t b = 0; b < nb; ++b) {
+        std::vector<int64_t> rbs;
+        bool ok = true;
+        for (int k = 0; k < dasp::WARPS_PER_BLOCK && ok; ++k) {
+            const size_t gi = static_cast<size_t>(b * dasp::WARPS_PER_BLOCK + k);
+            if (gi >= warp_word.size() || warp_word[gi] == ~0ull) { ok = false; break; }
+            const dasp::PanelDesc& d = desc[warp_word[gi] >> 32];
+            const int64_t w = static_cast<int64_t>(warp_word[gi] & 0xffffffffu);
+            if (w >= d.nmwd) { ok = false; break; }
+            // the row-blocks of wide warp w (kernels.cu medium_warp)
+            const int64_t rbe = d.rb0 + d.rbm, gw = w & ~int64_t(dasp::WARPS_PER_BLOCK - 1);
+            const int64_t stg = wide_il ? std::min<int64_t>(dasp::WARPS_PER_BLOCK, d.nmwd - gw) : 1;
+            const int64_t r0 = wide_il ? d.rb0 + gw * rbw + (w - gw) : d.rb0 + w * rbw;
+            const int64_t r1 = std::min(r0 - (w - gw) * (wide_il != 0) + stg * rbw, rbe);
+            for (int64_t rb = r0; rb < r1; rb += stg) rbs.push_back(rb);
+        }
+        if (!ok || rbs.empty()) continue;
+        int64_t tmin = INT64_MAX, tmax = -1, gathers = 0;
+        auto each_col = [&](auto&& fn) {
+            for (int64_t rb : rbs) {
+                for (int64_t e = rbp[rb]; e < rbp[rb + 1]; ++e) fn(rc[e]);
+                for (int64_t e = ip[8 * rb]; e < ip[8 * rb + 8]; ++e) fn(ic[e]);
+            }
+        };
+        each_col([&](int32_t c) {
+            if (c < 0 || c / STAGE_T >= full_tiles) return;
+            const int64_t t = c / STAGE_T;
+            tmin = std::min(tmin, t); tmax = std::max(tmax, t); ++gathers;
+        });
+        if (tmax < 0 || tmax - tmin + 1 > dasp::STAGE_MAX_SPAN) continue;
+        const int span = static_cast<int>(tmax - tmin + 1);
+        std::vector<uint8_t> used(static_cast<size_t>(span), 0);
+        each_col([&](int32_t c) {
+            if (c < 0 || c / STAGE_T >= full_tiles) return;
+            used[static_cast<size_t>(c / STAGE_T - tmin)] = 1;
+        });
+        std::vector<std::pair<int, int>> runs;   // [t0, t1)
+        for (int i = 0; i < span; ++i) {
+            if (!used[i]) continue;
+            if (!runs.empty() && runs.back().second == i) runs.back().second = i + 1;
+            else runs.push_back({i, i + 1});
+        }
+        int64_t distinct = 0;
+        for (auto& r : runs) distinct += r.second - r.first;
+        while (static_cast<int>(runs.size()) > dasp::STAGE_RUNS) {   // merge the smallest gap
+            size_t g = 0;
+            for (size_t k = 1; k + 1 < runs.size(); ++k)
+                if (runs[k + 1].first - runs[k].second < runs[g + 1].first - runs[g].second) g = k;
+            runs[g].second = runs[g + 1].second;
+            runs.erase(runs.begin() + static_cast<std::ptrdiff_t>(g) + 1);
+        }
+        int slots = 0;
+        for (auto& r : runs) slots += r.second - r.first;
+        if (slots > dasp::STAGE_MAX_SLOTS || static_cast<double>(gathers) < kStageReuse * distinct * STAGE_T) continue;
+        dasp::StageEnt& e = st[static_cast<size_t>(b)];
+        e.xbase = static_cast<int32_t>(tmin * STAGE_T);
+        e.ntile = span;
+        e.meta = static_cast<int32_t>(runs.size()) | (slots << 8);
+        for (size_t r = 0; r < runs.size(); ++r) {
+            e.run_t0[r] = static_cast<uint16_t>(runs[r].first);
+            e.run_nt[r] = static_cast<uint16_t>(runs[r].second - runs[r].first);
+        }
+        ++staged;
+        mspan = std::max(mspan, span);
+        mslots = std::max(mslots, slots);
+    }
+    *max_span = mspan;
+    *max_slots = mslots;
+    return staged;
 }
 
 dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_t* panel_table,
@@ -339,6 +448,20 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
             for (int64_t w = 0; w < d.nunits; ++w) unit_order[d.unit0 + cnt[bucket(d.unit0 + w)]++] = static_cast<int32_t>(d.unit0 + w);
         }
     }
+    // x-window staging (x_stage: 0 automatic -- on when at least a quarter of the main blocks
+    // qualify --, 1 off, 2 wherever a block qualifies); host-built CUDA-core plans only
+    p->stage_blocks = 0;
+    p->stage_smem = p->stage_map_bytes = 0;
+    std::vector<dasp::StageEnt> stab;
+    if (o.x_stage != 1 && p->variant == DASP_VARIANT_CUDACORE && f.arr[DASP_ARR_REG_COL].ptr && p->blocks > 0) {
+        int mspan = 0, mslots = 0;
+        const int64_t ns = build_stage_table(f, warp_word, desc, p->rbw, p->wide_il, stab, &mspan, &mslots);
+        if (ns > 0 && (o.x_stage == 2 || (DASP_X_STAGE_AUTO && 4 * ns >= p->blocks))) {
+            p->stage_blocks = ns;
+            p->stage_map_bytes = (mspan + 127) / 128 * 128;
+            p->stage_smem = p->stage_map_bytes + mslots * dasp::STAGE_T * sx(p->dtype);
+        }
+    }
     if (p->device < 0) return DASP_OK;
 
     auto upload = [&](void** dst, const void* src, size_t bytes) -> dasp_status_t {
@@ -354,6 +477,21 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     if ((st = upload(&p->d_panels, desc.data(), desc.size() * sizeof(dasp::PanelDesc))) != DASP_OK) return st;
     if ((st = upload(&p->d_warp_word, warp_word.data(), warp_word.size() * 8)) != DASP_OK) return st;
     if ((st = upload(&p->d_unit_order, unit_order.data(), unit_order.size() * 4)) != DASP_OK) return st;
+    if (p->stage_blocks > 0) {
+        // tile maps: span tile -> slot (runs back to back), 0xff elsewhere; 16-byte aligned per block
+        std::vector<unsigned char> maps;
+        for (auto& e : stab) {
+            if (e.ntile <= 0) continue;
+            e.map16 = static_cast<int32_t>(maps.size() / 16);
+            const size_t at = maps.size();
+            maps.resize(at + ((static_cast<size_t>(e.ntile) + 15) & ~size_t(15)), 0xff);
+            int slot = 0;
+            for (int r = 0; r < (e.meta & 0xff); ++r)
+                for (int k = 0; k < e.run_nt[r]; ++k) maps[at + e.run_t0[r] + k] = static_cast<unsigned char>(slot++);
+        }
+        if ((st = upload(&p->d_stage, stab.data(), stab.size() * sizeof(dasp::StageEnt))) != DASP_OK) return st;
+        if ((st = upload(&p->d_stage_map, maps.data(), maps.size())) != DASP_OK) return st;
+    }
 
     return DASP_OK;
 }
@@ -624,8 +762,17 @@ static dasp_status_t spmv_impl(dasp_plan_t p, const void* x, void* y, const dasp
     mp.n0 = n0;
     mp.fin_warps = dasp::finish_warps(mp.row_long, n0);
     const int64_t fin_blocks = (mp.fin_warps + dasp::WARPS_PER_BLOCK - 1) / dasp::WARPS_PER_BLOCK;
+    // x-window staging: CUDA-core calls without scatter destinations whose x is 16-byte aligned
+    // (cp.async.bulk source alignment); any other call runs the unstaged instantiation
+    int stage_smem = 0;
+    if (p->d_stage && variant == DASP_VARIANT_CUDACORE && extra.n == 0 && (reinterpret_cast<uintptr_t>(x) & 15) == 0) {
+        mp.stage = static_cast<const dasp::StageEnt*>(p->d_stage);
+        mp.stage_map = static_cast<const unsigned char*>(p->d_stage_map);
+        mp.stage_map_bytes = p->stage_map_bytes;
+        stage_smem = p->stage_smem;
+    }
     e = timed(p, DASP_K_MAIN, s, on, [&] {
-        return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s, p->occ5);
+        return dasp::launch_main(mp, p->dtype, variant, p->blocks + fin_blocks, s, p->occ5, stage_smem);
     });
     if (e != cudaSuccess) return DASP_ERR_CUDA;
     return DASP_OK;
@@ -753,6 +900,8 @@ dasp_status_t dasp_plan_get_info(dasp_plan_t p, dasp_plan_info_t* o) {
     o->narrow_rb_per_warp = p->nrw;
     o->main_blocks_per_sm = p->occ5 ? 5 : 4;
     o->short_tiles_per_warp = p->tpw;
+    o->x_stage_blocks = p->stage_blocks;
+    o->x_stage_smem = p->stage_smem;
     o->max_len = f.max_len;
     o->threshold = f.tau;
     o->build_ms = p->build_ms;

@@ -45,6 +45,36 @@
 #ifndef DASP_CHUNK_PIPE_F32
 #define DASP_CHUNK_PIPE_F32 0
 #endif
+//   CHUNK_U2  : CUDA-core wide medium path: two 4-block chunks per load / gather round trip
+//   RAGGED_FIRST: CUDA-core wide medium path: ragged chunk + first irregular element accumulated first
+#ifndef DASP_RAGGED_FIRST_F64
+#define DASP_RAGGED_FIRST_F64 0
+#endif
+#ifndef DASP_RAGGED_FIRST_F32
+#define DASP_RAGGED_FIRST_F32 0
+#endif
+#ifndef DASP_RAGGED_FIRST_F16
+#define DASP_RAGGED_FIRST_F16 1   // C3 FP16 main -4.4 %, C2+ -1.4 %, C2 +-0, C5 +0.9 %; spill-free 5-block kernel (same file)
+#endif
+//   PEEL      : CUDA-core wide medium path: chunk 0, ragged chunk and first irregular element gathered in one round
+#ifndef DASP_PEEL_F64
+#define DASP_PEEL_F64 1   // C2 FP64 main -3.5 %, C2+ -3.6 %, C3 -0.8 %, C5 -0.6 % (profiles/r02/peel_ragged_first_ab.jsonl)
+#endif
+#ifndef DASP_PEEL_F32
+#define DASP_PEEL_F32 0
+#endif
+#ifndef DASP_PEEL_F16
+#define DASP_PEEL_F16 0
+#endif
+#ifndef DASP_CHUNK_U2_F64
+#define DASP_CHUNK_U2_F64 0
+#endif
+#ifndef DASP_CHUNK_U2_F16
+#define DASP_CHUNK_U2_F16 0
+#endif
+#ifndef DASP_CHUNK_U2_F32
+#define DASP_CHUNK_U2_F32 0
+#endif
 #ifndef DASP_SHORT_TPW_F64
 #define DASP_SHORT_TPW_F64 2
 #endif
@@ -66,10 +96,12 @@ constexpr unsigned FULL = 0xffffffffu;
 // variant template argument: bits 0-1 the block-dot path, bit 2 the scatter epilogue
 // (dasp_spmv_scatter), bit 3 the FP16 CUDA-core instantiation at 5 blocks / 48 registers per
 // thread (VAR_OCC5, plans without a wide-medium majority: main_occ5), each instantiated separately
-enum { VAR_MMA = 1, VAR_CUDACORE = 2, VAR_SCATTER = 4, VAR_OCC5 = 8 };
+// bit 4 the x-window staging instantiation (VAR_STAGE, CUDA-core only: x_stage plans)
+enum { VAR_MMA = 1, VAR_CUDACORE = 2, VAR_SCATTER = 4, VAR_OCC5 = 8, VAR_STAGE = 16 };
 __host__ __device__ constexpr int vk(int v) { return v & 3; }
 __host__ __device__ constexpr bool vs(int v) { return (v & VAR_SCATTER) != 0; }
 __host__ __device__ constexpr bool vo(int v) { return (v & VAR_OCC5) != 0; }
+__host__ __device__ constexpr bool vst(int v) { return (v & VAR_STAGE) != 0; }
 
 // ------------------------------------------------------------------------------------------
 // memory helpers
@@ -155,6 +187,85 @@ __device__ __forceinline__ uint32_t ld1_b32(const void* a, uint64_t pol) {
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
     return v;
 }
+// ------------------------------------------------------------------------------------------
+// x-window staging (StageEnt, kernels.cuh): one thread of a staged block arms an mbarrier with
+// the byte count and issues up to STAGE_RUNS cp.async.bulk copies (TMA, UBLKCP) of runs of
+// STAGE_T-column tiles of x into dynamic shared memory; the block fills the span's tile map;
+// the wide medium warps wait on the mbarrier (parity 0) before their first gather and read a
+// staged column from shared memory, any other column from global memory.
+// ------------------------------------------------------------------------------------------
+struct StageSm {
+    unsigned long long bar;
+    int32_t xbase, ntile;
+};
+__shared__ StageSm s_stage;
+extern __shared__ __align__(128) unsigned char s_dyn[];
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+
+// every thread of a staged-instantiation main block (not a finish block) calls this once.  Thread 0
+// initialises the mbarrier (no memory dependency) and the block synchronises once; then thread 0
+// reads the block's entry, publishes xbase / ntile and arms the barrier with the bytes of the tile
+// map and the runs (or arrives without bytes for an unstaged block), while the other warps go on
+// to their metadata and stream loads.  Gathering warps wait on phase 0 (stage_wait).
+__device__ __forceinline__ void stage_prologue(const MainParams& P, int64_t sb, int sx) {
+    const uint32_t bar = smem_u32(&s_stage.bar);
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const StageEnt* e = P.stage + sb;
+        const int ntile = __ldg(&e->ntile);
+        s_stage.ntile = ntile;
+        s_stage.xbase = __ldg(&e->xbase);
+        if (ntile > 0) {
+            const int meta = __ldg(&e->meta), nrun = meta & 0xff;
+            const uint32_t mapb = (static_cast<uint32_t>(ntile) + 15u) & ~15u;
+            const uint32_t tx = mapb + static_cast<uint32_t>(meta >> 8) * STAGE_T * sx;
+            asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(tx) : "memory");
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                         ::"r"(smem_u32(s_dyn)), "l"(P.stage_map + static_cast<int64_t>(__ldg(&e->map16)) * 16), "r"(mapb),
+                           "r"(bar)
+                         : "memory");
+            const char* xg = static_cast<const char*>(P.x) + static_cast<int64_t>(__ldg(&e->xbase)) * sx;
+            uint32_t dst = smem_u32(s_dyn + P.stage_map_bytes);
+            for (int r = 0; r < nrun; ++r) {
+                const uint32_t t0 = __ldg(&e->run_t0[r]), nt = __ldg(&e->run_nt[r]);
+                const uint32_t bytes = nt * STAGE_T * sx;
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(dst), "l"(xg + static_cast<int64_t>(t0) * STAGE_T * sx), "r"(bytes), "r"(bar)
+                             : "memory");
+                dst += bytes;
+            }
+        } else {
+            asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+        }
+    }
+}
+// gathering warps: wait for phase 0 (the copies, or thread 0's plain arrive); returns xbase / ntile
+__device__ __forceinline__ void stage_wait(int32_t& xbase, int32_t& ntile) {
+    const uint32_t bar = smem_u32(&s_stage.bar);
+    asm volatile("{\n\t.reg .pred P1;\nWAIT_%=:\n\t"
+                 "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 P1, [%0], 0;\n\t"
+                 "@!P1 bra WAIT_%=;\n\t}" ::"r"(bar) : "memory");
+    xbase = s_stage.xbase;
+    ntile = s_stage.ntile;
+}
+// staged gather: shared memory when the column's tile is staged, else the read-only path
+template <typename X>
+__device__ __forceinline__ X stage_x(const X* x, const MainParams& P, uint32_t c, int32_t xbase, int32_t ntile) {
+    if (static_cast<int32_t>(c) < 0) return X(0);
+    const uint32_t d = c - static_cast<uint32_t>(xbase);
+    const uint32_t ti = d / STAGE_T;
+    if (ti < static_cast<uint32_t>(ntile)) {
+        const uint32_t slot = s_dyn[ti];
+        if (slot != 0xffu)
+            return reinterpret_cast<const X*>(s_dyn + P.stage_map_bytes)[slot * STAGE_T + (d % STAGE_T)];
+    }
+    return __ldg(x + c);
+}
+
 // x gather through the read-only path; column -1 (pad, R12) reads 0 without touching memory
 #ifndef DASP_EXP_NOX
 #define DASP_EXP_NOX 0   // experiment only: every x gather reads x[c & 255] (cache-resident) -- wrong results
@@ -450,8 +561,96 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
     const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val) + M.base;
     const int32_t* rc = P.reg_col + M.base;
     const typename IO::T* x = static_cast<const typename IO::T*>(P.x);
+    // x gather: through shared memory in a staged block (VAR_STAGE), else the read-only path
+    int32_t sxb = 0, snt = 0;
+    if constexpr (vst(VAR)) stage_wait(sxb, snt);
+    auto G = [&](uint32_t c) -> double {
+        if constexpr (vst(VAR)) return static_cast<double>(stage_x<typename IO::T>(x, P, c, sxb, snt));
+        else return IO::gx(x, c);
+    };
     double c0 = 0.0, c1 = 0.0, part = 0.0;
-    if constexpr (FULL) {
+    // CUDA-core RAGGED_FIRST: the ragged last chunk and the first irregular element (loaded in the
+    // first round with chunk 0) are gathered and accumulated before the full chunks, so their gathers
+    // travel with chunk 0's instead of after the chunk loop, and their registers are free during it
+    constexpr bool RF = vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_RAGGED_FIRST) != 0;
+    auto ragged_irr = [&]() {
+        double xr[3];
+#pragma unroll
+        for (int j = 0; j < 3; ++j) xr[j] = G(L.cr[j]);   // pads / unused slots read 0
+        const double xi = G(L.ci);
+#pragma unroll
+        for (int j = 0; j < 3; ++j) {
+            if (j < rem) {                                     // rem is warp-uniform
+                if constexpr (vk(VAR) == VAR_MMA) dmma(c0, c1, IO::cv(L.vr[j]), xr[j]);
+                else part = fma(IO::cv(L.vr[j]), xr[j], part);
+            }
+        }
+        if constexpr (vk(VAR) == VAR_MMA) {                        // Alg. 3 l.13-17: diagonal -> quad g
+            const double d = diag_to_quad(c0, c1, lane);
+            part = t == 0 ? d : 0.0;
+        }
+        part = fma(IO::cv(L.vi), xi, part);                    // Alg. 3 l.20-24: irregular part
+    };
+    if constexpr (RF) ragged_irr();
+    if constexpr (FULL && vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_PEEL) != 0) {
+        // CUDA-core PEEL: chunk 0's gathers, the ragged chunk's and the first irregular element's
+        // go out in one round (all were loaded together in the first round); accumulation order
+        // chunk 0, ragged, irregular element, chunks 1..nfull-1
+        if (nfull > 0) {
+            double xa[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) xa[j] = G(L.ca[j]);
+            double xr[3];
+#pragma unroll
+            for (int j = 0; j < 3; ++j) xr[j] = G(L.cr[j]);
+            const double xi = G(L.ci);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) part = fma(IO::cv(L.va[j]), xa[j], part);
+#pragma unroll
+            for (int j = 0; j < 3; ++j)
+                if (j < rem) part = fma(IO::cv(L.vr[j]), xr[j], part);
+            part = fma(IO::cv(L.vi), xi, part);
+            for (int ch = 1; ch < nfull; ++ch) {
+                typename IO::R va[4];
+                uint32_t ca[4];
+                IO::ld4r(rv + ch * 128 + lane * 4, pol, va);
+                ld4_b32(rc + ch * 128 + lane * 4, pol, ca);
+                double xv[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) xv[j] = G(ca[j]);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xv[j], part);
+            }
+        } else {
+            ragged_irr();
+        }
+    } else if constexpr (FULL && vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_CHUNK_U2) != 0) {
+        // two chunks per round trip: chunk ch+1's stream loads are issued together with chunk ch's
+        // (ch > 0), then the 8 gathers, then 8 FMAs in slot order (the same per-lane order as one
+        // chunk at a time, so the result is bitwise unchanged)
+        typename IO::R va[4], vb[4];
+        uint32_t ca[4], cb[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) { va[j] = L.va[j]; ca[j] = L.ca[j]; }
+        for (int ch = 0; ch < nfull; ch += 2) {
+            if (ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
+            const bool two = ch + 1 < nfull;                   // warp-uniform
+#pragma unroll
+            for (int j = 0; j < 4; ++j) { vb[j] = 0; cb[j] = 0xffffffffu; }
+            if (two) { IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vb); ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cb); }
+            double xa[4], xb[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) xa[j] = G(ca[j]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) xb[j] = G(cb[j]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xa[j], part);
+            if (two) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) part = fma(IO::cv(vb[j]), xb[j], part);
+            }
+        }
+    } else if constexpr (FULL) {
         typename IO::R va[4];
         uint32_t ca[4];
 #pragma unroll
@@ -462,7 +661,7 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
             if (!DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
             double xv[4];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) xv[j] = IO::gx(x, ca[j]);
+            for (int j = 0; j < 4; ++j) xv[j] = G(ca[j]);
             typename IO::R vn[4];
             uint32_t cn[4];
             if (DASP_BY_DT(DT, DASP_CHUNK_PIPE) && ch + 1 < nfull) {
@@ -480,25 +679,10 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
             }
         }
     }
-    double xr[3];
-#pragma unroll
-    for (int j = 0; j < 3; ++j) xr[j] = IO::gx(x, L.cr[j]);   // pads / unused slots read 0
-    const double xi = IO::gx(x, L.ci);
-#pragma unroll
-    for (int j = 0; j < 3; ++j) {
-        if (j < rem) {                                     // rem is warp-uniform
-            if constexpr (vk(VAR) == VAR_MMA) dmma(c0, c1, IO::cv(L.vr[j]), xr[j]);
-            else part = fma(IO::cv(L.vr[j]), xr[j], part);
-        }
-    }
-    if constexpr (vk(VAR) == VAR_MMA) {                        // Alg. 3 l.13-17: diagonal -> quad g
-        const double d = diag_to_quad(c0, c1, lane);
-        part = t == 0 ? d : 0.0;
-    }
-    part = fma(IO::cv(L.vi), xi, part);                    // Alg. 3 l.20-24: irregular part
+    if constexpr (!RF && !(FULL && vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_PEEL) != 0)) ragged_irr();
     const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
     for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
-        part = fma(IO::ld1(iv + k, pol), IO::gx(x, ld1_b32(P.irr_col + k, pol)), part);
+        part = fma(IO::ld1(iv + k, pol), G(ld1_b32(P.irr_col + k, pol)), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
     if (t == 0) store_y<DT, VAR>(P, M.orow, part);              // Alg. 3 l.25 through the output map (R9)
@@ -540,6 +724,12 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
     const int32_t* rc = P.reg_col + M.base;
     const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
     const uint16_t* x = static_cast<const uint16_t*>(P.x);
+    int32_t sxb = 0, snt = 0;
+    if constexpr (vst(VAR)) stage_wait(sxb, snt);
+    auto GH = [&](uint32_t c) -> uint16_t {
+        if constexpr (vst(VAR)) return stage_x<unsigned short>(reinterpret_cast<const unsigned short*>(x), P, c, sxb, snt);
+        else return gxh(x, c);
+    };
     float c0 = 0.f, c1 = 0.f, part = 0.f;
     // one 8x8 block: this lane's two slots 2t, 2t+1 of row g
     auto blockx = [&](uint32_t a, uint16_t xa, uint16_t xb) {
@@ -551,8 +741,75 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
             part = fmaf(av.y, h2f(xb), part);
         }
     };
-    auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) { blockx(a, gxh(x, ca), gxh(x, cb)); };
-    if constexpr (FULL) {
+    auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) { blockx(a, GH(ca), GH(cb)); };
+    // CUDA-core RAGGED_FIRST / CHUNK_U2: as in medium_finish_f64
+    constexpr bool RF = vk(VAR) == VAR_CUDACORE && DASP_RAGGED_FIRST_F16 != 0;
+    auto ragged_irr = [&]() {
+#pragma unroll
+        for (int j = 0; j < 3; ++j)
+            if (j < rem) block(L.vr[j], L.cr[2 * j], L.cr[2 * j + 1]);   // rem is warp-uniform
+        if constexpr (vk(VAR) == VAR_MMA) {
+            const float d = diag_to_quad(c0, c1, lane);
+            part = t == 0 ? d : 0.f;
+        }
+        part = fmaf(h2f(L.vi), h2f(GH(L.ci)), part);
+    };
+    if constexpr (RF) ragged_irr();
+    constexpr bool PEEL = FULL && vk(VAR) == VAR_CUDACORE && DASP_PEEL_F16 != 0;
+    if constexpr (PEEL) {
+        if (nfull > 0) {
+            uint16_t xa[8], xr[6];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) xa[e] = GH(L.ca[e]);
+#pragma unroll
+            for (int e = 0; e < 6; ++e) xr[e] = GH(L.cr[e]);
+            const uint16_t xi = GH(L.ci);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) blockx(L.va[j], xa[2 * j], xa[2 * j + 1]);
+#pragma unroll
+            for (int j = 0; j < 3; ++j)
+                if (j < rem) blockx(L.vr[j], xr[2 * j], xr[2 * j + 1]);
+            part = fmaf(h2f(L.vi), h2f(xi), part);
+            for (int ch = 1; ch < nfull; ++ch) {
+                uint32_t va[4], ca[8];
+                ld4_b32(rv + ch * 256 + lane * 8, pol, va);
+                ld8_b32(rc + ch * 256 + lane * 8, pol, ca);
+                uint16_t xh[8];
+#pragma unroll
+                for (int e = 0; e < 8; ++e) xh[e] = GH(ca[e]);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) blockx(va[j], xh[2 * j], xh[2 * j + 1]);
+            }
+        } else {
+            ragged_irr();
+        }
+    } else if constexpr (FULL && vk(VAR) == VAR_CUDACORE && DASP_CHUNK_U2_F16 != 0) {
+        uint32_t va[4], ca[8], vb[4], cb[8];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) va[j] = L.va[j];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) ca[e] = L.ca[e];
+        for (int ch = 0; ch < nfull; ch += 2) {
+            if (ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
+            const bool two = ch + 1 < nfull;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) vb[j] = 0u;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) cb[e] = 0xffffffffu;
+            if (two) { ld4_b32(rv + (ch + 1) * 256 + lane * 8, pol, vb); ld8_b32(rc + (ch + 1) * 256 + lane * 8, pol, cb); }
+            uint16_t xa[8], xb[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) xa[e] = GH(ca[e]);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) xb[e] = GH(cb[e]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) blockx(va[j], xa[2 * j], xa[2 * j + 1]);
+            if (two) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) blockx(vb[j], xb[2 * j], xb[2 * j + 1]);
+            }
+        }
+    } else if constexpr (FULL) {
         uint32_t va[4], ca[8];
 #pragma unroll
         for (int j = 0; j < 4; ++j) va[j] = L.va[j];
@@ -562,7 +819,7 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
             if (!DASP_CHUNK_PIPE_F16 && ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
             uint16_t xh[8];
 #pragma unroll
-            for (int e = 0; e < 8; ++e) xh[e] = gxh(x, ca[e]);
+            for (int e = 0; e < 8; ++e) xh[e] = GH(ca[e]);
             uint32_t vn[4], cn[8];
             if (DASP_CHUNK_PIPE_F16 && ch + 1 < nfull) { ld4_b32(rv + (ch + 1) * 256 + lane * 8, pol, vn); ld8_b32(rc + (ch + 1) * 256 + lane * 8, pol, cn); }
 #pragma unroll
@@ -575,16 +832,9 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
             }
         }
     }
-#pragma unroll
-    for (int j = 0; j < 3; ++j)
-        if (j < rem) block(L.vr[j], L.cr[2 * j], L.cr[2 * j + 1]);   // rem is warp-uniform
-    if constexpr (vk(VAR) == VAR_MMA) {
-        const float d = diag_to_quad(c0, c1, lane);
-        part = t == 0 ? d : 0.f;
-    }
-    part = fmaf(h2f(L.vi), h2f(gxh(x, L.ci)), part);
+    if constexpr (!RF && !PEEL) ragged_irr();
     for (int64_t k = M.ib + t + 4; k < M.ib + M.ilen; k += 4)
-        part = fmaf(h2f(__ldg(iv + k)), h2f(gxh(x, ld1_b32(P.irr_col + k, pol))), part);
+        part = fmaf(h2f(__ldg(iv + k)), h2f(GH(ld1_b32(P.irr_col + k, pol))), part);
     part += __shfl_xor_sync(FULL, part, 1);
     part += __shfl_xor_sync(FULL, part, 2);
     if (t == 0) store_y<1, VAR>(P, M.orow, part);
@@ -1251,20 +1501,11 @@ dasp_long_kernel(const MainParams P, int64_t n_units) {
     else long_unit_f64<DT, VAR>(P, u, lane, pol);
 }
 
-// medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
+// one main-kernel warp after the finish blocks: its role inside its panel (MainParams::warp_word);
+// the descriptor fields are loaded only on the branch that needs them so they do not stay live
+// (register pressure = occupancy)
 template <int DT, int VAR>
-__global__ void __launch_bounds__(MAIN_THREADS, vo(VAR) ? 5
-                                                         : (DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32)))
-dasp_main_kernel(const MainParams P) {
-    const int lane = threadIdx.x & 31;
-    const int64_t fin_blocks = (P.fin_warps + WARPS_PER_BLOCK - 1) / WARPS_PER_BLOCK;
-    if (blockIdx.x < fin_blocks) {                       // long-row phase 2 + empty rows
-        const int64_t fw = static_cast<int64_t>(blockIdx.x) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
-        if (fw < P.fin_warps) finish_warp<DT, VAR>(P, fw, lane);
-        return;
-    }
-    // role of this warp inside its panel (MainParams::warp_word); the descriptor fields are loaded
-    // only on the branch that needs them so they do not stay live (register pressure = occupancy)
+__device__ __forceinline__ void main_warp(const MainParams& P, int64_t fin_blocks, int lane) {
     const int64_t gw = (static_cast<int64_t>(blockIdx.x) - fin_blocks) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
     if (gw >= P.n_mwarps) return;
     const uint64_t ww = __ldg(P.warp_word + gw);
@@ -1279,6 +1520,29 @@ dasp_main_kernel(const MainParams P) {
         return;
     }
     short_item<DT, VAR>(P, D, w - nmw, lane, pol);
+}
+
+// medium row-blocks and short tiles of every panel (panel order; Alg. 3-5)
+template <int DT, int VAR>
+__global__ void __launch_bounds__(MAIN_THREADS, vo(VAR) ? 5
+                                                         : (DT == 0 ? DASP_MIN_BLOCKS : (DT == 1 ? DASP_MIN_BLOCKS_F16 : DASP_MIN_BLOCKS_F32)))
+dasp_main_kernel(const MainParams P) {
+    const int lane = threadIdx.x & 31;
+    const int64_t fin_blocks = (P.fin_warps + WARPS_PER_BLOCK - 1) / WARPS_PER_BLOCK;
+    if (blockIdx.x < fin_blocks) {                       // long-row phase 2 + empty rows
+        const int64_t fw = static_cast<int64_t>(blockIdx.x) * WARPS_PER_BLOCK + (threadIdx.x >> 5);
+        if (fw < P.fin_warps) finish_warp<DT, VAR>(P, fw, lane);
+        return;
+    }
+    if constexpr (vst(VAR)) {                            // x-window staging: before any warp returns
+        stage_prologue(P, static_cast<int64_t>(blockIdx.x) - fin_blocks, static_cast<int>(sizeof(typename Tr<DT>::X)));
+        main_warp<DT, VAR>(P, fin_blocks, lane);
+        // the block's shared memory must outlive its bulk copies (a block whose warps gathered
+        // nothing would otherwise exit with copies in flight)
+        if (threadIdx.x == 0) { int32_t a, b; stage_wait(a, b); }
+    } else {
+        main_warp<DT, VAR>(P, fin_blocks, lane);
+    }
 }
 
 
@@ -1322,7 +1586,18 @@ int short_tiles_per_warp(int dtype, bool occ5) { return occ5 ? DASP_SHORT_TPW_OC
 int narrow_rb_per_warp(int) { return DASP_NARROW_RB; }
 
 template <int DT>
-static cudaError_t launch_main_dt(const MainParams& p, int variant, bool scatter, bool occ5, unsigned nb, cudaStream_t s) {
+static cudaError_t launch_main_dt(const MainParams& p, int variant, bool scatter, bool occ5, unsigned nb, cudaStream_t s,
+                                  int stage_smem) {
+    if (stage_smem > 0 && variant == VAR_CUDACORE && !scatter) {   // x-window staging instantiation
+        if constexpr (DT == 1) {
+            if (occ5) {
+                dasp_main_kernel<DT, VAR_CUDACORE | VAR_OCC5 | VAR_STAGE><<<nb, MAIN_THREADS, stage_smem, s>>>(p);
+                return cudaGetLastError();
+            }
+        }
+        dasp_main_kernel<DT, VAR_CUDACORE | VAR_STAGE><<<nb, MAIN_THREADS, stage_smem, s>>>(p);
+        return cudaGetLastError();
+    }
     if constexpr (DT == 1) {
         if (occ5 && variant != VAR_MMA) {
             if (scatter) dasp_main_kernel<1, VAR_CUDACORE | VAR_SCATTER | VAR_OCC5><<<nb, MAIN_THREADS, 0, s>>>(p);
@@ -1340,14 +1615,16 @@ static cudaError_t launch_main_dt(const MainParams& p, int variant, bool scatter
     return cudaGetLastError();
 }
 
-cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s, bool occ5) {
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s, bool occ5,
+                        int stage_smem) {
     if (blocks <= 0) return cudaSuccess;
     if (blocks > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     const unsigned nb = static_cast<unsigned>(blocks);
     const bool scatter = p.extra.n > 0;
-    if (dtype == 0) return launch_main_dt<0>(p, variant, scatter, false, nb, s);
-    if (dtype == 1) return launch_main_dt<1>(p, variant, scatter, occ5, nb, s);
-    return launch_main_dt<2>(p, variant, scatter, false, nb, s);
+    if (!p.stage) stage_smem = 0;
+    if (dtype == 0) return launch_main_dt<0>(p, variant, scatter, false, nb, s, stage_smem);
+    if (dtype == 1) return launch_main_dt<1>(p, variant, scatter, occ5, nb, s, stage_smem);
+    return launch_main_dt<2>(p, variant, scatter, false, nb, s, stage_smem);
 }
 
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s) {

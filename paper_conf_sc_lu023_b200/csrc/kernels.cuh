@@ -36,6 +36,27 @@ struct PanelDesc {
     int64_t rbm, rbn, nmwd, nmwm;
 };
 
+// Shared-memory staging of x windows (north_star (3): "shared-memory or TMA staging where reuse
+// exists").  One entry per main-kernel block (after the finish blocks).  A staged
+// block's wide medium warps gather x from shared memory: the block's referenced columns, in tiles
+// of STAGE_T consecutive columns, are copied by cp.async.bulk (TMA) at block start as up to
+// STAGE_RUNS runs of consecutive tiles, together with the block's tile map (plan-built, in the
+// stage_map array at 16-byte offset map16): span tile i (columns xbase + STAGE_T i ..) lives in
+// slot tmap[i] (0xff = not staged: gathered from global memory).
+constexpr int STAGE_T = 32;          // columns per tile
+constexpr int STAGE_RUNS = 4;        // bulk copies per block
+constexpr int STAGE_MAX_SPAN = 4096; // tiles in a block's span (one byte of tile map each)
+constexpr int STAGE_MAX_SLOTS = 96;  // staged tiles per block (FP64: 24 KB)
+struct StageEnt {
+    int32_t xbase;                   // first column of span tile 0 (a multiple of STAGE_T)
+    int32_t ntile;                   // span tiles; 0 = block not staged
+    uint16_t run_t0[STAGE_RUNS];     // run r: span tiles [run_t0[r], run_t0[r] + run_nt[r]),
+    uint16_t run_nt[STAGE_RUNS];     //   stored in slots after the previous runs'
+    int32_t meta;                    // nrun | slots << 8
+    int32_t map16;                   // tile map offset in stage_map, 16-byte units
+};
+static_assert(sizeof(StageEnt) == 32, "StageEnt layout");
+
 // Everything the long-row and main kernels read.
 struct MainParams {
     const void* long_val;
@@ -73,6 +94,11 @@ struct MainParams {
     const int32_t* long_out;
     const int32_t* empty_rows;
     int64_t row_long, n0, fin_warps;
+    // x-window staging (staged instantiation only): per-block table and the tile-map bytes that
+    // precede the staged tiles in dynamic shared memory
+    const StageEnt* stage;
+    const unsigned char* stage_map;   // every staged block's tile map (16-byte aligned each)
+    int32_t stage_map_bytes;
 };
 // finish work of the fused main kernel: 4 long rows per warp, then 128 empty rows per warp
 inline int64_t finish_warps(int64_t row_long, int64_t n0) { return (row_long + 3) / 4 + (n0 + 127) / 128; }
@@ -80,7 +106,10 @@ inline int64_t finish_warps(int64_t row_long, int64_t n0) { return (row_long + 3
 // variant: 1 = MMA (DMMA/HMMA diagonal trick), 2 = CUDA-core.  dtype: 0 = FP64, 1 = FP16, 2 = FP32.
 // occ5: FP16 CUDA-core plans without a wide-medium majority run the 5-block / 48-register
 // instantiation (its short warps take DASP_SHORT_TPW_OCC5 tiles: short_tiles_per_warp(dtype, true))
-cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s, bool occ5 = false);
+// stage_smem > 0 (with p.stage set): the x-window staging instantiation, that many bytes of dynamic
+// shared memory per block
+cudaError_t launch_main(const MainParams& p, int dtype, int variant, int64_t blocks, cudaStream_t s, bool occ5 = false,
+                        int stage_smem = 0);
 cudaError_t launch_long(const MainParams& p, int dtype, int variant, int64_t n_units, cudaStream_t s);
 // short tiles one main-kernel warp processes (build knobs DASP_SHORT_TPW_*)
 int short_tiles_per_warp(int dtype, bool occ5 = false);

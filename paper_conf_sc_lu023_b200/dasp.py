@@ -44,7 +44,7 @@ class Options(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("variant", ctypes.c_int32), ("validate", ctypes.c_int32),
                 ("keep_host", ctypes.c_int32), ("medium_rb_per_warp", ctypes.c_int32),
                 ("num_threads", ctypes.c_int32), ("panel_rows", ctypes.c_int64),
-                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double)]
+                ("max_len", ctypes.c_int32), ("threshold", ctypes.c_double), ("x_stage", ctypes.c_int32)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -60,7 +60,8 @@ class PlanInfo(ctypes.Structure):
                 ("max_len", ctypes.c_int64), ("threshold", ctypes.c_double),
                 ("build_ms", ctypes.c_double), ("upload_ms", ctypes.c_double),
                 ("rowblocks_mid", ctypes.c_int64), ("rowblocks_narrow", ctypes.c_int64), ("narrow_rb_per_warp", ctypes.c_int32),
-                ("main_blocks_per_sm", ctypes.c_int32), ("short_tiles_per_warp", ctypes.c_int32)]
+                ("main_blocks_per_sm", ctypes.c_int32), ("short_tiles_per_warp", ctypes.c_int32),
+                ("x_stage_blocks", ctypes.c_int64), ("x_stage_smem", ctypes.c_int32)]
 
     def as_dict(self):
         return {name: getattr(self, name) for name, _ in self._fields_}
@@ -162,12 +163,12 @@ class Plan:
 def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", device: int = 0,
                      variant: int = DASP_VARIANT_CUDACORE, validate: bool = True, keep_host: bool = False,
                      medium_rb_per_warp: int = 0, num_threads: int = 0, panel_rows: int = 0,
-                     max_len: int = 256, threshold: float = 0.75) -> Plan:
+                     max_len: int = 256, threshold: float = 0.75, x_stage: int = 0) -> Plan:
     """Build the DASP format of a host CSR matrix and upload it (device=-1: host-only plan).
 
     row_ptr int64[m+1], col_idx int32[nnz], val float64[nnz] (dtype "f64") or float16[nnz]
     (dtype "f16"; passed as binary16 bits) or float32[nnz] (dtype "f32").  panel_rows: 0 automatic,
-    -1 one global panel."""
+    -1 one global panel.  x_stage: shared-memory x-window staging, 0 automatic, 1 off, 2 on."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     if dtype == "f64":
@@ -193,6 +194,7 @@ def dasp_plan_create(row_ptr, col_idx, val, m: int, n: int, dtype: str = "f64", 
     opts.keep_host, opts.medium_rb_per_warp, opts.num_threads = int(keep_host), medium_rb_per_warp, num_threads
     opts.panel_rows = panel_rows
     opts.max_len, opts.threshold = int(max_len), float(threshold)
+    opts.x_stage = int(x_stage)
     h = ctypes.c_void_p()
     st = _lib.dasp_plan_create(ctypes.byref(h), m, n, nnz, _ptr(row_ptr), _ptr(col_idx), _ptr(val), dt,
                                ctypes.byref(opts))

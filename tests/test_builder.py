@@ -228,3 +228,26 @@ def test_binding_rejects_short_and_mistyped_host_buffers():
         dasp.dasp_spmv_host_stream(p, np.zeros(2 * A.n - 1), A.n, np.zeros(2 * A.m), A.m, 2)
     with pytest.raises(ValueError):
         dasp.dasp_spmv_host_stream(p, np.zeros(2 * A.n), A.n, np.zeros(2 * A.m - 1), A.m, 2)
+
+
+def test_x_stage_table_selection():
+    """x-window staging is chosen from the plan's own columns: the wide medium blocks of
+    a 27-point stencil gather from three dense plane windows (staged); a power-law matrix's blocks
+    gather from all of x (never staged); FP16 stencil rows (27 <= 4K = 32 slots) are mid row-blocks,
+    not wide ones; x_stage = 1 turns it off; the MMA default variant never stages."""
+    st = synth.generate(synth.config("c2", scale=0.25))
+    for dt, sx in (("f64", 8), ("f32", 4)):
+        val = st.val.astype(np.float64 if dt == "f64" else np.float32)
+        info = dasp.dasp_plan_create(st.row_ptr, st.col, val, st.m, st.n, dt, device=-1, x_stage=2).info
+        assert info["x_stage_blocks"] > 0
+        # tile map (one byte per span tile, 128-B rounded) + staged tiles of 32 columns
+        assert info["x_stage_smem"] >= 3 * 32 * sx and (info["x_stage_smem"] - 32 * sx * 96) <= 4096
+        off = dasp.dasp_plan_create(st.row_ptr, st.col, val, st.m, st.n, dt, device=-1, x_stage=1).info
+        assert off["x_stage_blocks"] == 0 and off["x_stage_smem"] == 0
+    mma = dasp.dasp_plan_create(st.row_ptr, st.col, st.val, st.m, st.n, "f64", device=-1,
+                                variant=dasp.DASP_VARIANT_MMA, x_stage=2).info
+    assert mma["x_stage_blocks"] == 0
+    h = dasp.dasp_plan_create(st.row_ptr, st.col, st.val.astype(np.float16), st.m, st.n, "f16", device=-1, x_stage=2).info
+    assert h["x_stage_blocks"] == 0 and h["rowblocks_mid"] > 0
+    pl = synth.generate(synth.config("c3", scale=0.02))
+    assert dasp.dasp_plan_create(pl.row_ptr, pl.col, pl.val, pl.m, pl.n, "f64", device=-1, x_stage=2).info["x_stage_blocks"] == 0

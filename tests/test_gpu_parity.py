@@ -475,3 +475,78 @@ def test_fp16_occupancy5_layout(name, expect5):
     assert mplan.info["main_blocks_per_sm"] == 4
     for v in VARIANTS:
         assert np.array_equal(run(mplan, x, "f16", variant=v), y_ref), (name, VNAME[v])
+
+
+# x-window staging (north_star (3) "shared-memory or TMA staging where reuse exists"):
+# a staged block gathers the same x values from shared memory, so its y is bitwise the unstaged y
+def _band_windows(m, n, windows, width, seed):
+    """rows of `windows` clusters of `width` consecutive columns, cluster k at offset k * (n - m) /
+    (windows - 1) from the row index (a stencil-like window structure with more windows than runs)"""
+    rng = np.random.default_rng(seed)
+    step = (n - m - width) // max(1, windows - 1)
+    rows = []
+    for i in range(m):
+        cols = np.concatenate([i + k * step + np.arange(width) for k in range(windows)])
+        rows.append(np.unique(np.clip(cols, 0, n - 1)))
+    rp = np.zeros(m + 1, dtype=np.int64)
+    rp[1:] = np.cumsum([len(r) for r in rows])
+    col = np.concatenate(rows).astype(np.int32)
+    val = rng.integers(-3, 4, len(col)).astype(np.float64)
+    return synth.CSR(m, n, rp, col, val, name="band")
+
+
+def _stage_cases():
+    yield "c2_32", synth.generate(synth.config("c2", scale=0.25, val_mode=synth.VAL_INT))
+    yield "c2_64", synth.generate(synth.config("c2", scale=0.5, val_mode=synth.VAL_INT))
+    yield "band6", _band_windows(40000, 40000 + 6 * 700 + 33, 6, 5, 3)        # 6 windows -> merged runs
+    yield "band3_odd", _band_windows(30001, 30001 + 2 * 900 + 41, 3, 7, 4)    # n not a multiple of 32
+
+
+STAGE_CASES = list(_stage_cases())
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+@pytest.mark.parametrize("name,A", STAGE_CASES, ids=[c[0] for c in STAGE_CASES])
+def test_x_stage_bitwise_equal_to_unstaged(name, A, dt):
+    staged, plain = make(A, dt, x_stage=2), make(A, dt, x_stage=1)
+    assert staged.info["x_stage_blocks"] > 0 and staged.info["x_stage_smem"] > 0, name
+    assert plain.info["x_stage_blocks"] == 0
+    for seed, mode in ((11, synth.VAL_INT), (12, synth.VAL_UNIFORM)):
+        x = synth.vector(seed, A.n, mode)
+        y0 = synth.vector(seed + 1, A.m, mode)
+        for alpha, beta in ((1.0, 0.0), (-0.5, 2.0)):
+            ys = run(staged, x, dt, alpha, beta, y0 if beta else None, variant=dasp.DASP_VARIANT_CUDACORE)
+            yp = run(plain, x, dt, alpha, beta, y0 if beta else None, variant=dasp.DASP_VARIANT_CUDACORE)
+            assert np.array_equal(ys, yp), (name, dt, seed, alpha)
+            y_ref, s = oracle_ref(A, x, dt, alpha, beta, y0 if beta else None)
+            if mode == synth.VAL_INT:
+                assert np.array_equal(ys, y_ref), (name, dt)
+            else:
+                assert oracle.tolerance_ok(ys, y_ref, s, dt).all(), (name, dt)
+        # the MMA variant of a staged plan runs the unstaged kernel: same values
+        ym = run(staged, x, dt, variant=dasp.DASP_VARIANT_MMA)
+        y_ref, s = oracle_ref(A, x, dt)
+        assert oracle.tolerance_ok(ym, y_ref, s, dt).all()
+
+
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+def test_x_stage_misaligned_x_falls_back(dt):
+    """x that is not 16-byte aligned (a view at an odd element offset) cannot be the cp.async.bulk
+    source: the call runs the unstaged kernel and gives the same y"""
+    A = STAGE_CASES[0][1]
+    plan = make(A, dt, x_stage=2)
+    assert plan.info["x_stage_blocks"] > 0
+    x = synth.vector(21, A.n, synth.VAL_INT).astype(NP_VAL[dt])
+    buf = torch.zeros(A.n + 1, dtype=torch.float64 if dt == "f64" else torch.float32, device="cuda")
+    buf[1:] = torch.from_numpy(x).cuda()
+    xv = buf[1:]
+    assert xv.data_ptr() % 16 != 0
+    ydt = torch.float64 if dt == "f64" else torch.float32
+    y1 = torch.empty(A.m, dtype=ydt, device="cuda")
+    y2 = torch.empty(A.m, dtype=ydt, device="cuda")
+    dasp.dasp_spmv(plan, xv, y1, 1.0, 0.0)
+    dasp.dasp_spmv(plan, torch.from_numpy(x).cuda(), y2, 1.0, 0.0)
+    torch.cuda.synchronize()
+    assert torch.equal(y1, y2)
+    y_ref, _ = oracle_ref(A, x.astype(np.float64), dt)
+    assert np.array_equal(y1.cpu().numpy().astype(np.float64), y_ref)
