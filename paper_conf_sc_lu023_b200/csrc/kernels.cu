@@ -75,6 +75,16 @@
 #ifndef DASP_CHUNK_U2_F32
 #define DASP_CHUNK_U2_F32 0
 #endif
+// 1: wide medium warps (CUDA-core) load the next row-block's metadata with this one's streams
+#ifndef DASP_WIDE_META_PF_F64
+#define DASP_WIDE_META_PF_F64 0
+#endif
+#ifndef DASP_WIDE_META_PF_F16
+#define DASP_WIDE_META_PF_F16 0
+#endif
+#ifndef DASP_WIDE_META_PF_F32
+#define DASP_WIDE_META_PF_F32 0
+#endif
 #ifndef DASP_SHORT_TPW_F64
 #define DASP_SHORT_TPW_F64 2
 #endif
@@ -888,6 +898,23 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
             else medium_rb_f64<DT, VAR>(P, MA, lane, pol);
             rb += st;
         }
+    } else if constexpr (vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_WIDE_META_PF) != 0) {
+        // the next row-block's metadata loads are issued with this row-block's stream loads
+        RbMeta Mn = rb_meta(P, rb0, lane);
+        for (int64_t rb = rb0; rb < rb1; rb += st) {
+            const RbMeta M = Mn;
+            if constexpr (DT == 1) {
+                MedLdH L;
+                medium_load_f16(P, M, lane, pol, L);
+                if (rb + st < rb1) Mn = rb_meta(P, rb + st, lane);
+                medium_finish_f16<VAR>(P, M, L, lane, pol);
+            } else {
+                MedLd<DT> L;
+                medium_load_f64<DT>(P, M, lane, pol, L);
+                if (rb + st < rb1) Mn = rb_meta(P, rb + st, lane);
+                medium_finish_f64<DT, VAR>(P, M, L, lane, pol);
+            }
+        }
     } else {
 #if DASP_EXP_TRACE
         Trace tr;
@@ -1260,6 +1287,16 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 // 1: the next pass's stream loads are issued before this pass's gathers.  Measured
 // (profiles/r01d/narrow_pipe.jsonl): FP16 C3 main kernel -3 %, stencils -1 %; FP64 +6 % (spills at
 // 64 registers), FP32 neutral -- so FP16 only.
+// 1: narrow / mid warps load the next pass's row metadata with this pass's streams
+#ifndef DASP_NARROW_META_PF_F64
+#define DASP_NARROW_META_PF_F64 0
+#endif
+#ifndef DASP_NARROW_META_PF_F16
+#define DASP_NARROW_META_PF_F16 0
+#endif
+#ifndef DASP_NARROW_META_PF_F32
+#define DASP_NARROW_META_PF_F32 0
+#endif
 #ifndef DASP_NARROW_PIPE_F64
 #define DASP_NARROW_PIPE_F64 0
 #endif
@@ -1279,6 +1316,70 @@ template <> struct NarLd<1> {                      // FP16: two octets
     uint32_t c[2][8];
     int32_t orow;
 };
+// a narrow lane's row metadata: regular region start, irregular start / length, output row, nreg
+struct NarMeta {
+    int64_t base, ib;
+    int32_t ilen, orow, nreg;
+};
+template <int DT>
+__device__ __forceinline__ NarMeta narrow_meta(const MainParams& P, int64_t rq, bool act, int g) {
+    if (!act) return NarMeta{0, 0, 0, -1, 0};
+    const int64_t i = rq * 8 + g;
+    const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
+    return NarMeta{base, ib, static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i),
+                   static_cast<int32_t>((__ldg(P.rb_ptr + rq + 1) - base) >> (DT == 1 ? 6 : 5))};
+}
+// stream loads of one lane's row (metadata M; M.orow = -1: inactive) for its groups 2 sub, 2 sub + 1
+template <int DT>
+__device__ __forceinline__ void narrow_load_m(const MainParams& P, const NarMeta& M, int g, int sub, uint64_t pol,
+                                              NarLd<DT>& L) {
+    L.orow = M.orow;
+    const int64_t base = M.base, ib = M.ib;
+    const int ilen = M.ilen, nreg = M.nreg;
+    if constexpr (DT == 1) {
+        const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
+        const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int q = 2 * sub + h;
+            if (q < nreg) {
+                const int64_t off = base + (nreg >= 4 ? 32 * g + 16 * sub + 8 * h : 64 * q + 8 * g);
+                ld4_b32(rv + off, pol, L.v[h]);
+                ld8_b32(P.reg_col + off, pol, L.c[h]);
+            } else {
+                const int k0 = 8 * (q - nreg);
+#pragma unroll
+                for (int e = 0; e < 8; e += 2) {
+                    uint32_t lo = 0, hi = 0;
+                    L.c[h][e] = L.c[h][e + 1] = 0xffffffffu;
+                    if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); L.c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                    if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); L.c[h][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
+                    L.v[h][e >> 1] = lo | (hi << 16);
+                }
+            }
+        }
+    } else {
+        using IO = ValIO<DT>;
+        const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
+        const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int q = 2 * sub + h;
+            if (q < nreg) {
+                const int64_t off = base + (nreg >= 4 ? 16 * g + 8 * sub + 4 * h : 32 * q + 4 * g);
+                IO::ld4r(rv + off, pol, L.v[h]);
+                ld4_b32(P.reg_col + off, pol, L.c[h]);
+            } else {
+                const int k0 = 4 * (q - nreg);
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    L.v[h][e] = 0; L.c[h][e] = 0xffffffffu;
+                    if (k0 + e < ilen) { L.v[h][e] = IO::ld1r(iv + ib + k0 + e, pol); L.c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
+                }
+            }
+        }
+    }
+}
 // stream loads of row g of row-block rq (rq < rbe) for this lane's groups 2 sub, 2 sub + 1
 template <int DT>
 __device__ __forceinline__ void narrow_load(const MainParams& P, int64_t rq, bool act, int g, int sub, uint64_t pol,
@@ -1405,6 +1506,18 @@ __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t gb, i
             narrow_load<DT>(P, rn, ps + 1 < passes && rn < rbe, g, sub, pol, B);
             narrow_finish<DT, VAR, LPR>(P, A, sub);
             A = B;
+        }
+    } else if constexpr (DASP_BY_DT(DT, DASP_NARROW_META_PF) != 0) {
+        // the next pass's metadata loads are issued with this pass's stream loads, so every pass
+        // after the first costs two dependent round trips (streams, gathers) instead of three
+        NarMeta Mn = narrow_meta<DT>(P, r0, r0 < rbe, g);
+        for (int64_t ps = 0; ps < passes; ++ps) {
+            NarLd<DT> A;
+            const NarMeta M = Mn;
+            narrow_load_m<DT>(P, M, g, sub, pol, A);
+            const int64_t rn = r0 + (ps + 1) * step;
+            Mn = narrow_meta<DT>(P, rn, ps + 1 < passes && rn < rbe, g);
+            narrow_finish<DT, VAR, LPR>(P, A, sub);
         }
     } else {
 #if DASP_EXP_TRACE
