@@ -77,7 +77,7 @@
 #endif
 // 1: wide medium warps (CUDA-core) load the next row-block's metadata with this one's streams
 #ifndef DASP_WIDE_META_PF_F64
-#define DASP_WIDE_META_PF_F64 0
+#define DASP_WIDE_META_PF_F64 1   // C2 main -1.8 %, C2+ -3.8 %, C5 -0.7 %, C3 +-0; FP32 C3 +2.6 %, FP16 +-0 (off there; profiles/r02b/meta_prefetch_ab.jsonl)
 #endif
 #ifndef DASP_WIDE_META_PF_F16
 #define DASP_WIDE_META_PF_F16 0
@@ -898,7 +898,7 @@ __device__ __forceinline__ void medium_rbs(const MainParams& P, int64_t rb0, int
             else medium_rb_f64<DT, VAR>(P, MA, lane, pol);
             rb += st;
         }
-    } else if constexpr (vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_WIDE_META_PF) != 0) {
+    } else if constexpr (vk(VAR) == VAR_CUDACORE && !vst(VAR) && DASP_BY_DT(DT, DASP_WIDE_META_PF) != 0) {
         // the next row-block's metadata loads are issued with this row-block's stream loads
         RbMeta Mn = rb_meta(P, rb0, lane);
         for (int64_t rb = rb0; rb < rb1; rb += st) {

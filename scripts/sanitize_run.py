@@ -1,6 +1,6 @@
 """Workload for compute-sanitizer (scripts/sanitize.sh): every row class on small matrices, both
 compute variants, all three dtypes, beta = 0 and beta != 0, the scatter epilogue, the host-buffer
-calls and the device builder.  Checks results against the oracle so a silent corruption fails too."""
+calls, the device builder and the x-window staging instantiation.  Checks results against the oracle so a silent corruption fails too."""
 import os
 import sys
 
@@ -48,6 +48,24 @@ def main():
                 assert np.array_equal(dasp.dasp_plan_copy_array(dplan, arr), dasp.dasp_plan_copy_array(plan, arr)), arr
             dplan.destroy()
             plan.destroy()
+    # x-window staging instantiation (cp.async.bulk + mbarrier): stencil blocks, FP64 / FP32
+    A = synth.generate(synth.config("c2", scale=0.25))
+    x = synth.vector(5, A.n)
+    for dt in ("f64", "f32"):
+        val = A.val.astype(NP[dt])
+        xv = x.astype(NP[dt])
+        st = dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dt, device=0, x_stage=2)
+        pl = dasp.dasp_plan_create(A.row_ptr, A.col, val, A.m, A.n, dt, device=0, x_stage=1)
+        assert st.info["x_stage_blocks"] > 0
+        xd = torch.from_numpy(xv).cuda()
+        ydt = torch.float64 if dt == "f64" else torch.float32
+        ys, yp = torch.zeros(A.m, dtype=ydt, device="cuda"), torch.zeros(A.m, dtype=ydt, device="cuda")
+        dasp.dasp_spmv(st, xd, ys, 1.0, 0.0)
+        dasp.dasp_spmv(pl, xd, yp, 1.0, 0.0)
+        torch.cuda.synchronize()
+        assert torch.equal(ys, yp), dt
+        st.destroy()
+        pl.destroy()
     torch.cuda.synchronize()
     torch.cuda.empty_cache()   # torch's caching allocator keeps its blocks otherwise (reported as leaks)
     print("sanitize workload ok")
