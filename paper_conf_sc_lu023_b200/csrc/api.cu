@@ -76,7 +76,7 @@ int sa(int dtype) { return dtype == DASP_R_16F ? 4 : 8; }   // long-group partia
 // ~50 MB of L2 that data shared by all SMs gets on B200 (profiles/r01 L2 probe)
 constexpr int64_t kAutoPanelRows = int64_t(1) << 20;
 #ifndef DASP_COL_BUCKETS
-#define DASP_COL_BUCKETS 16
+#define DASP_COL_BUCKETS 256   // long-unit column buckets: C3 FP16 long -2.6 %, C5 -1.1 %, C7 -1.7 %, C3 FP64 -0.5 % vs 16 (profiles/r02b/long_col_buckets.jsonl)
 #endif
 #ifndef DASP_LONG_ORDER
 #define DASP_LONG_ORDER 2   // long-unit schedule: 0 memory order, 1 column buckets per panel, 2 global buckets (C3 long -6 %, profiles/r02/long_order.jsonl)
