@@ -66,6 +66,16 @@
 #ifndef DASP_PEEL_F16
 #define DASP_PEEL_F16 0
 #endif
+//   PEEL_U2   : with PEEL, chunks 1.. two per load / gather round trip
+#ifndef DASP_PEEL_U2_F64
+#define DASP_PEEL_U2_F64 0
+#endif
+#ifndef DASP_PEEL_U2_F32
+#define DASP_PEEL_U2_F32 0
+#endif
+#ifndef DASP_PEEL_U2_F16
+#define DASP_PEEL_U2_F16 0
+#endif
 #ifndef DASP_CHUNK_U2_F64
 #define DASP_CHUNK_U2_F64 0
 #endif
@@ -620,7 +630,28 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
             for (int j = 0; j < 3; ++j)
                 if (j < rem) part = fma(IO::cv(L.vr[j]), xr[j], part);
             part = fma(IO::cv(L.vi), xi, part);
-            for (int ch = 1; ch < nfull; ++ch) {
+            int ch = 1;
+            if constexpr (DASP_BY_DT(DT, DASP_PEEL_U2) != 0) {
+                // chunks 1.. two per round trip (both chunks' streams, then both chunks' gathers)
+                for (; ch + 1 < nfull; ch += 2) {
+                    typename IO::R va[4], vb[4];
+                    uint32_t ca[4], cb[4];
+                    IO::ld4r(rv + ch * 128 + lane * 4, pol, va);
+                    ld4_b32(rc + ch * 128 + lane * 4, pol, ca);
+                    IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vb);
+                    ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cb);
+                    double xa[4], xb[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) xa[j] = G(ca[j]);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) xb[j] = G(cb[j]);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xa[j], part);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) part = fma(IO::cv(vb[j]), xb[j], part);
+                }
+            }
+            for (; ch < nfull; ++ch) {
                 typename IO::R va[4];
                 uint32_t ca[4];
                 IO::ld4r(rv + ch * 128 + lane * 4, pol, va);
@@ -1180,11 +1211,47 @@ __device__ __forceinline__ void empty_row(void* yv, int32_t row, double beta, co
         for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[row] = r;
 }
 // finish warp fw of the fused main kernel: long rows 4fw..4fw+3, or empty rows (4 per lane)
+// a row of more than kHugeGroups groups is summed by the whole warp (32 lanes, 8 accumulators each:
+// 256 partials per round) instead of 8 lanes with 4 (32 per round): a row of 10^5 nonzeros (1563
+// groups) takes 7 dependent rounds instead of 49, a row of 10^7 610 instead of 4883.  Lane l sums
+// partials g0 + l + 32 j into accumulator j mod 8, then (a0+a1)+(a2+a3) ... and a 5-step shuffle
+// tree: a fixed order, deterministic.
+constexpr int64_t kHugeGroups = 128;
+template <int DT>
+__device__ __forceinline__ typename Tr<DT>::A long_row_sum_warp(const void* partial, int64_t g0, int64_t g1, int lane) {
+    using A = typename Tr<DT>::A;
+    const A* part = static_cast<const A*>(partial);
+    A a[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) a[j] = 0;
+    int64_t k = g0 + lane;
+    for (; k + 7 * 32 < g1; k += 8 * 32) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) a[j] += part[k + 32 * j];
+    }
+    for (int j = 0; k < g1; k += 32, ++j) a[j & 7] += part[k];
+    A s = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+    return s;
+}
 template <int DT, int VAR>
 __device__ __forceinline__ void finish_warp(const MainParams& P, int64_t fw, int lane) {
     const int64_t lw = (P.row_long + 3) / 4;
     if (fw < lw) {
         const int64_t r = fw * 4 + (lane >> 3);
+        // the warp's 4 rows: any huge one?  (lane 8q reads row q's range; warp-uniform vote)
+        bool huge = false;
+        if ((lane & 7) == 0 && r < P.row_long) huge = __ldg(P.group_ptr + r + 1) - __ldg(P.group_ptr + r) > kHugeGroups;
+        if (__any_sync(FULL, huge)) {
+            for (int q = 0; q < 4; ++q) {
+                const int64_t rq = fw * 4 + q;
+                if (rq >= P.row_long) break;
+                const auto s = long_row_sum_warp<DT>(P.partial, __ldg(P.group_ptr + rq), __ldg(P.group_ptr + rq + 1), lane);
+                if (lane == 0) store_y<DT, VAR>(P, __ldg(P.long_out + rq), s);
+            }
+            return;
+        }
         const auto s = long_row_sum<DT>(P.partial, P.group_ptr, r, P.row_long, lane);
         if ((lane & 7) == 0 && r < P.row_long) store_y<DT, VAR>(P, __ldg(P.long_out + r), s);
         return;
