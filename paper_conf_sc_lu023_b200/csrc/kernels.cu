@@ -95,6 +95,16 @@
 #ifndef DASP_WIDE_META_PF_F32
 #define DASP_WIDE_META_PF_F32 0
 #endif
+// 1: short tiles gather x by cp.async into shared memory (register-free gathers), FP64 / FP32
+#ifndef DASP_SHORT_ASYNC_F64
+#define DASP_SHORT_ASYNC_F64 0
+#endif
+#ifndef DASP_SHORT_ASYNC_F32
+#define DASP_SHORT_ASYNC_F32 0
+#endif
+#ifndef DASP_SHORT_ASYNC_F16
+#define DASP_SHORT_ASYNC_F16 0
+#endif
 #ifndef DASP_SHORT_TPW_F64
 #define DASP_SHORT_TPW_F64 2
 #endif
@@ -1273,7 +1283,8 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
     const int tpw = (DT == 1 && !vo(VAR)) ? P.tpw : TPW;   // only FP16 layouts vary (main_occ5)
     const int64_t t0 = ws * tpw;
     if (t0 >= nt || !(P.class_mask & 4)) return;
-    if constexpr (TPW > 2) {   // generic: every tile's loads, then every tile's gathers, then the math
+    constexpr bool ASYNC = DT != 1 && DASP_BY_DT(DT, DASP_SHORT_ASYNC) != 0 && !vo(VAR);
+    if constexpr (TPW > 2 || ASYNC) {   // generic: every tile's loads, then every tile's gathers, then the math
         ShortRef R[TPW];
         const int64_t te = min(t0 + tpw, nt);           // this warp's tiles [t0, te)
 #pragma unroll
@@ -1287,6 +1298,42 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
             for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_gather_f16(P, L[k], xh[k]);
 #pragma unroll
             for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_math_f16<VAR>(P, R[k].cat, L[k], xh[k], lane);
+        } else if constexpr (ASYNC) {
+            // register-free gathers: each lane's x values go to a per-warp shared buffer by 4/8-byte
+            // cp.async (LDGSTS; a pad column copies 0 bytes = zero fill), so during the gather round trip
+            // the warp holds only the values and the output map in registers
+            using X = typename Tr<DT>::X;
+            __shared__ X s_xg[WARPS_PER_BLOCK][TPW * 4][32];
+            const int wib = threadIdx.x >> 5;
+            const X* x = static_cast<const X*>(P.x);
+            ShortLd<DT> L[TPW];
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_load_f64<DT>(P, R[k], lane, pol, L[k]);
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) {
+                if (t0 + k < te) {
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int32_t c = static_cast<int32_t>(L[k].c[j]);
+                        const uint32_t dst = smem_u32(&s_xg[wib][k * 4 + j][lane]);
+                        asm volatile("cp.async.ca.shared.global [%0], [%1], %2, %3;"
+                                     ::"r"(dst), "l"(x + (c >= 0 ? c : 0)), "n"(static_cast<int>(sizeof(X))),
+                                       "r"(c >= 0 ? static_cast<int>(sizeof(X)) : 0)
+                                     : "memory");
+                    }
+                }
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+#pragma unroll
+            for (int k = 0; k < TPW; ++k) {
+                if (t0 + k < te) {
+                    double xv[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) xv[j] = static_cast<double>(s_xg[wib][k * 4 + j][lane]);
+                    short_math_f64<DT, VAR>(P, R[k].cat, L[k], xv, lane);
+                }
+            }
         } else {
             ShortLd<DT> L[TPW];
             double xv[TPW][4];
