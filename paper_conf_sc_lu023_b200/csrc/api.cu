@@ -348,6 +348,13 @@ int64_t build_stage_table(const HostFormat& f, const std::vector<uint64_t>& warp
     return staged;
 }
 
+// mid (two-lanes-per-row) row-blocks: rows spanning at most mid_max_slots(K) slots; experiment knob
+// DASP_MID_MUL_F16 (FP16, K = 8): the multiple of K up to which row-blocks go to the mid path
+#ifndef DASP_MID_MUL_F16
+#define DASP_MID_MUL_F16 4
+#endif
+inline int mid_slots(int K) { return K == 8 ? DASP_MID_MUL_F16 * K : dasp::mid_max_slots(K); }
+
 dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_t* panel_table,
                            const std::vector<int32_t>& unit_first_col, const std::vector<int32_t>& nslots) {
     HostFormat& f = p->host;
@@ -374,7 +381,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
         const int64_t* e = panel_table + q * dasp::PANEL_FIELDS;
         int64_t rbm = e[5];
         if (nrw > 0)
-            while (rbm > 0 && nslots[e[4] + rbm - 1] <= dasp::mid_max_slots(f.geo.K)) --rbm;
+            while (rbm > 0 && nslots[e[4] + rbm - 1] <= mid_slots(f.geo.K)) --rbm;
         wide_rbs += rbm;
     }
     p->occ5 = p->dtype == DASP_R_16F && p->variant == DASP_VARIANT_CUDACORE && 4 * wide_rbs <= f.nrb;
@@ -389,7 +396,7 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
             while (d.rbn > 0 && nslots[d.rb0 + d.rbn - 1] <= dasp::narrow_max_slots(f.geo.K)) --d.rbn;
         d.rbm = d.rbn;
         if (nrw > 0)
-            while (d.rbm > 0 && nslots[d.rb0 + d.rbm - 1] <= dasp::mid_max_slots(f.geo.K)) --d.rbm;
+            while (d.rbm > 0 && nslots[d.rb0 + d.rbm - 1] <= mid_slots(f.geo.K)) --d.rbm;
         d.nmwd = (d.rbm + p->rbw - 1) / p->rbw;
         d.nmwm = d.nmwd + (nrw > 0 ? (d.rbn - d.rbm + nrw - 1) / nrw : 0);
         d.nmw = d.nmwm + (nrw > 0 ? (d.nrb - d.rbn + nrw - 1) / nrw : 0);
