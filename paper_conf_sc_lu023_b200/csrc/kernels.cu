@@ -66,6 +66,16 @@
 #ifndef DASP_PEEL_F16
 #define DASP_PEEL_F16 0
 #endif
+//   PEEL_PIPE : with PEEL, chunk ch+1's streams issued with chunk ch's gathers
+#ifndef DASP_PEEL_PIPE_F64
+#define DASP_PEEL_PIPE_F64 0
+#endif
+#ifndef DASP_PEEL_PIPE_F32
+#define DASP_PEEL_PIPE_F32 0
+#endif
+#ifndef DASP_PEEL_PIPE_F16
+#define DASP_PEEL_PIPE_F16 0
+#endif
 //   PEEL_U2   : with PEEL, chunks 1.. two per load / gather round trip
 #ifndef DASP_PEEL_U2_F64
 #define DASP_PEEL_U2_F64 0
@@ -634,6 +644,41 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
 #pragma unroll
             for (int j = 0; j < 3; ++j) xr[j] = G(L.cr[j]);
             const double xi = G(L.ci);
+            if constexpr (DASP_BY_DT(DT, DASP_PEEL_PIPE) != 0) {
+                // software pipeline: chunk ch+1's streams are issued while chunk ch's gathers are
+                // in flight (chunk 1's with the first round's gathers), one round trip per chunk
+                typename IO::R vn[4];
+                uint32_t cn[4];
+                if (DASP_BY_DT(DT, DASP_PEEL_PIPE) == 1 && nfull > 1) {
+                    IO::ld4r(rv + 128 + lane * 4, pol, vn);
+                    ld4_b32(rc + 128 + lane * 4, pol, cn);
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) part = fma(IO::cv(L.va[j]), xa[j], part);
+#pragma unroll
+                for (int j = 0; j < 3; ++j)
+                    if (j < rem) part = fma(IO::cv(L.vr[j]), xr[j], part);
+                part = fma(IO::cv(L.vi), xi, part);
+                if (DASP_BY_DT(DT, DASP_PEEL_PIPE) == 2 && nfull > 1) {   // 2: chunk 1 after the first round
+                    IO::ld4r(rv + 128 + lane * 4, pol, vn);
+                    ld4_b32(rc + 128 + lane * 4, pol, cn);
+                }
+                for (int ch = 1; ch < nfull; ++ch) {
+                    typename IO::R va[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) va[j] = vn[j];
+                    double xv[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) xv[j] = G(cn[j]);
+                    if (ch + 1 < nfull) {
+                        IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vn);
+                        ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cn);
+                    }
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xv[j], part);
+                }
+                goto peel_done;
+            }
 #pragma unroll
             for (int j = 0; j < 4; ++j) part = fma(IO::cv(L.va[j]), xa[j], part);
 #pragma unroll
@@ -675,6 +720,7 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
         } else {
             ragged_irr();
         }
+    peel_done:;
     } else if constexpr (FULL && vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_CHUNK_U2) != 0) {
         // two chunks per round trip: chunk ch+1's stream loads are issued together with chunk ch's
         // (ch > 0), then the 8 gathers, then 8 FMAs in slot order (the same per-lane order as one
