@@ -45,7 +45,6 @@
 #ifndef DASP_CHUNK_PIPE_F32
 #define DASP_CHUNK_PIPE_F32 0
 #endif
-//   CHUNK_U2  : CUDA-core wide medium path: two 4-block chunks per load / gather round trip
 //   RAGGED_FIRST: CUDA-core wide medium path: ragged chunk + first irregular element accumulated first
 #ifndef DASP_RAGGED_FIRST_F64
 #define DASP_RAGGED_FIRST_F64 0
@@ -66,35 +65,6 @@
 #ifndef DASP_PEEL_F16
 #define DASP_PEEL_F16 0
 #endif
-//   PEEL_PIPE : with PEEL, chunk ch+1's streams issued with chunk ch's gathers
-#ifndef DASP_PEEL_PIPE_F64
-#define DASP_PEEL_PIPE_F64 0
-#endif
-#ifndef DASP_PEEL_PIPE_F32
-#define DASP_PEEL_PIPE_F32 0
-#endif
-#ifndef DASP_PEEL_PIPE_F16
-#define DASP_PEEL_PIPE_F16 0
-#endif
-//   PEEL_U2   : with PEEL, chunks 1.. two per load / gather round trip
-#ifndef DASP_PEEL_U2_F64
-#define DASP_PEEL_U2_F64 0
-#endif
-#ifndef DASP_PEEL_U2_F32
-#define DASP_PEEL_U2_F32 0
-#endif
-#ifndef DASP_PEEL_U2_F16
-#define DASP_PEEL_U2_F16 0
-#endif
-#ifndef DASP_CHUNK_U2_F64
-#define DASP_CHUNK_U2_F64 0
-#endif
-#ifndef DASP_CHUNK_U2_F16
-#define DASP_CHUNK_U2_F16 0
-#endif
-#ifndef DASP_CHUNK_U2_F32
-#define DASP_CHUNK_U2_F32 0
-#endif
 // 1: wide medium warps (CUDA-core) load the next row-block's metadata with this one's streams
 #ifndef DASP_WIDE_META_PF_F64
 #define DASP_WIDE_META_PF_F64 1   // C2 main -1.8 %, C2+ -3.8 %, C5 -0.7 %, C3 +-0; FP32 C3 +2.6 %, FP16 +-0 (off there; profiles/r02b/meta_prefetch_ab.jsonl)
@@ -104,16 +74,6 @@
 #endif
 #ifndef DASP_WIDE_META_PF_F32
 #define DASP_WIDE_META_PF_F32 0
-#endif
-// 1: short tiles gather x by cp.async into shared memory (register-free gathers), FP64 / FP32
-#ifndef DASP_SHORT_ASYNC_F64
-#define DASP_SHORT_ASYNC_F64 0
-#endif
-#ifndef DASP_SHORT_ASYNC_F32
-#define DASP_SHORT_ASYNC_F32 0
-#endif
-#ifndef DASP_SHORT_ASYNC_F16
-#define DASP_SHORT_ASYNC_F16 0
 #endif
 #ifndef DASP_SHORT_TPW_F64
 #define DASP_SHORT_TPW_F64 2
@@ -644,69 +604,13 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
 #pragma unroll
             for (int j = 0; j < 3; ++j) xr[j] = G(L.cr[j]);
             const double xi = G(L.ci);
-            if constexpr (DASP_BY_DT(DT, DASP_PEEL_PIPE) != 0) {
-                // software pipeline: chunk ch+1's streams are issued while chunk ch's gathers are
-                // in flight (chunk 1's with the first round's gathers), one round trip per chunk
-                typename IO::R vn[4];
-                uint32_t cn[4];
-                if (DASP_BY_DT(DT, DASP_PEEL_PIPE) == 1 && nfull > 1) {
-                    IO::ld4r(rv + 128 + lane * 4, pol, vn);
-                    ld4_b32(rc + 128 + lane * 4, pol, cn);
-                }
-#pragma unroll
-                for (int j = 0; j < 4; ++j) part = fma(IO::cv(L.va[j]), xa[j], part);
-#pragma unroll
-                for (int j = 0; j < 3; ++j)
-                    if (j < rem) part = fma(IO::cv(L.vr[j]), xr[j], part);
-                part = fma(IO::cv(L.vi), xi, part);
-                if (DASP_BY_DT(DT, DASP_PEEL_PIPE) == 2 && nfull > 1) {   // 2: chunk 1 after the first round
-                    IO::ld4r(rv + 128 + lane * 4, pol, vn);
-                    ld4_b32(rc + 128 + lane * 4, pol, cn);
-                }
-                for (int ch = 1; ch < nfull; ++ch) {
-                    typename IO::R va[4];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) va[j] = vn[j];
-                    double xv[4];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) xv[j] = G(cn[j]);
-                    if (ch + 1 < nfull) {
-                        IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vn);
-                        ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cn);
-                    }
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xv[j], part);
-                }
-                goto peel_done;
-            }
 #pragma unroll
             for (int j = 0; j < 4; ++j) part = fma(IO::cv(L.va[j]), xa[j], part);
 #pragma unroll
             for (int j = 0; j < 3; ++j)
                 if (j < rem) part = fma(IO::cv(L.vr[j]), xr[j], part);
             part = fma(IO::cv(L.vi), xi, part);
-            int ch = 1;
-            if constexpr (DASP_BY_DT(DT, DASP_PEEL_U2) != 0) {
-                // chunks 1.. two per round trip (both chunks' streams, then both chunks' gathers)
-                for (; ch + 1 < nfull; ch += 2) {
-                    typename IO::R va[4], vb[4];
-                    uint32_t ca[4], cb[4];
-                    IO::ld4r(rv + ch * 128 + lane * 4, pol, va);
-                    ld4_b32(rc + ch * 128 + lane * 4, pol, ca);
-                    IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vb);
-                    ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cb);
-                    double xa[4], xb[4];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) xa[j] = G(ca[j]);
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) xb[j] = G(cb[j]);
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xa[j], part);
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) part = fma(IO::cv(vb[j]), xb[j], part);
-                }
-            }
-            for (; ch < nfull; ++ch) {
+            for (int ch = 1; ch < nfull; ++ch) {
                 typename IO::R va[4];
                 uint32_t ca[4];
                 IO::ld4r(rv + ch * 128 + lane * 4, pol, va);
@@ -719,33 +623,6 @@ __device__ __forceinline__ void medium_finish_f64(const MainParams& P, const RbM
             }
         } else {
             ragged_irr();
-        }
-    peel_done:;
-    } else if constexpr (FULL && vk(VAR) == VAR_CUDACORE && DASP_BY_DT(DT, DASP_CHUNK_U2) != 0) {
-        // two chunks per round trip: chunk ch+1's stream loads are issued together with chunk ch's
-        // (ch > 0), then the 8 gathers, then 8 FMAs in slot order (the same per-lane order as one
-        // chunk at a time, so the result is bitwise unchanged)
-        typename IO::R va[4], vb[4];
-        uint32_t ca[4], cb[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) { va[j] = L.va[j]; ca[j] = L.ca[j]; }
-        for (int ch = 0; ch < nfull; ch += 2) {
-            if (ch > 0) { IO::ld4r(rv + ch * 128 + lane * 4, pol, va); ld4_b32(rc + ch * 128 + lane * 4, pol, ca); }
-            const bool two = ch + 1 < nfull;                   // warp-uniform
-#pragma unroll
-            for (int j = 0; j < 4; ++j) { vb[j] = 0; cb[j] = 0xffffffffu; }
-            if (two) { IO::ld4r(rv + (ch + 1) * 128 + lane * 4, pol, vb); ld4_b32(rc + (ch + 1) * 128 + lane * 4, pol, cb); }
-            double xa[4], xb[4];
-#pragma unroll
-            for (int j = 0; j < 4; ++j) xa[j] = G(ca[j]);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) xb[j] = G(cb[j]);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) part = fma(IO::cv(va[j]), xa[j], part);
-            if (two) {
-#pragma unroll
-                for (int j = 0; j < 4; ++j) part = fma(IO::cv(vb[j]), xb[j], part);
-            }
         }
     } else if constexpr (FULL) {
         typename IO::R va[4];
@@ -839,7 +716,7 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
         }
     };
     auto block = [&](uint32_t a, uint32_t ca, uint32_t cb) { blockx(a, GH(ca), GH(cb)); };
-    // CUDA-core RAGGED_FIRST / CHUNK_U2: as in medium_finish_f64
+    // CUDA-core RAGGED_FIRST: as in medium_finish_f64
     constexpr bool RF = vk(VAR) == VAR_CUDACORE && DASP_RAGGED_FIRST_F16 != 0;
     auto ragged_irr = [&]() {
 #pragma unroll
@@ -879,32 +756,6 @@ __device__ __forceinline__ void medium_finish_f16(const MainParams& P, const RbM
             }
         } else {
             ragged_irr();
-        }
-    } else if constexpr (FULL && vk(VAR) == VAR_CUDACORE && DASP_CHUNK_U2_F16 != 0) {
-        uint32_t va[4], ca[8], vb[4], cb[8];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) va[j] = L.va[j];
-#pragma unroll
-        for (int e = 0; e < 8; ++e) ca[e] = L.ca[e];
-        for (int ch = 0; ch < nfull; ch += 2) {
-            if (ch > 0) { ld4_b32(rv + ch * 256 + lane * 8, pol, va); ld8_b32(rc + ch * 256 + lane * 8, pol, ca); }
-            const bool two = ch + 1 < nfull;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) vb[j] = 0u;
-#pragma unroll
-            for (int e = 0; e < 8; ++e) cb[e] = 0xffffffffu;
-            if (two) { ld4_b32(rv + (ch + 1) * 256 + lane * 8, pol, vb); ld8_b32(rc + (ch + 1) * 256 + lane * 8, pol, cb); }
-            uint16_t xa[8], xb[8];
-#pragma unroll
-            for (int e = 0; e < 8; ++e) xa[e] = GH(ca[e]);
-#pragma unroll
-            for (int e = 0; e < 8; ++e) xb[e] = GH(cb[e]);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) blockx(va[j], xa[2 * j], xa[2 * j + 1]);
-            if (two) {
-#pragma unroll
-                for (int j = 0; j < 4; ++j) blockx(vb[j], xb[2 * j], xb[2 * j + 1]);
-            }
         }
     } else if constexpr (FULL) {
         uint32_t va[4], ca[8];
@@ -1329,8 +1180,7 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
     const int tpw = (DT == 1 && !vo(VAR)) ? P.tpw : TPW;   // only FP16 layouts vary (main_occ5)
     const int64_t t0 = ws * tpw;
     if (t0 >= nt || !(P.class_mask & 4)) return;
-    constexpr bool ASYNC = DT != 1 && DASP_BY_DT(DT, DASP_SHORT_ASYNC) != 0 && !vo(VAR);
-    if constexpr (TPW > 2 || ASYNC) {   // generic: every tile's loads, then every tile's gathers, then the math
+    if constexpr (TPW > 2) {   // generic: every tile's loads, then every tile's gathers, then the math
         ShortRef R[TPW];
         const int64_t te = min(t0 + tpw, nt);           // this warp's tiles [t0, te)
 #pragma unroll
@@ -1344,42 +1194,6 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
             for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_gather_f16(P, L[k], xh[k]);
 #pragma unroll
             for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_math_f16<VAR>(P, R[k].cat, L[k], xh[k], lane);
-        } else if constexpr (ASYNC) {
-            // register-free gathers: each lane's x values go to a per-warp shared buffer by 4/8-byte
-            // cp.async (LDGSTS; a pad column copies 0 bytes = zero fill), so during the gather round trip
-            // the warp holds only the values and the output map in registers
-            using X = typename Tr<DT>::X;
-            __shared__ X s_xg[WARPS_PER_BLOCK][TPW * 4][32];
-            const int wib = threadIdx.x >> 5;
-            const X* x = static_cast<const X*>(P.x);
-            ShortLd<DT> L[TPW];
-#pragma unroll
-            for (int k = 0; k < TPW; ++k) if (t0 + k < te) short_load_f64<DT>(P, R[k], lane, pol, L[k]);
-#pragma unroll
-            for (int k = 0; k < TPW; ++k) {
-                if (t0 + k < te) {
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int32_t c = static_cast<int32_t>(L[k].c[j]);
-                        const uint32_t dst = smem_u32(&s_xg[wib][k * 4 + j][lane]);
-                        asm volatile("cp.async.ca.shared.global [%0], [%1], %2, %3;"
-                                     ::"r"(dst), "l"(x + (c >= 0 ? c : 0)), "n"(static_cast<int>(sizeof(X))),
-                                       "r"(c >= 0 ? static_cast<int>(sizeof(X)) : 0)
-                                     : "memory");
-                    }
-                }
-            }
-            asm volatile("cp.async.commit_group;" ::: "memory");
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-#pragma unroll
-            for (int k = 0; k < TPW; ++k) {
-                if (t0 + k < te) {
-                    double xv[4];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) xv[j] = static_cast<double>(s_xg[wib][k * 4 + j][lane]);
-                    short_math_f64<DT, VAR>(P, R[k].cat, L[k], xv, lane);
-                }
-            }
         } else {
             ShortLd<DT> L[TPW];
             double xv[TPW][4];
@@ -1447,16 +1261,6 @@ __device__ __forceinline__ void short_item(const MainParams& P, const PanelDesc*
 // 1: the next pass's stream loads are issued before this pass's gathers.  Measured
 // (profiles/r01d/narrow_pipe.jsonl): FP16 C3 main kernel -3 %, stencils -1 %; FP64 +6 % (spills at
 // 64 registers), FP32 neutral -- so FP16 only.
-// 1: narrow / mid warps load the next pass's row metadata with this pass's streams
-#ifndef DASP_NARROW_META_PF_F64
-#define DASP_NARROW_META_PF_F64 0
-#endif
-#ifndef DASP_NARROW_META_PF_F16
-#define DASP_NARROW_META_PF_F16 0
-#endif
-#ifndef DASP_NARROW_META_PF_F32
-#define DASP_NARROW_META_PF_F32 0
-#endif
 #ifndef DASP_NARROW_PIPE_F64
 #define DASP_NARROW_PIPE_F64 0
 #endif
@@ -1476,70 +1280,6 @@ template <> struct NarLd<1> {                      // FP16: two octets
     uint32_t c[2][8];
     int32_t orow;
 };
-// a narrow lane's row metadata: regular region start, irregular start / length, output row, nreg
-struct NarMeta {
-    int64_t base, ib;
-    int32_t ilen, orow, nreg;
-};
-template <int DT>
-__device__ __forceinline__ NarMeta narrow_meta(const MainParams& P, int64_t rq, bool act, int g) {
-    if (!act) return NarMeta{0, 0, 0, -1, 0};
-    const int64_t i = rq * 8 + g;
-    const int64_t base = __ldg(P.rb_ptr + rq), ib = __ldg(P.irr_ptr + i);
-    return NarMeta{base, ib, static_cast<int32_t>(__ldg(P.irr_ptr + i + 1) - ib), __ldg(P.med_out + i),
-                   static_cast<int32_t>((__ldg(P.rb_ptr + rq + 1) - base) >> (DT == 1 ? 6 : 5))};
-}
-// stream loads of one lane's row (metadata M; M.orow = -1: inactive) for its groups 2 sub, 2 sub + 1
-template <int DT>
-__device__ __forceinline__ void narrow_load_m(const MainParams& P, const NarMeta& M, int g, int sub, uint64_t pol,
-                                              NarLd<DT>& L) {
-    L.orow = M.orow;
-    const int64_t base = M.base, ib = M.ib;
-    const int ilen = M.ilen, nreg = M.nreg;
-    if constexpr (DT == 1) {
-        const uint16_t* rv = static_cast<const uint16_t*>(P.reg_val);
-        const unsigned short* iv = static_cast<const unsigned short*>(P.irr_val);
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const int q = 2 * sub + h;
-            if (q < nreg) {
-                const int64_t off = base + (nreg >= 4 ? 32 * g + 16 * sub + 8 * h : 64 * q + 8 * g);
-                ld4_b32(rv + off, pol, L.v[h]);
-                ld8_b32(P.reg_col + off, pol, L.c[h]);
-            } else {
-                const int k0 = 8 * (q - nreg);
-#pragma unroll
-                for (int e = 0; e < 8; e += 2) {
-                    uint32_t lo = 0, hi = 0;
-                    L.c[h][e] = L.c[h][e + 1] = 0xffffffffu;
-                    if (k0 + e < ilen) { lo = __ldg(iv + ib + k0 + e); L.c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
-                    if (k0 + e + 1 < ilen) { hi = __ldg(iv + ib + k0 + e + 1); L.c[h][e + 1] = ld1_b32(P.irr_col + ib + k0 + e + 1, pol); }
-                    L.v[h][e >> 1] = lo | (hi << 16);
-                }
-            }
-        }
-    } else {
-        using IO = ValIO<DT>;
-        const typename IO::T* rv = static_cast<const typename IO::T*>(P.reg_val);
-        const typename IO::T* iv = static_cast<const typename IO::T*>(P.irr_val);
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const int q = 2 * sub + h;
-            if (q < nreg) {
-                const int64_t off = base + (nreg >= 4 ? 16 * g + 8 * sub + 4 * h : 32 * q + 4 * g);
-                IO::ld4r(rv + off, pol, L.v[h]);
-                ld4_b32(P.reg_col + off, pol, L.c[h]);
-            } else {
-                const int k0 = 4 * (q - nreg);
-#pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                    L.v[h][e] = 0; L.c[h][e] = 0xffffffffu;
-                    if (k0 + e < ilen) { L.v[h][e] = IO::ld1r(iv + ib + k0 + e, pol); L.c[h][e] = ld1_b32(P.irr_col + ib + k0 + e, pol); }
-                }
-            }
-        }
-    }
-}
 // stream loads of row g of row-block rq (rq < rbe) for this lane's groups 2 sub, 2 sub + 1
 template <int DT>
 __device__ __forceinline__ void narrow_load(const MainParams& P, int64_t rq, bool act, int g, int sub, uint64_t pol,
@@ -1666,18 +1406,6 @@ __device__ __forceinline__ void medium_narrow(const MainParams& P, int64_t gb, i
             narrow_load<DT>(P, rn, ps + 1 < passes && rn < rbe, g, sub, pol, B);
             narrow_finish<DT, VAR, LPR>(P, A, sub);
             A = B;
-        }
-    } else if constexpr (DASP_BY_DT(DT, DASP_NARROW_META_PF) != 0) {
-        // the next pass's metadata loads are issued with this pass's stream loads, so every pass
-        // after the first costs two dependent round trips (streams, gathers) instead of three
-        NarMeta Mn = narrow_meta<DT>(P, r0, r0 < rbe, g);
-        for (int64_t ps = 0; ps < passes; ++ps) {
-            NarLd<DT> A;
-            const NarMeta M = Mn;
-            narrow_load_m<DT>(P, M, g, sub, pol, A);
-            const int64_t rn = r0 + (ps + 1) * step;
-            Mn = narrow_meta<DT>(P, rn, ps + 1 < passes && rn < rbe, g);
-            narrow_finish<DT, VAR, LPR>(P, A, sub);
         }
     } else {
 #if DASP_EXP_TRACE
