@@ -1118,29 +1118,34 @@ __device__ __forceinline__ void empty_row(void* yv, int32_t row, double beta, co
         for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[row] = r;
 }
 // finish warp fw of the fused main kernel: long rows 4fw..4fw+3, or empty rows (4 per lane)
-// a row of more than kHugeGroups groups is summed by the whole warp (32 lanes, 8 accumulators each:
-// 256 partials per round) instead of 8 lanes with 4 (32 per round): a row of 10^5 nonzeros (1563
-// groups) takes 7 dependent rounds instead of 49, a row of 10^7 610 instead of 4883.  Lane l sums
-// partials g0 + l + 32 j into accumulator j mod 8, then (a0+a1)+(a2+a3) ... and a 5-step shuffle
-// tree: a fixed order, deterministic.
+// a row of more than kHugeGroups groups is summed by the whole warp (32 lanes, 4 accumulators each:
+// 128 partials per round) instead of 8 lanes with 4 (32 per round): a row of 10^5 nonzeros (1563
+// groups) takes 13 dependent rounds instead of 49, a row of 10^7 1221 instead of 4883.  Lane l sums
+// partials g0 + l + 32 j into accumulator j mod 4 while 4 more remain, the rest into accumulator 0,
+// then (a0+a1)+(a2+a3) and a 5-step shuffle tree: a fixed order, deterministic.
 constexpr int64_t kHugeGroups = 128;
 template <int DT>
 __device__ __forceinline__ typename Tr<DT>::A long_row_sum_warp(const void* partial, int64_t g0, int64_t g1, int lane) {
     using A = typename Tr<DT>::A;
     const A* part = static_cast<const A*>(partial);
-    A a[8];
-#pragma unroll
-    for (int j = 0; j < 8; ++j) a[j] = 0;
+    A a0 = 0, a1 = 0, a2 = 0, a3 = 0;
     int64_t k = g0 + lane;
-    for (; k + 7 * 32 < g1; k += 8 * 32) {
-#pragma unroll
-        for (int j = 0; j < 8; ++j) a[j] += part[k + 32 * j];
-    }
-    for (int j = 0; k < g1; k += 32, ++j) a[j & 7] += part[k];
-    A s = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+    for (; k + 3 * 32 < g1; k += 4 * 32) { a0 += part[k]; a1 += part[k + 32]; a2 += part[k + 64]; a3 += part[k + 96]; }
+    for (; k < g1; k += 32) a0 += part[k];                 // the < 4 remaining partials of this lane
+    A s = (a0 + a1) + (a2 + a3);
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
     return s;
+}
+// the 4 rows of a finish warp that holds a huge row, one after the other on all 32 lanes
+template <int DT, int VAR>
+__device__ __forceinline__ void finish_huge(const MainParams& P, int64_t fw, int lane) {
+    for (int q = 0; q < 4; ++q) {
+        const int64_t rq = fw * 4 + q;
+        if (rq >= P.row_long) break;
+        const auto s = long_row_sum_warp<DT>(P.partial, __ldg(P.group_ptr + rq), __ldg(P.group_ptr + rq + 1), lane);
+        if (lane == 0) store_y<DT, VAR>(P, __ldg(P.long_out + rq), s);
+    }
 }
 template <int DT, int VAR>
 __device__ __forceinline__ void finish_warp(const MainParams& P, int64_t fw, int lane) {
@@ -1151,12 +1156,7 @@ __device__ __forceinline__ void finish_warp(const MainParams& P, int64_t fw, int
         bool huge = false;
         if ((lane & 7) == 0 && r < P.row_long) huge = __ldg(P.group_ptr + r + 1) - __ldg(P.group_ptr + r) > kHugeGroups;
         if (__any_sync(FULL, huge)) {
-            for (int q = 0; q < 4; ++q) {
-                const int64_t rq = fw * 4 + q;
-                if (rq >= P.row_long) break;
-                const auto s = long_row_sum_warp<DT>(P.partial, __ldg(P.group_ptr + rq), __ldg(P.group_ptr + rq + 1), lane);
-                if (lane == 0) store_y<DT, VAR>(P, __ldg(P.long_out + rq), s);
-            }
+            finish_huge<DT, VAR>(P, fw, lane);
             return;
         }
         const auto s = long_row_sum<DT>(P.partial, P.group_ptr, r, P.row_long, lane);
