@@ -460,7 +460,8 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     p->stage_blocks = 0;
     p->stage_smem = p->stage_map_bytes = 0;
     std::vector<dasp::StageEnt> stab;
-    if (o.x_stage != 1 && p->variant == DASP_VARIANT_CUDACORE && f.arr[DASP_ARR_REG_COL].ptr && p->blocks > 0) {
+    const bool want_stage = o.x_stage == 2 || (o.x_stage == 0 && DASP_X_STAGE_AUTO);
+    if (want_stage && p->variant == DASP_VARIANT_CUDACORE && f.arr[DASP_ARR_REG_COL].ptr && p->blocks > 0) {
         int mspan = 0, mslots = 0;
         const int64_t ns = build_stage_table(f, warp_word, desc, p->rbw, p->wide_il, stab, &mspan, &mslots);
         if (ns > 0 && (o.x_stage == 2 || (DASP_X_STAGE_AUTO && 4 * ns >= p->blocks))) {
