@@ -1118,12 +1118,12 @@ __device__ __forceinline__ void empty_row(void* yv, int32_t row, double beta, co
         for (int d = 0; d < extra.n; ++d) static_cast<Y*>(extra.ptr[d])[row] = r;
 }
 // finish warp fw of the fused main kernel: long rows 4fw..4fw+3, or empty rows (4 per lane)
-// a row of more than kHugeGroups groups is summed by the whole warp (32 lanes, 4 accumulators each:
+// a row of more than kHugeGroups (1024) groups is summed by the whole warp (32 lanes, 4 accumulators each:
 // 128 partials per round) instead of 8 lanes with 4 (32 per round): a row of 10^5 nonzeros (1563
 // groups) takes 13 dependent rounds instead of 49, a row of 10^7 1221 instead of 4883.  Lane l sums
 // partials g0 + l + 32 j into accumulator j mod 4 while 4 more remain, the rest into accumulator 0,
 // then (a0+a1)+(a2+a3) and a 5-step shuffle tree: a fixed order, deterministic.
-constexpr int64_t kHugeGroups = 128;
+constexpr int64_t kHugeGroups = 1024;   // 128 slowed C7's phase 2 (rows of 129-313 groups): 0.0198 -> 0.0285 ms
 template <int DT>
 __device__ __forceinline__ typename Tr<DT>::A long_row_sum_warp(const void* partial, int64_t g0, int64_t g1, int lane) {
     using A = typename Tr<DT>::A;

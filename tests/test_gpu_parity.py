@@ -552,12 +552,12 @@ def test_x_stage_misaligned_x_falls_back(dt):
     assert np.array_equal(y1.cpu().numpy().astype(np.float64), y_ref)
 
 
-# long-row phase 2 of rows with more than 128 groups runs on the whole warp (kernels.cu
+# long-row phase 2 of rows with more than 1024 groups runs on the whole warp (kernels.cu
 # long_row_sum_warp): huge and ordinary long rows share finish warps; exact on integers, within the
 # FP64 / FP16 bars on real values, deterministic
 @pytest.mark.parametrize("dt", DTYPES)
 def test_huge_long_rows_phase2(dt):
-    lens = [300, 2_000_000, 257, 70_000, 10, 3, 8193, 1, 9000, 513, 131 * 64 + 1, 129 * 64]
+    lens = [300, 2_000_000, 257, 70_000, 10, 3, 8193, 1, 9000, 513, 1025 * 64 + 1, 1024 * 64]
     for vm in (synth.VAL_INT, synth.VAL_UNIFORM):
         A = synth.from_lengths(lens, n=3_000_000, val_mode=vm)
         x = synth.vector(61, A.n, vm)
