@@ -579,7 +579,7 @@ def run_single(args, local):
                  "nnz": {"short": info["nnz_short"], "medium": info["nnz_medium"], "long": info["nnz_long"]},
                  "fill_rate": (info["nnz_long_new"] + info["nnz_reg_new"] + info["nnz_irreg"]
                                + info["nnz_short_new"]) / max(info["nnz"], 1) - 1.0,
-                 "medium_rb_per_warp": info["medium_rb_per_warp"]},
+                 "medium_rb_per_warp": info["medium_rb_per_warp"], "x_stage_blocks": info.get("x_stage_blocks")},
     }
     print(json.dumps(line))
 
