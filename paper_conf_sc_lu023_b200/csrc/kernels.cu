@@ -906,8 +906,17 @@ __device__ __forceinline__ ShortRef short_ref(const PanelDesc* D, int64_t t) {
     return r;
 }
 // the output map: singles 4 consecutive outputs per lane; two-output tiles L and L+32; len-4 L
+#ifndef DASP_EXP_SHORT_YSEQ
+#define DASP_EXP_SHORT_YSEQ 0   // experiment only: short outputs go to consecutive y slots (no output map; wrong y)
+#endif
 __device__ __forceinline__ void short_load_out(const MainParams& P, const ShortRef& T, int lane, uint64_t pol,
                                                int32_t (&o)[4]) {
+    if (DASP_EXP_SHORT_YSEQ) {
+        const int32_t b = static_cast<int32_t>(T.obase % (1 << 23));
+        if (T.cat == 3) { for (int j = 0; j < 4; ++j) o[j] = b + lane * 4 + j; }
+        else { o[0] = b + lane; o[1] = T.cat != 1 ? b + 32 + lane : -1; o[2] = o[3] = -1; }
+        return;
+    }
     if (T.cat == 3) {
         ld4_b32(P.short_out + T.obase + lane * 4, pol, *reinterpret_cast<uint32_t(*)[4]>(&o));
     } else {
@@ -934,7 +943,8 @@ __device__ __forceinline__ void short_load_f64(const MainParams& P, const ShortR
         for (int j = 0; j < 4; ++j) {
             L.v[j] = IO::ld1r(sv + 32 * j + lane, pol);
             L.c[j] = ld1_b32(P.short_col + T.tile * 128 + 32 * j + lane, pol);
-            L.o[j] = static_cast<int32_t>(ld1_b32(P.short_out + T.obase + 32 * j + lane, pol));
+            L.o[j] = DASP_EXP_SHORT_YSEQ ? static_cast<int32_t>(T.obase % (1 << 23)) + 32 * j + lane
+                                         : static_cast<int32_t>(ld1_b32(P.short_out + T.obase + 32 * j + lane, pol));
         }
         return;
     }
