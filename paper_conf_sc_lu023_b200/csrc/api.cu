@@ -95,6 +95,9 @@ constexpr int64_t kAllocPad = dasp::kDeviceArrayPad;   // vector loads may read 
 #ifndef DASP_PACK_WARPS
 #define DASP_PACK_WARPS 1   // 1: panels' warps packed back to back in the main grid; 0: each panel padded to whole blocks
 #endif
+#ifndef DASP_HEAVY_FIRST_F16
+#define DASP_HEAVY_FIRST_F16 8   // FP16: C3 main -3.2 % (3 reps), C5 +-0 vs 16 (profiles/r02b/heavy_first_f16.jsonl)
+#endif
 #ifndef DASP_HEAVY_FIRST
 #define DASP_HEAVY_FIRST 16  // leading blocks of every panel dispatched at the start of the main grid (C3 FP16 -2.7 %, FP64 -0.1..-0.8 %, others +-0.8 %: profiles/r02/heavy_first_ab.jsonl, chunk_units_removed_and_heavy_first.jsonl)
 #endif
@@ -415,7 +418,8 @@ dasp_status_t setup_launch(dasp_plan_s* p, const dasp_options_t& o, const int64_
     // the launch.  Panels are packed back to back (DASP_PACK_WARPS) or each padded to whole blocks.
     std::vector<uint64_t> warp_word;
     {
-        const int64_t heavy = (f.n_panels > 1 ? DASP_HEAVY_FIRST : 0) * dasp::WARPS_PER_BLOCK;
+        const int64_t heavy = (f.n_panels > 1 ? (p->dtype == DASP_R_16F ? DASP_HEAVY_FIRST_F16 : DASP_HEAVY_FIRST) : 0) *
+                              dasp::WARPS_PER_BLOCK;
         auto emit = [&](int64_t q, int64_t w0, int64_t w1) {
             for (int64_t w = w0; w < w1; ++w) warp_word.push_back((static_cast<uint64_t>(q) << 32) | static_cast<uint64_t>(w));
             if (!DASP_PACK_WARPS)
