@@ -3,6 +3,8 @@ long, an occasional row of 10^4-10^5 nonzeros), rectangular shapes, banded and s
 unsorted columns and duplicate entries, random panel sizes, both compute variants, all dtypes and the
 x-window staging path -- on small integer values, so every y must equal the CPU oracle bit for bit
 ("fuzz recipe").  P:L77-93 (Alg. 1) defines y for every row whatever the class mix."""
+import os
+
 import numpy as np
 import pytest
 
@@ -15,6 +17,7 @@ pytestmark = pytest.mark.gpu
 from paper_conf_sc_lu023_b200 import dasp  # noqa: E402
 
 NP_VAL = {"f64": np.float64, "f16": np.float16, "f32": np.float32}
+N_SEEDS = int(os.environ.get("DASP_FUZZ_SEEDS", "32"))   # a longer one-off run: DASP_FUZZ_SEEDS=256
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -63,7 +66,7 @@ def random_csr(seed):
 
 
 @pytest.mark.parametrize("dt", ["f64", "f16", "f32"])
-@pytest.mark.parametrize("seed", range(32))
+@pytest.mark.parametrize("seed", range(N_SEEDS))
 def test_fuzz_bit_exact(seed, dt):
     A, rng = random_csr(seed)
     x = rng.integers(-3, 4, A.n).astype(np.float64)
